@@ -1,0 +1,411 @@
+"""bench.py -- ConcatBatch encoder forward throughput on B200 (non-pad tokens/s).
+
+Contract (driver): ``python bench.py --gpus N --steps K --warmup W [--impl reference]``;
+for N > 1 launched under torchrun, one rank per GPU.  Prints ONE JSON line on rank 0.
+
+A step = one pass of the whole hot path -- pack_embed -> S x [QKV GEMM -> segment-masked
+attention -> W_O GEMM + residual -> LN -> FFN1 + act -> FFN2 + residual -> LN] -> unpack --
+over one packed batch of B rows x L slots per GPU (BASELINE.json configs[1]: Transformer-
+base, L = 128, ParaCrawl-like lengths, bf16, B = 256 rows per GPU).  Weak scaling: each
+rank packs its own seeded request stream (seed + 1000 * rank); weights are generated on
+rank 0 and broadcast once (NCCL); there is no per-step collective.
+
+value: device time (CUDA events on the launching stream), inputs resident in HBM, the
+       forward replayed from a CUDA graph, L2 flushed (256 MiB write) between steps,
+       max over ranks; value = sum of non-pad tokens over ranks / max time.
+e2e:   the same metric through the public API from host memory: per step tcb_pack (C++),
+       H2D of the segment table + token ids from pinned memory, forward, unpack, D2H of the
+       per-request outputs [T, d] into pinned memory; host wall clock, synchronised.
+roofline: the dominant kernel (the tcgen05 GEMM class) measured live with CUDA events
+       around each launch (tcb_profile_*), algorithmic flops = 24 d^2 S T per forward.
+cpu_baseline / --impl reference: the float64 oracle (oracle/, test infrastructure) on a
+       bounded sample of the same workload, on this host's cores.
+"""
+from __future__ import annotations
+
+import argparse
+import json
+import os
+import subprocess
+import sys
+import threading
+import time
+
+import numpy as np
+
+ROOT = os.path.dirname(os.path.abspath(__file__))
+sys.path.insert(0, ROOT)
+
+import tcb_workload as wl  # noqa: E402
+
+METRIC = "non-pad tokens/s, ConcatBatch encoder fwd at 1/2/4/8 B200; % TC peak"
+UNIT = "tokens/s"
+
+
+def _peaks():
+    try:
+        return json.load(open(os.path.join(ROOT, "MEASURED_PEAKS.json"))), "measured"
+    except Exception:
+        return {"hbm_gbs": 6650.0, "bf16_tflops": 1590.0, "bf16_tflops_sustained": 1400.0,
+                "sm_max_mhz": 1965.0}, "fallback"
+
+
+class ClockSampler:
+    """nvidia-smi clocks / throttle reasons sampled during the timed region."""
+
+    Q = ("index,clocks.sm,clocks.max.sm,power.draw,clocks_event_reasons.active,"
+         "clocks_event_reasons.hw_slowdown,clocks_event_reasons.hw_thermal_slowdown,"
+         "clocks_event_reasons.sw_thermal_slowdown,clocks_event_reasons.sw_power_cap")
+
+    def __init__(self, gpu: int):
+        self.gpu = gpu
+        self.rows = []
+        self._stop = threading.Event()
+        self._t = None
+
+    def _run(self):
+        while not self._stop.is_set():
+            try:
+                out = subprocess.run(["nvidia-smi", "-i", str(self.gpu),
+                                      f"--query-gpu={self.Q}", "--format=csv,noheader,nounits"],
+                                     capture_output=True, text=True, timeout=5).stdout
+                for line in out.strip().splitlines():
+                    self.rows.append([x.strip() for x in line.split(",")])
+            except Exception:
+                pass
+            self._stop.wait(0.2)
+
+    def __enter__(self):
+        self._t = threading.Thread(target=self._run, daemon=True)
+        self._t.start()
+        return self
+
+    def __exit__(self, *a):
+        self._stop.set()
+        if self._t:
+            self._t.join(timeout=10)
+
+    def summary(self):
+        if not self.rows:
+            return {"sm_mhz": None, "sm_max_mhz": None, "reasons": ["nvidia-smi unavailable"],
+                    "samples": 0}
+        sm = [float(r[1]) for r in self.rows if r[1].replace(".", "").isdigit()]
+        mx = [float(r[2]) for r in self.rows if r[2].replace(".", "").isdigit()]
+        names = ["hw_slowdown", "hw_thermal_slowdown", "sw_thermal_slowdown", "sw_power_cap"]
+        reasons = sorted({names[i] for r in self.rows for i in range(4)
+                          if len(r) > 5 + i and r[5 + i].lower() == "active"})
+        pw = [float(r[3]) for r in self.rows if r[3].replace(".", "").isdigit()]
+        return {"sm_mhz": float(np.median(sm)) if sm else None,
+                "sm_max_mhz": max(mx) if mx else None, "reasons": reasons,
+                "power_w_max": max(pw) if pw else None, "samples": len(self.rows)}
+
+
+def make_batches(key: str, rank: int, nbatches: int):
+    """Seeded packed batches for this rank: (lengths, ids) filling B rows of L slots."""
+    wlc = wl.WORKLOADS[key]
+    out = []
+    for b in range(nbatches):
+        seed = wlc.seeds[0] + 1000 * rank + 97 * b
+        lengths = wl.lengths_filling(wlc.lengths, wlc.rows, wlc.row_len, seed, 0.995)
+        ids = wl.draw_token_ids(int(lengths.sum()), wlc.model.vocab, wlc.seeds[1] + 1000 * rank + 97 * b)
+        out.append((lengths, ids))
+    return out
+
+
+def cpu_oracle_sample(key: str, lengths, ids, weights, budget_s: float = 12.0, max_rows=16):
+    """Time the f64 oracle (as it stands) row by row on this host until ~budget_s."""
+    import oracle
+    wlc = wl.WORKLOADS[key]
+    model = wlc.model
+    names = wl.weight_names(model)
+    pk = oracle.pack(lengths, wlc.row_len, wlc.rows)
+    lay = oracle.layout(lengths, pk["req_row"], pk["req_col"], pk["num_rows"], wlc.row_len)
+    seg = lay["segment_ids"]
+    L = wlc.row_len
+    tokens, elapsed, rows = 0, 0.0, 0
+    while elapsed < budget_s and rows < min(max_rows, pk["num_rows"]):
+        t0 = time.perf_counter()
+        oracle.encoder_rows(model, weights, names, ids, lay, L, [rows])
+        elapsed += time.perf_counter() - t0
+        tokens += int(np.sum(seg[rows * L:(rows + 1) * L] >= 0))
+        rows += 1
+    cores = len(os.sched_getaffinity(0)) if hasattr(os, "sched_getaffinity") else os.cpu_count()
+    return {"value": tokens / elapsed, "unit": UNIT, "cores": int(os.environ.get("OMP_NUM_THREADS", cores)),
+            "kind": "oracle",
+            "sample": f"first {rows} packed rows ({tokens} non-pad tokens) of the rank-0 batch, "
+                      f"{model.name} L={L}, float64, {elapsed:.1f} s"}
+
+
+def run_reference(args):
+    """--impl reference: the f64 oracle timed as it stands, rank 0 only."""
+    rank = int(os.environ.get("RANK", 0))
+    world = int(os.environ.get("WORLD_SIZE", 1))
+    if rank != 0:
+        return 0
+    key = args.workload
+    wlc = wl.WORKLOADS[key]
+    (lengths, ids), = make_batches(key, 0, 1)
+    weights = wl.draw_weights(wlc.model, wlc.seeds[2])
+    import oracle
+    names = wl.weight_names(wlc.model)
+    pk = oracle.pack(lengths, wlc.row_len, wlc.rows)
+    lay = oracle.layout(lengths, pk["req_row"], pk["req_col"], pk["num_rows"], wlc.row_len)
+    L = wlc.row_len
+    seg = lay["segment_ids"]
+    # each step: a bounded sample (one packed row) of the workload
+    def step(i):
+        r = i % pk["num_rows"]
+        oracle.encoder_rows(wlc.model, weights, names, ids, lay, L, [r])
+        return int(np.sum(seg[r * L:(r + 1) * L] >= 0))
+    for i in range(args.warmup):
+        step(i)
+    toks, t0 = 0, time.perf_counter()
+    for i in range(args.steps):
+        toks += step(args.warmup + i)
+    el = time.perf_counter() - t0
+    v = toks / el
+    cores = len(os.sched_getaffinity(0)) if hasattr(os, "sched_getaffinity") else os.cpu_count()
+    line = {"metric": METRIC, "value": v, "unit": UNIT, "n_gpus": world, "steps": args.steps,
+            "warmup": args.warmup, "ms_per_step": 1e3 * el / max(args.steps, 1),
+            "higher_is_better": True, "scaling": "weak", "vs_baseline": None, "dtype": "f64",
+            "data": "synthetic", "impl": "reference",
+            "config": {"workload": wlc.name, "model": wlc.model.name, "row_len": L,
+                       "rows_per_gpu": wlc.rows, "sample_per_step": "one packed row"},
+            "cpu_baseline": {"value": v, "unit": UNIT, "cores": cores, "kind": "oracle",
+                             "sample": "one packed row per step of the rank-0 batch"},
+            "e2e": {"value": v, "unit": UNIT, "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0}}
+    print(json.dumps(line), flush=True)
+    return 0
+
+
+def main():
+    ap = argparse.ArgumentParser()
+    ap.add_argument("--gpus", type=int, default=1)
+    ap.add_argument("--steps", type=int, default=20)
+    ap.add_argument("--warmup", type=int, default=5)
+    ap.add_argument("--impl", default="ours", choices=["ours", "reference"])
+    ap.add_argument("--workload", default="c2", choices=sorted(wl.WORKLOADS))
+    ap.add_argument("--no-cpu-baseline", action="store_true")
+    ap.add_argument("--no-graph", action="store_true")
+    args = ap.parse_args()
+    args.warmup = max(args.warmup, 3)
+    if args.impl == "reference":
+        return run_reference(args)
+
+    import torch
+    import torch.distributed as dist
+
+    import paper_conf_icpp_fuc0z22_b200 as tcb
+    from paper_conf_icpp_fuc0z22_b200 import dist as tdist
+
+    rank, world = tdist.init("nccl")
+    local = int(os.environ.get("LOCAL_RANK", 0))
+    torch.cuda.set_device(local)
+    dev = torch.device("cuda", local)
+    key = args.workload
+    wlc = wl.WORKLOADS[key]
+    model = wlc.model
+    names = wl.weight_names(model)
+    L, B = wlc.row_len, wlc.rows
+
+    # weights: drawn on rank 0, one NCCL broadcast of the flat buffers
+    weights_np = wl.draw_weights(model, wlc.seeds[2]) if rank == 0 else None
+    views = tdist.broadcast_weights(model, names, weights_np, dev)
+    enc = tcb.Encoder(model, None, names, device=str(dev), tensors=views)
+
+    batches = make_batches(key, rank, 4)
+    plans = [tcb.tcb_pack(l, L, B) for l, _ in batches]
+    plan = plans[0]
+    info = plan.info
+    M = info["num_slots"]
+    assert info["num_rows"] == B, info
+    tokens_rank = info["placed_tokens"]
+    d_segtab = torch.from_numpy(plan.segtab()).to(dev)
+    d_ids = torch.from_numpy(batches[0][1]).to(dev)
+    rows = enc.alloc_rows(M)
+    out = torch.empty((info["total_tokens"], model.d_model), dtype=enc.dtype, device=dev)
+    stream = torch.cuda.Stream(device=dev)
+    flush = torch.empty(256 * 1024 * 1024, dtype=torch.uint8, device=dev)
+
+    def fwd():
+        enc.encoder_forward(plan, d_segtab, d_ids, rows, stream=stream)
+        enc.unpack(plan, d_segtab, rows, out, stream=stream)
+
+    # launches per step (counted from the library's own counter on one eager step)
+    c0 = tcb.launch_count()
+    with torch.cuda.stream(stream):
+        fwd()
+    stream.synchronize()
+    launches_per_step = tcb.launch_count() - c0
+
+    graph = None
+    if not args.no_graph:
+        with torch.cuda.stream(stream):
+            fwd()
+        stream.synchronize()
+        graph = torch.cuda.CUDAGraph()
+        with torch.cuda.graph(graph, stream=stream):
+            fwd()
+
+    def step():
+        if graph is not None:
+            graph.replay()
+        else:
+            fwd()
+
+    with torch.cuda.stream(stream):
+        for _ in range(args.warmup):
+            step()
+    stream.synchronize()
+
+    # ---- timed region: device time, L2 flushed between steps -----------------------------
+    ev = [(torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True))
+          for _ in range(args.steps)]
+    if world > 1:
+        dist.barrier()
+    torch.cuda.synchronize()
+    with ClockSampler(local) as clk:
+        with torch.cuda.stream(stream):
+            for i in range(args.steps):
+                flush.zero_()
+                ev[i][0].record(stream)
+                step()
+                ev[i][1].record(stream)
+        torch.cuda.synchronize()
+    if world > 1:
+        dist.barrier()
+    ms = sum(a.elapsed_time(b) for a, b in ev)
+    t_local = torch.tensor([ms, float(tokens_rank)], dtype=torch.float64, device=dev)
+    if world > 1:
+        tmax = t_local.clone()
+        dist.all_reduce(tmax, op=dist.ReduceOp.MAX)
+        tsum = t_local.clone()
+        dist.all_reduce(tsum, op=dist.ReduceOp.SUM)
+        ms_max, tokens_all = float(tmax[0]), float(tsum[1])
+    else:
+        ms_max, tokens_all = ms, float(tokens_rank)
+    value = tokens_all * args.steps / (ms_max / 1e3)
+    ms_per_step = ms_max / args.steps
+
+    # ---- roofline: per-kernel-class CUDA-event durations over K eager steps ----------------
+    tcb.profile_enable(True)
+    with torch.cuda.stream(stream):
+        for _ in range(args.steps):
+            flush.zero_()
+            fwd()
+    stream.synchronize()
+    prof = tcb.profile_collect()
+    tcb.profile_enable(False)
+    peaks, peak_src = _peaks()
+    d, S = model.d_model, model.num_layers
+    gemm_cls = ["gemm_qkv", "gemm_o", "gemm_ffn1", "gemm_ffn2"]
+    gemm_ms = sum(prof[c][0] for c in gemm_cls) / args.steps
+    gemm_launches = sum(prof[c][1] for c in gemm_cls) / args.steps
+    total_prof_ms = sum(v[0] for v in prof.values()) / args.steps
+    gemm_flops = 2.0 * tokens_rank * S * (3 * d * d + d * d + 2 * d * model.d_ff)
+    attn_flops = 4.0 * d * S * info["useful_score_elems"]
+    achieved_tf = gemm_flops / (gemm_ms / 1e3) / 1e12
+    peak_tf = peaks.get("bf16_tflops_sustained", peaks["bf16_tflops"])
+    traffic = None
+    tpath = os.path.join(ROOT, "profiles", "traffic.json")
+    if os.path.exists(tpath):
+        try:
+            traffic = json.load(open(tpath)).get(key, {}).get("gemm_dram_bytes_per_launch")
+        except Exception:
+            traffic = None
+    roofline = {"bound": "tensor", "kernel": "linear_tc_kernel (tcgen05 GEMMs: QKV, W_O, FFN1, FFN2)",
+                "achieved": achieved_tf, "peak": peak_tf, "unit": "TFLOP/s",
+                "frac": achieved_tf / peak_tf, "traffic": traffic,
+                "peak_source": f"{peak_src} bf16_tflops_sustained (kernel timed inside a long step)",
+                "frac_of_burst_peak": achieved_tf / peaks["bf16_tflops"],
+                "gemm_share_of_step": gemm_ms / total_prof_ms if total_prof_ms else None,
+                "launches_per_step": gemm_launches,
+                "per_class_ms_per_step": {k: v[0] / args.steps for k, v in prof.items()}}
+    whole_tc = (gemm_flops + attn_flops) / (ms_per_step / 1e3) / 1e12
+
+    # ---- e2e: public API from host memory, every step -------------------------------------
+    pinned_ids = [torch.from_numpy(i).pin_memory() for _, i in batches]
+    out_host = torch.empty((max(p.info["total_tokens"] for p in plans), model.d_model),
+                           dtype=enc.dtype).pin_memory()
+    e2e_rows = enc.alloc_rows(M)
+    e2e_ids = torch.empty(max(len(i) for _, i in batches), dtype=torch.int32, device=dev)
+    e2e_seg = torch.empty(max(p.segtab().size for p in plans), dtype=torch.int32, device=dev)
+    e2e_out = torch.empty((out_host.shape[0], model.d_model), dtype=enc.dtype, device=dev)
+    seg_pin = torch.empty(e2e_seg.numel(), dtype=torch.int32).pin_memory()
+    h2d = d2h = 0
+
+    def e2e_step(i):
+        nonlocal h2d, d2h
+        lengths, ids = batches[i % len(batches)]
+        p = tcb.tcb_pack(lengths, L, B)                         # host packer (C++)
+        st = p.segtab()
+        seg_pin[:st.size].copy_(torch.from_numpy(st))
+        with torch.cuda.stream(stream):
+            e2e_seg[:st.size].copy_(seg_pin[:st.size], non_blocking=True)
+            e2e_ids[:len(ids)].copy_(pinned_ids[i % len(batches)], non_blocking=True)
+            enc.encoder_forward(p, e2e_seg, e2e_ids, e2e_rows, stream=stream)
+            T = p.info["total_tokens"]
+            enc.unpack(p, e2e_seg, e2e_rows, e2e_out, stream=stream)
+            out_host[:T].copy_(e2e_out[:T], non_blocking=True)
+        stream.synchronize()
+        h2d += st.size * 4 + len(ids) * 4
+        d2h += T * model.d_model * e2e_out.element_size()
+
+    for i in range(args.warmup):
+        e2e_step(i)
+    h2d = d2h = 0
+    if world > 1:
+        dist.barrier()
+    t0 = time.perf_counter()
+    for i in range(args.steps):
+        e2e_step(i)
+    e2e_s = time.perf_counter() - t0
+    e2e_t = torch.tensor([e2e_s], dtype=torch.float64, device=dev)
+    if world > 1:
+        dist.all_reduce(e2e_t, op=dist.ReduceOp.MAX)
+    e2e_tokens = sum(plans[i % len(plans)].info["placed_tokens"] for i in range(args.steps))
+    e2e_value = e2e_tokens * world / float(e2e_t[0])
+
+    cpu = None
+    if rank == 0 and world == 1 and not args.no_cpu_baseline:
+        cpu = cpu_oracle_sample(key, batches[0][0], batches[0][1],
+                                wl.draw_weights(model, wlc.seeds[2]))
+
+    if rank == 0:
+        line = {
+            "metric": METRIC, "value": value, "unit": UNIT, "n_gpus": world,
+            "steps": args.steps, "warmup": args.warmup, "ms_per_step": ms_per_step,
+            "higher_is_better": True, "scaling": "weak", "vs_baseline": None, "dtype": "bf16",
+            "data": "synthetic (seeded ParaCrawl-like lengths, random-init weights)",
+            "config": {"workload": wlc.name, "model": model.name, "layers": S, "d_model": d,
+                       "heads": model.num_heads, "d_ff": model.d_ff, "row_len": L,
+                       "rows_per_gpu": B, "global_batch_rows": B * world,
+                       "non_pad_tokens_per_gpu": tokens_rank,
+                       "padding_fraction": 1.0 - tokens_rank / M,
+                       "attention_tiles_skipped_128": 1.0 - info["kv_tiles_visited"] / info["kv_tiles_dense"]
+                       if info["kv_tiles_dense"] > 0 else None,
+                       "attention_score_elems_executed_vs_dense": info["executed_score_elems"] / (B * L * L),
+                       "attention_useful_fraction_of_executed": info["useful_score_elems"] / max(info["executed_score_elems"], 1),
+                       "parallelism": f"dp{world} (rows sharded, weights broadcast once)",
+                       "l2": "flushed (256 MiB write) between timed steps",
+                       "cuda_graph": graph is not None},
+            "tc_frac_whole_step": whole_tc / peaks["bf16_tflops"],
+            "tc_whole_step_tflops": whole_tc,
+            "gpu_launches": int(launches_per_step * args.steps),
+            "roofline": roofline,
+            "e2e": {"value": e2e_value, "unit": UNIT, "h2d_bytes_per_step": h2d // args.steps,
+                    "d2h_bytes_per_step": d2h // args.steps,
+                    "path": "tcb_pack + pinned H2D + tcb_encoder_forward + tcb_unpack + D2H, sync per step"},
+            "clocks": clk.summary(),
+            "cpu_baseline": cpu,
+            "paper_context": "paper reports only end-to-end serving on 1x V100 (<~4e3 tok/s incl. decoder); no encoder tokens/s",
+        }
+        print(json.dumps(line), flush=True)
+    if world > 1:
+        dist.barrier()
+        dist.destroy_process_group()
+    return 0
+
+
+if __name__ == "__main__":
+    sys.exit(main())

@@ -1,0 +1,247 @@
+"""B200-native ConcatBatching encoder (TCB, Fu et al., ICPP'22) -- Python binding.
+
+Thin layer over libtcb.so (include/tcb.h): PyTorch supplies device memory and streams;
+every step of the path (pack_embed, tcgen05 GEMMs, segment-masked attention, LayerNorm,
+unpack) runs in the library's sm_100a kernels.  Names follow the C ABI:
+
+    plan = tcb_pack(lengths, row_len, max_rows, policy)          # host, C++
+    enc  = Encoder(model_cfg, weights)                           # device weights
+    rows = enc.encoder_forward(plan, d_segtab, d_token_ids)      # [B*L, d] on the GPU
+    out  = enc.unpack(plan, d_segtab, rows)                      # [total_tokens, d]
+"""
+from __future__ import annotations
+
+import ctypes
+from typing import Dict, Optional, Sequence
+
+import numpy as np
+
+from . import _lib
+from ._lib import KCLASSES, POLICIES, TcbError, check, lib
+
+__all__ = ["Plan", "Encoder", "tcb_pack", "op_linear", "op_attention", "op_layernorm",
+           "launch_count", "profile_enable", "profile_collect", "TcbError", "KCLASSES"]
+
+_DTYPES = {"fp32": 0, "bf16": 1}
+_ACTS = {"gelu": 0, "relu": 1}
+_PES = {"sin_paper": 0, "sin_vaswani": 1, "learned": 2}
+_VEC_WEIGHTS = ("type_emb", "emb_ln_g", "emb_ln_b", "b_qkv", "b_o", "ln1_g", "ln1_b", "b_1",
+                "b_2", "ln2_g", "ln2_b")
+
+
+def _ptr(a) -> ctypes.c_void_p:
+    if a is None:
+        return None
+    if isinstance(a, np.ndarray):
+        return a.ctypes.data_as(ctypes.c_void_p)
+    return ctypes.c_void_p(a.data_ptr())  # torch tensor
+
+
+def _stream_ptr(stream) -> ctypes.c_void_p:
+    if stream is None:
+        import torch
+        stream = torch.cuda.current_stream()
+    return ctypes.c_void_p(stream.cuda_stream)
+
+
+class Plan:
+    """A packed batch (host): row assignment + segment table.  Wraps tcb_plan*."""
+
+    def __init__(self, handle: ctypes.c_void_p):
+        self._h = handle
+        info = _lib.PlanInfo()
+        check(lib().tcb_plan_info_get(self._h, ctypes.byref(info)))
+        self.info = info.as_dict()
+
+    def __del__(self):
+        h, self._h = getattr(self, "_h", None), None
+        if h and _lib._lib is not None:
+            _lib._lib.tcb_plan_destroy(h)
+
+    @property
+    def handle(self):
+        return self._h
+
+    @property
+    def num_slots(self) -> int:
+        return self.info["num_slots"]
+
+    def arrays(self) -> Dict[str, np.ndarray]:
+        i = self.info
+        n, S, M, Q = i["num_requests"], i["num_segments"], i["num_slots"], i["qtiles"]
+        out = {"req_row": np.zeros(max(n, 1), np.int32), "req_col": np.zeros(max(n, 1), np.int32),
+               "seg_req": np.zeros(max(S, 1), np.int32), "seg_start": np.zeros(max(S, 1), np.int32),
+               "cu_seqlens": np.zeros(S + 1, np.int32),
+               "segment_ids": np.zeros(max(M, 1), np.int32),
+               "positions": np.zeros(max(M, 1), np.int32),
+               "qtile_kv": np.zeros(max(2 * Q, 1), np.int32)}
+        check(lib().tcb_plan_copy(self._h, *[_ptr(out[k]) for k in (
+            "req_row", "req_col", "seg_req", "seg_start", "cu_seqlens", "segment_ids",
+            "positions", "qtile_kv")]))
+        out["req_row"], out["req_col"] = out["req_row"][:n], out["req_col"][:n]
+        out["seg_req"], out["seg_start"] = out["seg_req"][:S], out["seg_start"][:S]
+        out["segment_ids"], out["positions"] = out["segment_ids"][:M], out["positions"][:M]
+        out["qtile_kv"] = out["qtile_kv"][:2 * Q].reshape(Q, 2)
+        return out
+
+    def segtab(self) -> np.ndarray:
+        """The device form of the plan (int32 words; copy it to the GPU as-is)."""
+        words = int(lib().tcb_plan_segtab_words(self._h))
+        buf = np.zeros(words, np.int32)
+        check(lib().tcb_plan_write_segtab(self._h, _ptr(buf), words))
+        return buf
+
+
+def tcb_pack(lengths: Sequence[int], row_len: int, max_rows: int = 0,
+             policy: str = "first_fit") -> Plan:
+    """Assign requests to rows (C++ packer).  See include/tcb.h tcb_pack."""
+    arr = np.ascontiguousarray(np.asarray(lengths, dtype=np.int32))
+    h = ctypes.c_void_p()
+    check(lib().tcb_pack(_ptr(arr) if len(arr) else None, len(arr), int(row_len),
+                         int(max_rows), POLICIES[policy], ctypes.byref(h)))
+    return Plan(h)
+
+
+def launch_count() -> int:
+    return int(lib().tcb_launch_count())
+
+
+def profile_enable(on: bool) -> None:
+    check(lib().tcb_profile_enable(1 if on else 0))
+
+
+def profile_collect() -> Dict[str, tuple]:
+    ms = np.zeros(len(KCLASSES), np.float64)
+    n = np.zeros(len(KCLASSES), np.int64)
+    check(lib().tcb_profile_collect(_ptr(ms), _ptr(n)))
+    return {k: (float(ms[i]), int(n[i])) for i, k in enumerate(KCLASSES)}
+
+
+class Encoder:
+    """Device weights + workspace for one model config; runs the C-ABI device calls.
+
+    ``model`` is any object with tcb_workload.ModelConfig attributes; ``weights`` maps the
+    canonical names (tcb_workload.weight_names) to fp32 numpy arrays (already rounded to
+    bf16 values for bf16 models).  Matrices are uploaded in the model dtype, vectors fp32.
+    """
+
+    def __init__(self, model, weights: Dict[str, np.ndarray], names: Sequence[str],
+                 device: str = "cuda", tensors: Optional[list] = None):
+        import torch
+        self.model = model
+        self.device = torch.device(device)
+        self.dtype = torch.float32 if model.dtype == "fp32" else torch.bfloat16
+        self.cfg = _lib.ModelConfig(model.num_layers, model.d_model, model.num_heads,
+                                    model.d_ff, model.vocab, model.max_pos, _DTYPES[model.dtype],
+                                    _ACTS[model.act], _PES[model.pe], int(model.emb_ln),
+                                    int(model.use_type_emb), model.ln_eps, model.emb_ln_eps,
+                                    model.emb_scale)
+        if tensors is None:
+            tensors = []
+            for n in names:
+                base = n.split(".")[-1]
+                dt = torch.float32 if base in _VEC_WEIGHTS else self.dtype
+                tensors.append(torch.from_numpy(np.ascontiguousarray(weights[n]))
+                               .to(device=self.device, dtype=dt).contiguous())
+        self.tensors = tensors
+        ptrs = (ctypes.c_void_p * len(tensors))(*[t.data_ptr() for t in tensors])
+        h = ctypes.c_void_p()
+        check(lib().tcb_weights_create(ctypes.byref(self.cfg), ptrs, len(tensors),
+                                       ctypes.byref(h)))
+        self._h = h
+        self._ws = None
+
+    @staticmethod
+    def weight_dtypes(model, names):
+        """(name, is_matrix) for each canonical tensor (used by the broadcast runtime)."""
+        return [(n, n.split(".")[-1] not in _VEC_WEIGHTS) for n in names]
+
+    def __del__(self):
+        h, self._h = getattr(self, "_h", None), None
+        if h and _lib._lib is not None:
+            _lib._lib.tcb_weights_destroy(h)
+
+    def workspace_bytes(self, num_slots: int) -> int:
+        b = ctypes.c_size_t(0)
+        check(lib().tcb_workspace_size(ctypes.byref(self.cfg), int(num_slots), ctypes.byref(b)))
+        return int(b.value)
+
+    def workspace(self, num_slots: int):
+        import torch
+        need = self.workspace_bytes(num_slots)
+        if self._ws is None or self._ws.numel() < need:
+            self._ws = torch.empty(need, dtype=torch.uint8, device=self.device)
+        return self._ws
+
+    def alloc_rows(self, num_slots: int):
+        import torch
+        return torch.empty((num_slots, self.model.d_model), dtype=self.dtype, device=self.device)
+
+    def embed(self, plan: Plan, d_segtab, d_ids, rows, d_seg=None, d_pos=None, stream=None):
+        check(lib().tcb_embed(self._h, plan.handle, _ptr(d_segtab), _ptr(d_ids), _ptr(rows),
+                              _ptr(d_seg), _ptr(d_pos), _stream_ptr(stream)))
+        return rows
+
+    def encoder_forward(self, plan: Plan, d_segtab, d_ids, rows=None, stream=None):
+        M = plan.num_slots
+        if rows is None:
+            rows = self.alloc_rows(M)
+        ws = self.workspace(M)
+        check(lib().tcb_encoder_forward(self._h, plan.handle, _ptr(d_segtab), _ptr(d_ids),
+                                        _ptr(rows), _ptr(ws), ws.numel(), _stream_ptr(stream)))
+        return rows
+
+    def unpack(self, plan: Plan, d_segtab, rows, out=None, stream=None):
+        import torch
+        if out is None:
+            out = torch.zeros((plan.info["total_tokens"], self.model.d_model), dtype=self.dtype,
+                              device=self.device)
+        check(lib().tcb_unpack(self._h, plan.handle, _ptr(d_segtab), _ptr(rows), _ptr(out),
+                               _stream_ptr(stream)))
+        return out
+
+    def run(self, lengths, token_ids, row_len: int, max_rows: int = 0,
+            policy: str = "first_fit"):
+        """Host arrays in, device outputs out: pack -> H2D -> forward -> unpack."""
+        import torch
+        plan = tcb_pack(lengths, row_len, max_rows, policy)
+        d_segtab = torch.from_numpy(plan.segtab()).to(self.device)
+        d_ids = torch.from_numpy(np.ascontiguousarray(token_ids, dtype=np.int32)).to(self.device)
+        rows = self.encoder_forward(plan, d_segtab, d_ids)
+        out = self.unpack(plan, d_segtab, rows)
+        return plan, rows, out
+
+
+def op_linear(A, W, bias, R=None, epilogue: str = "bias", out=None, stream=None):
+    import torch
+    M, K = A.shape
+    N = W.shape[0]
+    if out is None:
+        out = torch.empty((M, N), dtype=A.dtype, device=A.device)
+    dt = 0 if A.dtype == torch.float32 else 1
+    check(lib().tcb_op_linear(dt, M, N, K, _ptr(A), _ptr(W), _ptr(bias), _ptr(R),
+                              _lib.EPILOGUES[epilogue], _ptr(out), _stream_ptr(stream)))
+    return out
+
+
+def op_attention(qkv, seg_ids, d_segtab, num_heads: int, out=None, stream=None):
+    import torch
+    M, three_d = qkv.shape
+    d = three_d // 3
+    if out is None:
+        out = torch.empty((M, d), dtype=qkv.dtype, device=qkv.device)
+    dt = 0 if qkv.dtype == torch.float32 else 1
+    check(lib().tcb_op_attention(dt, M, d, num_heads, _ptr(qkv), _ptr(seg_ids), _ptr(d_segtab),
+                                 _ptr(out), _stream_ptr(stream)))
+    return out
+
+
+def op_layernorm(Z, g, b, eps: float, seg_ids=None, out=None, stream=None):
+    import torch
+    rows, d = Z.shape
+    if out is None:
+        out = torch.empty_like(Z)
+    dt = 0 if Z.dtype == torch.float32 else 1
+    check(lib().tcb_op_layernorm(dt, rows, d, _ptr(Z), _ptr(g), _ptr(b), float(eps),
+                                 _ptr(seg_ids), _ptr(out), _stream_ptr(stream)))
+    return out

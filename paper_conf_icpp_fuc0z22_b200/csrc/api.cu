@@ -1,0 +1,501 @@
+// api.cu -- the device half of the libtcb C ABI (include/tcb.h, include/tcb_ops.h):
+// weights handle, workspace layout, tcb_embed / tcb_encoder_forward / tcb_unpack, the
+// op-level entry points and the launch/profiling instrumentation.  Host code only; every
+// arithmetic step runs in the kernels of elementwise.cu, linear_tc.cu, linear_f32.cu and
+// attention.cu.  There is no CPU fallback: without an sm_100 device every device call
+// returns TCB_ERR_NO_DEVICE.
+#include <cuda.h>
+#include <cuda_runtime.h>
+
+#include <atomic>
+#include <cstdlib>
+#include <cstring>
+#include <mutex>
+#include <new>
+#include <string>
+#include <vector>
+
+#include "kernels.h"
+#include "tcb_internal.h"
+
+using tcb::fail;
+
+namespace {
+
+std::atomic<int64_t> g_launches{0};
+
+// ---- profiling: CUDA event pairs around each launch ----------------------------------------
+struct ProfRec {
+  int cls;
+  cudaEvent_t a, b;
+};
+std::mutex g_prof_mu;
+bool g_prof_on = false;
+std::vector<ProfRec> g_prof;
+std::vector<cudaEvent_t> g_event_pool;
+
+cudaEvent_t pool_event() {
+  if (!g_event_pool.empty()) {
+    cudaEvent_t e = g_event_pool.back();
+    g_event_pool.pop_back();
+    return e;
+  }
+  cudaEvent_t e = nullptr;
+  cudaEventCreate(&e);
+  return e;
+}
+
+struct ProfScope {
+  bool on;
+  int cls;
+  cudaStream_t s;
+  cudaEvent_t a = nullptr, b = nullptr;
+  ProfScope(int c, cudaStream_t st) : on(false), cls(c), s(st) {
+    std::lock_guard<std::mutex> g(g_prof_mu);
+    if (!g_prof_on) return;
+    on = true;
+    a = pool_event();
+    b = pool_event();
+    cudaEventRecord(a, s);
+  }
+  ~ProfScope() {
+    if (!on) return;
+    cudaEventRecord(b, s);
+    std::lock_guard<std::mutex> g(g_prof_mu);
+    g_prof.push_back({cls, a, b});
+  }
+};
+
+tcb_status cuda_fail(cudaError_t e, const char* what) {
+  return fail(TCB_ERR_CUDA, std::string(what) + ": " + cudaGetErrorString(e));
+}
+
+#define TCB_LAUNCH(cls, stream, expr)                                 \
+  do {                                                                \
+    ProfScope _ps((cls), (stream));                                   \
+    cudaError_t _e = (expr);                                          \
+    g_launches.fetch_add(1, std::memory_order_relaxed);               \
+    if (_e != cudaSuccess) return cuda_fail(_e, #expr);               \
+  } while (0)
+
+tcb_status check_device() {
+  int n = 0;
+  if (cudaGetDeviceCount(&n) != cudaSuccess || n == 0) {
+    cudaGetLastError();
+    return fail(TCB_ERR_NO_DEVICE, "no CUDA device visible (libtcb has no CPU fallback)");
+  }
+  int dev = 0, major = 0;
+  cudaGetDevice(&dev);
+  cudaDeviceGetAttribute(&major, cudaDevAttrComputeCapabilityMajor, dev);
+  if (major != 10)
+    return fail(TCB_ERR_NO_DEVICE, "libtcb is built for sm_100a (B200); device has major " +
+                                       std::to_string(major));
+  return TCB_OK;
+}
+
+constexpr size_t align256(size_t x) { return (x + 255) & ~static_cast<size_t>(255); }
+
+struct WsLayout {
+  size_t seg, qkv, att, z, x1, h, total;
+};
+WsLayout ws_layout(const tcb_model_config& c, int64_t M) {
+  const size_t es = c.dtype == 0 ? 4 : 2;
+  WsLayout L{};
+  size_t off = 0;
+  L.seg = off; off += align256(sizeof(int32_t) * static_cast<size_t>(M));
+  L.qkv = off; off += align256(es * static_cast<size_t>(M) * 3 * c.d_model);
+  L.att = off; off += align256(es * static_cast<size_t>(M) * c.d_model);
+  L.z = off;   off += align256(es * static_cast<size_t>(M) * c.d_model);
+  L.x1 = off;  off += align256(es * static_cast<size_t>(M) * c.d_model);
+  L.h = off;   off += align256(es * static_cast<size_t>(M) * c.d_ff);
+  L.total = off;
+  return L;
+}
+
+tcb_status validate_cfg(const tcb_model_config* c) {
+  if (!c) return fail(TCB_ERR_INVALID_ARGUMENT, "config is NULL");
+  if (c->num_layers < 0 || c->d_model <= 0 || c->num_heads <= 0 || c->d_ff <= 0 ||
+      c->vocab <= 0 || c->max_pos <= 0 || (c->dtype != 0 && c->dtype != 1) ||
+      (c->act != 0 && c->act != 1) || c->pe < 0 || c->pe > 2)
+    return fail(TCB_ERR_INVALID_ARGUMENT, "invalid model config field");
+  if (c->d_model % c->num_heads != 0)
+    return fail(TCB_ERR_UNSUPPORTED, "d_model % num_heads != 0");
+  const int dh = c->d_model / c->num_heads;
+  if (c->dtype == 1) {
+    if (dh != 64 || c->d_model % 64 != 0 || c->d_ff % 64 != 0 || c->d_model > 2048)
+      return fail(TCB_ERR_UNSUPPORTED,
+                  "bf16 path needs d_head == 64, d_model % 64 == 0, d_ff % 64 == 0, d_model <= 2048");
+  } else {
+    if (dh > 64 || dh % 2 != 0 || c->d_model % 4 != 0 || c->d_model > 1024)
+      return fail(TCB_ERR_UNSUPPORTED,
+                  "fp32 path needs d_head <= 64 and even, d_model % 4 == 0, d_model <= 1024");
+  }
+  return TCB_OK;
+}
+
+}  // namespace
+
+struct tcb_weights {
+  tcb_model_config cfg{};
+  std::vector<const void*> t;
+  float* pe_table = nullptr;
+  struct LayerMaps {
+    CUtensorMap qkv, o, w1, w2;
+  };
+  std::vector<LayerMaps> maps;
+  // activation TMA descriptors, rebuilt when the (rows, workspace) pointers change
+  std::mutex mu;
+  const void* c_rows = nullptr;
+  const void* c_ws = nullptr;
+  int64_t c_M = -1;
+  CUtensorMap mX{}, mAtt{}, mX1{}, mH{};
+
+  const void* tok_emb() const { return t[0]; }
+  const void* pos_emb() const { return t[1]; }
+  const float* type_emb() const { return static_cast<const float*>(t[2]); }
+  const float* emb_ln_g() const { return static_cast<const float*>(t[3]); }
+  const float* emb_ln_b() const { return static_cast<const float*>(t[4]); }
+  const void* L(int layer, int i) const { return t[5 + 12 * layer + i]; }
+  const float* Lf(int layer, int i) const { return static_cast<const float*>(L(layer, i)); }
+};
+
+namespace {
+
+enum { W_QKV = 0, B_QKV, W_O, B_O, LN1_G, LN1_B, W_1, B_1, W_2, B_2, LN2_G, LN2_B };
+
+tcb_status embed_impl(const tcb_weights* w, int64_t M, const int32_t* d_segtab,
+                      const int32_t* d_ids, void* d_rows, int32_t* d_seg, int32_t* d_pos,
+                      cudaStream_t s) {
+  const tcb_model_config& c = w->cfg;
+  tcb::k::EmbedArgs a{};
+  a.segtab = reinterpret_cast<const int4*>(d_segtab);
+  a.ids = d_ids;
+  a.tok_emb = w->tok_emb();
+  a.pos_emb = c.pe == 2 ? w->pos_emb() : nullptr;
+  a.pe_table = c.pe == 2 ? nullptr : w->pe_table;
+  a.type_emb = c.use_type_emb ? w->type_emb() : nullptr;
+  a.ln_g = c.emb_ln ? w->emb_ln_g() : nullptr;
+  a.ln_b = c.emb_ln ? w->emb_ln_b() : nullptr;
+  a.emb_scale = c.emb_scale;
+  a.ln_eps = c.emb_ln_eps;
+  a.d = c.d_model;
+  a.max_pos = c.max_pos;
+  a.num_slots = M;
+  a.X = d_rows;
+  a.seg_ids = d_seg;
+  a.positions = d_pos;
+  TCB_LAUNCH(TCB_K_EMBED, s, tcb::k::launch_embed(c.dtype, a, s));
+  return TCB_OK;
+}
+
+tcb_status validate_plan_for(const tcb_weights* w, const tcb_plan* p) {
+  if (!w || !p) return fail(TCB_ERR_INVALID_ARGUMENT, "weights or plan is NULL");
+  if (p->info.num_slots > INT32_MAX)
+    return fail(TCB_ERR_UNSUPPORTED, "more than 2^31 slots in one forward");
+  if (p->num_rows > 0 && p->row_len > w->cfg.max_pos)
+    return fail(TCB_ERR_UNSUPPORTED, "row_len " + std::to_string(p->row_len) +
+                                         " exceeds max_pos " + std::to_string(w->cfg.max_pos));
+  return TCB_OK;
+}
+
+}  // namespace
+
+extern "C" {
+
+int64_t tcb_launch_count(void) { return g_launches.load(); }
+
+tcb_status tcb_profile_enable(int32_t on) {
+  tcb::clear_error();
+  std::lock_guard<std::mutex> g(g_prof_mu);
+  g_prof_on = on != 0;
+  return TCB_OK;
+}
+
+tcb_status tcb_profile_collect(double* ms, int64_t* launches) {
+  tcb::clear_error();
+  std::lock_guard<std::mutex> g(g_prof_mu);
+  if (ms) for (int i = 0; i < TCB_KCLASS_COUNT; ++i) ms[i] = 0.0;
+  if (launches) for (int i = 0; i < TCB_KCLASS_COUNT; ++i) launches[i] = 0;
+  tcb_status st = TCB_OK;
+  for (const ProfRec& r : g_prof) {
+    float t = 0.f;
+    cudaError_t e = cudaEventSynchronize(r.b);
+    if (e == cudaSuccess) e = cudaEventElapsedTime(&t, r.a, r.b);
+    if (e != cudaSuccess) st = cuda_fail(e, "tcb_profile_collect");
+    if (ms) ms[r.cls] += t;
+    if (launches) launches[r.cls] += 1;
+    g_event_pool.push_back(r.a);
+    g_event_pool.push_back(r.b);
+  }
+  g_prof.clear();
+  return st;
+}
+
+int32_t tcb_weights_count(const tcb_model_config* cfg) {
+  return cfg ? 5 + 12 * cfg->num_layers : -1;
+}
+
+tcb_status tcb_workspace_size(const tcb_model_config* cfg, int64_t num_slots, size_t* bytes) {
+  tcb::clear_error();
+  if (tcb_status st = validate_cfg(cfg)) return st;
+  if (!bytes || num_slots < 0) return fail(TCB_ERR_INVALID_ARGUMENT, "tcb_workspace_size");
+  *bytes = ws_layout(*cfg, num_slots).total;
+  return TCB_OK;
+}
+
+tcb_status tcb_weights_create(const tcb_model_config* cfg, const void* const* tensors,
+                              int32_t num_tensors, tcb_weights** out) {
+  tcb::clear_error();
+  if (!out) return fail(TCB_ERR_INVALID_ARGUMENT, "tcb_weights_create: out is NULL");
+  *out = nullptr;
+  if (tcb_status st = validate_cfg(cfg)) return st;
+  if (!tensors || num_tensors != tcb_weights_count(cfg))
+    return fail(TCB_ERR_INVALID_ARGUMENT, "tcb_weights_create: expected " +
+                                              std::to_string(tcb_weights_count(cfg)) + " tensors");
+  for (int i = 0; i < num_tensors; ++i) {
+    if (!tensors[i] || (reinterpret_cast<uintptr_t>(tensors[i]) & 15))
+      return fail(TCB_ERR_INVALID_ARGUMENT,
+                  "tcb_weights_create: tensor " + std::to_string(i) + " is NULL or not 16-byte aligned");
+  }
+  if (tcb_status st = check_device()) return st;
+  tcb_weights* w = new (std::nothrow) tcb_weights();
+  if (!w) return fail(TCB_ERR_OUT_OF_MEMORY, "tcb_weights_create");
+  w->cfg = *cfg;
+  w->t.assign(tensors, tensors + num_tensors);
+  const tcb_model_config& c = *cfg;
+  if (c.pe != 2) {
+    cudaError_t e = cudaMalloc(&w->pe_table, sizeof(float) * static_cast<size_t>(c.max_pos) * c.d_model);
+    if (e != cudaSuccess) { delete w; return fail(TCB_ERR_OUT_OF_MEMORY, "PE table allocation"); }
+    e = tcb::k::launch_pe_table(w->pe_table, c.max_pos, c.d_model, c.pe, nullptr);
+    g_launches.fetch_add(1);
+    if (e == cudaSuccess) e = cudaDeviceSynchronize();
+    if (e != cudaSuccess) { cudaFree(w->pe_table); delete w; return cuda_fail(e, "PE table"); }
+  }
+  if (c.dtype == 1) {
+    w->maps.resize(c.num_layers);
+    for (int l = 0; l < c.num_layers; ++l) {
+      const int d = c.d_model, f = c.d_ff;
+      bool ok = tcb::k::make_tmap_bf16(&w->maps[l].qkv, w->L(l, W_QKV), 3 * d, d,
+                                       tcb::k::linear_tc_block_n(3 * d)) &&
+                tcb::k::make_tmap_bf16(&w->maps[l].o, w->L(l, W_O), d, d,
+                                       tcb::k::linear_tc_block_n(d)) &&
+                tcb::k::make_tmap_bf16(&w->maps[l].w1, w->L(l, W_1), f, d,
+                                       tcb::k::linear_tc_block_n(f)) &&
+                tcb::k::make_tmap_bf16(&w->maps[l].w2, w->L(l, W_2), d, f,
+                                       tcb::k::linear_tc_block_n(d));
+      if (!ok) {
+        if (w->pe_table) cudaFree(w->pe_table);
+        delete w;
+        return fail(TCB_ERR_CUDA, "cuTensorMapEncodeTiled failed for a weight matrix");
+      }
+    }
+  }
+  *out = w;
+  return TCB_OK;
+}
+
+void tcb_weights_destroy(tcb_weights* w) {
+  if (!w) return;
+  if (w->pe_table) cudaFree(w->pe_table);
+  delete w;
+}
+
+tcb_status tcb_embed(const tcb_weights* w, const tcb_plan* plan, const int32_t* d_segtab,
+                     const int32_t* d_token_ids, void* d_rows, int32_t* d_segment_ids,
+                     int32_t* d_positions, tcb_stream_t stream) {
+  tcb::clear_error();
+  if (tcb_status st = validate_plan_for(w, plan)) return st;
+  const int64_t M = plan->info.num_slots;
+  if (M == 0) return TCB_OK;
+  if (!d_segtab || !d_rows || (plan->info.total_tokens > 0 && !d_token_ids))
+    return fail(TCB_ERR_INVALID_ARGUMENT, "tcb_embed: NULL device pointer");
+  return embed_impl(w, M, d_segtab, d_token_ids, d_rows, d_segment_ids, d_positions,
+                    reinterpret_cast<cudaStream_t>(stream));
+}
+
+tcb_status tcb_encoder_forward(const tcb_weights* wc, const tcb_plan* plan,
+                               const int32_t* d_segtab, const int32_t* d_token_ids,
+                               void* d_rows, void* d_ws, size_t ws_bytes, tcb_stream_t stream) {
+  tcb::clear_error();
+  if (tcb_status st = validate_plan_for(wc, plan)) return st;
+  tcb_weights* w = const_cast<tcb_weights*>(wc);
+  const tcb_model_config& c = w->cfg;
+  const int64_t M = plan->info.num_slots;
+  if (M == 0) return TCB_OK;
+  if (!d_segtab || !d_rows || !d_ws || (plan->info.total_tokens > 0 && !d_token_ids))
+    return fail(TCB_ERR_INVALID_ARGUMENT, "tcb_encoder_forward: NULL device pointer");
+  const WsLayout L = ws_layout(c, M);
+  if (ws_bytes < L.total)
+    return fail(TCB_ERR_WORKSPACE_TOO_SMALL, "tcb_encoder_forward: workspace " +
+                                                 std::to_string(ws_bytes) + " < " +
+                                                 std::to_string(L.total) + " bytes");
+  cudaStream_t s = reinterpret_cast<cudaStream_t>(stream);
+  uint8_t* ws = static_cast<uint8_t*>(d_ws);
+  int32_t* seg = reinterpret_cast<int32_t*>(ws + L.seg);
+  void* qkv = ws + L.qkv;
+  void* att = ws + L.att;
+  void* z = ws + L.z;
+  void* x1 = ws + L.x1;
+  void* hbuf = ws + L.h;
+  const int d = c.d_model, f = c.d_ff;
+  const int act_epi = c.act == 0 ? TCB_EPI_BIAS_GELU : TCB_EPI_BIAS_RELU;
+  const int4* segtab = reinterpret_cast<const int4*>(d_segtab);
+
+  if (tcb_status st = embed_impl(w, M, d_segtab, d_token_ids, d_rows, seg, nullptr, s)) return st;
+
+  if (c.dtype == 1) {
+    {
+      std::lock_guard<std::mutex> g(w->mu);
+      if (w->c_rows != d_rows || w->c_ws != d_ws || w->c_M != M) {
+        const bool ok = tcb::k::make_tmap_bf16(&w->mX, d_rows, M, d, 128) &&
+                        tcb::k::make_tmap_bf16(&w->mAtt, att, M, d, 128) &&
+                        tcb::k::make_tmap_bf16(&w->mX1, x1, M, d, 128) &&
+                        tcb::k::make_tmap_bf16(&w->mH, hbuf, M, f, 128);
+        if (!ok) return fail(TCB_ERR_CUDA, "cuTensorMapEncodeTiled failed for an activation");
+        w->c_rows = d_rows;
+        w->c_ws = d_ws;
+        w->c_M = M;
+      }
+    }
+    for (int l = 0; l < c.num_layers; ++l) {
+      const auto& mp = w->maps[l];
+      TCB_LAUNCH(TCB_K_GEMM_QKV, s, tcb::k::launch_linear_bf16_tc(w->mX, mp.qkv, M, 3 * d, d,
+                                                                  w->Lf(l, B_QKV), nullptr,
+                                                                  TCB_EPI_BIAS, qkv, s));
+      TCB_LAUNCH(TCB_K_ATTN, s, tcb::k::launch_attention_bf16(M, d, c.num_heads, qkv, seg,
+                                                              segtab, att, s));
+      TCB_LAUNCH(TCB_K_GEMM_O, s, tcb::k::launch_linear_bf16_tc(w->mAtt, mp.o, M, d, d,
+                                                                w->Lf(l, B_O), d_rows,
+                                                                TCB_EPI_BIAS_RESIDUAL, z, s));
+      TCB_LAUNCH(TCB_K_LN, s, tcb::k::launch_layernorm(1, M, d, z, w->Lf(l, LN1_G),
+                                                       w->Lf(l, LN1_B), c.ln_eps, seg, x1, s));
+      TCB_LAUNCH(TCB_K_GEMM_FFN1, s, tcb::k::launch_linear_bf16_tc(w->mX1, mp.w1, M, f, d,
+                                                                   w->Lf(l, B_1), nullptr,
+                                                                   act_epi, hbuf, s));
+      TCB_LAUNCH(TCB_K_GEMM_FFN2, s, tcb::k::launch_linear_bf16_tc(w->mH, mp.w2, M, d, f,
+                                                                   w->Lf(l, B_2), x1,
+                                                                   TCB_EPI_BIAS_RESIDUAL, z, s));
+      TCB_LAUNCH(TCB_K_LN, s, tcb::k::launch_layernorm(1, M, d, z, w->Lf(l, LN2_G),
+                                                       w->Lf(l, LN2_B), c.ln_eps, seg, d_rows, s));
+    }
+  } else {
+    float* X = static_cast<float*>(d_rows);
+    for (int l = 0; l < c.num_layers; ++l) {
+      TCB_LAUNCH(TCB_K_GEMM_QKV, s, tcb::k::launch_linear_f32(
+                                        M, 3 * d, d, X, static_cast<const float*>(w->L(l, W_QKV)),
+                                        w->Lf(l, B_QKV), nullptr, TCB_EPI_BIAS,
+                                        static_cast<float*>(qkv), s));
+      TCB_LAUNCH(TCB_K_ATTN, s, tcb::k::launch_attention_f32(M, d, c.num_heads,
+                                                             static_cast<const float*>(qkv), seg,
+                                                             segtab, static_cast<float*>(att), s));
+      TCB_LAUNCH(TCB_K_GEMM_O, s, tcb::k::launch_linear_f32(
+                                      M, d, d, static_cast<const float*>(att),
+                                      static_cast<const float*>(w->L(l, W_O)), w->Lf(l, B_O), X,
+                                      TCB_EPI_BIAS_RESIDUAL, static_cast<float*>(z), s));
+      TCB_LAUNCH(TCB_K_LN, s, tcb::k::launch_layernorm(0, M, d, z, w->Lf(l, LN1_G),
+                                                       w->Lf(l, LN1_B), c.ln_eps, seg, x1, s));
+      TCB_LAUNCH(TCB_K_GEMM_FFN1, s, tcb::k::launch_linear_f32(
+                                         M, f, d, static_cast<const float*>(x1),
+                                         static_cast<const float*>(w->L(l, W_1)), w->Lf(l, B_1),
+                                         nullptr, act_epi, static_cast<float*>(hbuf), s));
+      TCB_LAUNCH(TCB_K_GEMM_FFN2, s, tcb::k::launch_linear_f32(
+                                         M, d, f, static_cast<const float*>(hbuf),
+                                         static_cast<const float*>(w->L(l, W_2)), w->Lf(l, B_2),
+                                         static_cast<const float*>(x1), TCB_EPI_BIAS_RESIDUAL,
+                                         static_cast<float*>(z), s));
+      TCB_LAUNCH(TCB_K_LN, s, tcb::k::launch_layernorm(0, M, d, z, w->Lf(l, LN2_G),
+                                                       w->Lf(l, LN2_B), c.ln_eps, seg, X, s));
+    }
+  }
+  if (std::getenv("TCB_DEBUG_SYNC")) {
+    cudaError_t e = cudaStreamSynchronize(s);
+    if (e != cudaSuccess) return cuda_fail(e, "tcb_encoder_forward (TCB_DEBUG_SYNC)");
+  }
+  return TCB_OK;
+}
+
+tcb_status tcb_unpack(const tcb_weights* w, const tcb_plan* plan, const int32_t* d_segtab,
+                      const void* d_rows, void* d_out, tcb_stream_t stream) {
+  tcb::clear_error();
+  if (tcb_status st = validate_plan_for(w, plan)) return st;
+  const int64_t M = plan->info.num_slots;
+  if (M == 0) return TCB_OK;
+  if (!d_segtab || !d_rows || !d_out) return fail(TCB_ERR_INVALID_ARGUMENT, "tcb_unpack: NULL");
+  cudaStream_t s = reinterpret_cast<cudaStream_t>(stream);
+  TCB_LAUNCH(TCB_K_UNPACK, s, tcb::k::launch_unpack(w->cfg.dtype,
+                                                    reinterpret_cast<const int4*>(d_segtab), M,
+                                                    w->cfg.d_model, d_rows, d_out, s));
+  return TCB_OK;
+}
+
+// ---- op-level entry points (include/tcb_ops.h) ---------------------------------------------
+tcb_status tcb_op_linear(int32_t dtype, int64_t M, int32_t N, int32_t K, const void* A,
+                         const void* W, const float* bias, const void* R, int32_t epi, void* C,
+                         tcb_stream_t stream) {
+  tcb::clear_error();
+  if (M < 0 || N <= 0 || K <= 0 || epi < 0 || epi > 3 || (dtype != 0 && dtype != 1))
+    return fail(TCB_ERR_INVALID_ARGUMENT, "tcb_op_linear: bad shape / dtype / epilogue");
+  if (M == 0) return TCB_OK;
+  if (!A || !W || !bias || !C || (epi == TCB_EPI_BIAS_RESIDUAL && !R))
+    return fail(TCB_ERR_INVALID_ARGUMENT, "tcb_op_linear: NULL pointer");
+  if (tcb_status st = check_device()) return st;
+  cudaStream_t s = reinterpret_cast<cudaStream_t>(stream);
+  if (dtype == 0) {
+    TCB_LAUNCH(TCB_K_GEMM_QKV, s, tcb::k::launch_linear_f32(
+                                      M, N, K, static_cast<const float*>(A),
+                                      static_cast<const float*>(W), bias,
+                                      static_cast<const float*>(R), epi, static_cast<float*>(C), s));
+    return TCB_OK;
+  }
+  if (K % 64 != 0 || N % 64 != 0 || M > INT32_MAX)
+    return fail(TCB_ERR_UNSUPPORTED, "tcb_op_linear (bf16): needs K % 64 == 0 and N % 64 == 0");
+  CUtensorMap ma, mw;
+  if (!tcb::k::make_tmap_bf16(&ma, A, M, K, 128) ||
+      !tcb::k::make_tmap_bf16(&mw, W, N, K, tcb::k::linear_tc_block_n(N)))
+    return fail(TCB_ERR_CUDA, "tcb_op_linear: cuTensorMapEncodeTiled failed (alignment?)");
+  TCB_LAUNCH(TCB_K_GEMM_QKV, s, tcb::k::launch_linear_bf16_tc(ma, mw, M, N, K, bias, R, epi, C, s));
+  return TCB_OK;
+}
+
+tcb_status tcb_op_attention(int32_t dtype, int64_t num_slots, int32_t d_model,
+                            int32_t num_heads, const void* qkv, const int32_t* d_seg,
+                            const int32_t* d_segtab, void* O, tcb_stream_t stream) {
+  tcb::clear_error();
+  if (num_slots < 0 || d_model <= 0 || num_heads <= 0 || d_model % num_heads != 0 ||
+      (dtype != 0 && dtype != 1))
+    return fail(TCB_ERR_INVALID_ARGUMENT, "tcb_op_attention: bad shape / dtype");
+  if (num_slots == 0) return TCB_OK;
+  if (!qkv || !d_seg || !d_segtab || !O) return fail(TCB_ERR_INVALID_ARGUMENT, "tcb_op_attention: NULL");
+  const int dh = d_model / num_heads;
+  if ((dtype == 1 && dh != 64) || (dtype == 0 && dh > 64))
+    return fail(TCB_ERR_UNSUPPORTED, "tcb_op_attention: unsupported head dim");
+  if (tcb_status st = check_device()) return st;
+  cudaStream_t s = reinterpret_cast<cudaStream_t>(stream);
+  const int4* segtab = reinterpret_cast<const int4*>(d_segtab);
+  if (dtype == 1)
+    TCB_LAUNCH(TCB_K_ATTN, s, tcb::k::launch_attention_bf16(num_slots, d_model, num_heads, qkv,
+                                                            d_seg, segtab, O, s));
+  else
+    TCB_LAUNCH(TCB_K_ATTN, s, tcb::k::launch_attention_f32(num_slots, d_model, num_heads,
+                                                           static_cast<const float*>(qkv), d_seg,
+                                                           segtab, static_cast<float*>(O), s));
+  return TCB_OK;
+}
+
+tcb_status tcb_op_layernorm(int32_t dtype, int64_t rows, int32_t d, const void* Z,
+                            const float* g, const float* b, float eps, const int32_t* d_seg,
+                            void* Y, tcb_stream_t stream) {
+  tcb::clear_error();
+  if (rows < 0 || d <= 0 || (dtype != 0 && dtype != 1))
+    return fail(TCB_ERR_INVALID_ARGUMENT, "tcb_op_layernorm: bad shape / dtype");
+  if (rows == 0) return TCB_OK;
+  if (!Z || !g || !b || !Y) return fail(TCB_ERR_INVALID_ARGUMENT, "tcb_op_layernorm: NULL");
+  if (d % (dtype == 1 ? 8 : 4) != 0 || d > (dtype == 1 ? 2048 : 1024))
+    return fail(TCB_ERR_UNSUPPORTED, "tcb_op_layernorm: d unsupported");
+  if (tcb_status st = check_device()) return st;
+  cudaStream_t s = reinterpret_cast<cudaStream_t>(stream);
+  TCB_LAUNCH(TCB_K_LN, s, tcb::k::launch_layernorm(dtype, rows, d, Z, g, b, eps, d_seg, Y, s));
+  return TCB_OK;
+}
+
+}  // extern "C"

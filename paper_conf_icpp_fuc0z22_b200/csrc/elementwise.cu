@@ -1,0 +1,287 @@
+// elementwise.cu -- HBM-bound kernels of the ConcatBatching path (sm_100a):
+//   pack_embed : gather token embeddings, add the separate positional encoding (positions
+//                restart at each request, §4.1.1, Eq. (1)-(2) P:329-333), write
+//                the per-slot segment metadata; optional BERT type-0 + LayerNorm (R5).
+//   layernorm  : warp-per-row two-pass LayerNorm (post-LN encoder, R10).
+//   unpack     : scatter the rows back per request (Concat of Eq. (8)).
+//   pe_table   : the sinusoidal table PE[pos, dim] (Eq. (1)-(2); R1 variant flag).
+// One warp owns one slot / row; each lane moves 16-byte vectors so a warp touches whole
+// 512-byte spans (coalesced); rows are kept in registers between the reduction passes.
+#include <cuda_bf16.h>
+
+#include <cmath>
+
+#include "kernels.h"
+
+namespace tcb {
+namespace k {
+namespace {
+
+constexpr int kWarpsPerBlock = 8;
+constexpr int kMaxVecPerLane = 8;  // 16-byte vectors per lane: d <= 8*32*8 = 2048 (bf16)
+
+template <typename T> struct Vec;
+template <> struct Vec<float> {
+  static constexpr int N = 4;
+  __device__ static void load(const float* p, float* v) {
+    float4 x = *reinterpret_cast<const float4*>(p);
+    v[0] = x.x; v[1] = x.y; v[2] = x.z; v[3] = x.w;
+  }
+  __device__ static void store(float* p, const float* v) {
+    *reinterpret_cast<float4*>(p) = make_float4(v[0], v[1], v[2], v[3]);
+  }
+};
+template <> struct Vec<__nv_bfloat16> {
+  static constexpr int N = 8;
+  __device__ static void load(const __nv_bfloat16* p, float* v) {
+    uint4 x = *reinterpret_cast<const uint4*>(p);
+    const __nv_bfloat162* h = reinterpret_cast<const __nv_bfloat162*>(&x);
+#pragma unroll
+    for (int i = 0; i < 4; ++i) {
+      float2 f = __bfloat1622float2(h[i]);
+      v[2 * i] = f.x; v[2 * i + 1] = f.y;
+    }
+  }
+  __device__ static void store(__nv_bfloat16* p, const float* v) {
+    uint4 x;
+    __nv_bfloat162* h = reinterpret_cast<__nv_bfloat162*>(&x);
+#pragma unroll
+    for (int i = 0; i < 4; ++i) h[i] = __floats2bfloat162_rn(v[2 * i], v[2 * i + 1]);
+    *reinterpret_cast<uint4*>(p) = x;
+  }
+};
+
+__device__ __forceinline__ float warp_sum(float v) {
+#pragma unroll
+  for (int o = 16; o > 0; o >>= 1) v += __shfl_xor_sync(0xffffffffu, v, o);
+  return v;
+}
+
+// Segment containing `slot` (binary search over the records' slot_start), or -1 for pad.
+__device__ __forceinline__ int find_segment(const int4* segtab, int64_t slot, int4* rec_out) {
+  const int S = segtab[0].x;
+  int lo = 0, hi = S - 1, found = -1;
+  while (lo <= hi) {
+    const int mid = (lo + hi) >> 1;
+    const int4 r = __ldg(&segtab[1 + mid]);
+    if (r.x <= slot) { found = mid; lo = mid + 1; } else { hi = mid - 1; }
+  }
+  if (found < 0) return -1;
+  const int4 r = __ldg(&segtab[1 + found]);
+  if (slot >= r.x + r.y) return -1;
+  *rec_out = r;
+  return found;
+}
+
+template <typename T>
+__global__ void __launch_bounds__(kWarpsPerBlock * 32) pack_embed_kernel(EmbedArgs a) {
+  constexpr int V = Vec<T>::N;
+  const int lane = threadIdx.x & 31;
+  const int64_t slot = static_cast<int64_t>(blockIdx.x) * kWarpsPerBlock + (threadIdx.x >> 5);
+  if (slot >= a.num_slots) return;
+  const int d = a.d;
+  const int nvec = d / V;
+  T* x = reinterpret_cast<T*>(a.X) + slot * d;
+  int4 rec;
+  const int seg = find_segment(a.segtab, slot, &rec);
+  if (seg < 0) {  // pad slot: zeros, segment -1, position -1 (R12)
+    float z[V] = {};
+    for (int i = lane; i < nvec; i += 32) Vec<T>::store(x + i * V, z);
+    if (lane == 0) {
+      if (a.seg_ids) a.seg_ids[slot] = -1;
+      if (a.positions) a.positions[slot] = -1;
+    }
+    return;
+  }
+  const int pos = static_cast<int>(slot - rec.x);           // restarts at 0 per request
+  const int tok = rec.z + pos;
+  const int id = __ldg(&a.ids[tok]);
+  if (lane == 0) {
+    if (a.seg_ids) a.seg_ids[slot] = seg;
+    if (a.positions) a.positions[slot] = pos;
+  }
+  const T* e = reinterpret_cast<const T*>(a.tok_emb) + static_cast<int64_t>(id) * d;
+  float v[kMaxVecPerLane][V];
+  float sum = 0.f;
+#pragma unroll
+  for (int j = 0; j < kMaxVecPerLane; ++j) {
+    const int i = lane + 32 * j;
+    if (i < nvec) {
+      Vec<T>::load(e + i * V, v[j]);
+      float p[V];
+      if (a.pe_table) {
+        const float* pt = a.pe_table + static_cast<int64_t>(pos) * d + i * V;
+#pragma unroll
+        for (int c = 0; c < V; c += 4) {
+          float4 q = *reinterpret_cast<const float4*>(pt + c);
+          p[c] = q.x; p[c + 1] = q.y; p[c + 2] = q.z; p[c + 3] = q.w;
+        }
+      } else {
+        Vec<T>::load(reinterpret_cast<const T*>(a.pos_emb) + static_cast<int64_t>(pos) * d + i * V, p);
+      }
+#pragma unroll
+      for (int c = 0; c < V; ++c) {
+        float t = v[j][c] * a.emb_scale + p[c];
+        if (a.type_emb) t += __ldg(&a.type_emb[i * V + c]);
+        v[j][c] = t;
+        sum += t;
+      }
+    }
+  }
+  if (a.ln_g) {
+    const float mean = warp_sum(sum) / d;
+    float sq = 0.f;
+#pragma unroll
+    for (int j = 0; j < kMaxVecPerLane; ++j)
+      if (lane + 32 * j < nvec)
+#pragma unroll
+        for (int c = 0; c < V; ++c) { const float t = v[j][c] - mean; sq += t * t; }
+    const float rstd = rsqrtf(warp_sum(sq) / d + a.ln_eps);
+#pragma unroll
+    for (int j = 0; j < kMaxVecPerLane; ++j) {
+      const int i = lane + 32 * j;
+      if (i < nvec)
+#pragma unroll
+        for (int c = 0; c < V; ++c)
+          v[j][c] = (v[j][c] - mean) * rstd * __ldg(&a.ln_g[i * V + c]) + __ldg(&a.ln_b[i * V + c]);
+    }
+  }
+#pragma unroll
+  for (int j = 0; j < kMaxVecPerLane; ++j) {
+    const int i = lane + 32 * j;
+    if (i < nvec) Vec<T>::store(x + i * V, v[j]);
+  }
+}
+
+template <typename T>
+__global__ void __launch_bounds__(kWarpsPerBlock * 32)
+layernorm_kernel(int64_t rows, int d, const T* __restrict__ Z, const float* __restrict__ g,
+                 const float* __restrict__ b, float eps, const int32_t* __restrict__ seg_ids,
+                 T* __restrict__ Y) {
+  constexpr int V = Vec<T>::N;
+  const int lane = threadIdx.x & 31;
+  const int64_t row = static_cast<int64_t>(blockIdx.x) * kWarpsPerBlock + (threadIdx.x >> 5);
+  if (row >= rows) return;
+  const int nvec = d / V;
+  T* y = Y + row * d;
+  if (seg_ids && __ldg(&seg_ids[row]) < 0) {  // pad row -> 0 (R12)
+    float z[V] = {};
+    for (int i = lane; i < nvec; i += 32) Vec<T>::store(y + i * V, z);
+    return;
+  }
+  const T* z = Z + row * d;
+  float v[kMaxVecPerLane][V];
+  float sum = 0.f;
+#pragma unroll
+  for (int j = 0; j < kMaxVecPerLane; ++j) {
+    const int i = lane + 32 * j;
+    if (i < nvec) {
+      Vec<T>::load(z + i * V, v[j]);
+#pragma unroll
+      for (int c = 0; c < V; ++c) sum += v[j][c];
+    }
+  }
+  const float mean = warp_sum(sum) / d;
+  float sq = 0.f;
+#pragma unroll
+  for (int j = 0; j < kMaxVecPerLane; ++j)
+    if (lane + 32 * j < nvec)
+#pragma unroll
+      for (int c = 0; c < V; ++c) { const float t = v[j][c] - mean; sq += t * t; }
+  const float rstd = rsqrtf(warp_sum(sq) / d + eps);
+#pragma unroll
+  for (int j = 0; j < kMaxVecPerLane; ++j) {
+    const int i = lane + 32 * j;
+    if (i < nvec) {
+      float o[V];
+      const float4* gg = reinterpret_cast<const float4*>(g + i * V);
+      const float4* bb = reinterpret_cast<const float4*>(b + i * V);
+#pragma unroll
+      for (int c = 0; c < V; c += 4) {
+        const float4 g4 = __ldg(gg + c / 4), b4 = __ldg(bb + c / 4);
+        o[c] = (v[j][c] - mean) * rstd * g4.x + b4.x;
+        o[c + 1] = (v[j][c + 1] - mean) * rstd * g4.y + b4.y;
+        o[c + 2] = (v[j][c + 2] - mean) * rstd * g4.z + b4.z;
+        o[c + 3] = (v[j][c + 3] - mean) * rstd * g4.w + b4.w;
+      }
+      Vec<T>::store(y + i * V, o);
+    }
+  }
+}
+
+template <typename T>
+__global__ void __launch_bounds__(kWarpsPerBlock * 32)
+unpack_kernel(const int4* __restrict__ segtab, int64_t num_slots, int d,
+              const T* __restrict__ rows, T* __restrict__ out) {
+  constexpr int V = Vec<T>::N;
+  const int lane = threadIdx.x & 31;
+  const int64_t slot = static_cast<int64_t>(blockIdx.x) * kWarpsPerBlock + (threadIdx.x >> 5);
+  if (slot >= num_slots) return;
+  int4 rec;
+  if (find_segment(segtab, slot, &rec) < 0) return;
+  const int64_t tok = rec.z + (slot - rec.x);
+  const uint4* src = reinterpret_cast<const uint4*>(rows + slot * d);
+  uint4* dst = reinterpret_cast<uint4*>(out + tok * d);
+  const int nvec = d / V;
+  for (int i = lane; i < nvec; i += 32) dst[i] = __ldg(src + i);
+}
+
+__global__ void pe_table_kernel(float* table, int max_pos, int d, int variant) {
+  const int64_t i = static_cast<int64_t>(blockIdx.x) * blockDim.x + threadIdx.x;
+  if (i >= static_cast<int64_t>(max_pos) * d) return;
+  const int pos = static_cast<int>(i / d), dim = static_cast<int>(i % d);
+  const int e = dim / 2;
+  // Eq. (1)-(2): PE(pos,2e) = sin(pos/10000^(2e/d)); PE(pos,2e+1) = cos(pos/10000^((2e+1)/d))
+  // (literal, R1; variant 1 uses 2e/d for both).  Evaluated in double, stored as fp32.
+  const double expo = (dim % 2 == 0 || variant == 1) ? (2.0 * e) / d : (2.0 * e + 1.0) / d;
+  const double ang = pos / pow(10000.0, expo);
+  table[i] = static_cast<float>(dim % 2 == 0 ? sin(ang) : cos(ang));
+}
+
+}  // namespace
+
+cudaError_t launch_embed(int dtype, const EmbedArgs& a, cudaStream_t s) {
+  if (a.num_slots == 0) return cudaSuccess;
+  const unsigned grid = static_cast<unsigned>((a.num_slots + kWarpsPerBlock - 1) / kWarpsPerBlock);
+  if (dtype == 0) pack_embed_kernel<float><<<grid, kWarpsPerBlock * 32, 0, s>>>(a);
+  else pack_embed_kernel<__nv_bfloat16><<<grid, kWarpsPerBlock * 32, 0, s>>>(a);
+  return cudaGetLastError();
+}
+
+cudaError_t launch_layernorm(int dtype, int64_t rows, int d, const void* Z, const float* g,
+                             const float* b, float eps, const int32_t* seg_ids, void* Y,
+                             cudaStream_t s) {
+  if (rows == 0) return cudaSuccess;
+  const unsigned grid = static_cast<unsigned>((rows + kWarpsPerBlock - 1) / kWarpsPerBlock);
+  if (dtype == 0)
+    layernorm_kernel<float><<<grid, kWarpsPerBlock * 32, 0, s>>>(
+        rows, d, static_cast<const float*>(Z), g, b, eps, seg_ids, static_cast<float*>(Y));
+  else
+    layernorm_kernel<__nv_bfloat16><<<grid, kWarpsPerBlock * 32, 0, s>>>(
+        rows, d, static_cast<const __nv_bfloat16*>(Z), g, b, eps, seg_ids,
+        static_cast<__nv_bfloat16*>(Y));
+  return cudaGetLastError();
+}
+
+cudaError_t launch_unpack(int dtype, const int4* segtab, int64_t num_slots, int d,
+                          const void* rows, void* out, cudaStream_t s) {
+  if (num_slots == 0) return cudaSuccess;
+  const unsigned grid = static_cast<unsigned>((num_slots + kWarpsPerBlock - 1) / kWarpsPerBlock);
+  if (dtype == 0)
+    unpack_kernel<float><<<grid, kWarpsPerBlock * 32, 0, s>>>(
+        segtab, num_slots, d, static_cast<const float*>(rows), static_cast<float*>(out));
+  else
+    unpack_kernel<__nv_bfloat16><<<grid, kWarpsPerBlock * 32, 0, s>>>(
+        segtab, num_slots, d, static_cast<const __nv_bfloat16*>(rows),
+        static_cast<__nv_bfloat16*>(out));
+  return cudaGetLastError();
+}
+
+cudaError_t launch_pe_table(float* table, int max_pos, int d, int variant, cudaStream_t s) {
+  const int64_t n = static_cast<int64_t>(max_pos) * d;
+  pe_table_kernel<<<static_cast<unsigned>((n + 255) / 256), 256, 0, s>>>(table, max_pos, d, variant);
+  return cudaGetLastError();
+}
+
+}  // namespace k
+}  // namespace tcb

@@ -1,0 +1,63 @@
+// kernels.h -- launchers of the sm_100a kernels of libtcb (device code lives in *.cu).
+#pragma once
+
+#include <cuda.h>
+#include <cuda_runtime.h>
+#include <cstdint>
+
+namespace tcb {
+namespace k {
+
+// Embedding / metadata / elementwise (elementwise.cu) -------------------------------------
+struct EmbedArgs {
+  const int4* segtab;          // device segment table (header + records)
+  const int32_t* ids;          // [total_tokens]
+  const void* tok_emb;         // [vocab, d] dtype
+  const void* pos_emb;         // [max_pos, d] dtype (learned PE) or nullptr
+  const float* pe_table;       // [max_pos, d] fp32 sinusoidal table or nullptr
+  const float* type_emb;       // [d] or nullptr
+  const float* ln_g;           // [d] or nullptr (no embedding LN)
+  const float* ln_b;
+  float emb_scale, ln_eps;
+  int32_t d, max_pos;
+  int64_t num_slots;
+  void* X;                     // out [num_slots, d] dtype
+  int32_t* seg_ids;            // out [num_slots] or nullptr
+  int32_t* positions;          // out [num_slots] or nullptr
+};
+cudaError_t launch_embed(int dtype, const EmbedArgs& a, cudaStream_t s);
+
+cudaError_t launch_layernorm(int dtype, int64_t rows, int d, const void* Z, const float* g,
+                             const float* b, float eps, const int32_t* seg_ids, void* Y,
+                             cudaStream_t s);
+
+cudaError_t launch_unpack(int dtype, const int4* segtab, int64_t num_slots, int d,
+                          const void* rows, void* out, cudaStream_t s);
+
+cudaError_t launch_pe_table(float* table, int max_pos, int d, int variant, cudaStream_t s);
+
+// Linear layers --------------------------------------------------------------------------
+cudaError_t launch_linear_f32(int64_t M, int N, int K, const float* A, const float* W,
+                              const float* bias, const float* R, int epi, float* C,
+                              cudaStream_t s);
+
+// Host-side TMA descriptor for a row-major bf16 matrix [rows, cols] (cols contiguous),
+// box = box_rows x 64 columns, 128-byte swizzle.  Returns false on failure.
+bool make_tmap_bf16(CUtensorMap* map, const void* ptr, uint64_t rows, uint64_t cols,
+                    uint32_t box_rows);
+// The box_rows the tensor-core GEMM needs for its B (weight) operand at this N.
+int linear_tc_block_n(int N);
+cudaError_t launch_linear_bf16_tc(const CUtensorMap& tmA, const CUtensorMap& tmW, int64_t M,
+                                  int N, int K, const float* bias, const void* R, int epi,
+                                  void* C, cudaStream_t s);
+
+// Attention ------------------------------------------------------------------------------
+cudaError_t launch_attention_bf16(int64_t num_slots, int d_model, int num_heads,
+                                  const void* qkv, const int32_t* seg_ids, const int4* segtab,
+                                  void* O, cudaStream_t s);
+cudaError_t launch_attention_f32(int64_t num_slots, int d_model, int num_heads,
+                                 const float* qkv, const int32_t* seg_ids, const int4* segtab,
+                                 float* O, cudaStream_t s);
+
+}  // namespace k
+}  // namespace tcb

@@ -1,0 +1,38 @@
+// tcb_internal.h -- shared declarations of libtcb (host code + kernel launchers).
+#pragma once
+
+#include <cstdint>
+#include <cstddef>
+#include <string>
+#include <vector>
+
+#include "../../include/tcb.h"
+#include "../../include/tcb_ops.h"
+
+// Geometry of the segment-masked attention kernel (attn.cu); the host plan uses it to
+// report how many score elements the kernel evaluates (tcb_plan_info).
+constexpr int kAttnQBlock = 64;    // query slots per CTA (4 warps x 16 rows)
+constexpr int kAttnWarpRows = 16;  // query rows per warp (one m16 MMA tile)
+constexpr int kAttnKSub = 16;      // keys per skip decision (one k16 MMA step of P.V)
+
+namespace tcb {
+
+// Error reporting -------------------------------------------------------------------------
+void set_error(const std::string& msg);
+void clear_error();
+tcb_status fail(tcb_status st, const std::string& msg);
+
+// Segment-table record (16 bytes), see tcb.h "device form of a plan".
+struct SegRec {
+  int32_t start, len, tok, req;
+};
+
+}  // namespace tcb
+
+struct tcb_plan {
+  int32_t n = 0, row_len = 0, num_rows = 0, max_rows = 0, policy = 0;
+  std::vector<int32_t> lengths, req_row, req_col;
+  std::vector<int64_t> tok_off;          // request-order offset of each request's tokens
+  std::vector<int32_t> seg_req, seg_start;
+  tcb_plan_info info{};
+};

@@ -1,0 +1,164 @@
+"""CPU tests of the C ABI (no GPU needed): libtcb.so loads and exports every declared
+symbol; the C++ packer (tcb_pack) is bit-exact against the oracle's packer and layout on
+random and golden inputs, for every policy; error conventions; plan counters against a
+brute-force tile enumeration (P9); device calls without a GPU fail loudly (no fallback).
+"""
+import json
+import os
+import re
+
+import numpy as np
+import pytest
+
+import oracle
+import tcb_workload as wl
+import paper_conf_icpp_fuc0z22_b200 as tcb
+from paper_conf_icpp_fuc0z22_b200 import _lib
+
+ROOT = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+
+
+def _declared_symbols():
+    names = set()
+    for h in ("tcb.h", "tcb_ops.h"):
+        src = open(os.path.join(ROOT, "include", h)).read()
+        src = re.sub(r"/\*.*?\*/", "", src, flags=re.S)
+        names |= set(re.findall(r"\b(tcb_[a-z_0-9]+)\s*\(", src))
+    return names
+
+
+def test_library_exports_every_declared_symbol():
+    L = _lib.lib()
+    declared = _declared_symbols()
+    assert declared == set(_lib.EXPORTS), declared ^ set(_lib.EXPORTS)
+    for name in declared:
+        assert hasattr(L, name), name
+    assert b"sm_100a" in L.tcb_version()
+
+
+def _plan_vs_oracle(lengths, L, max_rows, policy):
+    plan = tcb.tcb_pack(lengths, L, max_rows, policy)
+    pk = oracle.pack(lengths, L, max_rows, policy)
+    lay = oracle.layout(lengths, pk["req_row"], pk["req_col"], pk["num_rows"], L, 128)
+    a = plan.arrays()
+    assert plan.info["num_rows"] == pk["num_rows"]
+    assert a["req_row"].tolist() == pk["req_row"].tolist()
+    assert a["req_col"].tolist() == pk["req_col"].tolist()
+    for k in ("seg_req", "seg_start", "cu_seqlens", "segment_ids", "positions"):
+        assert a[k].tolist() == lay[k].tolist(), k
+    assert a["qtile_kv"].tolist() == lay["qtile_kv"].tolist()
+    return plan, lay
+
+
+@pytest.mark.parametrize("policy", list(oracle.POLICIES))
+@pytest.mark.parametrize("seed", range(12))
+def test_pack_bit_exact_vs_oracle_random(policy, seed):
+    rng = np.random.default_rng(500 + seed)
+    L = int(rng.choice([8, 32, 64, 128, 256]))
+    n = int(rng.integers(0, 200))
+    lengths = rng.integers(1, L + 1, size=n).astype(np.int32)
+    max_rows = int(rng.choice([0, 0, 3, 20]))
+    _plan_vs_oracle(lengths, L, max_rows, policy)
+
+
+@pytest.mark.parametrize("dist,L", [("paracrawl", 128), ("dia", 512), ("mixed_8_512", 512),
+                                    ("wmt", 256), ("paper_normal_20", 128)])
+def test_pack_bit_exact_vs_oracle_workloads(dist, L):
+    lengths = np.minimum(wl.draw_lengths(dist, 800, 77), L).astype(np.int32)
+    _plan_vs_oracle(lengths, L, 64, "first_fit")
+
+
+def test_pack_golden_f1(golden_dir):
+    f1 = json.load(open(os.path.join(golden_dir, "f1_layout.json")))
+    plan = tcb.tcb_pack(f1["lengths"], f1["row_len"])
+    a = plan.arrays()
+    assert a["req_row"].tolist() == f1["req_row"]
+    assert a["req_col"].tolist() == f1["req_col"]
+    assert a["seg_start"].tolist() == f1["seg_start"]
+    assert a["cu_seqlens"].tolist() == f1["cu_seqlens"]
+    assert a["qtile_kv"].tolist() == f1["qtile_kv_128"]
+    st = plan.segtab()
+    assert st[:4].tolist() == [8, 64, 32, 58]
+    recs = st[4:].reshape(-1, 4)
+    assert recs[:, 0].tolist() == f1["seg_start"]
+    assert recs[:, 1].tolist() == [f1["lengths"][r] for r in f1["seg_req"]]
+    cu_req = np.concatenate([[0], np.cumsum(f1["lengths"])])
+    assert recs[:, 2].tolist() == [int(cu_req[r]) for r in f1["seg_req"]]
+    assert recs[:, 3].tolist() == f1["seg_req"]
+    assert plan.info["placed_tokens"] == 58 and plan.info["num_slots"] == 64
+
+
+def test_pack_errors():
+    with pytest.raises(tcb.TcbError) as e:
+        tcb.tcb_pack([3, 40], 32)
+    assert e.value.status == -2 and "request 1" in str(e.value)
+    with pytest.raises(tcb.TcbError) as e:
+        tcb.tcb_pack([3, 0], 32)
+    assert e.value.status == -1
+    with pytest.raises(tcb.TcbError) as e:
+        tcb.tcb_pack([3], 30)          # row_len % 8 != 0
+    assert e.value.status == -1
+    with pytest.raises(tcb.TcbError):
+        tcb.tcb_pack([3], 32, -1)
+    p = tcb.tcb_pack([], 32)
+    assert p.info["num_rows"] == 0 and p.info["num_slots"] == 0
+    assert p.segtab().tolist() == [0, 0, 32, 0]
+
+
+def test_plan_counters_vs_brute_force():
+    """P9 on the product's plan counters: 128x128 tiles touching a diagonal block, the
+    dense count, sum l^2, and the kernel's executed 16x16 sub-blocks (re-derived here from
+    its stated geometry: 64-slot CTAs, 16-row warps, 16-key sub-blocks from the CTA start)."""
+    lengths = np.minimum(wl.draw_lengths("dia", 300, 5), 512).astype(np.int32)
+    plan = tcb.tcb_pack(lengths, 512, 16)
+    a = plan.arrays()
+    seg = a["segment_ids"]
+    M = len(seg)
+    T = 128
+    visited = 0
+    for qt in range(M // T):
+        q = set(seg[qt * T:(qt + 1) * T].tolist()) - {-1}
+        for kt in range(M // T):
+            k = set(seg[kt * T:(kt + 1) * T].tolist()) - {-1}
+            if (qt * T) // 512 == (kt * T) // 512 and q & k:
+                visited += 1
+    info = plan.info
+    assert info["kv_tiles_visited"] == visited
+    assert info["kv_tiles_dense"] == info["num_rows"] * 16
+    placed = a["req_row"] >= 0
+    assert info["useful_score_elems"] == int(np.sum(lengths[placed].astype(np.int64) ** 2))
+    starts, lens = a["seg_start"], lengths[a["seg_req"]]
+    ex = 0
+    for q0 in range(0, M, 64):
+        iv = []
+        for w in range(4):
+            ss = [s for s in seg[q0 + 16 * w:q0 + 16 * w + 16] if s >= 0]
+            iv.append((min(starts[s] for s in ss), max(starts[s] + lens[s] for s in ss))
+                      if ss else None)
+        real = [x for x in iv if x]
+        if not real:
+            continue
+        clo, chi = min(x[0] for x in real), max(x[1] for x in real)
+        for x in real:
+            ex += 256 * sum(1 for kb in range(clo, chi, 16) if kb < x[1] and kb + 16 > x[0])
+    assert info["executed_score_elems"] == ex
+    assert info["useful_score_elems"] <= ex
+
+
+def test_device_calls_fail_loudly_without_gpu():
+    import torch
+    if torch.cuda.is_available():
+        pytest.skip("a GPU is visible")
+    m = wl.MODELS["toy"]
+    cfg = _lib.ModelConfig(m.num_layers, m.d_model, m.num_heads, m.d_ff, m.vocab, m.max_pos,
+                           0, 0, 0, 0, 0, 1e-5, 1e-5, 1.0)
+    import ctypes
+    n = _lib.lib().tcb_weights_count(ctypes.byref(cfg))
+    assert n == 5 + 12 * m.num_layers
+    fake = (ctypes.c_void_p * n)(*([4096] * n))
+    h = ctypes.c_void_p()
+    st = _lib.lib().tcb_weights_create(ctypes.byref(cfg), fake, n, ctypes.byref(h))
+    assert st == -7   # TCB_ERR_NO_DEVICE: there is no CPU fallback
+    assert b"no CPU fallback" in _lib.lib().tcb_last_error()
+    st = _lib.lib().tcb_op_linear(1, 128, 64, 64, 4096, 4096, 4096, None, 0, 4096, None)
+    assert st == -7

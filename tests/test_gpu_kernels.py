@@ -1,0 +1,191 @@
+"""Per-kernel parity of the CUDA path against the float64 oracle (GPU, sm_100a).
+
+Each kernel is called through the C ABI (include/tcb.h, include/tcb_ops.h) on seeded
+inputs; the oracle computes the same step in f64 on the identical (bf16-representable)
+values.  Integer metadata must be bit-exact.
+"""
+import numpy as np
+import pytest
+
+import oracle
+import tcb_workload as wl
+
+torch = pytest.importorskip("torch")
+pytestmark = pytest.mark.gpu
+
+import paper_conf_icpp_fuc0z22_b200 as tcb  # noqa: E402
+from _helpers import small_model  # noqa: E402
+
+
+def _dev(x, dtype=None):
+    t = torch.from_numpy(np.ascontiguousarray(x))
+    return t.to("cuda", dtype=dtype) if dtype is not None else t.to("cuda")
+
+
+def _bf16(x):
+    return wl.round_to_bf16(np.asarray(x, np.float32))
+
+
+# ------------------------------------------------------------------------------ linear --
+LIN_SHAPES = [(1, 64, 64), (100, 128, 64), (128, 256, 512), (1000, 192, 128),
+              (4133, 1536, 512), (777, 768, 768), (2048, 512, 2048), (300, 3072, 1024)]
+
+
+@pytest.mark.parametrize("M,N,K", LIN_SHAPES)
+@pytest.mark.parametrize("epi", ["bias", "bias_gelu", "bias_relu", "bias_residual"])
+def test_linear_bf16_tcgen05_vs_oracle(M, N, K, epi):
+    rng = np.random.default_rng(M * 7 + N * 3 + K)
+    A = _bf16(rng.normal(size=(M, K)))
+    W = _bf16(rng.uniform(-1, 1, size=(N, K)) * np.sqrt(3.0 / K))
+    b = _bf16(rng.normal(0, 0.1, size=N))
+    R = _bf16(rng.normal(size=(M, N))) if epi == "bias_residual" else None
+    out = tcb.op_linear(_dev(A, torch.bfloat16), _dev(W, torch.bfloat16), _dev(b, torch.float32),
+                        _dev(R, torch.bfloat16) if R is not None else None, epi)
+    torch.cuda.synchronize()
+    got = out.float().cpu().numpy()
+    act = {"bias_gelu": "gelu", "bias_relu": "relu"}.get(epi, "none")
+    ref = oracle.linear(A, W, b, R, act)
+    # one bf16 rounding of the output (2^-8 relative) + fp32 accumulation-order noise
+    err = np.abs(got - ref)
+    bound = 2.0 ** -8 * np.abs(ref) + 1e-3 * np.max(np.abs(ref)) + 1e-6
+    assert np.all(err <= bound), float(np.max(err / bound))
+
+
+@pytest.mark.parametrize("M,N,K", [(64, 192, 64), (130, 256, 64), (37, 64, 256)])
+@pytest.mark.parametrize("epi", ["bias", "bias_gelu", "bias_residual"])
+def test_linear_f32_simt_vs_oracle(M, N, K, epi):
+    rng = np.random.default_rng(11 + M + N + K)
+    A = rng.normal(size=(M, K)).astype(np.float32)
+    W = (rng.uniform(-1, 1, size=(N, K)) * np.sqrt(3.0 / K)).astype(np.float32)
+    b = rng.normal(0, 0.1, size=N).astype(np.float32)
+    R = rng.normal(size=(M, N)).astype(np.float32) if epi == "bias_residual" else None
+    out = tcb.op_linear(_dev(A), _dev(W), _dev(b), _dev(R) if R is not None else None, epi)
+    torch.cuda.synchronize()
+    ref = oracle.linear(A, W, b, R, {"bias_gelu": "gelu"}.get(epi, "none"))
+    assert np.max(np.abs(out.cpu().numpy() - ref)) <= 2e-5 * max(1.0, np.max(np.abs(ref)))
+
+
+def test_linear_deterministic_and_m_zero():
+    rng = np.random.default_rng(3)
+    A = _dev(_bf16(rng.normal(size=(999, 512))), torch.bfloat16)
+    W = _dev(_bf16(rng.normal(size=(1536, 512)) * 0.05), torch.bfloat16)
+    b = _dev(np.zeros(1536, np.float32))
+    o1 = tcb.op_linear(A, W, b)
+    o2 = tcb.op_linear(A, W, b)
+    torch.cuda.synchronize()
+    assert torch.equal(o1, o2)
+    e = tcb.op_linear(A[:0], W, b)
+    assert e.shape == (0, 1536)
+
+
+# --------------------------------------------------------------------------- attention --
+def _attn_case(lengths, L, d, h, dtype, seed, max_rows=0):
+    rng = np.random.default_rng(seed)
+    plan = tcb.tcb_pack(lengths, L, max_rows)
+    arr = plan.arrays()
+    M = plan.num_slots
+    qkv = rng.normal(size=(M, 3 * d)).astype(np.float32)
+    if dtype == "bf16":
+        qkv = _bf16(qkv)
+    tdt = torch.bfloat16 if dtype == "bf16" else torch.float32
+    seg = _dev(arr["segment_ids"])
+    segtab = _dev(plan.segtab())
+    out = tcb.op_attention(_dev(qkv, tdt), seg, segtab, h)
+    torch.cuda.synchronize()
+    ref = oracle.attention(qkv, arr["segment_ids"], plan.info["num_rows"], L, d, h)
+    return out.float().cpu().numpy(), ref, arr["segment_ids"]
+
+
+@pytest.mark.parametrize("case", [
+    ("uniform_3_16", 40, 32), ("paracrawl", 300, 128), ("dia", 60, 512), ("wmt", 200, 256),
+    ("mixed_8_512", 80, 512)])
+def test_attention_bf16_vs_oracle(case):
+    dist, n, L = case
+    lengths = np.minimum(wl.draw_lengths(dist, n, 9), L).astype(np.int32)
+    got, ref, seg = _attn_case(lengths, L, 256, 4, "bf16", 1)
+    real = seg >= 0
+    # P is rounded to bf16 before P.V and O to bf16 on store: ~2^-8 relative
+    for s in np.unique(seg[real]):
+        rows = seg == s
+        e = np.max(np.abs(got[rows] - ref[rows])) / np.max(np.abs(ref[rows]))
+        assert e <= 1.5e-2, (s, e)
+    assert np.all(got[~real] == 0)
+
+
+def test_attention_bf16_single_long_request_and_tail():
+    """One request filling a 512 row (textbook SDPA) + a ragged last row + pad tail."""
+    got, ref, seg = _attn_case(np.array([512, 77, 3], np.int32), 512, 128, 2, "bf16", 4)
+    real = seg >= 0
+    assert np.max(np.abs(got[real] - ref[real])) / np.max(np.abs(ref[real])) <= 1.5e-2
+    assert np.all(got[~real] == 0)
+
+
+def test_attention_f32_vs_oracle():
+    lengths = wl.draw_lengths("uniform_3_16", 8, 0)
+    got, ref, seg = _attn_case(lengths, 32, 64, 2, "fp32", 2)
+    assert np.max(np.abs(got - ref)) <= 2e-6
+
+
+# ------------------------------------------------------------------- layernorm / embed --
+@pytest.mark.parametrize("d", [512, 768, 1024])
+def test_layernorm_bf16_vs_oracle(d):
+    rng = np.random.default_rng(d)
+    Z = _bf16(rng.normal(1.0, 3.0, size=(1031, d)))
+    g = _bf16(1 + rng.normal(0, 0.1, size=d))
+    b = _bf16(rng.normal(0, 0.1, size=d))
+    seg = np.zeros(1031, np.int32)
+    seg[-5:] = -1
+    out = tcb.op_layernorm(_dev(Z, torch.bfloat16), _dev(g), _dev(b), 1e-5, _dev(seg))
+    torch.cuda.synchronize()
+    got = out.float().cpu().numpy()
+    ref = oracle.layernorm(Z, g, b, 1e-5)
+    assert np.all(np.abs(got[:-5] - ref[:-5]) <= 2.0 ** -8 * np.abs(ref[:-5]) + 2e-3)
+    assert np.all(got[-5:] == 0)
+
+
+@pytest.mark.parametrize("mkey", ["toy", "transformer-base", "bert-base"])
+def test_pack_embed_metadata_bit_exact_and_values(mkey):
+    model = wl.MODELS[mkey]
+    w = wl.draw_weights(model, 2)
+    names = wl.weight_names(model)
+    L = 32 if mkey == "toy" else 128
+    lengths = np.minimum(wl.draw_lengths("paracrawl", 90, 4), L).astype(np.int32)
+    ids = wl.draw_token_ids(int(lengths.sum()), model.vocab, 5)
+    enc = tcb.Encoder(model, w, names)
+    plan = tcb.tcb_pack(lengths, L, 0)
+    M = plan.num_slots
+    segtab = _dev(plan.segtab())
+    d_ids = _dev(ids)
+    rows = enc.alloc_rows(M)
+    seg = torch.full((M,), 7, dtype=torch.int32, device="cuda")
+    pos = torch.full((M,), 7, dtype=torch.int32, device="cuda")
+    enc.embed(plan, segtab, d_ids, rows, seg, pos)
+    torch.cuda.synchronize()
+    pk = oracle.pack(lengths, L)
+    lay = oracle.layout(lengths, pk["req_row"], pk["req_col"], pk["num_rows"], L)
+    assert seg.cpu().numpy().tolist() == lay["segment_ids"].tolist()
+    assert pos.cpu().numpy().tolist() == lay["positions"].tolist()
+    ref = oracle.embed(model, w, ids, lay)
+    got = rows.float().cpu().numpy()
+    tol = 1e-6 if model.dtype == "fp32" else 2.0 ** -8
+    assert np.all(np.abs(got - ref) <= tol * np.abs(ref) + (1e-6 if model.dtype == "fp32" else 1e-3))
+
+
+def test_unpack_roundtrip_exact():
+    model = small_model(dtype="bf16", d=128, h=2, f=256)
+    w = wl.draw_weights(model, 1)
+    enc = tcb.Encoder(model, w, wl.weight_names(model))
+    lengths = np.array([5, 17, 3, 30, 1, 8], np.int32)
+    plan = tcb.tcb_pack(lengths, 32, 0, "first_fit_decreasing")
+    segtab = _dev(plan.segtab())
+    M = plan.num_slots
+    rows = torch.randn(M, 128, device="cuda").to(torch.bfloat16)
+    out = enc.unpack(plan, segtab, rows)
+    torch.cuda.synchronize()
+    a = plan.arrays()
+    cu = np.concatenate([[0], np.cumsum(lengths)])
+    r = rows.cpu()
+    o = out.cpu()
+    for s, req in enumerate(a["seg_req"]):
+        st = a["seg_start"][s]
+        assert torch.equal(o[cu[req]:cu[req + 1]], r[st:st + lengths[req]])
