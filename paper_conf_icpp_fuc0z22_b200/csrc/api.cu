@@ -140,15 +140,17 @@ struct tcb_weights {
   std::vector<const void*> t;
   float* pe_table = nullptr;
   struct LayerMaps {
-    CUtensorMap qkv, o, w1, w2;
+    CUtensorMap qkv, o, w1, w2;  // W operands (built once)
   };
   std::vector<LayerMaps> maps;
-  // activation TMA descriptors, rebuilt when the (rows, workspace) pointers change
+  // activation TMA descriptors, rebuilt when the (rows, workspace) pointers change:
+  // A-role (GEMM input) and C-role (GEMM output / residual input) views of each buffer
   std::mutex mu;
   const void* c_rows = nullptr;
   const void* c_ws = nullptr;
   int64_t c_M = -1;
-  CUtensorMap mX{}, mAtt{}, mX1{}, mH{};
+  CUtensorMap aX{}, aAtt{}, aX1{}, aH{};
+  CUtensorMap cQkv{}, cZ{}, cH{}, cX{}, cX1{};
 
   const void* tok_emb() const { return t[0]; }
   const void* pos_emb() const { return t[1]; }
@@ -275,14 +277,10 @@ tcb_status tcb_weights_create(const tcb_model_config* cfg, const void* const* te
     w->maps.resize(c.num_layers);
     for (int l = 0; l < c.num_layers; ++l) {
       const int d = c.d_model, f = c.d_ff;
-      bool ok = tcb::k::make_tmap_bf16(&w->maps[l].qkv, w->L(l, W_QKV), 3 * d, d,
-                                       tcb::k::linear_tc_block_n(3 * d)) &&
-                tcb::k::make_tmap_bf16(&w->maps[l].o, w->L(l, W_O), d, d,
-                                       tcb::k::linear_tc_block_n(d)) &&
-                tcb::k::make_tmap_bf16(&w->maps[l].w1, w->L(l, W_1), f, d,
-                                       tcb::k::linear_tc_block_n(f)) &&
-                tcb::k::make_tmap_bf16(&w->maps[l].w2, w->L(l, W_2), d, f,
-                                       tcb::k::linear_tc_block_n(d));
+      bool ok = tcb::k::make_gemm_w_map(&w->maps[l].qkv, w->L(l, W_QKV), 3 * d, d) &&
+                tcb::k::make_gemm_w_map(&w->maps[l].o, w->L(l, W_O), d, d) &&
+                tcb::k::make_gemm_w_map(&w->maps[l].w1, w->L(l, W_1), f, d) &&
+                tcb::k::make_gemm_w_map(&w->maps[l].w2, w->L(l, W_2), d, f);
       if (!ok) {
         if (w->pe_table) cudaFree(w->pe_table);
         delete w;
@@ -347,10 +345,15 @@ tcb_status tcb_encoder_forward(const tcb_weights* wc, const tcb_plan* plan,
     {
       std::lock_guard<std::mutex> g(w->mu);
       if (w->c_rows != d_rows || w->c_ws != d_ws || w->c_M != M) {
-        const bool ok = tcb::k::make_tmap_bf16(&w->mX, d_rows, M, d, 128) &&
-                        tcb::k::make_tmap_bf16(&w->mAtt, att, M, d, 128) &&
-                        tcb::k::make_tmap_bf16(&w->mX1, x1, M, d, 128) &&
-                        tcb::k::make_tmap_bf16(&w->mH, hbuf, M, f, 128);
+        using namespace tcb::k;
+        const bool ok = make_gemm_a_map(&w->aX, d_rows, M, d) &&
+                        make_gemm_a_map(&w->aAtt, att, M, d) &&
+                        make_gemm_a_map(&w->aX1, x1, M, d) &&
+                        make_gemm_a_map(&w->aH, hbuf, M, f) &&
+                        make_gemm_c_map(&w->cQkv, qkv, M, 3 * d) &&
+                        make_gemm_c_map(&w->cZ, z, M, d) && make_gemm_c_map(&w->cH, hbuf, M, f) &&
+                        make_gemm_c_map(&w->cX, d_rows, M, d) &&
+                        make_gemm_c_map(&w->cX1, x1, M, d);
         if (!ok) return fail(TCB_ERR_CUDA, "cuTensorMapEncodeTiled failed for an activation");
         w->c_rows = d_rows;
         w->c_ws = d_ws;
@@ -359,22 +362,22 @@ tcb_status tcb_encoder_forward(const tcb_weights* wc, const tcb_plan* plan,
     }
     for (int l = 0; l < c.num_layers; ++l) {
       const auto& mp = w->maps[l];
-      TCB_LAUNCH(TCB_K_GEMM_QKV, s, tcb::k::launch_linear_bf16_tc(w->mX, mp.qkv, M, 3 * d, d,
-                                                                  w->Lf(l, B_QKV), nullptr,
-                                                                  TCB_EPI_BIAS, qkv, s));
+      const tcb::k::GemmMaps g_qkv{w->aX, mp.qkv, w->cQkv, w->cQkv};
+      const tcb::k::GemmMaps g_o{w->aAtt, mp.o, w->cZ, w->cX};
+      const tcb::k::GemmMaps g_1{w->aX1, mp.w1, w->cH, w->cH};
+      const tcb::k::GemmMaps g_2{w->aH, mp.w2, w->cZ, w->cX1};
+      TCB_LAUNCH(TCB_K_GEMM_QKV, s, tcb::k::launch_linear_bf16_tc(g_qkv, M, 3 * d, d,
+                                                                  w->Lf(l, B_QKV), TCB_EPI_BIAS, s));
       TCB_LAUNCH(TCB_K_ATTN, s, tcb::k::launch_attention_bf16(M, d, c.num_heads, qkv, seg,
                                                               segtab, att, s));
-      TCB_LAUNCH(TCB_K_GEMM_O, s, tcb::k::launch_linear_bf16_tc(w->mAtt, mp.o, M, d, d,
-                                                                w->Lf(l, B_O), d_rows,
-                                                                TCB_EPI_BIAS_RESIDUAL, z, s));
+      TCB_LAUNCH(TCB_K_GEMM_O, s, tcb::k::launch_linear_bf16_tc(g_o, M, d, d, w->Lf(l, B_O),
+                                                                TCB_EPI_BIAS_RESIDUAL, s));
       TCB_LAUNCH(TCB_K_LN, s, tcb::k::launch_layernorm(1, M, d, z, w->Lf(l, LN1_G),
                                                        w->Lf(l, LN1_B), c.ln_eps, seg, x1, s));
-      TCB_LAUNCH(TCB_K_GEMM_FFN1, s, tcb::k::launch_linear_bf16_tc(w->mX1, mp.w1, M, f, d,
-                                                                   w->Lf(l, B_1), nullptr,
-                                                                   act_epi, hbuf, s));
-      TCB_LAUNCH(TCB_K_GEMM_FFN2, s, tcb::k::launch_linear_bf16_tc(w->mH, mp.w2, M, d, f,
-                                                                   w->Lf(l, B_2), x1,
-                                                                   TCB_EPI_BIAS_RESIDUAL, z, s));
+      TCB_LAUNCH(TCB_K_GEMM_FFN1, s, tcb::k::launch_linear_bf16_tc(g_1, M, f, d, w->Lf(l, B_1),
+                                                                   act_epi, s));
+      TCB_LAUNCH(TCB_K_GEMM_FFN2, s, tcb::k::launch_linear_bf16_tc(g_2, M, d, f, w->Lf(l, B_2),
+                                                                   TCB_EPI_BIAS_RESIDUAL, s));
       TCB_LAUNCH(TCB_K_LN, s, tcb::k::launch_layernorm(1, M, d, z, w->Lf(l, LN2_G),
                                                        w->Lf(l, LN2_B), c.ln_eps, seg, d_rows, s));
     }
@@ -449,11 +452,12 @@ tcb_status tcb_op_linear(int32_t dtype, int64_t M, int32_t N, int32_t K, const v
   }
   if (K % 64 != 0 || N % 64 != 0 || M > INT32_MAX)
     return fail(TCB_ERR_UNSUPPORTED, "tcb_op_linear (bf16): needs K % 64 == 0 and N % 64 == 0");
-  CUtensorMap ma, mw;
-  if (!tcb::k::make_tmap_bf16(&ma, A, M, K, 128) ||
-      !tcb::k::make_tmap_bf16(&mw, W, N, K, tcb::k::linear_tc_block_n(N)))
+  tcb::k::GemmMaps maps;
+  if (!tcb::k::make_gemm_a_map(&maps.a, A, M, K) || !tcb::k::make_gemm_w_map(&maps.w, W, N, K) ||
+      !tcb::k::make_gemm_c_map(&maps.c, C, M, N) ||
+      !tcb::k::make_gemm_c_map(&maps.r, epi == TCB_EPI_BIAS_RESIDUAL ? R : C, M, N))
     return fail(TCB_ERR_CUDA, "tcb_op_linear: cuTensorMapEncodeTiled failed (alignment?)");
-  TCB_LAUNCH(TCB_K_GEMM_QKV, s, tcb::k::launch_linear_bf16_tc(ma, mw, M, N, K, bias, R, epi, C, s));
+  TCB_LAUNCH(TCB_K_GEMM_QKV, s, tcb::k::launch_linear_bf16_tc(maps, M, N, K, bias, epi, s));
   return TCB_OK;
 }
 

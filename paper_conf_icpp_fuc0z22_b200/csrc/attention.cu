@@ -78,7 +78,7 @@ attn_bf16_kernel(const __nv_bfloat16* __restrict__ qkv, const int32_t* __restric
   __shared__ alignas(128) __nv_bfloat16 sQ[QB * DH];
   __shared__ alignas(128) __nv_bfloat16 sK[2][KC * DH];
   __shared__ alignas(128) __nv_bfloat16 sV[2][KC * DH];
-  __shared__ int sSegK[2][KC];
+  __shared__ alignas(16) int sSegK[2][KC];
   __shared__ int sLo[4], sHi[4];
 
   const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
@@ -158,14 +158,19 @@ attn_bf16_kernel(const __nv_bfloat16* __restrict__ qkv, const int32_t* __restric
       cp_async_commit();
       cp_async_wait<1>();
       __syncthreads();
-      if (whi >= 0) {
-#pragma unroll 1
+      // sub-blocks [sb_lo, sb_hi) of this chunk intersect the warp's key interval; the
+      // others are cross-request (or beyond the row) and are skipped outright
+      const int lim = min(whi, chi);
+      const int sb_lo = wlo > kbase ? (wlo - kbase) >> 4 : 0;
+      const int sb_hi = lim > kbase ? min(KC / 16, (lim - kbase + 15) >> 4) : 0;
+      if (whi >= 0 && sb_lo < sb_hi) {
+        // S = Q K^T for 16 queries x up to 64 keys
+        float s[KC / 16][2][4];
+#pragma unroll
         for (int sb = 0; sb < KC / 16; ++sb) {
-          const int kb = kbase + sb * 16;
-          if (kb >= chi) break;
-          if (kb >= whi || kb + 16 <= wlo) continue;  // cross-request sub-block: skipped
-          // S = Q K^T for 16 queries x 16 keys
-          float s[2][4] = {{0.f, 0.f, 0.f, 0.f}, {0.f, 0.f, 0.f, 0.f}};
+#pragma unroll
+          for (int j = 0; j < 2; ++j) s[sb][j][0] = s[sb][j][1] = s[sb][j][2] = s[sb][j][3] = 0.f;
+          if (sb < sb_lo || sb >= sb_hi) continue;   // warp-uniform
 #pragma unroll
           for (int ks = 0; ks < 4; ++ks) {
             const int mi = lane >> 3;
@@ -173,49 +178,58 @@ attn_bf16_kernel(const __nv_bfloat16* __restrict__ qkv, const int32_t* __restric
             const int c = 2 * ks + (mi & 1);
             uint32_t k0, k1, k2, k3;
             ldsm_x4(smem_u32(&sK[buf][swz(r, c)]), k0, k1, k2, k3);
-            mma_bf16(s[0], qf[ks], k0, k1);
-            mma_bf16(s[1], qf[ks], k2, k3);
+            mma_bf16(s[sb][0], qf[ks], k0, k1);
+            mma_bf16(s[sb][1], qf[ks], k2, k3);
           }
-          // mask (M of Eq. (6)) + scale into the log2 domain
-          float bmA = -INFINITY, bmB = -INFINITY;
+        }
+        // mask M of Eq. (6) (pairs of different requests -> -inf) + scale to log2 domain
+        float bmA = -INFINITY, bmB = -INFINITY;
+#pragma unroll
+        for (int sb = 0; sb < KC / 16; ++sb) {
 #pragma unroll
           for (int j = 0; j < 2; ++j) {
             const int kl = sb * 16 + j * 8 + 2 * t4;
-            const int sk0 = sSegK[buf][kl], sk1 = sSegK[buf][kl + 1];
-            s[j][0] = (segA >= 0 && sk0 == segA) ? s[j][0] * scale_log2 : -INFINITY;
-            s[j][1] = (segA >= 0 && sk1 == segA) ? s[j][1] * scale_log2 : -INFINITY;
-            s[j][2] = (segB >= 0 && sk0 == segB) ? s[j][2] * scale_log2 : -INFINITY;
-            s[j][3] = (segB >= 0 && sk1 == segB) ? s[j][3] * scale_log2 : -INFINITY;
-            bmA = fmaxf(bmA, fmaxf(s[j][0], s[j][1]));
-            bmB = fmaxf(bmB, fmaxf(s[j][2], s[j][3]));
+            const int2 sk = *reinterpret_cast<const int2*>(&sSegK[buf][kl]);
+            const bool live = sb >= sb_lo && sb < sb_hi;
+            s[sb][j][0] = (live && sk.x == segA) ? s[sb][j][0] * scale_log2 : -INFINITY;
+            s[sb][j][1] = (live && sk.y == segA) ? s[sb][j][1] * scale_log2 : -INFINITY;
+            s[sb][j][2] = (live && sk.x == segB) ? s[sb][j][2] * scale_log2 : -INFINITY;
+            s[sb][j][3] = (live && sk.y == segB) ? s[sb][j][3] * scale_log2 : -INFINITY;
+            bmA = fmaxf(bmA, fmaxf(s[sb][j][0], s[sb][j][1]));
+            bmB = fmaxf(bmB, fmaxf(s[sb][j][2], s[sb][j][3]));
           }
-          bmA = fmaxf(bmA, __shfl_xor_sync(0xffffffffu, bmA, 1));
-          bmA = fmaxf(bmA, __shfl_xor_sync(0xffffffffu, bmA, 2));
-          bmB = fmaxf(bmB, __shfl_xor_sync(0xffffffffu, bmB, 1));
-          bmB = fmaxf(bmB, __shfl_xor_sync(0xffffffffu, bmB, 2));
-          const float nmA = fmaxf(mA, bmA), nmB = fmaxf(mB, bmB);
-          const float uA = nmA == -INFINITY ? 0.f : nmA;
-          const float uB = nmB == -INFINITY ? 0.f : nmB;
+        }
+        bmA = fmaxf(bmA, __shfl_xor_sync(0xffffffffu, bmA, 1));
+        bmA = fmaxf(bmA, __shfl_xor_sync(0xffffffffu, bmA, 2));
+        bmB = fmaxf(bmB, __shfl_xor_sync(0xffffffffu, bmB, 1));
+        bmB = fmaxf(bmB, __shfl_xor_sync(0xffffffffu, bmB, 2));
+        const float nmA = fmaxf(mA, bmA), nmB = fmaxf(mB, bmB);
+        const float uA = nmA == -INFINITY ? 0.f : nmA;
+        const float uB = nmB == -INFINITY ? 0.f : nmB;
+        if (nmA != mA || nmB != mB) {          // rescale only when a running max moved
           const float aA = exp2f(mA - uA), aB = exp2f(mB - uB);
-          mA = nmA;
-          mB = nmB;
-          float p[2][4];
-          float sumA = 0.f, sumB = 0.f;
-#pragma unroll
-          for (int j = 0; j < 2; ++j) {
-            p[j][0] = exp2f(s[j][0] - uA);
-            p[j][1] = exp2f(s[j][1] - uA);
-            p[j][2] = exp2f(s[j][2] - uB);
-            p[j][3] = exp2f(s[j][3] - uB);
-            sumA += p[j][0] + p[j][1];
-            sumB += p[j][2] + p[j][3];
-          }
-          lA = lA * aA + sumA;
-          lB = lB * aB + sumB;
+          lA *= aA;
+          lB *= aB;
 #pragma unroll
           for (int j = 0; j < 8; ++j) {
             acc[j][0] *= aA; acc[j][1] *= aA;
             acc[j][2] *= aB; acc[j][3] *= aB;
+          }
+          mA = nmA;
+          mB = nmB;
+        }
+#pragma unroll
+        for (int sb = 0; sb < KC / 16; ++sb) {
+          if (sb < sb_lo || sb >= sb_hi) continue;   // warp-uniform
+          float p[2][4];
+#pragma unroll
+          for (int j = 0; j < 2; ++j) {
+            p[j][0] = exp2f(s[sb][j][0] - uA);
+            p[j][1] = exp2f(s[sb][j][1] - uA);
+            p[j][2] = exp2f(s[sb][j][2] - uB);
+            p[j][3] = exp2f(s[sb][j][3] - uB);
+            lA += p[j][0] + p[j][1];
+            lB += p[j][2] + p[j][3];
           }
           const uint32_t pa[4] = {pack_bf16(p[0][0], p[0][1]), pack_bf16(p[0][2], p[0][3]),
                                   pack_bf16(p[1][0], p[1][1]), pack_bf16(p[1][2], p[1][3])};
@@ -235,6 +249,7 @@ attn_bf16_kernel(const __nv_bfloat16* __restrict__ qkv, const int32_t* __restric
       __syncthreads();
     }
   }
+  cp_async_wait<0>();
   // --- 3. normalise and store (pad / empty rows -> 0) ------------------------------------
   lA += __shfl_xor_sync(0xffffffffu, lA, 1);
   lA += __shfl_xor_sync(0xffffffffu, lA, 2);

@@ -10,6 +10,7 @@
 #include <cuda_bf16.h>
 
 #include <cmath>
+#include <type_traits>
 
 #include "kernels.h"
 
@@ -18,7 +19,6 @@ namespace k {
 namespace {
 
 constexpr int kWarpsPerBlock = 8;
-constexpr int kMaxVecPerLane = 8;  // 16-byte vectors per lane: d <= 8*32*8 = 2048 (bf16)
 
 template <typename T> struct Vec;
 template <> struct Vec<float> {
@@ -73,7 +73,7 @@ __device__ __forceinline__ int find_segment(const int4* segtab, int64_t slot, in
   return found;
 }
 
-template <typename T>
+template <typename T, int NV>
 __global__ void __launch_bounds__(kWarpsPerBlock * 32) pack_embed_kernel(EmbedArgs a) {
   constexpr int V = Vec<T>::N;
   const int lane = threadIdx.x & 31;
@@ -101,10 +101,10 @@ __global__ void __launch_bounds__(kWarpsPerBlock * 32) pack_embed_kernel(EmbedAr
     if (a.positions) a.positions[slot] = pos;
   }
   const T* e = reinterpret_cast<const T*>(a.tok_emb) + static_cast<int64_t>(id) * d;
-  float v[kMaxVecPerLane][V];
+  float v[NV][V];
   float sum = 0.f;
 #pragma unroll
-  for (int j = 0; j < kMaxVecPerLane; ++j) {
+  for (int j = 0; j < NV; ++j) {
     const int i = lane + 32 * j;
     if (i < nvec) {
       Vec<T>::load(e + i * V, v[j]);
@@ -132,13 +132,13 @@ __global__ void __launch_bounds__(kWarpsPerBlock * 32) pack_embed_kernel(EmbedAr
     const float mean = warp_sum(sum) / d;
     float sq = 0.f;
 #pragma unroll
-    for (int j = 0; j < kMaxVecPerLane; ++j)
+    for (int j = 0; j < NV; ++j)
       if (lane + 32 * j < nvec)
 #pragma unroll
         for (int c = 0; c < V; ++c) { const float t = v[j][c] - mean; sq += t * t; }
     const float rstd = rsqrtf(warp_sum(sq) / d + a.ln_eps);
 #pragma unroll
-    for (int j = 0; j < kMaxVecPerLane; ++j) {
+    for (int j = 0; j < NV; ++j) {
       const int i = lane + 32 * j;
       if (i < nvec)
 #pragma unroll
@@ -147,64 +147,82 @@ __global__ void __launch_bounds__(kWarpsPerBlock * 32) pack_embed_kernel(EmbedAr
     }
   }
 #pragma unroll
-  for (int j = 0; j < kMaxVecPerLane; ++j) {
+  for (int j = 0; j < NV; ++j) {
     const int i = lane + 32 * j;
     if (i < nvec) Vec<T>::store(x + i * V, v[j]);
   }
 }
 
-template <typename T>
+// LayerNorm: each warp normalises kLnRows rows; all their 16-byte loads are issued before
+// the first reduction so each lane keeps kLnRows * NV loads in flight.
+constexpr int kLnRows = 2;
+
+template <typename T, int NV>
 __global__ void __launch_bounds__(kWarpsPerBlock * 32)
 layernorm_kernel(int64_t rows, int d, const T* __restrict__ Z, const float* __restrict__ g,
                  const float* __restrict__ b, float eps, const int32_t* __restrict__ seg_ids,
                  T* __restrict__ Y) {
   constexpr int V = Vec<T>::N;
   const int lane = threadIdx.x & 31;
-  const int64_t row = static_cast<int64_t>(blockIdx.x) * kWarpsPerBlock + (threadIdx.x >> 5);
-  if (row >= rows) return;
+  const int64_t row0 =
+      (static_cast<int64_t>(blockIdx.x) * kWarpsPerBlock + (threadIdx.x >> 5)) * kLnRows;
+  if (row0 >= rows) return;
   const int nvec = d / V;
-  T* y = Y + row * d;
-  if (seg_ids && __ldg(&seg_ids[row]) < 0) {  // pad row -> 0 (R12)
-    float z[V] = {};
-    for (int i = lane; i < nvec; i += 32) Vec<T>::store(y + i * V, z);
-    return;
-  }
-  const T* z = Z + row * d;
-  float v[kMaxVecPerLane][V];
-  float sum = 0.f;
+  float v[kLnRows][NV][V];
+  bool pad[kLnRows];
 #pragma unroll
-  for (int j = 0; j < kMaxVecPerLane; ++j) {
-    const int i = lane + 32 * j;
-    if (i < nvec) {
-      Vec<T>::load(z + i * V, v[j]);
+  for (int rr = 0; rr < kLnRows; ++rr) {
+    const int64_t row = row0 + rr;
+    pad[rr] = row >= rows || (seg_ids && __ldg(&seg_ids[row]) < 0);
+    if (row >= rows) continue;
+    const T* z = Z + row * d;
 #pragma unroll
-      for (int c = 0; c < V; ++c) sum += v[j][c];
+    for (int j = 0; j < NV; ++j) {
+      const int i = lane + 32 * j;
+      if (i < nvec) Vec<T>::load(z + i * V, v[rr][j]);
     }
   }
-  const float mean = warp_sum(sum) / d;
-  float sq = 0.f;
 #pragma unroll
-  for (int j = 0; j < kMaxVecPerLane; ++j)
-    if (lane + 32 * j < nvec)
+  for (int rr = 0; rr < kLnRows; ++rr) {
+    const int64_t row = row0 + rr;
+    if (row >= rows) break;
+    T* y = Y + row * d;
+    if (pad[rr]) {  // pad row -> 0 (R12)
+      float zero[V] = {};
+      for (int i = lane; i < nvec; i += 32) Vec<T>::store(y + i * V, zero);
+      continue;
+    }
+    float sum = 0.f;
 #pragma unroll
-      for (int c = 0; c < V; ++c) { const float t = v[j][c] - mean; sq += t * t; }
-  const float rstd = rsqrtf(warp_sum(sq) / d + eps);
+    for (int j = 0; j < NV; ++j)
+      if (lane + 32 * j < nvec)
 #pragma unroll
-  for (int j = 0; j < kMaxVecPerLane; ++j) {
-    const int i = lane + 32 * j;
-    if (i < nvec) {
-      float o[V];
-      const float4* gg = reinterpret_cast<const float4*>(g + i * V);
-      const float4* bb = reinterpret_cast<const float4*>(b + i * V);
+        for (int c = 0; c < V; ++c) sum += v[rr][j][c];
+    const float mean = warp_sum(sum) / d;
+    float sq = 0.f;
 #pragma unroll
-      for (int c = 0; c < V; c += 4) {
-        const float4 g4 = __ldg(gg + c / 4), b4 = __ldg(bb + c / 4);
-        o[c] = (v[j][c] - mean) * rstd * g4.x + b4.x;
-        o[c + 1] = (v[j][c + 1] - mean) * rstd * g4.y + b4.y;
-        o[c + 2] = (v[j][c + 2] - mean) * rstd * g4.z + b4.z;
-        o[c + 3] = (v[j][c + 3] - mean) * rstd * g4.w + b4.w;
+    for (int j = 0; j < NV; ++j)
+      if (lane + 32 * j < nvec)
+#pragma unroll
+        for (int c = 0; c < V; ++c) { const float t = v[rr][j][c] - mean; sq += t * t; }
+    const float rstd = rsqrtf(warp_sum(sq) / d + eps);
+#pragma unroll
+    for (int j = 0; j < NV; ++j) {
+      const int i = lane + 32 * j;
+      if (i < nvec) {
+        float o[V];
+        const float4* gg = reinterpret_cast<const float4*>(g + i * V);
+        const float4* bb = reinterpret_cast<const float4*>(b + i * V);
+#pragma unroll
+        for (int c = 0; c < V; c += 4) {
+          const float4 g4 = __ldg(gg + c / 4), b4 = __ldg(bb + c / 4);
+          o[c] = (v[rr][j][c] - mean) * rstd * g4.x + b4.x;
+          o[c + 1] = (v[rr][j][c + 1] - mean) * rstd * g4.y + b4.y;
+          o[c + 2] = (v[rr][j][c + 2] - mean) * rstd * g4.z + b4.z;
+          o[c + 3] = (v[rr][j][c + 3] - mean) * rstd * g4.w + b4.w;
+        }
+        Vec<T>::store(y + i * V, o);
       }
-      Vec<T>::store(y + i * V, o);
     }
   }
 }
@@ -238,13 +256,34 @@ __global__ void pe_table_kernel(float* table, int max_pos, int d, int variant) {
   table[i] = static_cast<float>(dim % 2 == 0 ? sin(ang) : cos(ang));
 }
 
+// Runtime -> compile-time vectors-per-lane (registers hold exactly the row).
+template <typename F>
+bool dispatch_nv(int nv, F&& f) {
+  switch (nv) {
+    case 1: f(std::integral_constant<int, 1>{}); return true;
+    case 2: f(std::integral_constant<int, 2>{}); return true;
+    case 3: f(std::integral_constant<int, 3>{}); return true;
+    case 4: f(std::integral_constant<int, 4>{}); return true;
+    case 5: f(std::integral_constant<int, 5>{}); return true;
+    case 6: f(std::integral_constant<int, 6>{}); return true;
+    case 7: f(std::integral_constant<int, 7>{}); return true;
+    case 8: f(std::integral_constant<int, 8>{}); return true;
+    default: return false;
+  }
+}
+
 }  // namespace
 
 cudaError_t launch_embed(int dtype, const EmbedArgs& a, cudaStream_t s) {
   if (a.num_slots == 0) return cudaSuccess;
   const unsigned grid = static_cast<unsigned>((a.num_slots + kWarpsPerBlock - 1) / kWarpsPerBlock);
-  if (dtype == 0) pack_embed_kernel<float><<<grid, kWarpsPerBlock * 32, 0, s>>>(a);
-  else pack_embed_kernel<__nv_bfloat16><<<grid, kWarpsPerBlock * 32, 0, s>>>(a);
+  const int nv = (a.d / (dtype == 0 ? 4 : 8) + 31) / 32;
+  auto go = [&](auto tag) {
+    constexpr int NV = decltype(tag)::value;
+    if (dtype == 0) pack_embed_kernel<float, NV><<<grid, kWarpsPerBlock * 32, 0, s>>>(a);
+    else pack_embed_kernel<__nv_bfloat16, NV><<<grid, kWarpsPerBlock * 32, 0, s>>>(a);
+  };
+  if (!dispatch_nv(nv, go)) return cudaErrorInvalidValue;
   return cudaGetLastError();
 }
 
@@ -252,14 +291,20 @@ cudaError_t launch_layernorm(int dtype, int64_t rows, int d, const void* Z, cons
                              const float* b, float eps, const int32_t* seg_ids, void* Y,
                              cudaStream_t s) {
   if (rows == 0) return cudaSuccess;
-  const unsigned grid = static_cast<unsigned>((rows + kWarpsPerBlock - 1) / kWarpsPerBlock);
-  if (dtype == 0)
-    layernorm_kernel<float><<<grid, kWarpsPerBlock * 32, 0, s>>>(
-        rows, d, static_cast<const float*>(Z), g, b, eps, seg_ids, static_cast<float*>(Y));
-  else
-    layernorm_kernel<__nv_bfloat16><<<grid, kWarpsPerBlock * 32, 0, s>>>(
-        rows, d, static_cast<const __nv_bfloat16*>(Z), g, b, eps, seg_ids,
-        static_cast<__nv_bfloat16*>(Y));
+  const int64_t per_block = static_cast<int64_t>(kWarpsPerBlock) * kLnRows;
+  const unsigned grid = static_cast<unsigned>((rows + per_block - 1) / per_block);
+  const int nv = (d / (dtype == 0 ? 4 : 8) + 31) / 32;
+  auto go = [&](auto tag) {
+    constexpr int NV = decltype(tag)::value;
+    if (dtype == 0)
+      layernorm_kernel<float, NV><<<grid, kWarpsPerBlock * 32, 0, s>>>(
+          rows, d, static_cast<const float*>(Z), g, b, eps, seg_ids, static_cast<float*>(Y));
+    else
+      layernorm_kernel<__nv_bfloat16, NV><<<grid, kWarpsPerBlock * 32, 0, s>>>(
+          rows, d, static_cast<const __nv_bfloat16*>(Z), g, b, eps, seg_ids,
+          static_cast<__nv_bfloat16*>(Y));
+  };
+  if (!dispatch_nv(nv, go)) return cudaErrorInvalidValue;
   return cudaGetLastError();
 }
 

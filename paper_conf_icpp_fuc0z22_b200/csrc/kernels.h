@@ -41,15 +41,23 @@ cudaError_t launch_linear_f32(int64_t M, int N, int K, const float* A, const flo
                               const float* bias, const float* R, int epi, float* C,
                               cudaStream_t s);
 
-// Host-side TMA descriptor for a row-major bf16 matrix [rows, cols] (cols contiguous),
-// box = box_rows x 64 columns, 128-byte swizzle.  Returns false on failure.
+// Tensor-core GEMM (linear_tc.cu).  TMA descriptors are built on the host: A [M, K]
+// (128-row boxes, 128B swizzle), W [N, K] (BN/CG-row boxes), C / R [M, N] (32 x 32 boxes,
+// 64B swizzle; R is read only by the residual epilogue).
+struct GemmMaps {
+  CUtensorMap a, w, c, r;
+};
+struct GemmShape {
+  int cg, bn;  // CTAs per MMA tile (cta_group) and tile width in N
+};
+GemmShape linear_tc_shape(int N);
 bool make_tmap_bf16(CUtensorMap* map, const void* ptr, uint64_t rows, uint64_t cols,
-                    uint32_t box_rows);
-// The box_rows the tensor-core GEMM needs for its B (weight) operand at this N.
-int linear_tc_block_n(int N);
-cudaError_t launch_linear_bf16_tc(const CUtensorMap& tmA, const CUtensorMap& tmW, int64_t M,
-                                  int N, int K, const float* bias, const void* R, int epi,
-                                  void* C, cudaStream_t s);
+                    uint32_t box_rows, uint32_t box_cols, int swizzle_bytes);
+bool make_gemm_a_map(CUtensorMap* map, const void* A, uint64_t M, uint64_t K);
+bool make_gemm_w_map(CUtensorMap* map, const void* W, uint64_t N, uint64_t K);
+bool make_gemm_c_map(CUtensorMap* map, const void* C, uint64_t M, uint64_t N);
+cudaError_t launch_linear_bf16_tc(const GemmMaps& maps, int64_t M, int N, int K,
+                                  const float* bias, int epi, cudaStream_t s);
 
 // Attention ------------------------------------------------------------------------------
 cudaError_t launch_attention_bf16(int64_t num_slots, int d_model, int num_heads,

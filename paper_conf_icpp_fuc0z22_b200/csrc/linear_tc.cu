@@ -1,22 +1,29 @@
 // linear_tc.cu -- bf16 linear layers on the 5th-generation tensor cores (sm_100a):
 //   C[M, N] = epi(A[M, K] . W[N, K]^T + bias[N]) (+ R[M, N]),  fp32 accumulation in TMEM.
-// The QKV projection (Eq. (3), with W_Q|W_K|W_V stacked along N), W_O and the two
-// FFN linears of every encoder layer.  These are the dense contractions of the
-// path, so they run on tcgen05.mma:
-//   * persistent CTAs (one per SM), tiles of 128 x BN walked M-major-inner so the weight
-//     tile stays hot in L2 and consecutive CTAs share A rows;
-//   * warp 0: TMA producer (cp.async.bulk.tensor, 128B swizzle) into a STAGES-deep ring of
-//     {A 128x64, W BNx64} bf16 tiles guarded by full/empty mbarriers;
-//   * warp 1: one elected thread issues tcgen05.mma.cta_group::1.kind::f16 (M=128, N=BN,
-//     K=16) from shared-memory descriptors into a double-buffered TMEM accumulator
-//     (2 x BN fp32 columns) and tcgen05.commit's the smem slot / accumulator barriers;
-//   * warp 2: TMEM allocator;
-//   * warps 4..11: epilogue -- tcgen05.ld 32 lanes x 32 columns, + bias, GELU(erf)/ReLU or
-//     + residual, round to bf16, 16-byte stores; overlaps the next tile's MMAs.
+// The QKV projection (Eq. (3), W_Q|W_K|W_V stacked along N), W_O and the two FFN
+// linears of every encoder layer -- the dense contractions of the path.
+//
+// Design (persistent, warp-specialised, one CTA per SM):
+//   * CG = 2 (default): a cluster of 2 CTAs (a TPC pair) computes a 256 x BN tile with
+//     tcgen05.mma.cta_group::2 (M = 256): each CTA TMA-loads its own 128 rows of A and
+//     BN/2 rows of W into a STAGES-deep smem ring; the even CTA's single MMA thread issues
+//     the MMAs for the pair and tcgen05.commit's (multicast) the smem-slot and accumulator
+//     barriers of both CTAs.  Per SM this halves the W traffic of a 1-CTA 128 x BN tile.
+//     CG = 1: the same with 128 x BN tiles on one SM.
+//   * TMEM: double-buffered 2 x BN fp32 accumulator columns, so the epilogue of tile i
+//     overlaps the MMAs of tile i+1.
+//   * Epilogue (8 warps; warp w owns TMEM lanes 32*(w%4).. and one half of the columns):
+//     tcgen05.ld 32 lanes x 32 columns (the next chunk's load overlaps this chunk's math)
+//     -> + bias -> GELU(erf) / ReLU or + residual -> bf16 -> 64B-swizzled smem staging ->
+//     TMA bulk tensor store (coalesced; clips the M tail).  Each warp has one 2 KB staging
+//     buffer per chunk of a tile; the residual chunks of a tile are TMA-prefetched into
+//     them before the accumulator is ready, so their latency hides behind the MMAs.
 #include <cuda_bf16.h>
 #include <cudaTypedefs.h>
 
+#include <cstdlib>
 #include <mutex>
+#include <string>
 
 #include "kernels.h"
 #include "../../include/tcb_ops.h"
@@ -25,24 +32,50 @@ namespace tcb {
 namespace k {
 namespace {
 
-constexpr int BM = 128;
-constexpr int BK = 64;                 // 64 bf16 = 128 bytes = one swizzle-128B row
+constexpr int BK = 64;                  // 64 bf16 = 128 bytes = one swizzle-128B row
 constexpr int kEpiWarps = 8;
 constexpr int kThreads = (4 + kEpiWarps) * 32;
+constexpr int kStageRows = 32, kStageCols = 32;            // epilogue staging box
+constexpr int kStageBufBytes = kStageRows * kStageCols * 2;  // 2 KB
 
-template <int BN>
+template <int CG, int BN, int EPI>
 struct TcCfg {
-  static constexpr int kStages = BN == 256 ? 4 : 6;
-  static constexpr int kABytes = BM * BK * 2;
-  static constexpr int kBBytes = BN * BK * 2;
+  static constexpr int kRowsPerCta = 128;                   // A rows held by one CTA
+  static constexpr int kBRows = BN / CG;                    // W rows held by one CTA
+  static constexpr int kABytes = kRowsPerCta * BK * 2;
+  static constexpr int kBBytes = kBRows * BK * 2;
   static constexpr int kStageBytes = kABytes + kBBytes;
-  static constexpr int kTmemCols = 2 * BN;  // double-buffered accumulator
-  static constexpr int kSmemBytes = kStages * kStageBytes + 1024 /*align*/ + 256 /*barriers*/;
+  static constexpr int kChunksPerWarp = BN / 64;             // 32-column chunks per warp/tile
+  // staging buffers per epilogue warp: one per chunk when the residual tile is prefetched,
+  // else two (double-buffered TMA stores) so the freed smem deepens the operand ring
+  static constexpr int kBufs = EPI == TCB_EPI_BIAS_RESIDUAL ? kChunksPerWarp
+                               : (kChunksPerWarp < 2 ? kChunksPerWarp : 2);
+  static constexpr int kEpiBytes = kEpiWarps * kBufs * kStageBufBytes;
+  static constexpr int kStages = (225 * 1024 - kEpiBytes) / kStageBytes > 8
+                                     ? 8 : (225 * 1024 - kEpiBytes) / kStageBytes;
+  static constexpr int kTmemCols = 2 * BN;                  // double-buffered accumulator
+  static constexpr int kBarBytes = 8 * (2 * kStages + 4 + kBufs * kEpiWarps) + 16;
+  static constexpr int kSmemBytes = 1024 + kStages * kStageBytes + kEpiBytes + kBarBytes;
+  static_assert(kSmemBytes <= 232448, "shared memory budget");
+  static_assert(kTmemCols <= 512, "TMEM budget");
 };
 
 // ---- PTX helpers -------------------------------------------------------------------------
 __device__ __forceinline__ uint32_t smem_u32(const void* p) {
   return static_cast<uint32_t>(__cvta_generic_to_shared(p));
+}
+__device__ __forceinline__ uint32_t cluster_rank() {
+  uint32_t r;
+  asm volatile("mov.u32 %0, %%cluster_ctarank;" : "=r"(r));
+  return r;
+}
+__device__ __forceinline__ uint32_t map_to_rank0(uint32_t saddr) {
+  uint32_t r;
+  asm volatile("mapa.shared::cluster.u32 %0, %1, 0;" : "=r"(r) : "r"(saddr));
+  return r;
+}
+__device__ __forceinline__ void cluster_sync() {
+  asm volatile("barrier.cluster.arrive.release.aligned;\n\tbarrier.cluster.wait.acquire.aligned;" ::: "memory");
 }
 __device__ __forceinline__ void mbar_init(uint64_t* bar, uint32_t count) {
   asm volatile("mbarrier.init.shared::cta.b64 [%0], %1;" ::"r"(smem_u32(bar)), "r"(count));
@@ -51,9 +84,6 @@ __device__ __forceinline__ void mbar_expect_tx(uint64_t* bar, uint32_t bytes) {
   asm volatile("mbarrier.arrive.expect_tx.shared::cta.b64 _, [%0], %1;" ::"r"(smem_u32(bar)),
                "r"(bytes)
                : "memory");
-}
-__device__ __forceinline__ void mbar_arrive(uint64_t* bar) {
-  asm volatile("mbarrier.arrive.shared::cta.b64 _, [%0];" ::"r"(smem_u32(bar)) : "memory");
 }
 __device__ __forceinline__ void mbar_wait(uint64_t* bar, uint32_t parity) {
   const uint32_t addr = smem_u32(bar);
@@ -68,13 +98,34 @@ __device__ __forceinline__ void mbar_wait(uint64_t* bar, uint32_t parity) {
         : "memory");
   } while (!done);
 }
-__device__ __forceinline__ void tma_load_2d(void* dst, const CUtensorMap* map, uint64_t* bar,
-                                            int c0, int c1) {
-  asm volatile(
-      "cp.async.bulk.tensor.2d.shared::cluster.global.mbarrier::complete_tx::bytes"
-      " [%0], [%1, {%3, %4}], [%2];" ::"r"(smem_u32(dst)),
-      "l"(reinterpret_cast<uint64_t>(map)), "r"(smem_u32(bar)), "r"(c0), "r"(c1)
-      : "memory");
+// TMA load into this CTA's smem; completion bytes go to `bar_cluster` (own CTA for CG=1,
+// the even CTA of the pair for CG=2).
+template <int CG>
+__device__ __forceinline__ void tma_load_2d(void* dst, const CUtensorMap* map,
+                                            uint32_t bar_cluster, int c0, int c1) {
+  if constexpr (CG == 1) {
+    asm volatile(
+        "cp.async.bulk.tensor.2d.shared::cluster.global.mbarrier::complete_tx::bytes"
+        " [%0], [%1, {%3, %4}], [%2];" ::"r"(smem_u32(dst)),
+        "l"(reinterpret_cast<uint64_t>(map)), "r"(bar_cluster), "r"(c0), "r"(c1)
+        : "memory");
+  } else {
+    asm volatile(
+        "cp.async.bulk.tensor.2d.cta_group::2.shared::cluster.global.mbarrier::complete_tx::bytes"
+        " [%0], [%1, {%3, %4}], [%2];" ::"r"(smem_u32(dst)),
+        "l"(reinterpret_cast<uint64_t>(map)), "r"(bar_cluster), "r"(c0), "r"(c1)
+        : "memory");
+  }
+}
+template <int N>
+__device__ __forceinline__ void bulk_wait_read() {
+  asm volatile("cp.async.bulk.wait_group.read %0;" ::"n"(N) : "memory");
+}
+__device__ __forceinline__ void bulk_wait_all() {
+  asm volatile("cp.async.bulk.wait_group 0;" ::: "memory");
+}
+__device__ __forceinline__ void fence_async_smem() {
+  asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
 }
 __device__ __forceinline__ void tc_fence_before() {
   asm volatile("tcgen05.fence::before_thread_sync;" ::: "memory");
@@ -82,22 +133,39 @@ __device__ __forceinline__ void tc_fence_before() {
 __device__ __forceinline__ void tc_fence_after() {
   asm volatile("tcgen05.fence::after_thread_sync;" ::: "memory");
 }
+template <int CG>
 __device__ __forceinline__ void tc_commit(uint64_t* bar) {
-  asm volatile("tcgen05.commit.cta_group::1.mbarrier::arrive::one.shared::cluster.b64 [%0];" ::"r"(
-                   smem_u32(bar))
-               : "memory");
+  if constexpr (CG == 1) {
+    asm volatile("tcgen05.commit.cta_group::1.mbarrier::arrive::one.shared::cluster.b64 [%0];" ::"r"(
+                     smem_u32(bar))
+                 : "memory");
+  } else {
+    const uint16_t mask = 0x3;
+    asm volatile(
+        "tcgen05.commit.cta_group::2.mbarrier::arrive::one.shared::cluster.multicast::cluster.b64"
+        " [%0], %1;" ::"r"(smem_u32(bar)),
+        "h"(mask)
+        : "memory");
+  }
 }
+template <int CG>
 __device__ __forceinline__ void tc_mma(uint32_t tmem_d, uint64_t adesc, uint64_t bdesc,
                                        uint32_t idesc, uint32_t accumulate) {
-  asm volatile(
-      "{\n\t.reg .pred p;\n\t"
-      "setp.ne.b32 p, %4, 0;\n\t"
-      "tcgen05.mma.cta_group::1.kind::f16 [%0], %1, %2, %3, p;\n\t}" ::"r"(tmem_d),
-      "l"(adesc), "l"(bdesc), "r"(idesc), "r"(accumulate)
-      : "memory");
+  if constexpr (CG == 1) {
+    asm volatile(
+        "{\n\t.reg .pred p;\n\tsetp.ne.b32 p, %4, 0;\n\t"
+        "tcgen05.mma.cta_group::1.kind::f16 [%0], %1, %2, %3, p;\n\t}" ::"r"(tmem_d),
+        "l"(adesc), "l"(bdesc), "r"(idesc), "r"(accumulate)
+        : "memory");
+  } else {
+    asm volatile(
+        "{\n\t.reg .pred p;\n\tsetp.ne.b32 p, %4, 0;\n\t"
+        "tcgen05.mma.cta_group::2.kind::f16 [%0], %1, %2, %3, p;\n\t}" ::"r"(tmem_d),
+        "l"(adesc), "l"(bdesc), "r"(idesc), "r"(accumulate)
+        : "memory");
+  }
 }
-// 32 lanes x 32 consecutive fp32 columns: thread t of the warp gets lane (base + t).
-__device__ __forceinline__ void tmem_ld32(uint32_t taddr, uint32_t (&r)[32]) {
+__device__ __forceinline__ void tmem_ld32_nowait(uint32_t taddr, uint32_t (&r)[32]) {
   asm volatile(
       "tcgen05.ld.sync.aligned.32x32b.x32.b32 "
       "{%0,%1,%2,%3,%4,%5,%6,%7,%8,%9,%10,%11,%12,%13,%14,%15,"
@@ -108,7 +176,10 @@ __device__ __forceinline__ void tmem_ld32(uint32_t taddr, uint32_t (&r)[32]) {
         "=r"(r[19]), "=r"(r[20]), "=r"(r[21]), "=r"(r[22]), "=r"(r[23]), "=r"(r[24]),
         "=r"(r[25]), "=r"(r[26]), "=r"(r[27]), "=r"(r[28]), "=r"(r[29]), "=r"(r[30]),
         "=r"(r[31])
-      : "r"(taddr));
+      : "r"(taddr)
+      : "memory");
+}
+__device__ __forceinline__ void tmem_wait_ld() {
   asm volatile("tcgen05.wait::ld.sync.aligned;" ::: "memory");
 }
 
@@ -117,45 +188,90 @@ __device__ __forceinline__ void tmem_ld32(uint32_t taddr, uint32_t (&r)[32]) {
 __device__ __forceinline__ uint64_t sdesc_sw128(uint32_t saddr) {
   uint64_t d = 0;
   d |= static_cast<uint64_t>((saddr & 0x3FFFFu) >> 4);
-  d |= static_cast<uint64_t>(1) << 16;             // LBO = 16 B (ignored)
-  d |= static_cast<uint64_t>(1024 >> 4) << 32;     // SBO = 1024 B
-  d |= static_cast<uint64_t>(1) << 46;             // descriptor version (sm_100)
-  d |= static_cast<uint64_t>(2) << 61;             // SWIZZLE_128B
+  d |= static_cast<uint64_t>(1) << 16;
+  d |= static_cast<uint64_t>(1024 >> 4) << 32;
+  d |= static_cast<uint64_t>(1) << 46;
+  d |= static_cast<uint64_t>(2) << 61;
   return d;
 }
 
-// Instruction descriptor, kind::f16: D fp32, A/B bf16, both K-major, M=128, N=BN.
-template <int BN>
+// Instruction descriptor, kind::f16: D fp32, A/B bf16, both K-major, M = 128*CG, N = BN.
+template <int CG, int BN>
 __device__ __forceinline__ constexpr uint32_t idesc_bf16() {
   return (1u << 4) | (1u << 7) | (1u << 10) | (static_cast<uint32_t>(BN >> 3) << 17) |
-         (static_cast<uint32_t>(BM >> 4) << 24);
+         (static_cast<uint32_t>((128 * CG) >> 4) << 24);
 }
 
 __device__ __forceinline__ float gelu_erf(float x) {
   return 0.5f * x * (1.f + erff(x * 0.70710678118654752f));
 }
 
-template <int BN, int EPI>
+__device__ __forceinline__ void st_shared_v4(uint32_t addr, uint4 v) {
+  asm volatile("st.shared.v4.b32 [%0], {%1, %2, %3, %4};" ::"r"(addr), "r"(v.x), "r"(v.y),
+               "r"(v.z), "r"(v.w)
+               : "memory");
+}
+__device__ __forceinline__ uint4 ld_shared_v4(uint32_t addr) {
+  uint4 v;
+  asm volatile("ld.shared.v4.b32 {%0, %1, %2, %3}, [%4];"
+               : "=r"(v.x), "=r"(v.y), "=r"(v.z), "=r"(v.w)
+               : "r"(addr)
+               : "memory");
+  return v;
+}
+__device__ __forceinline__ void mbar_arrive_remote(uint32_t cluster_addr) {
+  asm volatile("mbarrier.arrive.shared::cluster.b64 _, [%0];" ::"r"(cluster_addr) : "memory");
+}
+
+// byte offset of 16-byte chunk c of row r in a [32 rows x 64 B] 64B-swizzled box
+__device__ __forceinline__ uint32_t sw64(int r, int c) {
+  return static_cast<uint32_t>(r * 64 + ((c ^ ((r >> 1) & 3)) << 4));
+}
+
+// Tile rasterisation.  raster 0: N-major (concurrent clusters share the W tile, each
+// streams its own A rows); raster g > 0: groups of g M-blocks, inside a group M-blocks vary
+// fastest over all N-blocks, so concurrent clusters share both A and W tiles in L2.
+__device__ __forceinline__ void tile_coords(int tile, int m_blocks, int n_blocks, int raster,
+                                            int& m_blk, int& n_blk) {
+  if (raster <= 0) {
+    n_blk = tile / m_blocks;
+    m_blk = tile % m_blocks;
+    return;
+  }
+  const int per_group = raster * n_blocks;
+  const int g = tile / per_group, r = tile % per_group;
+  const int g_rows = min(raster, m_blocks - g * raster);
+  n_blk = r / g_rows;
+  m_blk = g * raster + r % g_rows;
+}
+
+template <int CG, int BN, int EPI>
 __global__ void __launch_bounds__(kThreads, 1)
 linear_tc_kernel(const __grid_constant__ CUtensorMap tmA, const __grid_constant__ CUtensorMap tmW,
-                 int M, int N, int K, const float* __restrict__ bias,
-                 const __nv_bfloat16* __restrict__ R, __nv_bfloat16* __restrict__ C) {
-  using Cfg = TcCfg<BN>;
+                 const __grid_constant__ CUtensorMap tmC, const __grid_constant__ CUtensorMap tmR,
+                 int M, int N, int K, const float* __restrict__ bias, int raster) {
+  using Cfg = TcCfg<CG, BN, EPI>;
   constexpr int S = Cfg::kStages;
+  constexpr int TILE_M = 128 * CG;
   extern __shared__ uint8_t smem_raw[];
   uint8_t* smem = reinterpret_cast<uint8_t*>((reinterpret_cast<uintptr_t>(smem_raw) + 1023) &
                                              ~static_cast<uintptr_t>(1023));
-  uint8_t* sA = smem;                               // S x [128 x 64] bf16
-  uint8_t* sB = smem + S * Cfg::kABytes;            // S x [BN x 64] bf16
-  uint64_t* full = reinterpret_cast<uint64_t*>(smem + S * Cfg::kStageBytes);
+  uint8_t* sA = smem;                                   // S x [128 x 64] bf16
+  uint8_t* sB = smem + S * Cfg::kABytes;                // S x [BN/CG x 64] bf16
+  uint8_t* sEpi = smem + S * Cfg::kStageBytes;          // 8 warps x 2 x 2 KB
+  uint64_t* full = reinterpret_cast<uint64_t*>(sEpi + Cfg::kEpiBytes);
   uint64_t* empty = full + S;
-  uint64_t* tfull = empty + S;                      // [2]
-  uint64_t* tempty = tfull + 2;                     // [2]
-  uint32_t* tmem_slot = reinterpret_cast<uint32_t*>(tempty + 2);
+  uint64_t* tfull = empty + S;                          // [2]
+  uint64_t* tempty = tfull + 2;                         // [2] (used on the even CTA)
+  uint64_t* rbar = tempty + 2;                          // [8 warps][chunks] residual loads
+  uint32_t* tmem_slot = reinterpret_cast<uint32_t*>(rbar + Cfg::kBufs * kEpiWarps);
 
   const int warp = threadIdx.x >> 5;
   const int lane = threadIdx.x & 31;
-  const int m_blocks = (M + BM - 1) / BM;
+  const uint32_t rank = CG == 2 ? cluster_rank() : 0;
+  const int cluster_id = blockIdx.x / CG;
+  const int num_clusters = gridDim.x / CG;
+  const int m_blocks = (M + TILE_M - 1) / TILE_M;
   const int n_blocks = N / BN;
   const int num_tiles = m_blocks * n_blocks;
   const int num_kb = K / BK;
@@ -163,145 +279,229 @@ linear_tc_kernel(const __grid_constant__ CUtensorMap tmA, const __grid_constant_
   if (warp == 0 && lane == 0) {
     asm volatile("prefetch.tensormap [%0];" ::"l"(reinterpret_cast<uint64_t>(&tmA)) : "memory");
     asm volatile("prefetch.tensormap [%0];" ::"l"(reinterpret_cast<uint64_t>(&tmW)) : "memory");
+    asm volatile("prefetch.tensormap [%0];" ::"l"(reinterpret_cast<uint64_t>(&tmC)) : "memory");
     for (int i = 0; i < S; ++i) { mbar_init(&full[i], 1); mbar_init(&empty[i], 1); }
-    for (int i = 0; i < 2; ++i) { mbar_init(&tfull[i], 1); mbar_init(&tempty[i], kEpiWarps); }
+    for (int i = 0; i < 2; ++i) { mbar_init(&tfull[i], 1); mbar_init(&tempty[i], CG * kEpiWarps); }
+    for (int i = 0; i < Cfg::kBufs * kEpiWarps; ++i) mbar_init(&rbar[i], 1);
     asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
   }
   if (warp == 2) {
-    asm volatile("tcgen05.alloc.cta_group::1.sync.aligned.shared::cta.b32 [%0], %1;" ::"r"(
-                     smem_u32(tmem_slot)),
-                 "r"(Cfg::kTmemCols)
-                 : "memory");
-    asm volatile("tcgen05.relinquish_alloc_permit.cta_group::1.sync.aligned;" ::: "memory");
+    if constexpr (CG == 1) {
+      asm volatile("tcgen05.alloc.cta_group::1.sync.aligned.shared::cta.b32 [%0], %1;" ::"r"(
+                       smem_u32(tmem_slot)), "r"(Cfg::kTmemCols) : "memory");
+      asm volatile("tcgen05.relinquish_alloc_permit.cta_group::1.sync.aligned;" ::: "memory");
+    } else {
+      asm volatile("tcgen05.alloc.cta_group::2.sync.aligned.shared::cta.b32 [%0], %1;" ::"r"(
+                       smem_u32(tmem_slot)), "r"(Cfg::kTmemCols) : "memory");
+      asm volatile("tcgen05.relinquish_alloc_permit.cta_group::2.sync.aligned;" ::: "memory");
+    }
   }
   tc_fence_before();
-  __syncthreads();
+  if constexpr (CG == 2) cluster_sync(); else __syncthreads();
   tc_fence_after();
   const uint32_t tmem_base = *tmem_slot;
 
   if (warp == 0) {
-    // ===== TMA producer =====
+    // ===== TMA producer (both CTAs of a pair load their own halves) =====
     if (lane == 0) {
+      const uint32_t full0 = CG == 2 ? map_to_rank0(smem_u32(full)) : smem_u32(full);
       int stage = 0;
       uint32_t phase = 0;
-      for (int tile = blockIdx.x; tile < num_tiles; tile += gridDim.x) {
-        const int n_blk = tile / m_blocks, m_blk = tile % m_blocks;
+      for (int tile = cluster_id; tile < num_tiles; tile += num_clusters) {
+        int m_blk, n_blk;
+        tile_coords(tile, m_blocks, n_blocks, raster, m_blk, n_blk);
+        const int a_row = m_blk * TILE_M + static_cast<int>(rank) * 128;
+        const int b_row = n_blk * BN + static_cast<int>(rank) * Cfg::kBRows;
         for (int kb = 0; kb < num_kb; ++kb) {
           mbar_wait(&empty[stage], phase ^ 1);
-          mbar_expect_tx(&full[stage], Cfg::kStageBytes);
-          tma_load_2d(sA + stage * Cfg::kABytes, &tmA, &full[stage], kb * BK, m_blk * BM);
-          tma_load_2d(sB + stage * Cfg::kBBytes, &tmW, &full[stage], kb * BK, n_blk * BN);
+          if (rank == 0) mbar_expect_tx(&full[stage], CG * Cfg::kStageBytes);
+          const uint32_t fb = full0 + 8u * stage;
+          tma_load_2d<CG>(sA + stage * Cfg::kABytes, &tmA, fb, kb * BK, a_row);
+          tma_load_2d<CG>(sB + stage * Cfg::kBBytes, &tmW, fb, kb * BK, b_row);
           if (++stage == S) { stage = 0; phase ^= 1; }
         }
       }
     }
   } else if (warp == 1) {
-    // ===== MMA issuer (one thread) =====
-    constexpr uint32_t idesc = idesc_bf16<BN>();
-    int stage = 0;
-    uint32_t phase = 0;
-    int acc = 0;
-    uint32_t acc_phase = 0;
-    for (int tile = blockIdx.x; tile < num_tiles; tile += gridDim.x) {
-      mbar_wait(&tempty[acc], acc_phase ^ 1);
-      tc_fence_after();
-      const uint32_t d_tmem = tmem_base + static_cast<uint32_t>(acc * BN);
-      for (int kb = 0; kb < num_kb; ++kb) {
-        mbar_wait(&full[stage], phase);
+    // ===== MMA issuer: one thread of the even CTA drives the pair =====
+    if (rank == 0) {
+#ifdef TCB_GEMM_PROBE
+      long long t_start = clock64(), t_full = 0, t_empty = 0, t_issue = 0;
+#endif
+      constexpr uint32_t idesc = idesc_bf16<CG, BN>();
+      int stage = 0;
+      uint32_t phase = 0;
+      int acc = 0;
+      uint32_t acc_phase = 0;
+      for (int tile = cluster_id; tile < num_tiles; tile += num_clusters) {
+#ifdef TCB_GEMM_PROBE
+        long long t0 = clock64();
+#endif
+        mbar_wait(&tempty[acc], acc_phase ^ 1);
+#ifdef TCB_GEMM_PROBE
+        t_empty += clock64() - t0;
+#endif
         tc_fence_after();
-        if (lane == 0) {
-          const uint32_t a0 = smem_u32(sA + stage * Cfg::kABytes);
-          const uint32_t b0 = smem_u32(sB + stage * Cfg::kBBytes);
+        const uint32_t d_tmem = tmem_base + static_cast<uint32_t>(acc * BN);
+        for (int kb = 0; kb < num_kb; ++kb) {
+#ifdef TCB_GEMM_PROBE
+          long long t1 = clock64();
+#endif
+          mbar_wait(&full[stage], phase);
+#ifdef TCB_GEMM_PROBE
+          long long t2 = clock64();
+          t_full += t2 - t1;
+#endif
+          tc_fence_after();
+          if (lane == 0) {
+            const uint32_t a0 = smem_u32(sA + stage * Cfg::kABytes);
+            const uint32_t b0 = smem_u32(sB + stage * Cfg::kBBytes);
 #pragma unroll
-          for (int k = 0; k < BK / 16; ++k) {
-            tc_mma(d_tmem, sdesc_sw128(a0 + k * 32), sdesc_sw128(b0 + k * 32), idesc,
-                   (kb | k) != 0 ? 1u : 0u);
+            for (int k = 0; k < BK / 16; ++k)
+              tc_mma<CG>(d_tmem, sdesc_sw128(a0 + k * 32), sdesc_sw128(b0 + k * 32), idesc,
+                         (kb | k) != 0 ? 1u : 0u);
+            tc_commit<CG>(&empty[stage]);
+            if (kb == num_kb - 1) tc_commit<CG>(&tfull[acc]);
           }
-          tc_commit(&empty[stage]);
-          if (kb == num_kb - 1) tc_commit(&tfull[acc]);
+          __syncwarp();
+#ifdef TCB_GEMM_PROBE
+          t_issue += clock64() - t2;
+#endif
+          if (++stage == S) { stage = 0; phase ^= 1; }
         }
-        __syncwarp();
-        if (++stage == S) { stage = 0; phase ^= 1; }
+        acc ^= 1;
+        if (acc == 0) acc_phase ^= 1;
       }
-      acc ^= 1;
-      if (acc == 0) acc_phase ^= 1;
+#ifdef TCB_GEMM_PROBE
+      if (lane == 0 && blockIdx.x < 8)
+        printf("probe cta %d total %lld wait_full %lld wait_tempty %lld issue %lld\n", blockIdx.x,
+               clock64() - t_start, t_full, t_empty, t_issue);
+#endif
     }
   } else if (warp >= 4) {
-    // ===== Epilogue =====
+    // ===== Epilogue: TMEM -> registers -> (bias, act | residual) -> bf16 -> TMA store =====
+    constexpr int NC = Cfg::kChunksPerWarp;
+    constexpr int NB = Cfg::kBufs;
+    const int ew = warp - 4;
     const int q = warp & 3;                 // TMEM lane quarter this warp may access
-    const int half = (warp - 4) >> 2;       // which half of the BN columns
-    const int row_in_tile = q * 32 + lane;
+    const int half = ew >> 2;               // which half of the BN columns
+    const uint32_t bufs = smem_u32(sEpi) + ew * NB * kStageBufBytes;
+    uint64_t* my_rbar = rbar + NB * ew;
+    uint32_t rphase = 0;                    // phase of this warp's residual barriers
+    const uint32_t tempty0 = CG == 2 ? map_to_rank0(smem_u32(tempty)) : smem_u32(tempty);
     int acc = 0;
     uint32_t acc_phase = 0;
-    for (int tile = blockIdx.x; tile < num_tiles; tile += gridDim.x) {
-      const int n_blk = tile / m_blocks, m_blk = tile % m_blocks;
-      mbar_wait(&tfull[acc], acc_phase);
-      tc_fence_after();
-      const int64_t gm = static_cast<int64_t>(m_blk) * BM + row_in_tile;
-      const bool row_ok = gm < M;
-#pragma unroll 1
-      for (int c = half * (BN / 2); c < (half + 1) * (BN / 2); c += 32) {
-        uint32_t r[32];
-        tmem_ld32(tmem_base + (static_cast<uint32_t>(q * 32) << 16) +
-                      static_cast<uint32_t>(acc * BN + c),
-                  r);
-        const int gn = n_blk * BN + c;
-        if (row_ok) {
-          float v[32];
-          const float4* b4 = reinterpret_cast<const float4*>(bias + gn);
+    for (int tile = cluster_id; tile < num_tiles; tile += num_clusters) {
+      int m_blk, n_blk;
+      tile_coords(tile, m_blocks, n_blocks, raster, m_blk, n_blk);
+      const int row0 = m_blk * TILE_M + static_cast<int>(rank) * 128 + q * 32;
+      const int col0 = n_blk * BN + half * (BN / 2);
+      if constexpr (EPI == TCB_EPI_BIAS_RESIDUAL) {
+        // every staging buffer is free once the previous tile's stores have read it; then
+        // prefetch this tile's residual chunks while the MMAs run
+        if (lane == 0) bulk_wait_read<0>();
+        __syncwarp();
+        if (lane == 0) {
 #pragma unroll
-          for (int j = 0; j < 8; ++j) {
-            const float4 bb = __ldg(b4 + j);
-            v[4 * j + 0] = __uint_as_float(r[4 * j + 0]) + bb.x;
-            v[4 * j + 1] = __uint_as_float(r[4 * j + 1]) + bb.y;
-            v[4 * j + 2] = __uint_as_float(r[4 * j + 2]) + bb.z;
-            v[4 * j + 3] = __uint_as_float(r[4 * j + 3]) + bb.w;
-          }
-          if (EPI == TCB_EPI_BIAS_GELU) {
-#pragma unroll
-            for (int j = 0; j < 32; ++j) v[j] = gelu_erf(v[j]);
-          } else if (EPI == TCB_EPI_BIAS_RELU) {
-#pragma unroll
-            for (int j = 0; j < 32; ++j) v[j] = fmaxf(v[j], 0.f);
-          } else if (EPI == TCB_EPI_BIAS_RESIDUAL) {
-            const uint4* rp = reinterpret_cast<const uint4*>(R + gm * N + gn);
-#pragma unroll
-            for (int j = 0; j < 4; ++j) {
-              uint4 x = __ldg(rp + j);
-              const __nv_bfloat162* h = reinterpret_cast<const __nv_bfloat162*>(&x);
-#pragma unroll
-              for (int e = 0; e < 4; ++e) {
-                const float2 f = __bfloat1622float2(h[e]);
-                v[8 * j + 2 * e] += f.x;
-                v[8 * j + 2 * e + 1] += f.y;
-              }
-            }
-          }
-          uint4* cp = reinterpret_cast<uint4*>(C + gm * N + gn);
-#pragma unroll
-          for (int j = 0; j < 4; ++j) {
-            uint4 x;
-            __nv_bfloat162* h = reinterpret_cast<__nv_bfloat162*>(&x);
-#pragma unroll
-            for (int e = 0; e < 4; ++e) h[e] = __floats2bfloat162_rn(v[8 * j + 2 * e], v[8 * j + 2 * e + 1]);
-            cp[j] = x;
+          for (int j = 0; j < NC; ++j) {
+            mbar_expect_tx(&my_rbar[j], kStageBufBytes);
+            asm volatile(
+                "cp.async.bulk.tensor.2d.shared::cluster.global.mbarrier::complete_tx::bytes"
+                " [%0], [%1, {%3, %4}], [%2];" ::"r"(bufs + j * kStageBufBytes),
+                "l"(reinterpret_cast<uint64_t>(&tmR)), "r"(smem_u32(&my_rbar[j])),
+                "r"(col0 + 32 * j), "r"(row0)
+                : "memory");
           }
         }
       }
+      mbar_wait(&tfull[acc], acc_phase);
+      tc_fence_after();
+      const uint32_t tbase = tmem_base + (static_cast<uint32_t>(q * 32) << 16) +
+                             static_cast<uint32_t>(acc * BN + half * (BN / 2));
+      uint32_t ra[32], rb[32];
+      tmem_ld32_nowait(tbase, ra);
+#pragma unroll
+      for (int j = 0; j < NC; ++j) {
+        uint32_t (&r)[32] = (j & 1) ? rb : ra;
+        uint32_t (&rn)[32] = (j & 1) ? ra : rb;
+        tmem_wait_ld();
+        if (j + 1 < NC) tmem_ld32_nowait(tbase + 32 * (j + 1), rn);   // overlap next load
+        const uint32_t buf = bufs + (j % NB) * kStageBufBytes;
+        const int gn = col0 + 32 * j;
+        if constexpr (EPI != TCB_EPI_BIAS_RESIDUAL) {
+          if (lane == 0) bulk_wait_read<NB - 1>();   // the store that last used `buf` read it
+          __syncwarp();
+        }
+        float v[32];
+        const float4* b4 = reinterpret_cast<const float4*>(bias + gn);
+#pragma unroll
+        for (int t = 0; t < 8; ++t) {
+          const float4 bb = __ldg(b4 + t);
+          v[4 * t + 0] = __uint_as_float(r[4 * t + 0]) + bb.x;
+          v[4 * t + 1] = __uint_as_float(r[4 * t + 1]) + bb.y;
+          v[4 * t + 2] = __uint_as_float(r[4 * t + 2]) + bb.z;
+          v[4 * t + 3] = __uint_as_float(r[4 * t + 3]) + bb.w;
+        }
+        if constexpr (EPI == TCB_EPI_BIAS_GELU) {
+#pragma unroll
+          for (int t = 0; t < 32; ++t) v[t] = gelu_erf(v[t]);
+        } else if constexpr (EPI == TCB_EPI_BIAS_RELU) {
+#pragma unroll
+          for (int t = 0; t < 32; ++t) v[t] = fmaxf(v[t], 0.f);
+        } else if constexpr (EPI == TCB_EPI_BIAS_RESIDUAL) {
+          mbar_wait(&my_rbar[j], rphase);
+#pragma unroll
+          for (int t = 0; t < 4; ++t) {
+            const uint4 x = ld_shared_v4(buf + sw64(lane, t));
+            const __nv_bfloat162* h = reinterpret_cast<const __nv_bfloat162*>(&x);
+#pragma unroll
+            for (int e = 0; e < 4; ++e) {
+              const float2 f = __bfloat1622float2(h[e]);
+              v[8 * t + 2 * e] += f.x;
+              v[8 * t + 2 * e + 1] += f.y;
+            }
+          }
+        }
+#pragma unroll
+        for (int t = 0; t < 4; ++t) {
+          uint4 x;
+          __nv_bfloat162* h = reinterpret_cast<__nv_bfloat162*>(&x);
+#pragma unroll
+          for (int e = 0; e < 4; ++e)
+            h[e] = __floats2bfloat162_rn(v[8 * t + 2 * e], v[8 * t + 2 * e + 1]);
+          st_shared_v4(buf + sw64(lane, t), x);
+        }
+        fence_async_smem();
+        __syncwarp();
+        if (lane == 0) {
+          asm volatile("cp.async.bulk.tensor.2d.global.shared::cta.bulk_group [%0, {%2, %3}], [%1];" ::"l"(
+                           reinterpret_cast<uint64_t>(&tmC)),
+                       "r"(buf), "r"(gn), "r"(row0)
+                       : "memory");
+          asm volatile("cp.async.bulk.commit_group;" ::: "memory");
+        }
+      }
+      rphase ^= 1;
+      // all TMEM reads of this accumulator are complete (last tcgen05.wait::ld above)
       tc_fence_before();
       __syncwarp();
-      if (lane == 0) mbar_arrive(&tempty[acc]);
+      if (lane == 0) mbar_arrive_remote(tempty0 + 8u * acc);
       acc ^= 1;
       if (acc == 0) acc_phase ^= 1;
     }
+    if (lane == 0) bulk_wait_all();
   }
+  __syncwarp();
   tc_fence_before();
-  __syncthreads();
+  if constexpr (CG == 2) cluster_sync(); else __syncthreads();
   tc_fence_after();
   if (warp == 2) {
-    asm volatile("tcgen05.dealloc.cta_group::1.sync.aligned.b32 %0, %1;" ::"r"(tmem_base),
-                 "r"(Cfg::kTmemCols)
-                 : "memory");
+    if constexpr (CG == 1)
+      asm volatile("tcgen05.dealloc.cta_group::1.sync.aligned.b32 %0, %1;" ::"r"(tmem_base),
+                   "r"(Cfg::kTmemCols) : "memory");
+    else
+      asm volatile("tcgen05.dealloc.cta_group::2.sync.aligned.b32 %0, %1;" ::"r"(tmem_base),
+                   "r"(Cfg::kTmemCols) : "memory");
   }
 }
 
@@ -322,41 +522,54 @@ PFN_cuTensorMapEncodeTiled_v12000 get_encode() {
   return g_encode;
 }
 
-template <int BN, int EPI>
-cudaError_t launch_tc(const CUtensorMap& tmA, const CUtensorMap& tmW, int M, int N, int K,
-                      const float* bias, const void* R, void* C, cudaStream_t s) {
-  using Cfg = TcCfg<BN>;
-  static bool attr_set = false;  // set once per instantiation (idempotent if raced)
+int num_sms() {
+  if (g_num_sms == 0) {
+    int dev = 0, n = 0;
+    cudaGetDevice(&dev);
+    cudaDeviceGetAttribute(&n, cudaDevAttrMultiProcessorCount, dev);
+    g_num_sms = n > 0 ? n : 148;
+  }
+  return g_num_sms;
+}
+
+template <int CG, int BN, int EPI>
+cudaError_t launch_tc(const GemmMaps& m, int M, int N, int K, const float* bias, cudaStream_t s) {
+  using Cfg = TcCfg<CG, BN, EPI>;
+  auto kern = linear_tc_kernel<CG, BN, EPI>;
+  static bool attr_set = false;  // idempotent if raced
   if (!attr_set) {
-    cudaError_t e = cudaFuncSetAttribute(linear_tc_kernel<BN, EPI>,
-                                         cudaFuncAttributeMaxDynamicSharedMemorySize,
+    cudaError_t e = cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize,
                                          Cfg::kSmemBytes);
     if (e != cudaSuccess) return e;
     attr_set = true;
   }
-  if (g_num_sms == 0) {
-    int dev = 0;
-    cudaGetDevice(&dev);
-    cudaDeviceGetAttribute(&g_num_sms, cudaDevAttrMultiProcessorCount, dev);
-    if (g_num_sms <= 0) g_num_sms = 148;
-  }
-  const int tiles = ((M + BM - 1) / BM) * (N / BN);
-  const int grid = tiles < g_num_sms ? tiles : g_num_sms;
-  linear_tc_kernel<BN, EPI><<<grid, kThreads, Cfg::kSmemBytes, s>>>(
-      tmA, tmW, M, N, K, bias, static_cast<const __nv_bfloat16*>(R),
-      static_cast<__nv_bfloat16*>(C));
-  return cudaGetLastError();
+  const int tiles = ((M + 128 * CG - 1) / (128 * CG)) * (N / BN);
+  int clusters = num_sms() / CG;
+  if (tiles < clusters) clusters = tiles;
+  cudaLaunchConfig_t cfg{};
+  cfg.gridDim = dim3(clusters * CG);
+  cfg.blockDim = dim3(kThreads);
+  cfg.dynamicSmemBytes = Cfg::kSmemBytes;
+  cfg.stream = s;
+  cudaLaunchAttribute attr[1];
+  attr[0].id = cudaLaunchAttributeClusterDimension;
+  attr[0].val.clusterDim.x = CG;
+  attr[0].val.clusterDim.y = 1;
+  attr[0].val.clusterDim.z = 1;
+  cfg.attrs = attr;
+  cfg.numAttrs = 1;
+  static const int raster = std::getenv("TCB_GEMM_RASTER") ? std::atoi(std::getenv("TCB_GEMM_RASTER")) : 8;
+  return cudaLaunchKernelEx(&cfg, kern, m.a, m.w, m.c, m.r, M, N, K, bias, raster);
 }
 
-template <int BN>
-cudaError_t dispatch_epi(const CUtensorMap& tmA, const CUtensorMap& tmW, int M, int N, int K,
-                         const float* bias, const void* R, int epi, void* C, cudaStream_t s) {
+template <int CG, int BN>
+cudaError_t dispatch_epi(const GemmMaps& m, int M, int N, int K, const float* bias, int epi,
+                         cudaStream_t s) {
   switch (epi) {
-    case TCB_EPI_BIAS: return launch_tc<BN, TCB_EPI_BIAS>(tmA, tmW, M, N, K, bias, R, C, s);
-    case TCB_EPI_BIAS_GELU: return launch_tc<BN, TCB_EPI_BIAS_GELU>(tmA, tmW, M, N, K, bias, R, C, s);
-    case TCB_EPI_BIAS_RELU: return launch_tc<BN, TCB_EPI_BIAS_RELU>(tmA, tmW, M, N, K, bias, R, C, s);
-    case TCB_EPI_BIAS_RESIDUAL:
-      return launch_tc<BN, TCB_EPI_BIAS_RESIDUAL>(tmA, tmW, M, N, K, bias, R, C, s);
+    case TCB_EPI_BIAS: return launch_tc<CG, BN, TCB_EPI_BIAS>(m, M, N, K, bias, s);
+    case TCB_EPI_BIAS_GELU: return launch_tc<CG, BN, TCB_EPI_BIAS_GELU>(m, M, N, K, bias, s);
+    case TCB_EPI_BIAS_RELU: return launch_tc<CG, BN, TCB_EPI_BIAS_RELU>(m, M, N, K, bias, s);
+    case TCB_EPI_BIAS_RESIDUAL: return launch_tc<CG, BN, TCB_EPI_BIAS_RESIDUAL>(m, M, N, K, bias, s);
     default: return cudaErrorInvalidValue;
   }
 }
@@ -364,35 +577,58 @@ cudaError_t dispatch_epi(const CUtensorMap& tmA, const CUtensorMap& tmW, int M, 
 }  // namespace
 
 bool make_tmap_bf16(CUtensorMap* map, const void* ptr, uint64_t rows, uint64_t cols,
-                    uint32_t box_rows) {
+                    uint32_t box_rows, uint32_t box_cols, int swizzle_bytes) {
   auto encode = get_encode();
   if (!encode || rows == 0) return false;
   cuuint64_t dims[2] = {cols, rows};
   cuuint64_t strides[1] = {cols * 2};
-  cuuint32_t box[2] = {static_cast<cuuint32_t>(BK), box_rows};
+  cuuint32_t box[2] = {box_cols, box_rows};
   cuuint32_t estr[2] = {1, 1};
+  const CUtensorMapSwizzle sw = swizzle_bytes == 128 ? CU_TENSOR_MAP_SWIZZLE_128B
+                                : swizzle_bytes == 64 ? CU_TENSOR_MAP_SWIZZLE_64B
+                                                      : CU_TENSOR_MAP_SWIZZLE_NONE;
   CUresult r = encode(map, CU_TENSOR_MAP_DATA_TYPE_BFLOAT16, 2, const_cast<void*>(ptr), dims,
-                      strides, box, estr, CU_TENSOR_MAP_INTERLEAVE_NONE,
-                      CU_TENSOR_MAP_SWIZZLE_128B, CU_TENSOR_MAP_L2_PROMOTION_L2_256B,
-                      CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE);
+                      strides, box, estr, CU_TENSOR_MAP_INTERLEAVE_NONE, sw,
+                      CU_TENSOR_MAP_L2_PROMOTION_L2_256B, CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE);
   return r == CUDA_SUCCESS;
 }
 
-int linear_tc_block_n(int N) {
-  if (N % 256 == 0) return 256;
-  if (N % 128 == 0) return 128;
-  return 64;
+bool make_gemm_a_map(CUtensorMap* map, const void* A, uint64_t M, uint64_t K) {
+  return make_tmap_bf16(map, A, M, K, 128, BK, 128);
+}
+bool make_gemm_w_map(CUtensorMap* map, const void* W, uint64_t N, uint64_t K) {
+  const GemmShape g = linear_tc_shape(static_cast<int>(N));
+  return make_tmap_bf16(map, W, N, K, static_cast<uint32_t>(g.bn / g.cg), BK, 128);
+}
+bool make_gemm_c_map(CUtensorMap* map, const void* C, uint64_t M, uint64_t N) {
+  return make_tmap_bf16(map, C, M, N, kStageRows, kStageCols, 64);
 }
 
-cudaError_t launch_linear_bf16_tc(const CUtensorMap& tmA, const CUtensorMap& tmW, int64_t M,
-                                  int N, int K, const float* bias, const void* R, int epi,
-                                  void* C, cudaStream_t s) {
-  if (M == 0) return cudaSuccess;
-  switch (linear_tc_block_n(N)) {
-    case 256: return dispatch_epi<256>(tmA, tmW, static_cast<int>(M), N, K, bias, R, epi, C, s);
-    case 128: return dispatch_epi<128>(tmA, tmW, static_cast<int>(M), N, K, bias, R, epi, C, s);
-    default: return dispatch_epi<64>(tmA, tmW, static_cast<int>(M), N, K, bias, R, epi, C, s);
+// Tile shape per N.  TCB_GEMM_VARIANT (tuning only; read once) forces cg1_256 / cg2_128 /
+// cg1_128 where N allows it.
+GemmShape linear_tc_shape(int N) {
+  static const char* forced = std::getenv("TCB_GEMM_VARIANT");
+  if (forced) {
+    const std::string f(forced);
+    if (f == "cg1_256" && N % 256 == 0) return {1, 256};
+    if (f == "cg1_128" && N % 128 == 0) return {1, 128};
+    if (f == "cg2_128" && N % 128 == 0) return {2, 128};
   }
+  if (N % 256 == 0) return {2, 256};
+  if (N % 128 == 0) return {2, 128};
+  return {1, 64};
+}
+
+cudaError_t launch_linear_bf16_tc(const GemmMaps& m, int64_t M, int N, int K, const float* bias,
+                                  int epi, cudaStream_t s) {
+  if (M == 0) return cudaSuccess;
+  const GemmShape g = linear_tc_shape(N);
+  const int Mi = static_cast<int>(M);
+  if (g.cg == 2 && g.bn == 256) return dispatch_epi<2, 256>(m, Mi, N, K, bias, epi, s);
+  if (g.cg == 2 && g.bn == 128) return dispatch_epi<2, 128>(m, Mi, N, K, bias, epi, s);
+  if (g.cg == 1 && g.bn == 256) return dispatch_epi<1, 256>(m, Mi, N, K, bias, epi, s);
+  if (g.cg == 1 && g.bn == 128) return dispatch_epi<1, 128>(m, Mi, N, K, bias, epi, s);
+  return dispatch_epi<1, 64>(m, Mi, N, K, bias, epi, s);
 }
 
 }  // namespace k
