@@ -55,8 +55,11 @@ class Plan:
 
     def __del__(self):
         h, self._h = getattr(self, "_h", None), None
-        if h and _lib._lib is not None:
-            _lib._lib.tcb_plan_destroy(h)
+        try:
+            if h and _lib._lib is not None:
+                _lib._lib.tcb_plan_destroy(h)
+        except Exception:  # interpreter shutdown
+            pass
 
     @property
     def handle(self):
@@ -158,8 +161,11 @@ class Encoder:
 
     def __del__(self):
         h, self._h = getattr(self, "_h", None), None
-        if h and _lib._lib is not None:
-            _lib._lib.tcb_weights_destroy(h)
+        try:
+            if h and _lib._lib is not None:
+                _lib._lib.tcb_weights_destroy(h)
+        except Exception:  # interpreter shutdown
+            pass
 
     def workspace_bytes(self, num_slots: int) -> int:
         b = ctypes.c_size_t(0)

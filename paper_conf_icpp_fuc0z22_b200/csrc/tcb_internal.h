@@ -11,7 +11,7 @@
 
 // Geometry of the segment-masked attention kernel (attn.cu); the host plan uses it to
 // report how many score elements the kernel evaluates (tcb_plan_info).
-constexpr int kAttnQBlock = 64;    // query slots per CTA (4 warps x 16 rows)
+constexpr int kAttnQBlock = 128;   // query slots per CTA (8 warps x 16 rows)
 constexpr int kAttnWarpRows = 16;  // query rows per warp (one m16 MMA tile)
 constexpr int kAttnKSub = 16;      // keys per skip decision (one k16 MMA step of P.V)
 

@@ -108,7 +108,7 @@ def test_pack_errors():
 def test_plan_counters_vs_brute_force():
     """P9 on the product's plan counters: 128x128 tiles touching a diagonal block, the
     dense count, sum l^2, and the kernel's executed 16x16 sub-blocks (re-derived here from
-    its stated geometry: 64-slot CTAs, 16-row warps, 16-key sub-blocks from the CTA start)."""
+    its stated geometry: 128-slot CTAs, 16-row warps, 16-key sub-blocks from the CTA start)."""
     lengths = np.minimum(wl.draw_lengths("dia", 300, 5), 512).astype(np.int32)
     plan = tcb.tcb_pack(lengths, 512, 16)
     a = plan.arrays()
@@ -129,9 +129,9 @@ def test_plan_counters_vs_brute_force():
     assert info["useful_score_elems"] == int(np.sum(lengths[placed].astype(np.int64) ** 2))
     starts, lens = a["seg_start"], lengths[a["seg_req"]]
     ex = 0
-    for q0 in range(0, M, 64):
+    for q0 in range(0, M, 128):
         iv = []
-        for w in range(4):
+        for w in range(8):
             ss = [s for s in seg[q0 + 16 * w:q0 + 16 * w + 16] if s >= 0]
             iv.append((min(starts[s] for s in ss), max(starts[s] + lens[s] for s in ss))
                       if ss else None)
