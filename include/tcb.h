@@ -114,15 +114,18 @@ tcb_status tcb_plan_copy(const tcb_plan* plan, int32_t* req_row, int32_t* req_co
                          int32_t* seg_req, int32_t* seg_start, int32_t* cu_seqlens,
                          int32_t* segment_ids, int32_t* positions, int32_t* qtile_kv);
 
-/* The device form of a plan: the segment table the kernels expand.  Layout (int32 words,
- * 16-byte records): header {num_segments, num_slots, row_len, total_tokens (low 31 bits)},
- * then one record per segment in (row, column) order:
- *   {slot_start, length, token_offset (request-order index of its first token), request}.
- * tcb_plan_segtab_words gives the word count (4 * (1 + num_segments)); tcb_plan_write_segtab
- * writes it into a HOST buffer of at least that many words; the caller copies it to the
- * device (16-byte aligned) and passes that pointer as d_segtab below.  A plan of the same
- * (num_rows, row_len) may later be written into the same device buffer and a captured CUDA
- * graph replayed: no kernel reads the host plan. */
+/* The device form of a plan: the segment table the kernels expand.  Layout (int32 words):
+ *   header (4 words)  {num_segments S, num_slots, row_len, total_tokens (low 31 bits)};
+ *   S records (4 words each, 16-byte aligned), one per segment in (row, column) order:
+ *                     {slot_start, length, token_offset (request-order index of its first
+ *                      token), request};
+ *   row index (num_rows + 1 words, padded to a multiple of 4): row_first[r] = index of the
+ *                     first segment of row r, row_first[num_rows] = S.
+ * tcb_plan_segtab_words gives the word count (4 * (1 + S) + round_up(num_rows + 1, 4));
+ * tcb_plan_write_segtab writes it into a HOST buffer of at least that many words; the caller
+ * copies it to the device (16-byte aligned) and passes that pointer as d_segtab below.  A
+ * plan of the same (num_rows, row_len) may later be written into the same device buffer (if
+ * it is large enough) and a captured CUDA graph replayed: no kernel reads the host plan. */
 int64_t tcb_plan_segtab_words(const tcb_plan* plan);
 tcb_status tcb_plan_write_segtab(const tcb_plan* plan, int32_t* host_dst, int64_t capacity_words);
 

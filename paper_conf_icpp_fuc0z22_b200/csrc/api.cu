@@ -165,7 +165,7 @@ namespace {
 
 enum { W_QKV = 0, B_QKV, W_O, B_O, LN1_G, LN1_B, W_1, B_1, W_2, B_2, LN2_G, LN2_B };
 
-tcb_status embed_impl(const tcb_weights* w, int64_t M, const int32_t* d_segtab,
+tcb_status embed_impl(const tcb_weights* w, const tcb_plan* plan, const int32_t* d_segtab,
                       const int32_t* d_ids, void* d_rows, int32_t* d_seg, int32_t* d_pos,
                       cudaStream_t s) {
   const tcb_model_config& c = w->cfg;
@@ -182,7 +182,9 @@ tcb_status embed_impl(const tcb_weights* w, int64_t M, const int32_t* d_segtab,
   a.ln_eps = c.emb_ln_eps;
   a.d = c.d_model;
   a.max_pos = c.max_pos;
-  a.num_slots = M;
+  a.num_rows = plan->num_rows;
+  a.row_len = plan->row_len;
+  a.num_slots = plan->info.num_slots;
   a.X = d_rows;
   a.seg_ids = d_seg;
   a.positions = d_pos;
@@ -307,7 +309,7 @@ tcb_status tcb_embed(const tcb_weights* w, const tcb_plan* plan, const int32_t* 
   if (M == 0) return TCB_OK;
   if (!d_segtab || !d_rows || (plan->info.total_tokens > 0 && !d_token_ids))
     return fail(TCB_ERR_INVALID_ARGUMENT, "tcb_embed: NULL device pointer");
-  return embed_impl(w, M, d_segtab, d_token_ids, d_rows, d_segment_ids, d_positions,
+  return embed_impl(w, plan, d_segtab, d_token_ids, d_rows, d_segment_ids, d_positions,
                     reinterpret_cast<cudaStream_t>(stream));
 }
 
@@ -339,7 +341,7 @@ tcb_status tcb_encoder_forward(const tcb_weights* wc, const tcb_plan* plan,
   const int act_epi = c.act == 0 ? TCB_EPI_BIAS_GELU : TCB_EPI_BIAS_RELU;
   const int4* segtab = reinterpret_cast<const int4*>(d_segtab);
 
-  if (tcb_status st = embed_impl(w, M, d_segtab, d_token_ids, d_rows, seg, nullptr, s)) return st;
+  if (tcb_status st = embed_impl(w, plan, d_segtab, d_token_ids, d_rows, seg, nullptr, s)) return st;
 
   if (c.dtype == 1) {
     {
@@ -426,7 +428,8 @@ tcb_status tcb_unpack(const tcb_weights* w, const tcb_plan* plan, const int32_t*
   if (!d_segtab || !d_rows || !d_out) return fail(TCB_ERR_INVALID_ARGUMENT, "tcb_unpack: NULL");
   cudaStream_t s = reinterpret_cast<cudaStream_t>(stream);
   TCB_LAUNCH(TCB_K_UNPACK, s, tcb::k::launch_unpack(w->cfg.dtype,
-                                                    reinterpret_cast<const int4*>(d_segtab), M,
+                                                    reinterpret_cast<const int4*>(d_segtab),
+                                                    plan->num_rows, plan->row_len,
                                                     w->cfg.d_model, d_rows, d_out, s));
   return TCB_OK;
 }

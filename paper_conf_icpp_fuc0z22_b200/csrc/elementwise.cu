@@ -57,99 +57,125 @@ __device__ __forceinline__ float warp_sum(float v) {
   return v;
 }
 
-// Segment containing `slot` (binary search over the records' slot_start), or -1 for pad.
-__device__ __forceinline__ int find_segment(const int4* segtab, int64_t slot, int4* rec_out) {
-  const int S = segtab[0].x;
-  int lo = 0, hi = S - 1, found = -1;
-  while (lo <= hi) {
-    const int mid = (lo + hi) >> 1;
-    const int4 r = __ldg(&segtab[1 + mid]);
-    if (r.x <= slot) { found = mid; lo = mid + 1; } else { hi = mid - 1; }
-  }
-  if (found < 0) return -1;
-  const int4 r = __ldg(&segtab[1 + found]);
-  if (slot >= r.x + r.y) return -1;
-  *rec_out = r;
-  return found;
-}
-
+// One CTA per (batch row, 64-slot chunk of it).  The row's segment records (row_first[] of
+// the device segment table gives them in O(1)) are staged in shared memory; each warp then
+// owns slots j = chunk*64 + warp, +8, ... and finds its segment by a binary search in smem.
+constexpr int kRowChunk = 64;
 template <typename T, int NV>
 __global__ void __launch_bounds__(kWarpsPerBlock * 32) pack_embed_kernel(EmbedArgs a) {
   constexpr int V = Vec<T>::N;
-  const int lane = threadIdx.x & 31;
-  const int64_t slot = static_cast<int64_t>(blockIdx.x) * kWarpsPerBlock + (threadIdx.x >> 5);
-  if (slot >= a.num_slots) return;
+  extern __shared__ int4 row_recs[];
+  const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
+  const int row = blockIdx.x;
+  const int S = a.segtab[0].x;
+  const int* row_first = reinterpret_cast<const int*>(a.segtab + 1 + S);
+  const int f = __ldg(&row_first[row]);
+  const int nseg = __ldg(&row_first[row + 1]) - f;
+  for (int i = threadIdx.x; i < nseg; i += blockDim.x) row_recs[i] = __ldg(&a.segtab[1 + f + i]);
+  // per-column vectors shared by every slot (BERT type-0 embedding, embedding LN) -> smem
+  float* s_type = reinterpret_cast<float*>(row_recs + a.row_len);
+  float* s_g = s_type + a.d;
+  float* s_b = s_g + a.d;
+  if (a.type_emb || a.ln_g) {
+    for (int i = threadIdx.x; i < a.d; i += blockDim.x) {
+      if (a.type_emb) s_type[i] = __ldg(&a.type_emb[i]);
+      if (a.ln_g) { s_g[i] = __ldg(&a.ln_g[i]); s_b[i] = __ldg(&a.ln_b[i]); }
+    }
+  }
+  __syncthreads();
   const int d = a.d;
   const int nvec = d / V;
-  T* x = reinterpret_cast<T*>(a.X) + slot * d;
-  int4 rec;
-  const int seg = find_segment(a.segtab, slot, &rec);
-  if (seg < 0) {  // pad slot: zeros, segment -1, position -1 (R12)
-    float z[V] = {};
-    for (int i = lane; i < nvec; i += 32) Vec<T>::store(x + i * V, z);
+  const int64_t row0 = static_cast<int64_t>(row) * a.row_len;
+  const int j_end = min(a.row_len, static_cast<int>(blockIdx.y + 1) * kRowChunk);
+  for (int j = static_cast<int>(blockIdx.y) * kRowChunk + warp; j < j_end; j += kWarpsPerBlock) {
+    const int64_t slot = row0 + j;
+    T* x = reinterpret_cast<T*>(a.X) + slot * d;
+    // last record with start <= slot
+    int lo = 0, hi = nseg - 1, k = -1;
+    while (lo <= hi) {
+      const int mid = (lo + hi) >> 1;
+      if (row_recs[mid].x <= slot) { k = mid; lo = mid + 1; } else { hi = mid - 1; }
+    }
+    const int4 rec = k >= 0 ? row_recs[k] : make_int4(0, 0, 0, 0);
+    if (k < 0 || slot >= rec.x + rec.y) {  // pad slot: zeros, segment -1, position -1 (R12)
+      float z[V] = {};
+      for (int i = lane; i < nvec; i += 32) Vec<T>::store(x + i * V, z);
+      if (lane == 0) {
+        if (a.seg_ids) a.seg_ids[slot] = -1;
+        if (a.positions) a.positions[slot] = -1;
+      }
+      continue;
+    }
+    const int seg = f + k;
+    const int pos = static_cast<int>(slot - rec.x);           // restarts at 0 per request
+    const int id = __ldg(&a.ids[rec.z + pos]);
     if (lane == 0) {
-      if (a.seg_ids) a.seg_ids[slot] = -1;
-      if (a.positions) a.positions[slot] = -1;
+      if (a.seg_ids) a.seg_ids[slot] = seg;
+      if (a.positions) a.positions[slot] = pos;
     }
-    return;
-  }
-  const int pos = static_cast<int>(slot - rec.x);           // restarts at 0 per request
-  const int tok = rec.z + pos;
-  const int id = __ldg(&a.ids[tok]);
-  if (lane == 0) {
-    if (a.seg_ids) a.seg_ids[slot] = seg;
-    if (a.positions) a.positions[slot] = pos;
-  }
-  const T* e = reinterpret_cast<const T*>(a.tok_emb) + static_cast<int64_t>(id) * d;
-  float v[NV][V];
-  float sum = 0.f;
+    const T* e = reinterpret_cast<const T*>(a.tok_emb) + static_cast<int64_t>(id) * d;
+    float v[NV][V];
+    float sum = 0.f;
 #pragma unroll
-  for (int j = 0; j < NV; ++j) {
-    const int i = lane + 32 * j;
-    if (i < nvec) {
-      Vec<T>::load(e + i * V, v[j]);
-      float p[V];
-      if (a.pe_table) {
-        const float* pt = a.pe_table + static_cast<int64_t>(pos) * d + i * V;
+    for (int jv = 0; jv < NV; ++jv) {
+      const int i = lane + 32 * jv;
+      if (i < nvec) {
+        Vec<T>::load(e + i * V, v[jv]);
+        float p[V];
+        if (a.pe_table) {
+          const float* pt = a.pe_table + static_cast<int64_t>(pos) * d + i * V;
 #pragma unroll
-        for (int c = 0; c < V; c += 4) {
-          float4 q = *reinterpret_cast<const float4*>(pt + c);
-          p[c] = q.x; p[c + 1] = q.y; p[c + 2] = q.z; p[c + 3] = q.w;
+          for (int c = 0; c < V; c += 4) {
+            float4 q = __ldg(reinterpret_cast<const float4*>(pt + c));
+            p[c] = q.x; p[c + 1] = q.y; p[c + 2] = q.z; p[c + 3] = q.w;
+          }
+        } else {
+          Vec<T>::load(reinterpret_cast<const T*>(a.pos_emb) + static_cast<int64_t>(pos) * d + i * V, p);
         }
-      } else {
-        Vec<T>::load(reinterpret_cast<const T*>(a.pos_emb) + static_cast<int64_t>(pos) * d + i * V, p);
-      }
+        if (a.type_emb) {
 #pragma unroll
-      for (int c = 0; c < V; ++c) {
-        float t = v[j][c] * a.emb_scale + p[c];
-        if (a.type_emb) t += __ldg(&a.type_emb[i * V + c]);
-        v[j][c] = t;
-        sum += t;
+          for (int c = 0; c < V; c += 4) {
+            const float4 ty = *reinterpret_cast<const float4*>(s_type + i * V + c);
+            p[c] += ty.x; p[c + 1] += ty.y; p[c + 2] += ty.z; p[c + 3] += ty.w;
+          }
+        }
+#pragma unroll
+        for (int c = 0; c < V; ++c) {
+          const float t = v[jv][c] * a.emb_scale + p[c];
+          v[jv][c] = t;
+          sum += t;
+        }
       }
     }
-  }
-  if (a.ln_g) {
-    const float mean = warp_sum(sum) / d;
-    float sq = 0.f;
+    if (a.ln_g) {
+      const float mean = warp_sum(sum) / d;
+      float sq = 0.f;
 #pragma unroll
-    for (int j = 0; j < NV; ++j)
-      if (lane + 32 * j < nvec)
+      for (int jv = 0; jv < NV; ++jv)
+        if (lane + 32 * jv < nvec)
 #pragma unroll
-        for (int c = 0; c < V; ++c) { const float t = v[j][c] - mean; sq += t * t; }
-    const float rstd = rsqrtf(warp_sum(sq) / d + a.ln_eps);
+          for (int c = 0; c < V; ++c) { const float t = v[jv][c] - mean; sq += t * t; }
+      const float rstd = rsqrtf(warp_sum(sq) / d + a.ln_eps);
 #pragma unroll
-    for (int j = 0; j < NV; ++j) {
-      const int i = lane + 32 * j;
-      if (i < nvec)
+      for (int jv = 0; jv < NV; ++jv) {
+        const int i = lane + 32 * jv;
+        if (i < nvec)
 #pragma unroll
-        for (int c = 0; c < V; ++c)
-          v[j][c] = (v[j][c] - mean) * rstd * __ldg(&a.ln_g[i * V + c]) + __ldg(&a.ln_b[i * V + c]);
+          for (int c = 0; c < V; c += 4) {
+            const float4 g4 = *reinterpret_cast<const float4*>(s_g + i * V + c);
+            const float4 b4 = *reinterpret_cast<const float4*>(s_b + i * V + c);
+            v[jv][c] = (v[jv][c] - mean) * rstd * g4.x + b4.x;
+            v[jv][c + 1] = (v[jv][c + 1] - mean) * rstd * g4.y + b4.y;
+            v[jv][c + 2] = (v[jv][c + 2] - mean) * rstd * g4.z + b4.z;
+            v[jv][c + 3] = (v[jv][c + 3] - mean) * rstd * g4.w + b4.w;
+          }
+      }
     }
-  }
 #pragma unroll
-  for (int j = 0; j < NV; ++j) {
-    const int i = lane + 32 * j;
-    if (i < nvec) Vec<T>::store(x + i * V, v[j]);
+    for (int jv = 0; jv < NV; ++jv) {
+      const int i = lane + 32 * jv;
+      if (i < nvec) Vec<T>::store(x + i * V, v[jv]);
+    }
   }
 }
 
@@ -227,21 +253,42 @@ layernorm_kernel(int64_t rows, int d, const T* __restrict__ Z, const float* __re
   }
 }
 
-template <typename T>
+// unpack: one CTA per (batch row, 64-slot chunk); the part of each segment inside the
+// chunk is a contiguous block in both the rows buffer and the request-order output, so the
+// CTA copies it with 16-byte vectors (4 independent loads in flight per thread).
 __global__ void __launch_bounds__(kWarpsPerBlock * 32)
-unpack_kernel(const int4* __restrict__ segtab, int64_t num_slots, int d,
-              const T* __restrict__ rows, T* __restrict__ out) {
-  constexpr int V = Vec<T>::N;
-  const int lane = threadIdx.x & 31;
-  const int64_t slot = static_cast<int64_t>(blockIdx.x) * kWarpsPerBlock + (threadIdx.x >> 5);
-  if (slot >= num_slots) return;
-  int4 rec;
-  if (find_segment(segtab, slot, &rec) < 0) return;
-  const int64_t tok = rec.z + (slot - rec.x);
-  const uint4* src = reinterpret_cast<const uint4*>(rows + slot * d);
-  uint4* dst = reinterpret_cast<uint4*>(out + tok * d);
-  const int nvec = d / V;
-  for (int i = lane; i < nvec; i += 32) dst[i] = __ldg(src + i);
+unpack_kernel(const int4* __restrict__ segtab, int row_len, int row_bytes_per_slot,
+              const uint8_t* __restrict__ rows, uint8_t* __restrict__ out) {
+  const int row = blockIdx.x;
+  const int S = segtab[0].x;
+  const int* row_first = reinterpret_cast<const int*>(segtab + 1 + S);
+  const int f = __ldg(&row_first[row]), e = __ldg(&row_first[row + 1]);
+  const int64_t c0 = static_cast<int64_t>(row) * row_len + blockIdx.y * kRowChunk;
+  const int64_t c1 = min(c0 + kRowChunk, static_cast<int64_t>(row + 1) * row_len);
+  constexpr int U = 4;
+  for (int sg = f; sg < e; ++sg) {
+    const int4 rec = __ldg(&segtab[1 + sg]);
+    const int64_t a0 = rec.x > c0 ? static_cast<int64_t>(rec.x) : c0;
+    const int64_t a1 = rec.x + rec.y < c1 ? static_cast<int64_t>(rec.x + rec.y) : c1;
+    if (a0 >= a1) continue;
+    const int64_t nvec = (a1 - a0) * row_bytes_per_slot / 16;
+    const uint4* src = reinterpret_cast<const uint4*>(rows + a0 * row_bytes_per_slot);
+    uint4* dst = reinterpret_cast<uint4*>(out + (rec.z + (a0 - rec.x)) * row_bytes_per_slot);
+    for (int64_t i0 = threadIdx.x; i0 < nvec; i0 += static_cast<int64_t>(blockDim.x) * U) {
+      uint4 t[U];
+#pragma unroll
+      for (int u = 0; u < U; ++u) {
+        const int64_t i = i0 + static_cast<int64_t>(u) * blockDim.x;
+        if (i < nvec) t[u] = __ldg(src + i);
+      }
+#pragma unroll
+      for (int u = 0; u < U; ++u) {
+        const int64_t i = i0 + static_cast<int64_t>(u) * blockDim.x;
+        if (i < nvec) dst[i] = t[u];
+      }
+    }
+  }
+  (void)row_len;
 }
 
 __global__ void pe_table_kernel(float* table, int max_pos, int d, int variant) {
@@ -276,14 +323,27 @@ bool dispatch_nv(int nv, F&& f) {
 
 cudaError_t launch_embed(int dtype, const EmbedArgs& a, cudaStream_t s) {
   if (a.num_slots == 0) return cudaSuccess;
-  const unsigned grid = static_cast<unsigned>((a.num_slots + kWarpsPerBlock - 1) / kWarpsPerBlock);
+  const dim3 grid(static_cast<unsigned>(a.num_rows), static_cast<unsigned>((a.row_len + kRowChunk - 1) / kRowChunk));
+  // <= row_len segment records + type embedding, LN gamma, LN beta (fp32, d each)
+  const size_t smem = static_cast<size_t>(a.row_len) * sizeof(int4) + 3 * sizeof(float) * a.d;
   const int nv = (a.d / (dtype == 0 ? 4 : 8) + 31) / 32;
+  cudaError_t attr_err = cudaSuccess;
   auto go = [&](auto tag) {
     constexpr int NV = decltype(tag)::value;
-    if (dtype == 0) pack_embed_kernel<float, NV><<<grid, kWarpsPerBlock * 32, 0, s>>>(a);
-    else pack_embed_kernel<__nv_bfloat16, NV><<<grid, kWarpsPerBlock * 32, 0, s>>>(a);
+    if (dtype == 0) {
+      if (smem > 48 * 1024)
+        attr_err = cudaFuncSetAttribute(pack_embed_kernel<float, NV>,
+                                        cudaFuncAttributeMaxDynamicSharedMemorySize, static_cast<int>(smem));
+      pack_embed_kernel<float, NV><<<grid, kWarpsPerBlock * 32, smem, s>>>(a);
+    } else {
+      if (smem > 48 * 1024)
+        attr_err = cudaFuncSetAttribute(pack_embed_kernel<__nv_bfloat16, NV>,
+                                        cudaFuncAttributeMaxDynamicSharedMemorySize, static_cast<int>(smem));
+      pack_embed_kernel<__nv_bfloat16, NV><<<grid, kWarpsPerBlock * 32, smem, s>>>(a);
+    }
   };
   if (!dispatch_nv(nv, go)) return cudaErrorInvalidValue;
+  if (attr_err != cudaSuccess) return attr_err;
   return cudaGetLastError();
 }
 
@@ -308,17 +368,13 @@ cudaError_t launch_layernorm(int dtype, int64_t rows, int d, const void* Z, cons
   return cudaGetLastError();
 }
 
-cudaError_t launch_unpack(int dtype, const int4* segtab, int64_t num_slots, int d,
+cudaError_t launch_unpack(int dtype, const int4* segtab, int num_rows, int row_len, int d,
                           const void* rows, void* out, cudaStream_t s) {
-  if (num_slots == 0) return cudaSuccess;
-  const unsigned grid = static_cast<unsigned>((num_slots + kWarpsPerBlock - 1) / kWarpsPerBlock);
-  if (dtype == 0)
-    unpack_kernel<float><<<grid, kWarpsPerBlock * 32, 0, s>>>(
-        segtab, num_slots, d, static_cast<const float*>(rows), static_cast<float*>(out));
-  else
-    unpack_kernel<__nv_bfloat16><<<grid, kWarpsPerBlock * 32, 0, s>>>(
-        segtab, num_slots, d, static_cast<const __nv_bfloat16*>(rows),
-        static_cast<__nv_bfloat16*>(out));
+  if (num_rows == 0) return cudaSuccess;
+  const int bytes_per_slot = d * (dtype == 0 ? 4 : 2);
+  const dim3 grid(static_cast<unsigned>(num_rows), static_cast<unsigned>((row_len + kRowChunk - 1) / kRowChunk));
+  unpack_kernel<<<grid, kWarpsPerBlock * 32, 0, s>>>(
+      segtab, row_len, bytes_per_slot, static_cast<const uint8_t*>(rows), static_cast<uint8_t*>(out));
   return cudaGetLastError();
 }
 

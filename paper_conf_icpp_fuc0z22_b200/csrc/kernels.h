@@ -20,6 +20,7 @@ struct EmbedArgs {
   const float* ln_b;
   float emb_scale, ln_eps;
   int32_t d, max_pos;
+  int32_t num_rows, row_len;
   int64_t num_slots;
   void* X;                     // out [num_slots, d] dtype
   int32_t* seg_ids;            // out [num_slots] or nullptr
@@ -31,7 +32,7 @@ cudaError_t launch_layernorm(int dtype, int64_t rows, int d, const void* Z, cons
                              const float* b, float eps, const int32_t* seg_ids, void* Y,
                              cudaStream_t s);
 
-cudaError_t launch_unpack(int dtype, const int4* segtab, int64_t num_slots, int d,
+cudaError_t launch_unpack(int dtype, const int4* segtab, int num_rows, int row_len, int d,
                           const void* rows, void* out, cudaStream_t s);
 
 cudaError_t launch_pe_table(float* table, int max_pos, int d, int variant, cudaStream_t s);

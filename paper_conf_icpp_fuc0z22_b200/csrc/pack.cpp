@@ -283,7 +283,7 @@ tcb_status tcb_plan_copy(const tcb_plan* p, int32_t* req_row, int32_t* req_col,
 
 int64_t tcb_plan_segtab_words(const tcb_plan* p) {
   if (!p) return -1;
-  return 4 * (1 + static_cast<int64_t>(p->seg_req.size()));
+  return 4 * (1 + static_cast<int64_t>(p->seg_req.size())) + (p->num_rows + 1 + 3) / 4 * 4;
 }
 
 tcb_status tcb_plan_write_segtab(const tcb_plan* p, int32_t* dst, int64_t capacity_words) {
@@ -308,6 +308,16 @@ tcb_status tcb_plan_write_segtab(const tcb_plan* p, int32_t* dst, int64_t capaci
     rec[2] = static_cast<int32_t>(p->tok_off[r]);
     rec[3] = r;
   }
+  // row index: segments are in (row, column) order, so row_first is a running count
+  int32_t* row_first = dst + 4 * (1 + p->seg_req.size());
+  const int32_t S = static_cast<int32_t>(p->seg_req.size());
+  int32_t s = 0;
+  for (int32_t k = 0; k <= p->num_rows; ++k) {
+    while (s < S && p->seg_start[s] < static_cast<int64_t>(k) * p->row_len) ++s;
+    row_first[k] = s;
+  }
+  const int64_t padded = (p->num_rows + 1 + 3) / 4 * 4;
+  for (int64_t k = p->num_rows + 1; k < padded; ++k) row_first[k] = S;
   return TCB_OK;
 }
 

@@ -79,7 +79,9 @@ def test_pack_golden_f1(golden_dir):
     assert a["qtile_kv"].tolist() == f1["qtile_kv_128"]
     st = plan.segtab()
     assert st[:4].tolist() == [8, 64, 32, 58]
-    recs = st[4:].reshape(-1, 4)
+    assert len(st) == 4 * 9 + 4
+    assert st[36:39].tolist() == [0, 3, 8]          # row_first: row 0 -> seg 0, row 1 -> 3, end
+    recs = st[4:36].reshape(-1, 4)
     assert recs[:, 0].tolist() == f1["seg_start"]
     assert recs[:, 1].tolist() == [f1["lengths"][r] for r in f1["seg_req"]]
     cu_req = np.concatenate([[0], np.cumsum(f1["lengths"])])
@@ -102,7 +104,7 @@ def test_pack_errors():
         tcb.tcb_pack([3], 32, -1)
     p = tcb.tcb_pack([], 32)
     assert p.info["num_rows"] == 0 and p.info["num_slots"] == 0
-    assert p.segtab().tolist() == [0, 0, 32, 0]
+    assert p.segtab().tolist() == [0, 0, 32, 0, 0, 0, 0, 0]
 
 
 def test_plan_counters_vs_brute_force():
