@@ -23,6 +23,17 @@ tcb_status tcb_op_linear(int32_t dtype, int64_t M, int32_t N, int32_t K, const v
                          const void* W, const float* bias, const void* R, int32_t epilogue,
                          void* C, tcb_stream_t stream);
 
+/* Fused post-LN residual block (R10): C = LN(A W^T + bias + R) * gamma + beta, row-wise
+ * over the N output columns (biased variance, two-pass, fp32) -- tcb_op_linear with
+ * TCB_EPI_BIAS_RESIDUAL followed by tcb_op_layernorm in one tcgen05 kernel.  bf16 only and
+ * N == 512 (a 2-CTA pair keeps complete 512-column rows in TMEM); K % 64 == 0.  Rows whose
+ * d_segment_ids entry is < 0 (pad slots) are written as 0; d_segment_ids may be NULL.
+ * Returns TCB_ERR_UNSUPPORTED for other shapes. */
+tcb_status tcb_op_linear_ln(int64_t M, int32_t N, int32_t K, const void* A, const void* W,
+                            const float* bias, const void* R, const float* gamma,
+                            const float* beta, float eps, const int32_t* d_segment_ids,
+                            void* C, tcb_stream_t stream);
+
 /* Segment-masked multi-head attention, Eq. (5)-(6) over packed rows:
  * O[i, h] = sum_j softmax_j(q_i.k_j / sqrt(d_head) + M_ij) v_j, M_ij = 0 iff slots i and j
  * hold the same request (the diagonal blocks Q_i K_i^T of Eq. (7)), -inf otherwise (R11:

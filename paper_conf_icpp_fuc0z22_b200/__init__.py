@@ -19,7 +19,7 @@ import numpy as np
 from . import _lib
 from ._lib import KCLASSES, POLICIES, TcbError, check, lib
 
-__all__ = ["Plan", "Encoder", "tcb_pack", "op_linear", "op_attention", "op_layernorm",
+__all__ = ["Plan", "Encoder", "tcb_pack", "op_linear", "op_linear_ln", "op_attention", "op_layernorm",
            "launch_count", "profile_enable", "profile_collect", "TcbError", "KCLASSES"]
 
 _DTYPES = {"fp32": 0, "bf16": 1}
@@ -227,6 +227,19 @@ def op_linear(A, W, bias, R=None, epilogue: str = "bias", out=None, stream=None)
     dt = 0 if A.dtype == torch.float32 else 1
     check(lib().tcb_op_linear(dt, M, N, K, _ptr(A), _ptr(W), _ptr(bias), _ptr(R),
                               _lib.EPILOGUES[epilogue], _ptr(out), _stream_ptr(stream)))
+    return out
+
+
+def op_linear_ln(A, W, bias, R, gamma, beta, eps: float, seg_ids=None, out=None, stream=None):
+    """C = LayerNorm(A W^T + bias + R) * gamma + beta (bf16, N == 512), one fused kernel."""
+    import torch
+    M, K = A.shape
+    N = W.shape[0]
+    if out is None:
+        out = torch.empty((M, N), dtype=A.dtype, device=A.device)
+    check(lib().tcb_op_linear_ln(M, N, K, _ptr(A), _ptr(W), _ptr(bias), _ptr(R), _ptr(gamma),
+                                 _ptr(beta), float(eps), _ptr(seg_ids), _ptr(out),
+                                 _stream_ptr(stream)))
     return out
 
 

@@ -28,7 +28,7 @@ EXPORTS = ["tcb_last_error", "tcb_version", "tcb_pack", "tcb_plan_destroy",
            "tcb_plan_write_segtab", "tcb_weights_count", "tcb_weights_create",
            "tcb_weights_destroy", "tcb_workspace_size", "tcb_embed", "tcb_encoder_forward",
            "tcb_unpack", "tcb_launch_count", "tcb_profile_enable", "tcb_profile_collect",
-           "tcb_op_linear", "tcb_op_attention", "tcb_op_layernorm"]
+           "tcb_op_linear", "tcb_op_linear_ln", "tcb_op_attention", "tcb_op_layernorm"]
 
 
 class TcbError(RuntimeError):
@@ -97,6 +97,7 @@ def lib() -> ctypes.CDLL:
         "tcb_profile_enable": (I32, [I32]),
         "tcb_profile_collect": (I32, [P, P]),
         "tcb_op_linear": (I32, [I32, I64, I32, I32, P, P, P, P, I32, P, P]),
+        "tcb_op_linear_ln": (I32, [I64, I32, I32, P, P, P, P, P, P, ctypes.c_float, P, P, P]),
         "tcb_op_attention": (I32, [I32, I64, I32, I32, P, P, P, P, P]),
         "tcb_op_layernorm": (I32, [I32, I64, I32, P, P, P, ctypes.c_float, P, P, P]),
     }

@@ -362,6 +362,10 @@ tcb_status tcb_encoder_forward(const tcb_weights* wc, const tcb_plan* plan,
         w->c_M = M;
       }
     }
+    // bias + residual + LayerNorm fused into the W_O / FFN2 GEMMs when a 2-CTA pair can hold
+    // complete rows in TMEM (d == 512); TCB_NO_LN_FUSION=1 forces the unfused kernels.
+    static const bool no_fusion = std::getenv("TCB_NO_LN_FUSION") != nullptr;
+    const bool fuse_ln = !no_fusion && tcb::k::linear_ln_supported(d);
     for (int l = 0; l < c.num_layers; ++l) {
       const auto& mp = w->maps[l];
       const tcb::k::GemmMaps g_qkv{w->aX, mp.qkv, w->cQkv, w->cQkv};
@@ -372,16 +376,30 @@ tcb_status tcb_encoder_forward(const tcb_weights* wc, const tcb_plan* plan,
                                                                   w->Lf(l, B_QKV), TCB_EPI_BIAS, s));
       TCB_LAUNCH(TCB_K_ATTN, s, tcb::k::launch_attention_bf16(M, d, c.num_heads, qkv, seg,
                                                               segtab, att, s));
-      TCB_LAUNCH(TCB_K_GEMM_O, s, tcb::k::launch_linear_bf16_tc(g_o, M, d, d, w->Lf(l, B_O),
-                                                                TCB_EPI_BIAS_RESIDUAL, s));
-      TCB_LAUNCH(TCB_K_LN, s, tcb::k::launch_layernorm(1, M, d, z, w->Lf(l, LN1_G),
-                                                       w->Lf(l, LN1_B), c.ln_eps, seg, x1, s));
+      if (fuse_ln) {   // W_O + bias + residual + LN1 in one kernel -> x1
+        const tcb::k::GemmMaps g_o_ln{w->aAtt, mp.o, w->cX1, w->cX};
+        TCB_LAUNCH(TCB_K_GEMM_O, s, tcb::k::launch_linear_ln_bf16_tc(
+                                        g_o_ln, M, d, d, w->Lf(l, B_O), w->Lf(l, LN1_G),
+                                        w->Lf(l, LN1_B), c.ln_eps, seg, s));
+      } else {
+        TCB_LAUNCH(TCB_K_GEMM_O, s, tcb::k::launch_linear_bf16_tc(g_o, M, d, d, w->Lf(l, B_O),
+                                                                  TCB_EPI_BIAS_RESIDUAL, s));
+        TCB_LAUNCH(TCB_K_LN, s, tcb::k::launch_layernorm(1, M, d, z, w->Lf(l, LN1_G),
+                                                         w->Lf(l, LN1_B), c.ln_eps, seg, x1, s));
+      }
       TCB_LAUNCH(TCB_K_GEMM_FFN1, s, tcb::k::launch_linear_bf16_tc(g_1, M, f, d, w->Lf(l, B_1),
                                                                    act_epi, s));
-      TCB_LAUNCH(TCB_K_GEMM_FFN2, s, tcb::k::launch_linear_bf16_tc(g_2, M, d, f, w->Lf(l, B_2),
-                                                                   TCB_EPI_BIAS_RESIDUAL, s));
-      TCB_LAUNCH(TCB_K_LN, s, tcb::k::launch_layernorm(1, M, d, z, w->Lf(l, LN2_G),
-                                                       w->Lf(l, LN2_B), c.ln_eps, seg, d_rows, s));
+      if (fuse_ln) {   // FFN2 + bias + residual + LN2 in one kernel -> X
+        const tcb::k::GemmMaps g_2_ln{w->aH, mp.w2, w->cX, w->cX1};
+        TCB_LAUNCH(TCB_K_GEMM_FFN2, s, tcb::k::launch_linear_ln_bf16_tc(
+                                           g_2_ln, M, d, f, w->Lf(l, B_2), w->Lf(l, LN2_G),
+                                           w->Lf(l, LN2_B), c.ln_eps, seg, s));
+      } else {
+        TCB_LAUNCH(TCB_K_GEMM_FFN2, s, tcb::k::launch_linear_bf16_tc(g_2, M, d, f, w->Lf(l, B_2),
+                                                                     TCB_EPI_BIAS_RESIDUAL, s));
+        TCB_LAUNCH(TCB_K_LN, s, tcb::k::launch_layernorm(1, M, d, z, w->Lf(l, LN2_G),
+                                                         w->Lf(l, LN2_B), c.ln_eps, seg, d_rows, s));
+      }
     }
   } else {
     float* X = static_cast<float*>(d_rows);
@@ -461,6 +479,28 @@ tcb_status tcb_op_linear(int32_t dtype, int64_t M, int32_t N, int32_t K, const v
       !tcb::k::make_gemm_c_map(&maps.r, epi == TCB_EPI_BIAS_RESIDUAL ? R : C, M, N))
     return fail(TCB_ERR_CUDA, "tcb_op_linear: cuTensorMapEncodeTiled failed (alignment?)");
   TCB_LAUNCH(TCB_K_GEMM_QKV, s, tcb::k::launch_linear_bf16_tc(maps, M, N, K, bias, epi, s));
+  return TCB_OK;
+}
+
+tcb_status tcb_op_linear_ln(int64_t M, int32_t N, int32_t K, const void* A, const void* W,
+                            const float* bias, const void* R, const float* gamma,
+                            const float* beta, float eps, const int32_t* d_seg, void* C,
+                            tcb_stream_t stream) {
+  tcb::clear_error();
+  if (M < 0 || N <= 0 || K <= 0) return fail(TCB_ERR_INVALID_ARGUMENT, "tcb_op_linear_ln: bad shape");
+  if (M == 0) return TCB_OK;
+  if (!A || !W || !bias || !R || !gamma || !beta || !C)
+    return fail(TCB_ERR_INVALID_ARGUMENT, "tcb_op_linear_ln: NULL pointer");
+  if (!tcb::k::linear_ln_supported(N) || K % 64 != 0 || M > INT32_MAX)
+    return fail(TCB_ERR_UNSUPPORTED, "tcb_op_linear_ln: needs N == 512 and K % 64 == 0");
+  if (tcb_status st = check_device()) return st;
+  cudaStream_t s = reinterpret_cast<cudaStream_t>(stream);
+  tcb::k::GemmMaps maps;
+  if (!tcb::k::make_gemm_a_map(&maps.a, A, M, K) || !tcb::k::make_gemm_w_map(&maps.w, W, N, K) ||
+      !tcb::k::make_gemm_c_map(&maps.c, C, M, N) || !tcb::k::make_gemm_c_map(&maps.r, R, M, N))
+    return fail(TCB_ERR_CUDA, "tcb_op_linear_ln: cuTensorMapEncodeTiled failed (alignment?)");
+  TCB_LAUNCH(TCB_K_GEMM_O, s, tcb::k::launch_linear_ln_bf16_tc(maps, M, N, K, bias, gamma, beta,
+                                                               eps, d_seg, s));
   return TCB_OK;
 }
 

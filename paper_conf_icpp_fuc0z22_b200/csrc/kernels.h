@@ -59,6 +59,11 @@ bool make_gemm_w_map(CUtensorMap* map, const void* W, uint64_t N, uint64_t K);
 bool make_gemm_c_map(CUtensorMap* map, const void* C, uint64_t M, uint64_t N);
 cudaError_t launch_linear_bf16_tc(const GemmMaps& maps, int64_t M, int N, int K,
                                   const float* bias, int epi, cudaStream_t s);
+// C = LayerNorm(A W^T + bias + R) * gamma + beta over rows of N = 512 columns (pad rows 0).
+bool linear_ln_supported(int N);
+cudaError_t launch_linear_ln_bf16_tc(const GemmMaps& maps, int64_t M, int N, int K,
+                                     const float* bias, const float* gamma, const float* beta,
+                                     float eps, const int32_t* seg_ids, cudaStream_t s);
 
 // Attention ------------------------------------------------------------------------------
 cudaError_t launch_attention_bf16(int64_t num_slots, int d_model, int num_heads,

@@ -505,6 +505,323 @@ linear_tc_kernel(const __grid_constant__ CUtensorMap tmA, const __grid_constant_
   }
 }
 
+// ---- GEMM + bias + residual + LayerNorm, fused (row width N = 512) -----------------------
+// Post-LN (R10): Y = LN(A W^T + b + R) * gamma + beta.  One 2-CTA pair owns a 256-row x
+// 512-column tile: per k-block each CTA loads its 128 rows of A once and both 128-row halves
+// of W (n-blocks 0 and 1), and the even CTA issues two M=256, N=256 MMAs into two TMEM
+// accumulators (all 512 columns).  The epilogue then holds complete rows: pass 1 adds bias
+// and the (TMA-prefetched) residual, writes z back to TMEM and accumulates the row moments
+// sum(z), sum(z^2); pass 2 normalises, rounds to bf16 and TMA-stores.  16 epilogue warps
+// (4 per TMEM lane quarter, 128 columns each) combine their row partials through shared
+// memory under a 128-thread named barrier.  Pad slots (segment id < 0) are written as 0
+// (R12).
+constexpr int kLnN = 512;
+constexpr int kLnEpiWarps = 16;                                      // 4 per TMEM lane quarter
+constexpr int kLnThreads = (4 + kLnEpiWarps) * 32;
+constexpr int kLnChunks = kLnN / 4 / 32;                             // 32-col chunks per warp
+constexpr int kLnStageBytes = 3 * 128 * BK * 2;                     // A + 2 W halves: 48 KB
+constexpr int kLnEpiBytes = kLnEpiWarps * 2 * kStageBufBytes;        // 64 KB
+constexpr int kLnStages = (227 * 1024 - 1024 - kLnEpiBytes - 4096) / kLnStageBytes;  // 3
+constexpr int kLnSmemBytes = 1024 + kLnStages * kLnStageBytes + kLnEpiBytes +
+                             8 * (2 * kLnStages + 2 + 2 * kLnEpiWarps) + 16 + 2 * 4 * 128 * 4;
+static_assert(kLnSmemBytes <= 232448, "shared memory budget");
+
+__device__ __forceinline__ void tmem_st32(uint32_t taddr, const float (&v)[32]) {
+  asm volatile(
+      "tcgen05.st.sync.aligned.32x32b.x32.b32 [%0], "
+      "{%1,%2,%3,%4,%5,%6,%7,%8,%9,%10,%11,%12,%13,%14,%15,%16,"
+      "%17,%18,%19,%20,%21,%22,%23,%24,%25,%26,%27,%28,%29,%30,%31,%32};" ::"r"(taddr),
+      "f"(v[0]), "f"(v[1]), "f"(v[2]), "f"(v[3]), "f"(v[4]), "f"(v[5]), "f"(v[6]), "f"(v[7]),
+      "f"(v[8]), "f"(v[9]), "f"(v[10]), "f"(v[11]), "f"(v[12]), "f"(v[13]), "f"(v[14]),
+      "f"(v[15]), "f"(v[16]), "f"(v[17]), "f"(v[18]), "f"(v[19]), "f"(v[20]), "f"(v[21]),
+      "f"(v[22]), "f"(v[23]), "f"(v[24]), "f"(v[25]), "f"(v[26]), "f"(v[27]), "f"(v[28]),
+      "f"(v[29]), "f"(v[30]), "f"(v[31])
+      : "memory");
+}
+__device__ __forceinline__ void named_bar(int id, int threads) {
+  asm volatile("bar.sync %0, %1;" ::"r"(id), "r"(threads) : "memory");
+}
+
+__global__ void __launch_bounds__(kLnThreads, 1)
+linear_ln_kernel(const __grid_constant__ CUtensorMap tmA, const __grid_constant__ CUtensorMap tmW,
+                 const __grid_constant__ CUtensorMap tmC, const __grid_constant__ CUtensorMap tmR,
+                 int M, int K, const float* __restrict__ bias, const float* __restrict__ gamma,
+                 const float* __restrict__ beta, float eps, const int32_t* __restrict__ seg_ids) {
+  constexpr int S = kLnStages;
+  constexpr int kHalfBytes = 128 * BK * 2;
+  extern __shared__ uint8_t smem_raw[];
+  uint8_t* smem = reinterpret_cast<uint8_t*>((reinterpret_cast<uintptr_t>(smem_raw) + 1023) &
+                                             ~static_cast<uintptr_t>(1023));
+  uint8_t* sStage = smem;                                   // S x {A, W half 0, W half 1}
+  uint8_t* sEpi = smem + S * kLnStageBytes;                 // 16 warps x 2 x 2 KB
+  uint64_t* full = reinterpret_cast<uint64_t*>(sEpi + kLnEpiBytes);
+  uint64_t* empty = full + S;
+  uint64_t* tfull = empty + S;
+  uint64_t* tempty = tfull + 1;
+  uint64_t* rbar = tempty + 1;                              // [16 warps][2]
+  uint32_t* tmem_slot = reinterpret_cast<uint32_t*>(rbar + 2 * kLnEpiWarps);
+  float* stats = reinterpret_cast<float*>(tmem_slot + 4);   // [4 parts][128 rows] x 2
+
+  const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
+  const uint32_t rank = cluster_rank();
+  const int cluster_id = blockIdx.x / 2, num_clusters = gridDim.x / 2;
+  const int num_tiles = (M + 255) / 256;
+  const int num_kb = K / BK;
+
+  if (warp == 0 && lane == 0) {
+    asm volatile("prefetch.tensormap [%0];" ::"l"(reinterpret_cast<uint64_t>(&tmA)) : "memory");
+    asm volatile("prefetch.tensormap [%0];" ::"l"(reinterpret_cast<uint64_t>(&tmW)) : "memory");
+    for (int i = 0; i < S; ++i) { mbar_init(&full[i], 1); mbar_init(&empty[i], 1); }
+    mbar_init(tfull, 1);
+    mbar_init(tempty, 2 * kLnEpiWarps);
+    for (int i = 0; i < 2 * kLnEpiWarps; ++i) mbar_init(&rbar[i], 1);
+    asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
+  }
+  if (warp == 2) {
+    asm volatile("tcgen05.alloc.cta_group::2.sync.aligned.shared::cta.b32 [%0], %1;" ::"r"(
+                     smem_u32(tmem_slot)), "r"(kLnN) : "memory");
+    asm volatile("tcgen05.relinquish_alloc_permit.cta_group::2.sync.aligned;" ::: "memory");
+  }
+  tc_fence_before();
+  cluster_sync();
+  tc_fence_after();
+  const uint32_t tmem_base = *tmem_slot;
+
+  if (warp == 0) {
+    // ===== TMA producer: A rows once, both W halves, per k-block =====
+    if (lane == 0) {
+      const uint32_t full0 = map_to_rank0(smem_u32(full));
+      int stage = 0;
+      uint32_t phase = 0;
+      for (int tile = cluster_id; tile < num_tiles; tile += num_clusters) {
+        const int a_row = tile * 256 + static_cast<int>(rank) * 128;
+        for (int kb = 0; kb < num_kb; ++kb) {
+          mbar_wait(&empty[stage], phase ^ 1);
+          if (rank == 0) mbar_expect_tx(&full[stage], 2 * kLnStageBytes);
+          const uint32_t fb = full0 + 8u * stage;
+          uint8_t* st = sStage + stage * kLnStageBytes;
+          tma_load_2d<2>(st, &tmA, fb, kb * BK, a_row);
+          tma_load_2d<2>(st + kHalfBytes, &tmW, fb, kb * BK, static_cast<int>(rank) * 128);
+          tma_load_2d<2>(st + 2 * kHalfBytes, &tmW, fb, kb * BK, 256 + static_cast<int>(rank) * 128);
+          if (++stage == S) { stage = 0; phase ^= 1; }
+        }
+      }
+    }
+  } else if (warp == 1) {
+    // ===== MMA issuer (even CTA): two N=256 halves per k-step =====
+    if (rank == 0) {
+      constexpr uint32_t idesc = idesc_bf16<2, 256>();
+      int stage = 0;
+      uint32_t phase = 0, tphase = 0;
+#ifdef TCB_GEMM_PROBE
+      long long t_start = clock64(), t_full = 0, t_empty = 0;
+#endif
+      for (int tile = cluster_id; tile < num_tiles; tile += num_clusters) {
+#ifdef TCB_GEMM_PROBE
+        long long t0 = clock64();
+#endif
+        mbar_wait(tempty, tphase ^ 1);
+#ifdef TCB_GEMM_PROBE
+        t_empty += clock64() - t0;
+#endif
+        tc_fence_after();
+        for (int kb = 0; kb < num_kb; ++kb) {
+#ifdef TCB_GEMM_PROBE
+          long long t1 = clock64();
+#endif
+          mbar_wait(&full[stage], phase);
+#ifdef TCB_GEMM_PROBE
+          t_full += clock64() - t1;
+#endif
+          tc_fence_after();
+          if (lane == 0) {
+            const uint32_t a0 = smem_u32(sStage + stage * kLnStageBytes);
+            const uint32_t b0 = a0 + kHalfBytes, b1 = a0 + 2 * kHalfBytes;
+#pragma unroll
+            for (int k = 0; k < BK / 16; ++k) {
+              const uint64_t ad = sdesc_sw128(a0 + k * 32);
+              tc_mma<2>(tmem_base, ad, sdesc_sw128(b0 + k * 32), idesc, (kb | k) != 0 ? 1u : 0u);
+              tc_mma<2>(tmem_base + 256, ad, sdesc_sw128(b1 + k * 32), idesc, (kb | k) != 0 ? 1u : 0u);
+            }
+            tc_commit<2>(&empty[stage]);
+            if (kb == num_kb - 1) tc_commit<2>(tfull);
+          }
+          __syncwarp();
+          if (++stage == S) { stage = 0; phase ^= 1; }
+        }
+        tphase ^= 1;
+      }
+#ifdef TCB_GEMM_PROBE
+      if (lane == 0 && blockIdx.x < 4)
+        printf("lnprobe mma cta %d total %lld wait_full %lld wait_tempty %lld\n", blockIdx.x,
+               clock64() - t_start, t_full, t_empty);
+#endif
+    }
+  } else if (warp >= 4) {
+    // ===== Epilogue: bias + residual + LayerNorm over complete 512-column rows =====
+    const int ew = warp - 4;
+    const int q = warp & 3;                       // TMEM lane quarter (rows 32q..32q+31)
+    const int part = ew >> 2;                     // 128-column quarter of the row
+    const uint32_t bufs = smem_u32(sEpi) + ew * 2 * kStageBufBytes;
+    uint64_t* my_rbar = rbar + 2 * ew;
+    uint32_t rph = 0;                             // bit b: phase of residual barrier b
+    const uint32_t tempty0 = map_to_rank0(smem_u32(tempty));
+    float* stat1 = stats;                         // [4][128]
+    float* stat2 = stats + 512;
+    const int srow = q * 32 + lane;               // row within this CTA's 128
+    uint32_t tphase = 0;
+    for (int tile = cluster_id; tile < num_tiles; tile += num_clusters) {
+      const int row0 = tile * 256 + static_cast<int>(rank) * 128 + q * 32;
+      const int64_t grow = static_cast<int64_t>(row0) + lane;
+      const bool pad = grow >= M || (seg_ids && __ldg(&seg_ids[grow]) < 0);
+      const int col0 = part * (kLnN / 4);
+      if (lane == 0) bulk_wait_read<0>();         // previous tile's stores have read the buffers
+      __syncwarp();
+      if (lane == 0) {
+#pragma unroll
+        for (int j = 0; j < 2; ++j) {
+          mbar_expect_tx(&my_rbar[j], kStageBufBytes);
+          asm volatile(
+              "cp.async.bulk.tensor.2d.shared::cluster.global.mbarrier::complete_tx::bytes"
+              " [%0], [%1, {%3, %4}], [%2];" ::"r"(bufs + j * kStageBufBytes),
+              "l"(reinterpret_cast<uint64_t>(&tmR)), "r"(smem_u32(&my_rbar[j])),
+              "r"(col0 + 32 * j), "r"(row0)
+              : "memory");
+        }
+      }
+#ifdef TCB_GEMM_PROBE
+      long long e0 = clock64();
+#endif
+      mbar_wait(tfull, tphase);
+#ifdef TCB_GEMM_PROBE
+      long long e1 = clock64();
+#endif
+      tc_fence_after();
+      const uint32_t tbase = tmem_base + (static_cast<uint32_t>(q * 32) << 16) + col0;
+      // pass 1: z = acc + bias + residual -> TMEM; row moments sum(z), sum(z^2)
+      float sum = 0.f, sumsq = 0.f;
+#pragma unroll 1
+      for (int j = 0; j < kLnChunks; ++j) {
+        const int b = j & 1;
+        const uint32_t buf = bufs + b * kStageBufBytes;
+        uint32_t r[32];
+        tmem_ld32_nowait(tbase + 32 * j, r);
+        tmem_wait_ld();
+        float* v = reinterpret_cast<float*>(r);
+        const float4* b4 = reinterpret_cast<const float4*>(bias + col0 + 32 * j);
+#pragma unroll
+        for (int t = 0; t < 8; ++t) {
+          const float4 bb = __ldg(b4 + t);
+          v[4 * t + 0] += bb.x;
+          v[4 * t + 1] += bb.y;
+          v[4 * t + 2] += bb.z;
+          v[4 * t + 3] += bb.w;
+        }
+        mbar_wait(&my_rbar[b], (rph >> b) & 1);
+        rph ^= 1u << b;
+#pragma unroll
+        for (int t = 0; t < 4; ++t) {
+          const uint4 x = ld_shared_v4(buf + sw64(lane, t));
+          const __nv_bfloat162* hh = reinterpret_cast<const __nv_bfloat162*>(&x);
+#pragma unroll
+          for (int e = 0; e < 4; ++e) {
+            const float2 f = __bfloat1622float2(hh[e]);
+            v[8 * t + 2 * e] += f.x;
+            v[8 * t + 2 * e + 1] += f.y;
+          }
+        }
+#pragma unroll
+        for (int t = 0; t < 32; ++t) {
+          sum += v[t];
+          sumsq = fmaf(v[t], v[t], sumsq);
+        }
+        tmem_st32(tbase + 32 * j, *reinterpret_cast<float(*)[32]>(v));
+        __syncwarp();                             // every lane has read buffer b
+        if (j + 2 < kLnChunks && lane == 0) {
+          mbar_expect_tx(&my_rbar[b], kStageBufBytes);
+          asm volatile(
+              "cp.async.bulk.tensor.2d.shared::cluster.global.mbarrier::complete_tx::bytes"
+              " [%0], [%1, {%3, %4}], [%2];" ::"r"(buf),
+              "l"(reinterpret_cast<uint64_t>(&tmR)), "r"(smem_u32(&my_rbar[b])),
+              "r"(col0 + 32 * (j + 2)), "r"(row0)
+              : "memory");
+        }
+      }
+      asm volatile("tcgen05.wait::st.sync.aligned;" ::: "memory");
+      stat1[part * 128 + srow] = sum;
+      stat2[part * 128 + srow] = sumsq;
+      named_bar(1 + q, 128);
+      // single-pass moments in fp32: |mean| is O(std) for these residual streams, so
+      // E[z^2] - mean^2 loses nothing material at the bf16 output precision
+      const float mean = (stat1[srow] + stat1[128 + srow] + stat1[256 + srow] + stat1[384 + srow]) *
+                         (1.f / kLnN);
+      const float ex2m = (stat2[srow] + stat2[128 + srow] + stat2[256 + srow] + stat2[384 + srow]) *
+                         (1.f / kLnN);
+      const float rstd = rsqrtf(fmaxf(ex2m - mean * mean, 0.f) + eps);
+      // pass 2: normalise, bf16, TMA store
+#pragma unroll 1
+      for (int j = 0; j < kLnChunks; ++j) {
+        const int b = j & 1;
+        const uint32_t buf = bufs + b * kStageBufBytes;
+        uint32_t r[32];
+        tmem_ld32_nowait(tbase + 32 * j, r);
+        tmem_wait_ld();
+        float* y = reinterpret_cast<float*>(r);
+        const float4* g4 = reinterpret_cast<const float4*>(gamma + col0 + 32 * j);
+        const float4* e4 = reinterpret_cast<const float4*>(beta + col0 + 32 * j);
+#pragma unroll
+        for (int t = 0; t < 8; ++t) {
+          const float4 gg = __ldg(g4 + t), ee = __ldg(e4 + t);
+          y[4 * t + 0] = pad ? 0.f : (y[4 * t + 0] - mean) * rstd * gg.x + ee.x;
+          y[4 * t + 1] = pad ? 0.f : (y[4 * t + 1] - mean) * rstd * gg.y + ee.y;
+          y[4 * t + 2] = pad ? 0.f : (y[4 * t + 2] - mean) * rstd * gg.z + ee.z;
+          y[4 * t + 3] = pad ? 0.f : (y[4 * t + 3] - mean) * rstd * gg.w + ee.w;
+        }
+        if (j >= 2) {
+          if (lane == 0) bulk_wait_read<1>();     // the store that last used `buf` read it
+          __syncwarp();
+        }
+#pragma unroll
+        for (int t = 0; t < 4; ++t) {
+          uint4 x;
+          __nv_bfloat162* hh = reinterpret_cast<__nv_bfloat162*>(&x);
+#pragma unroll
+          for (int e = 0; e < 4; ++e)
+            hh[e] = __floats2bfloat162_rn(y[8 * t + 2 * e], y[8 * t + 2 * e + 1]);
+          st_shared_v4(buf + sw64(lane, t), x);
+        }
+        fence_async_smem();
+        __syncwarp();
+        if (lane == 0) {
+          asm volatile("cp.async.bulk.tensor.2d.global.shared::cta.bulk_group [%0, {%2, %3}], [%1];" ::"l"(
+                           reinterpret_cast<uint64_t>(&tmC)),
+                       "r"(buf), "r"(col0 + 32 * j), "r"(row0)
+                       : "memory");
+          asm volatile("cp.async.bulk.commit_group;" ::: "memory");
+        }
+      }
+      // the stats slots are rewritten next tile only after all 4 warps passed this barrier
+      named_bar(1 + q, 128);
+      tc_fence_before();
+      __syncwarp();
+      if (lane == 0) mbar_arrive_remote(tempty0);
+#ifdef TCB_GEMM_PROBE
+      if (lane == 0 && blockIdx.x < 2 && warp == 4)
+        printf("lnprobe epi cta %d tile %d wait_tfull %lld epilogue %lld\n", blockIdx.x, tile, e1 - e0, clock64() - e1);
+#endif
+      tphase ^= 1;
+    }
+    if (lane == 0) bulk_wait_all();
+  }
+  __syncwarp();
+  tc_fence_before();
+  cluster_sync();
+  tc_fence_after();
+  if (warp == 2)
+    asm volatile("tcgen05.dealloc.cta_group::2.sync.aligned.b32 %0, %1;" ::"r"(tmem_base),
+                 "r"(kLnN) : "memory");
+}
+
 // ---- host side ---------------------------------------------------------------------------
 PFN_cuTensorMapEncodeTiled_v12000 g_encode = nullptr;
 std::once_flag g_encode_once;
@@ -575,6 +892,39 @@ cudaError_t dispatch_epi(const GemmMaps& m, int M, int N, int K, const float* bi
 }
 
 }  // namespace
+
+bool linear_ln_supported(int N) { return N == kLnN; }
+
+cudaError_t launch_linear_ln_bf16_tc(const GemmMaps& m, int64_t M, int N, int K,
+                                     const float* bias, const float* gamma, const float* beta,
+                                     float eps, const int32_t* seg_ids, cudaStream_t s) {
+  if (M == 0) return cudaSuccess;
+  if (N != kLnN) return cudaErrorInvalidValue;
+  static bool attr_set = false;
+  if (!attr_set) {
+    cudaError_t e = cudaFuncSetAttribute(linear_ln_kernel,
+                                         cudaFuncAttributeMaxDynamicSharedMemorySize, kLnSmemBytes);
+    if (e != cudaSuccess) return e;
+    attr_set = true;
+  }
+  const int tiles = static_cast<int>((M + 255) / 256);
+  int clusters = num_sms() / 2;
+  if (tiles < clusters) clusters = tiles;
+  cudaLaunchConfig_t cfg{};
+  cfg.gridDim = dim3(clusters * 2);
+  cfg.blockDim = dim3(kLnThreads);
+  cfg.dynamicSmemBytes = kLnSmemBytes;
+  cfg.stream = s;
+  cudaLaunchAttribute attr[1];
+  attr[0].id = cudaLaunchAttributeClusterDimension;
+  attr[0].val.clusterDim.x = 2;
+  attr[0].val.clusterDim.y = 1;
+  attr[0].val.clusterDim.z = 1;
+  cfg.attrs = attr;
+  cfg.numAttrs = 1;
+  return cudaLaunchKernelEx(&cfg, linear_ln_kernel, m.a, m.w, m.c, m.r, static_cast<int>(M), K,
+                            bias, gamma, beta, eps, seg_ids);
+}
 
 bool make_tmap_bf16(CUtensorMap* map, const void* ptr, uint64_t rows, uint64_t cols,
                     uint32_t box_rows, uint32_t box_cols, int swizzle_bytes) {

@@ -51,6 +51,32 @@ def test_linear_bf16_tcgen05_vs_oracle(M, N, K, epi):
     assert np.all(err <= bound), float(np.max(err / bound))
 
 
+@pytest.mark.parametrize("M,K", [(1, 512), (300, 512), (4133, 512), (1000, 2048), (32768, 512)])
+def test_linear_ln_fused_vs_oracle(M, K):
+    """W_O / FFN2 + bias + residual + LayerNorm in one tcgen05 kernel (N = 512)."""
+    N = 512
+    rng = np.random.default_rng(M + K)
+    A = _bf16(rng.normal(size=(M, K)))
+    W = _bf16(rng.uniform(-1, 1, size=(N, K)) * np.sqrt(3.0 / K))
+    b = _bf16(rng.normal(0, 0.1, size=N))
+    R = _bf16(rng.normal(size=(M, N)))
+    g = _bf16(1 + rng.normal(0, 0.1, size=N))
+    be = _bf16(rng.normal(0, 0.1, size=N))
+    seg = np.zeros(M, np.int32)
+    seg[::7] = -1
+    out = tcb.op_linear_ln(_dev(A, torch.bfloat16), _dev(W, torch.bfloat16), _dev(b, torch.float32),
+                           _dev(R, torch.bfloat16), _dev(g, torch.float32), _dev(be, torch.float32),
+                           1e-5, _dev(seg))
+    torch.cuda.synchronize()
+    got = out.float().cpu().numpy()
+    z = oracle.linear(A, W, b, R)
+    ref = oracle.layernorm(z, g, be, 1e-5)
+    real = seg >= 0
+    err = np.abs(got[real] - ref[real])
+    assert np.all(err <= 2.0 ** -8 * np.abs(ref[real]) + 2e-2), float(err.max())
+    assert np.all(got[~real] == 0)
+
+
 @pytest.mark.parametrize("M,N,K", [(64, 192, 64), (130, 256, 64), (37, 64, 256)])
 @pytest.mark.parametrize("epi", ["bias", "bias_gelu", "bias_residual"])
 def test_linear_f32_simt_vs_oracle(M, N, K, epi):
