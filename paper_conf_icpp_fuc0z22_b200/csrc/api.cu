@@ -165,6 +165,18 @@ namespace {
 
 enum { W_QKV = 0, B_QKV, W_O, B_O, LN1_G, LN1_B, W_1, B_1, W_2, B_2, LN2_G, LN2_B };
 
+// bf16 attention: tcgen05 kernel (attention_tc.cu); TCB_ATTN=mma selects the warp-level
+// mma.sync kernel (attention.cu) for A/B measurements.
+cudaError_t attention_bf16(int64_t M, int d, int heads, const void* qkv, const int32_t* seg,
+                           const int4* segtab, void* out, cudaStream_t s) {
+  static const bool use_mma = [] {
+    const char* v = std::getenv("TCB_ATTN");
+    return v && std::string(v) == "mma";
+  }();
+  return use_mma ? tcb::k::launch_attention_bf16(M, d, heads, qkv, seg, segtab, out, s)
+                 : tcb::k::launch_attention_bf16_tc(M, d, heads, qkv, seg, segtab, out, s);
+}
+
 tcb_status embed_impl(const tcb_weights* w, const tcb_plan* plan, const int32_t* d_segtab,
                       const int32_t* d_ids, void* d_rows, int32_t* d_seg, int32_t* d_pos,
                       cudaStream_t s) {
@@ -374,8 +386,7 @@ tcb_status tcb_encoder_forward(const tcb_weights* wc, const tcb_plan* plan,
       const tcb::k::GemmMaps g_2{w->aH, mp.w2, w->cZ, w->cX1};
       TCB_LAUNCH(TCB_K_GEMM_QKV, s, tcb::k::launch_linear_bf16_tc(g_qkv, M, 3 * d, d,
                                                                   w->Lf(l, B_QKV), TCB_EPI_BIAS, s));
-      TCB_LAUNCH(TCB_K_ATTN, s, tcb::k::launch_attention_bf16(M, d, c.num_heads, qkv, seg,
-                                                              segtab, att, s));
+      TCB_LAUNCH(TCB_K_ATTN, s, attention_bf16(M, d, c.num_heads, qkv, seg, segtab, att, s));
       if (fuse_ln) {   // W_O + bias + residual + LN1 in one kernel -> x1
         const tcb::k::GemmMaps g_o_ln{w->aAtt, mp.o, w->cX1, w->cX};
         TCB_LAUNCH(TCB_K_GEMM_O, s, tcb::k::launch_linear_ln_bf16_tc(
@@ -520,8 +531,7 @@ tcb_status tcb_op_attention(int32_t dtype, int64_t num_slots, int32_t d_model,
   cudaStream_t s = reinterpret_cast<cudaStream_t>(stream);
   const int4* segtab = reinterpret_cast<const int4*>(d_segtab);
   if (dtype == 1)
-    TCB_LAUNCH(TCB_K_ATTN, s, tcb::k::launch_attention_bf16(num_slots, d_model, num_heads, qkv,
-                                                            d_seg, segtab, O, s));
+    TCB_LAUNCH(TCB_K_ATTN, s, attention_bf16(num_slots, d_model, num_heads, qkv, d_seg, segtab, O, s));
   else
     TCB_LAUNCH(TCB_K_ATTN, s, tcb::k::launch_attention_f32(num_slots, d_model, num_heads,
                                                            static_cast<const float*>(qkv), d_seg,

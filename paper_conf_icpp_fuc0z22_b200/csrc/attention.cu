@@ -20,6 +20,7 @@
 #include <cuda_bf16.h>
 
 #include <cmath>
+#include <cstdio>
 
 #include "kernels.h"
 
@@ -96,15 +97,18 @@ __device__ __forceinline__ void mbar_expect_tx(uint32_t bar, uint32_t bytes) {
 __device__ __forceinline__ void mbar_arrive(uint32_t bar) {
   asm volatile("mbarrier.arrive.shared::cta.b64 _, [%0];" ::"r"(bar) : "memory");
 }
+// try_wait with a suspend-time hint: a waiting warp is parked by the hardware until the
+// phase completes (or ~10 us pass) instead of spinning and stealing issue slots from the
+// consumer warps that share its scheduler.
 __device__ __forceinline__ void mbar_wait(uint32_t bar, uint32_t parity) {
   uint32_t done = 0;
   do {
     asm volatile(
         "{\n\t.reg .pred p;\n\t"
-        "mbarrier.try_wait.parity.shared::cta.b64 p, [%1], %2;\n\t"
+        "mbarrier.try_wait.parity.shared::cta.b64 p, [%1], %2, %3;\n\t"
         "selp.u32 %0, 1, 0, p;\n\t}"
         : "=r"(done)
-        : "r"(bar), "r"(parity)
+        : "r"(bar), "r"(parity), "r"(10000)
         : "memory");
   } while (!done);
 }
@@ -272,11 +276,21 @@ attn_bf16_kernel(const __grid_constant__ CUtensorMap tmQKV, const int32_t* __res
   }
   int kv_stage = 0, q_stage = 0;
   uint32_t kv_phase = 0, q_phase = 0;
+#ifdef TCB_ATTN_PROBE
+  long long p_start = clock64(), p_q = 0, p_kv = 0;
+  int p_items = 0, p_chunks = 0;
+#endif
   for (int item = blockIdx.x; item < num_items; item += gridDim.x) {
     const int qb = item / num_heads, h = item % num_heads;
     const int64_t rowA = static_cast<int64_t>(qb) * AQ + warp * 16 + g, rowB = rowA + 8;
-
+#ifdef TCB_ATTN_PROBE
+    long long pq0 = clock64();
+#endif
     mbar_wait(q_full + 8 * q_stage, q_phase);
+#ifdef TCB_ATTN_PROBE
+    p_q += clock64() - pq0;
+    ++p_items;
+#endif
     const ItemInfo* inf = infos + q_stage;
     const int2 iv = inf->blk;
     const int4 wv = inf->warps[warp];              // union lo/hi, intersection lo/hi
@@ -303,7 +317,14 @@ attn_bf16_kernel(const __grid_constant__ CUtensorMap tmQKV, const int32_t* __res
       const int sb_hi = lim > kbase ? min(KC / 16, (lim - kbase + 15) >> 4) : 0;
       // always observe the slot's fill before releasing it (keeps the ring's phases exact
       // even when this warp skips the whole chunk)
+#ifdef TCB_ATTN_PROBE
+      long long pk0 = clock64();
+#endif
       mbar_wait(kv_full + 8 * kv_stage, kv_phase);
+#ifdef TCB_ATTN_PROBE
+      p_kv += clock64() - pk0;
+      ++p_chunks;
+#endif
       if (wv.y >= 0 && sb_lo < sb_hi) {
         const uint32_t kt = sK + kv_stage * kKVTileBytes, vt = sV + kv_stage * kKVTileBytes;
         float s[KC / 16][2][4];
@@ -408,6 +429,11 @@ attn_bf16_kernel(const __grid_constant__ CUtensorMap tmQKV, const int32_t* __res
         *reinterpret_cast<uint32_t*>(O + rowB * d_model + col) = pack_bf16(acc[j][2] * iB, acc[j][3] * iB);
     }
   }
+#ifdef TCB_ATTN_PROBE
+  if (lane == 0 && blockIdx.x < 2 && (warp == 0 || warp == 5))
+    printf("attnprobe cta %d warp %d total %lld wait_q %lld wait_kv %lld items %d chunks %d\n",
+           blockIdx.x, warp, clock64() - p_start, p_q, p_kv, p_items, p_chunks);
+#endif
 }
 
 // fp32 path: one warp per (query slot, head); keys restricted to the query's own request

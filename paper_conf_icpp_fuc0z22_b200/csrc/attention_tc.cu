@@ -1,0 +1,621 @@
+// attention_tc.cu -- segment-masked self-attention on the 5th-generation tensor cores.
+//
+// Eq. (5)-(6): Att_CB(Q,K,V) = softmax(QK^T/sqrt(d) + M) V with M = 0 on the
+// diagonal blocks Q_i K_i^T (Eq. (7)) and -inf elsewhere (R11).  Work item = (block of 128
+// query slots, head).  The block's key interval [start of its first request, end of its
+// last request) is walked in 128-key chunks; chunks outside it (other rows / other
+// requests) are never loaded or computed.  Per chunk:
+//   S = Q K^T       tcgen05.mma M=128 N=128 K=64 (Q, K K-major in smem) -> TMEM (fp32)
+//   softmax         8 warps: thread = one query row (its TMEM lane) x 64 of the 128 key
+//                   columns; mask = key outside the row's own request -> p = 0 exactly;
+//                   online max with lazy rescaling (O is only rescaled when the running
+//                   max grows by more than 2^8); p = 2^(s*log2e/sqrt(d) - m) in fp32, row
+//                   sum in fp32, P rounded to bf16 into smem (K-major, 128B swizzle)
+//   O += P V        tcgen05.mma M=128 N=64 K=128 (P K-major, V MN-major in smem) -> TMEM
+// Roles (one CTA per SM, persistent over items): warp 0 = item metadata + Q TMA, warp 1 =
+// MMA issuer (one thread), warp 2 = TMEM allocator, then K/V TMA producer, warps 4..11 =
+// softmax/epilogue.  Q/K/V rings and S/P double buffers are mbarrier-guarded, so loads,
+// QK^T of chunk c+1, softmax of chunk c and P V of chunk c-1 overlap.
+#include <cuda_bf16.h>
+#include <cudaTypedefs.h>
+
+#include <cmath>
+#include <cstdint>
+#include <cstdio>
+
+#include "kernels.h"
+
+namespace tcb {
+namespace k {
+namespace {
+
+constexpr int TQ = 128;                 // query slots per item (TMEM lanes)
+constexpr int TK = 128;                 // keys per chunk
+constexpr int DH = 64;                  // head dim
+constexpr int kSmWarps = 8;             // softmax warps (2 per TMEM lane quarter)
+constexpr int kThreads = (4 + kSmWarps) * 32;
+constexpr int kQStages = 3, kKVStages = 3;
+constexpr int kTileBytes = 128 * DH * 2;            // 16 KB: Q, K or V tile (128 rows x 128 B)
+constexpr int kPBytes = TQ * TK * 2;                // 32 KB: P tile (two 64-key K blocks)
+constexpr float kRescaleLog2 = 8.f;                 // lazy-rescale threshold (log2 units)
+
+struct ItemInfo {
+  int2 rows[TQ];   // [start, end) of the request of query slot q0 + r (empty for pads)
+  int kbase, nch;  // first key (8-aligned) and number of 128-key chunks
+};
+
+constexpr int kSmemBytes = 1024 + kQStages * kTileBytes + 2 * kKVStages * kTileBytes +
+                           2 * kPBytes + kQStages * static_cast<int>(sizeof(ItemInfo)) + 4096;
+
+__device__ __forceinline__ uint32_t smem_u32(const void* p) {
+  return static_cast<uint32_t>(__cvta_generic_to_shared(p));
+}
+__device__ __forceinline__ void mbar_init(uint32_t bar, uint32_t count) {
+  asm volatile("mbarrier.init.shared::cta.b64 [%0], %1;" ::"r"(bar), "r"(count));
+}
+__device__ __forceinline__ void mbar_expect_tx(uint32_t bar, uint32_t bytes) {
+  asm volatile("mbarrier.arrive.expect_tx.shared::cta.b64 _, [%0], %1;" ::"r"(bar), "r"(bytes)
+               : "memory");
+}
+__device__ __forceinline__ void mbar_arrive(uint32_t bar) {
+  asm volatile("mbarrier.arrive.shared::cta.b64 _, [%0];" ::"r"(bar) : "memory");
+}
+__device__ __forceinline__ void mbar_wait(uint32_t bar, uint32_t parity) {
+  uint32_t done = 0;
+  do {
+    asm volatile(
+        "{\n\t.reg .pred p;\n\t"
+        "mbarrier.try_wait.parity.shared::cta.b64 p, [%1], %2;\n\t"
+        "selp.u32 %0, 1, 0, p;\n\t}"
+        : "=r"(done)
+        : "r"(bar), "r"(parity)
+        : "memory");
+  } while (!done);
+}
+__device__ __forceinline__ void tma_load(uint32_t dst, const CUtensorMap* map, uint32_t bar,
+                                         int c0, int c1) {
+  asm volatile(
+      "cp.async.bulk.tensor.2d.shared::cluster.global.mbarrier::complete_tx::bytes"
+      " [%0], [%1, {%3, %4}], [%2];" ::"r"(dst),
+      "l"(reinterpret_cast<uint64_t>(map)), "r"(bar), "r"(c0), "r"(c1)
+      : "memory");
+}
+__device__ __forceinline__ void tc_fence_before() {
+  asm volatile("tcgen05.fence::before_thread_sync;" ::: "memory");
+}
+__device__ __forceinline__ void tc_fence_after() {
+  asm volatile("tcgen05.fence::after_thread_sync;" ::: "memory");
+}
+__device__ __forceinline__ void tc_commit(uint32_t bar) {
+  asm volatile("tcgen05.commit.cta_group::1.mbarrier::arrive::one.shared::cluster.b64 [%0];" ::"r"(bar)
+               : "memory");
+}
+__device__ __forceinline__ void tc_mma(uint32_t tmem_d, uint64_t adesc, uint64_t bdesc,
+                                       uint32_t idesc, uint32_t accumulate) {
+  asm volatile(
+      "{\n\t.reg .pred p;\n\tsetp.ne.b32 p, %4, 0;\n\t"
+      "tcgen05.mma.cta_group::1.kind::f16 [%0], %1, %2, %3, p;\n\t}" ::"r"(tmem_d),
+      "l"(adesc), "l"(bdesc), "r"(idesc), "r"(accumulate)
+      : "memory");
+}
+__device__ __forceinline__ void tmem_ld32(uint32_t taddr, uint32_t (&r)[32]) {
+  asm volatile(
+      "tcgen05.ld.sync.aligned.32x32b.x32.b32 "
+      "{%0,%1,%2,%3,%4,%5,%6,%7,%8,%9,%10,%11,%12,%13,%14,%15,"
+      "%16,%17,%18,%19,%20,%21,%22,%23,%24,%25,%26,%27,%28,%29,%30,%31}, [%32];"
+      : "=r"(r[0]), "=r"(r[1]), "=r"(r[2]), "=r"(r[3]), "=r"(r[4]), "=r"(r[5]), "=r"(r[6]),
+        "=r"(r[7]), "=r"(r[8]), "=r"(r[9]), "=r"(r[10]), "=r"(r[11]), "=r"(r[12]),
+        "=r"(r[13]), "=r"(r[14]), "=r"(r[15]), "=r"(r[16]), "=r"(r[17]), "=r"(r[18]),
+        "=r"(r[19]), "=r"(r[20]), "=r"(r[21]), "=r"(r[22]), "=r"(r[23]), "=r"(r[24]),
+        "=r"(r[25]), "=r"(r[26]), "=r"(r[27]), "=r"(r[28]), "=r"(r[29]), "=r"(r[30]),
+        "=r"(r[31])
+      : "r"(taddr)
+      : "memory");
+}
+__device__ __forceinline__ void tmem_wait_ld() { asm volatile("tcgen05.wait::ld.sync.aligned;" ::: "memory"); }
+__device__ __forceinline__ void tmem_st32(uint32_t taddr, const uint32_t (&v)[32]) {
+  asm volatile(
+      "tcgen05.st.sync.aligned.32x32b.x32.b32 [%0], "
+      "{%1,%2,%3,%4,%5,%6,%7,%8,%9,%10,%11,%12,%13,%14,%15,%16,"
+      "%17,%18,%19,%20,%21,%22,%23,%24,%25,%26,%27,%28,%29,%30,%31,%32};" ::"r"(taddr),
+      "r"(v[0]), "r"(v[1]), "r"(v[2]), "r"(v[3]), "r"(v[4]), "r"(v[5]), "r"(v[6]), "r"(v[7]),
+      "r"(v[8]), "r"(v[9]), "r"(v[10]), "r"(v[11]), "r"(v[12]), "r"(v[13]), "r"(v[14]),
+      "r"(v[15]), "r"(v[16]), "r"(v[17]), "r"(v[18]), "r"(v[19]), "r"(v[20]), "r"(v[21]),
+      "r"(v[22]), "r"(v[23]), "r"(v[24]), "r"(v[25]), "r"(v[26]), "r"(v[27]), "r"(v[28]),
+      "r"(v[29]), "r"(v[30]), "r"(v[31])
+      : "memory");
+}
+__device__ __forceinline__ void named_bar(int id, int threads) {
+  asm volatile("bar.sync %0, %1;" ::"r"(id), "r"(threads) : "memory");
+}
+__device__ __forceinline__ float ex2(float x) {
+  float y;
+  asm("ex2.approx.ftz.f32 %0, %1;" : "=f"(y) : "f"(x));
+  return y;
+}
+// K-major operand, rows of 128 B, 128B swizzle, 8-row groups 1024 B apart (SBO).
+__device__ __forceinline__ uint64_t desc_kmajor(uint32_t saddr) {
+  return static_cast<uint64_t>((saddr & 0x3FFFFu) >> 4) | (static_cast<uint64_t>(1) << 16) |
+         (static_cast<uint64_t>(1024 >> 4) << 32) | (static_cast<uint64_t>(1) << 46) |
+         (static_cast<uint64_t>(2) << 61);
+}
+// MN-major operand (V as the B of P.V): each 128 B row holds the 64 N-elements of one K
+// index; 8 K-rows form a 1024 B swizzle atom (SBO); a single 64-wide N block (LBO unused).
+__device__ __forceinline__ uint64_t desc_mnmajor(uint32_t saddr) {
+  return static_cast<uint64_t>((saddr & 0x3FFFFu) >> 4) | (static_cast<uint64_t>(1) << 16) |
+         (static_cast<uint64_t>(1024 >> 4) << 32) | (static_cast<uint64_t>(1) << 46) |
+         (static_cast<uint64_t>(2) << 61);
+}
+// kind::f16 instruction descriptors: fp32 D, bf16 A/B.
+constexpr uint32_t kIdescQK = (1u << 4) | (1u << 7) | (1u << 10) | ((128u >> 3) << 17) | ((128u >> 4) << 24);
+constexpr uint32_t kIdescPV = (1u << 4) | (1u << 7) | (1u << 10) | (1u << 16) | ((64u >> 3) << 17) |
+                              ((128u >> 4) << 24);
+
+__device__ void compute_info(ItemInfo* inf, const int32_t* __restrict__ seg_ids,
+                             const int4* __restrict__ segtab, int64_t q0, int64_t num_slots,
+                             int lane) {
+  int lo = INT_MAX, hi = -1;
+#pragma unroll
+  for (int i = 0; i < TQ / 32; ++i) {
+    const int64_t row = q0 + lane + 32 * i;
+    const int sg = row < num_slots ? __ldg(&seg_ids[row]) : -1;
+    int2 v = make_int2(0, 0);
+    if (sg >= 0) {
+      const int4 rec = __ldg(&segtab[1 + sg]);
+      v = make_int2(rec.x, rec.x + rec.y);
+      lo = min(lo, v.x);
+      hi = max(hi, v.y);
+    }
+    inf->rows[lane + 32 * i] = v;
+  }
+#pragma unroll
+  for (int o = 16; o > 0; o >>= 1) {
+    lo = min(lo, __shfl_xor_sync(0xffffffffu, lo, o));
+    hi = max(hi, __shfl_xor_sync(0xffffffffu, hi, o));
+  }
+  if (lane == 0) {
+    if (hi < 0) {
+      inf->kbase = 0;
+      inf->nch = 0;
+    } else {
+      const int kb = lo & ~7;
+      inf->kbase = kb;
+      inf->nch = (hi - kb + TK - 1) / TK;
+    }
+  }
+  __syncwarp();
+}
+
+__global__ void __launch_bounds__(kThreads, 1)
+attn_tc_kernel(const __grid_constant__ CUtensorMap tmQKV, const int32_t* __restrict__ seg_ids,
+               const int4* __restrict__ segtab, __nv_bfloat16* __restrict__ O,
+               int64_t num_slots, int d_model, int num_heads, int num_items, float scale_log2) {
+  extern __shared__ uint8_t smem_raw[];
+  const uint32_t raw = smem_u32(smem_raw);
+  const uint32_t base = (raw + 1023) & ~1023u;
+  const uint32_t sQ = base;                                    // [3][128 x 64]
+  const uint32_t sK = sQ + kQStages * kTileBytes;              // [3][128 x 64]
+  const uint32_t sV = sK + kKVStages * kTileBytes;             // [3][128 x 64]
+  const uint32_t sP = sV + kKVStages * kTileBytes;             // [2][2 blocks][128 x 64]
+  uint8_t* gen = smem_raw + (sP + 2 * kPBytes - raw);
+  ItemInfo* infos = reinterpret_cast<ItemInfo*>(gen);          // [3]
+  float* xch = reinterpret_cast<float*>(gen + kQStages * sizeof(ItemInfo));   // [2][128]
+  uint32_t* tmem_slot = reinterpret_cast<uint32_t*>(xch + 6 * TQ);   // [2 bufs][2][128] + l[2][128]
+  const uint32_t bars = (smem_u32(tmem_slot + 4) + 7) & ~7u;
+  const uint32_t q_full = bars, q_empty = q_full + 8 * kQStages;
+  const uint32_t kv_full = q_empty + 8 * kQStages, kv_empty = kv_full + 8 * kKVStages;
+  const uint32_t s_full = kv_empty + 8 * kKVStages, s_empty = s_full + 16;
+  const uint32_t p_full = s_empty + 16, p_empty = p_full + 16;
+  const uint32_t o_full = p_empty + 16, o_empty = o_full + 16;   // [2] each (O double buffer)
+  const uint32_t info_full = o_empty + 16;                     // [3]
+
+  const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
+  if (threadIdx.x == 0) {
+    for (int i = 0; i < kQStages; ++i) {
+      mbar_init(q_full + 8 * i, 1);
+      mbar_init(q_empty + 8 * i, 1 + kSmWarps + 1);   // MMA + softmax warps + K/V producer
+      mbar_init(info_full + 8 * i, 1);
+    }
+    for (int i = 0; i < kKVStages; ++i) { mbar_init(kv_full + 8 * i, 1); mbar_init(kv_empty + 8 * i, 1); }
+    for (int i = 0; i < 2; ++i) {
+      mbar_init(s_full + 8 * i, 1);
+      mbar_init(s_empty + 8 * i, kSmWarps);
+      mbar_init(p_full + 8 * i, kSmWarps);
+      mbar_init(p_empty + 8 * i, 1);
+    }
+    for (int i = 0; i < 2; ++i) { mbar_init(o_full + 8 * i, 1); mbar_init(o_empty + 8 * i, kSmWarps); }
+    asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
+  }
+  if (warp == 2) {
+    asm volatile("tcgen05.alloc.cta_group::1.sync.aligned.shared::cta.b32 [%0], %1;" ::"r"(
+                     smem_u32(tmem_slot)), "r"(512) : "memory");
+    asm volatile("tcgen05.relinquish_alloc_permit.cta_group::1.sync.aligned;" ::: "memory");
+  }
+  tc_fence_before();
+  __syncthreads();
+  tc_fence_after();
+  const uint32_t tmem = *tmem_slot;           // S0: +0, S1: +128, O: +256
+
+  if (warp == 0) {
+    // ================= item metadata + Q tile =================
+    if (lane == 0) asm volatile("prefetch.tensormap [%0];" ::"l"(reinterpret_cast<uint64_t>(&tmQKV)) : "memory");
+    int qs = 0;
+    uint32_t qph = 0;
+    for (int item = blockIdx.x; item < num_items; item += gridDim.x) {
+      const int qb = item / num_heads, h = item % num_heads;
+      const int64_t q0 = static_cast<int64_t>(qb) * TQ;
+      if (lane == 0) mbar_wait(q_empty + 8 * qs, qph ^ 1);
+      __syncwarp();
+      ItemInfo* inf = infos + qs;
+      compute_info(inf, seg_ids, segtab, q0, num_slots, lane);
+      if (lane == 0) {
+        mbar_arrive(info_full + 8 * qs);
+        if (inf->nch == 0) {
+          mbar_arrive(q_full + 8 * qs);
+        } else {
+          mbar_expect_tx(q_full + 8 * qs, kTileBytes);
+          tma_load(sQ + qs * kTileBytes, &tmQKV, q_full + 8 * qs, h * DH, static_cast<int>(q0));
+        }
+      }
+      if (++qs == kQStages) { qs = 0; qph ^= 1; }
+    }
+  } else if (warp == 2) {
+    // ================= K/V chunks =================
+    if (lane == 0) {
+      int qs = 0, ks = 0;
+      uint32_t qph = 0, kph = 0;
+      for (int item = blockIdx.x; item < num_items; item += gridDim.x) {
+        const int h = item % num_heads;
+        mbar_wait(info_full + 8 * qs, qph);
+        const int kbase = infos[qs].kbase, nch = infos[qs].nch;
+        mbar_arrive(q_empty + 8 * qs);
+        if (++qs == kQStages) { qs = 0; qph ^= 1; }
+        for (int c = 0; c < nch; ++c) {
+          mbar_wait(kv_empty + 8 * ks, kph ^ 1);
+          mbar_expect_tx(kv_full + 8 * ks, 2 * kTileBytes);
+          tma_load(sK + ks * kTileBytes, &tmQKV, kv_full + 8 * ks, d_model + h * DH, kbase + c * TK);
+          tma_load(sV + ks * kTileBytes, &tmQKV, kv_full + 8 * ks, 2 * d_model + h * DH, kbase + c * TK);
+          if (++ks == kKVStages) { ks = 0; kph ^= 1; }
+        }
+      }
+    }
+  } else if (warp == 1) {
+    // ================= MMA issuer =================
+    int qs = 0, ks = 0, ks_prev = 0;
+    uint32_t qph = 0, kph = 0;
+    uint32_t gc = 0;            // global chunk counter (S / P double buffers)
+    uint32_t it = 0;            // items with at least one chunk (O reuse)
+    for (int item = blockIdx.x; item < num_items; item += gridDim.x) {
+      mbar_wait(q_full + 8 * qs, qph);
+      const int nch = infos[qs].nch;
+      const uint32_t qaddr = sQ + qs * kTileBytes;
+      tc_fence_after();
+      auto pv = [&](uint32_t c_glob, int stage, bool first) {
+        const uint32_t b = c_glob & 1, u = c_glob >> 1;
+        mbar_wait(p_full + 8 * b, u & 1);
+        if (first) mbar_wait(o_empty + 8 * (it & 1), ((it >> 1) & 1) ^ 1);
+        tc_fence_after();
+        if (lane == 0) {
+          const uint32_t pa = sP + b * kPBytes, va = sV + stage * kTileBytes;
+#pragma unroll
+          for (int k = 0; k < TK / 16; ++k) {
+            const uint32_t a_addr = pa + (k >> 2) * kTileBytes + (k & 3) * 32;
+            tc_mma(tmem + 256 + (it & 1) * 64, desc_kmajor(a_addr), desc_mnmajor(va + k * 2048), kIdescPV,
+                   (!first || k > 0) ? 1u : 0u);
+          }
+          tc_commit(p_empty + 8 * b);
+          tc_commit(kv_empty + 8 * stage);
+        }
+        __syncwarp();
+      };
+      for (int c = 0; c < nch; ++c) {
+        const uint32_t b = gc & 1, u = gc >> 1;
+        mbar_wait(kv_full + 8 * ks, kph);
+        mbar_wait(s_empty + 8 * b, (u & 1) ^ 1);
+        tc_fence_after();
+        if (lane == 0) {
+          const uint32_t ka = sK + ks * kTileBytes;
+#pragma unroll
+          for (int k = 0; k < DH / 16; ++k)
+            tc_mma(tmem + b * 128, desc_kmajor(qaddr + k * 32), desc_kmajor(ka + k * 32), kIdescQK,
+                   k > 0 ? 1u : 0u);
+          tc_commit(s_full + 8 * b);
+          if (c == nch - 1) tc_commit(q_empty + 8 * qs);
+        }
+        __syncwarp();
+        if (c > 0) pv(gc - 1, ks_prev, c == 1);
+        ks_prev = ks;
+        if (++ks == kKVStages) { ks = 0; kph ^= 1; }
+        ++gc;
+      }
+      if (nch > 0) {
+        pv(gc - 1, ks_prev, nch == 1);
+        if (lane == 0) tc_commit(o_full + 8 * (it & 1));
+        __syncwarp();
+        ++it;
+      } else if (lane == 0) {
+        mbar_arrive(q_empty + 8 * qs);
+      }
+      if (++qs == kQStages) { qs = 0; qph ^= 1; }
+    }
+  } else if (warp >= 4) {
+    // ================= softmax + epilogue =================
+    const int sw = warp - 4;
+    const int q = warp & 3;                 // TMEM lane quarter
+    const int half = sw >> 2;               // key columns [64*half, 64*half+64) of a chunk
+    const int row = q * 32 + lane;
+    const uint32_t lane_off = static_cast<uint32_t>(q * 32) << 16;
+    int qs = 0;
+    uint32_t qph = 0, gc = 0, it = 0;
+#ifdef TCB_ATTN_PROBE
+    long long p_start = clock64(), p_sfull = 0, p_ld = 0, p_max = 0, p_pempty = 0, p_exp = 0, p_q = 0, p_fin = 0;
+#endif
+    // deferred epilogue state (previous item)
+    bool have_prev = false, p_real = false;
+    int p_qb = 0, p_h = 0, p_nch = 0;
+    float p_l = 0.f;
+    uint32_t p_it = 0;
+    auto finish = [&]() {
+      // ---- epilogue: O / l -> bf16 -> global (pad / empty rows -> 0) ----
+      const int64_t grow = static_cast<int64_t>(p_qb) * TQ + row;
+      float* xl = xch + 4 * TQ;              // separate from the per-chunk max exchange
+      xl[half * TQ + row] = p_l;
+      named_bar(1 + q, 64);
+      const float lt = xl[row] + xl[TQ + row];
+      named_bar(1 + q, 64);
+      uint32_t o[32];
+      if (p_nch > 0) {
+        const uint32_t os = p_it & 1;
+        mbar_wait(o_full + 8 * os, (p_it >> 1) & 1);
+        tc_fence_after();
+        tmem_ld32(tmem + lane_off + 256 + os * 64 + half * 32, o);
+        tmem_wait_ld();
+        tc_fence_before();
+        __syncwarp();
+        if (lane == 0) mbar_arrive(o_empty + 8 * os);
+      }
+      const float inv = (p_nch > 0 && p_real && lt > 0.f) ? 1.f / lt : 0.f;
+      if (grow < num_slots) {
+        uint4* dst = reinterpret_cast<uint4*>(O + grow * d_model + p_h * DH + half * 32);
+#pragma unroll
+        for (int t = 0; t < 4; ++t) {
+          uint4 x;
+          uint32_t* xp = reinterpret_cast<uint32_t*>(&x);
+#pragma unroll
+          for (int e = 0; e < 4; ++e) {
+            const int j = 8 * t + 2 * e;
+            const float a = inv == 0.f ? 0.f : __uint_as_float(o[j]) * inv;
+            const float bq = inv == 0.f ? 0.f : __uint_as_float(o[j + 1]) * inv;
+            __nv_bfloat162 hv = __floats2bfloat162_rn(a, bq);
+            xp[e] = *reinterpret_cast<uint32_t*>(&hv);
+          }
+          dst[t] = x;
+        }
+      }
+    };
+    for (int item = blockIdx.x; item < num_items; item += gridDim.x) {
+      const int qb = item / num_heads, h = item % num_heads;
+#ifdef TCB_ATTN_PROBE
+      long long tq = clock64();
+#endif
+      mbar_wait(q_full + 8 * qs, qph);
+#ifdef TCB_ATTN_PROBE
+      p_q += clock64() - tq;
+#endif
+      const ItemInfo* inf = infos + qs;
+      const int2 rr = inf->rows[row];
+      const int kbase = inf->kbase, nch = inf->nch;
+      __syncwarp();
+      if (lane == 0) mbar_arrive(q_empty + 8 * qs);   // metadata copied to registers
+      if (++qs == kQStages) { qs = 0; qph ^= 1; }
+      // key interval of this warp's 32 rows: union [ulo, uhi) and intersection [ilo, ihi)
+      // (a pad row empties the intersection)
+      const bool real = rr.y > rr.x;
+      int ulo = real ? rr.x : INT_MAX, uhi = real ? rr.y : -1;
+      int ilo = real ? rr.x : INT_MAX, ihi = real ? rr.y : -1;
+#pragma unroll
+      for (int o = 16; o > 0; o >>= 1) {
+        ulo = min(ulo, __shfl_xor_sync(0xffffffffu, ulo, o));
+        uhi = max(uhi, __shfl_xor_sync(0xffffffffu, uhi, o));
+        ilo = max(ilo, __shfl_xor_sync(0xffffffffu, ilo, o));
+        ihi = min(ihi, __shfl_xor_sync(0xffffffffu, ihi, o));
+      }
+      float m_used = -INFINITY, l = 0.f;
+      for (int c = 0; c < nch; ++c) {
+        const uint32_t b = gc & 1, u = gc >> 1;
+#ifdef TCB_ATTN_PROBE
+        long long t0 = clock64();
+#endif
+        mbar_wait(s_full + 8 * b, u & 1);
+#ifdef TCB_ATTN_PROBE
+        long long t1 = clock64();
+        p_sfull += t1 - t0;
+#endif
+        tc_fence_after();
+        uint32_t sr[64];
+        tmem_ld32(tmem + lane_off + b * 128 + half * 64, *reinterpret_cast<uint32_t(*)[32]>(&sr[0]));
+        tmem_ld32(tmem + lane_off + b * 128 + half * 64 + 32, *reinterpret_cast<uint32_t(*)[32]>(&sr[32]));
+        tmem_wait_ld();
+        tc_fence_before();
+        __syncwarp();
+        if (lane == 0) mbar_arrive(s_empty + 8 * b);
+#ifdef TCB_ATTN_PROBE
+        long long t2 = clock64();
+        p_ld += t2 - t1;
+#endif
+        // 32-key groups of this warp's half: dead (no key of any of its rows' requests:
+        // skipped, P = 0), interior (inside every row's request: no mask) or boundary
+        // (masked per element: key outside the row's own request -> -inf, R11)
+        const int k0 = kbase + c * TK + 64 * half;
+        const int jlo = max(rr.x - k0, 0), jhi = min(rr.y - k0, 64);
+        bool live[2], inner[2];
+#pragma unroll
+        for (int gi = 0; gi < 2; ++gi) {
+          const int gk = k0 + 32 * gi;
+          live[gi] = gk < uhi && gk + 32 > ulo;
+          inner[gi] = gk >= ilo && gk + 32 <= ihi;
+        }
+        // row max with 8 independent partial maxima (short dependency chains)
+        float mxp[8];
+#pragma unroll
+        for (int t = 0; t < 8; ++t) mxp[t] = -INFINITY;
+#pragma unroll
+        for (int gi = 0; gi < 2; ++gi) {
+          if (!live[gi]) continue;
+          if (inner[gi]) {
+#pragma unroll
+            for (int j = 32 * gi; j < 32 * gi + 32; ++j) mxp[j & 7] = fmaxf(mxp[j & 7], __uint_as_float(sr[j]));
+          } else {
+#pragma unroll
+            for (int j = 32 * gi; j < 32 * gi + 32; ++j) {
+              const float v = (j >= jlo && j < jhi) ? __uint_as_float(sr[j]) : -INFINITY;
+              sr[j] = __float_as_uint(v);
+              mxp[j & 7] = fmaxf(mxp[j & 7], v);
+            }
+          }
+        }
+        const float mx = fmaxf(fmaxf(fmaxf(mxp[0], mxp[1]), fmaxf(mxp[2], mxp[3])),
+                               fmaxf(fmaxf(mxp[4], mxp[5]), fmaxf(mxp[6], mxp[7])));
+        // row max across the two column halves (double-buffered exchange: one barrier)
+        float* xb = xch + (gc & 1) * 2 * TQ;
+        xb[half * TQ + row] = mx;
+        named_bar(1 + q, 64);
+        const float rmax = fmaxf(xb[row], xb[TQ + row]);
+#ifdef TCB_ATTN_PROBE
+        long long t3 = clock64();
+        p_max += t3 - t2;
+#endif
+        // lazy rescale: a row moves its max only when it grew by more than 2^8.  The O
+        // update uses warp-collective tcgen05.ld/st, so the decision is made per warp (any
+        // lane) and lanes that keep their max scale by 1.
+        bool grow = false;
+        if (rmax != -INFINITY) {
+          if (m_used == -INFINITY) m_used = rmax;   // nothing accumulated yet for this row
+          else grow = (rmax - m_used) * scale_log2 > kRescaleLog2;
+        }
+        if (__any_sync(0xffffffffu, grow)) {
+          // O must be current before it is rescaled: wait for P V of chunk c-1
+          const uint32_t pb = (gc - 1) & 1, pu = (gc - 1) >> 1;
+          mbar_wait(p_empty + 8 * pb, pu & 1);
+          tc_fence_after();
+          const float f = grow ? ex2((m_used - rmax) * scale_log2) : 1.f;
+          uint32_t o[32];
+          const uint32_t oaddr = tmem + lane_off + 256 + (it & 1) * 64 + half * 32;
+          tmem_ld32(oaddr, o);
+          tmem_wait_ld();
+#pragma unroll
+          for (int t = 0; t < 32; ++t) o[t] = __float_as_uint(__uint_as_float(o[t]) * f);
+          tmem_st32(oaddr, o);
+          asm volatile("tcgen05.wait::st.sync.aligned;" ::: "memory");
+          if (grow) {
+            l *= f;
+            m_used = rmax;
+          }
+        }
+        const float off = m_used == -INFINITY ? 0.f : -m_used * scale_log2;
+#ifdef TCB_ATTN_PROBE
+        long long t4 = clock64();
+#endif
+        // P buffer b is free once P V of chunk gc-2 is done
+        if (gc >= 2) mbar_wait(p_empty + 8 * b, (u & 1) ^ 1);
+#ifdef TCB_ATTN_PROBE
+        long long t5 = clock64();
+        p_pempty += t5 - t4;
+#endif
+        const uint32_t prow = sP + b * kPBytes + half * kTileBytes + row * 128;
+        float lp[4] = {0.f, 0.f, 0.f, 0.f};    // independent partial row sums
+#pragma unroll
+        for (int cch = 0; cch < 8; ++cch) {
+          uint32_t w4[4] = {0u, 0u, 0u, 0u};
+          if (live[cch >> 2]) {
+#pragma unroll
+            for (int e = 0; e < 4; ++e) {
+              const int j = cch * 8 + 2 * e;
+              // masked scores are -inf: 2^-inf = 0 exactly
+              const float p0 = ex2(fmaf(__uint_as_float(sr[j]), scale_log2, off));
+              const float p1 = ex2(fmaf(__uint_as_float(sr[j + 1]), scale_log2, off));
+              lp[e] += p0 + p1;
+              __nv_bfloat162 hv = __floats2bfloat162_rn(p0, p1);
+              w4[e] = *reinterpret_cast<uint32_t*>(&hv);
+            }
+          }
+          const uint32_t addr = prow + ((cch ^ (row & 7)) << 4);
+          asm volatile("st.shared.v4.b32 [%0], {%1, %2, %3, %4};" ::"r"(addr), "r"(w4[0]),
+                       "r"(w4[1]), "r"(w4[2]), "r"(w4[3])
+                       : "memory");
+        }
+        l += (lp[0] + lp[1]) + (lp[2] + lp[3]);
+#ifdef TCB_ATTN_PROBE
+        p_exp += clock64() - t5;
+#endif
+        asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
+        tc_fence_before();
+        __syncwarp();
+        if (lane == 0) mbar_arrive(p_full + 8 * b);
+        ++gc;
+      }
+      // the epilogue of the PREVIOUS item runs now, while the MMAs of this item's last chunk
+      // (and the next item's first) proceed -- O is double-buffered in TMEM
+#ifdef TCB_ATTN_PROBE
+      long long tf0 = clock64();
+#endif
+      if (have_prev) finish();
+#ifdef TCB_ATTN_PROBE
+      p_fin += clock64() - tf0;
+#endif
+      have_prev = true;
+      p_qb = qb;
+      p_h = h;
+      p_nch = nch;
+      p_real = rr.y > rr.x;
+      p_l = l;
+      p_it = it;
+      if (nch > 0) ++it;
+    }
+    if (have_prev) finish();
+#ifdef TCB_ATTN_PROBE
+    if (lane == 0 && blockIdx.x == 0 && (sw == 0 || sw == 5))
+      printf("tcprobe warp %d total %lld wait_q %lld wait_s %lld tmem_ld %lld max %lld wait_p %lld exp %lld finish %lld chunks %u\n",
+             warp, clock64() - p_start, p_q, p_sfull, p_ld, p_max, p_pempty, p_exp, p_fin, gc);
+#endif
+  }
+  __syncwarp();
+  tc_fence_before();
+  __syncthreads();
+  tc_fence_after();
+  if (warp == 2)
+    asm volatile("tcgen05.dealloc.cta_group::1.sync.aligned.b32 %0, %1;" ::"r"(tmem), "r"(512) : "memory");
+}
+
+}  // namespace
+
+cudaError_t launch_attention_bf16_tc(int64_t num_slots, int d_model, int num_heads,
+                                     const void* qkv, const int32_t* seg_ids,
+                                     const int4* segtab, void* O, cudaStream_t s) {
+  if (num_slots == 0) return cudaSuccess;
+  static bool attr = false;
+  static int sms = 0;
+  if (!attr) {
+    cudaError_t e = cudaFuncSetAttribute(attn_tc_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize,
+                                         kSmemBytes);
+    if (e != cudaSuccess) return e;
+    int dev = 0;
+    cudaGetDevice(&dev);
+    cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev);
+    attr = true;
+  }
+  CUtensorMap map;
+  if (!make_tmap_bf16(&map, qkv, static_cast<uint64_t>(num_slots), 3ull * d_model, 128, 64, 128))
+    return cudaErrorInvalidValue;
+  const int64_t qblocks = (num_slots + TQ - 1) / TQ;
+  const int items = static_cast<int>(qblocks * num_heads);
+  const unsigned grid = static_cast<unsigned>(items < sms ? items : sms);
+  const float scale_log2 = 1.4426950408889634f / sqrtf(static_cast<float>(DH));
+  attn_tc_kernel<<<grid, kThreads, kSmemBytes, s>>>(map, seg_ids, segtab,
+                                                    static_cast<__nv_bfloat16*>(O), num_slots,
+                                                    d_model, num_heads, items, scale_log2);
+  return cudaGetLastError();
+}
+
+}  // namespace k
+}  // namespace tcb

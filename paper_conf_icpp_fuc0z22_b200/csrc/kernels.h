@@ -69,6 +69,10 @@ cudaError_t launch_linear_ln_bf16_tc(const GemmMaps& maps, int64_t M, int N, int
 cudaError_t launch_attention_bf16(int64_t num_slots, int d_model, int num_heads,
                                   const void* qkv, const int32_t* seg_ids, const int4* segtab,
                                   void* O, cudaStream_t s);
+// tcgen05 variant (attention_tc.cu): S and O in TMEM, 128-query x 128-key chunks.
+cudaError_t launch_attention_bf16_tc(int64_t num_slots, int d_model, int num_heads,
+                                     const void* qkv, const int32_t* seg_ids, const int4* segtab,
+                                     void* O, cudaStream_t s);
 cudaError_t launch_attention_f32(int64_t num_slots, int d_model, int num_heads,
                                  const float* qkv, const int32_t* seg_ids, const int4* segtab,
                                  float* O, cudaStream_t s);

@@ -1,6 +1,6 @@
 cd $GRAFT_REPO_ROOT
 sed -i 's/FLAGS = \["-O3"/FLAGS = ["-DTCB_GEMM_PROBE", "-O3"/' paper_conf_icpp_fuc0z22_b200/_build.py
-python paper_conf_icpp_fuc0z22_b200/_build.py > /dev/null
+python -c "import sys; sys.path.insert(0,'paper_conf_icpp_fuc0z22_b200'); import _build; _build.build(force=True)" > /dev/null
 python - <<'PY'
 import sys; sys.path.insert(0,'.')
 import torch, paper_conf_icpp_fuc0z22_b200 as tcb

@@ -146,6 +146,34 @@ def test_attention_bf16_single_long_request_and_tail():
     assert np.all(got[~real] == 0)
 
 
+def test_attention_bf16_running_max_rescale():
+    """Scores that grow along the key axis force the online softmax to move its running
+    maximum across 128-key chunks (the lazy O-rescale path) -- with a mix of rows that do
+    and do not rescale inside the same warp."""
+    rng = np.random.default_rng(17)
+    lengths = np.array([500, 300, 200, 12], np.int32)
+    L, d, h = 512, 128, 2
+    plan = tcb.tcb_pack(lengths, L, 0)
+    arr = plan.arrays()
+    M = plan.num_slots
+    qkv = rng.normal(size=(M, 3 * d)).astype(np.float32)
+    pos = np.maximum(arr["positions"], 0).astype(np.float32)
+    qkv[:, :d] *= 2.0
+    qkv[:, d:2 * d] *= (1.0 + pos / 40.0)[:, None]      # key norms grow with position
+    qkv[::3, :d] *= 0.05                                 # some rows never rescale
+    qkv = _bf16(qkv)
+    out = tcb.op_attention(_dev(qkv, torch.bfloat16), _dev(arr["segment_ids"]),
+                           _dev(plan.segtab()), h)
+    torch.cuda.synchronize()
+    got = out.float().cpu().numpy()
+    ref = oracle.attention(qkv, arr["segment_ids"], plan.info["num_rows"], L, d, h)
+    seg = arr["segment_ids"]
+    for s_ in np.unique(seg[seg >= 0]):
+        rows = seg == s_
+        e = np.max(np.abs(got[rows] - ref[rows])) / np.max(np.abs(ref[rows]))
+        assert e <= 2e-2, (s_, e)
+
+
 def test_attention_f32_vs_oracle():
     lengths = wl.draw_lengths("uniform_3_16", 8, 0)
     got, ref, seg = _attn_case(lengths, 32, 64, 2, "fp32", 2)
