@@ -524,24 +524,29 @@ linear_tc_kernel(const __grid_constant__ CUtensorMap tmA, const __grid_constant_
 
 // ---- GEMM + bias + residual + LayerNorm, fused (row width N = 512) -----------------------
 // Post-LN (R10): Y = LN(A W^T + b + R) * gamma + beta.  One 2-CTA pair owns a 256-row x
-// 512-column tile: per k-block each CTA loads its 128 rows of A once and both 128-row halves
-// of W (n-blocks 0 and 1), and the even CTA issues two M=256, N=256 MMAs into two TMEM
-// accumulators (all 512 columns).  The epilogue then holds complete rows: pass 1 adds bias
-// and the (TMA-prefetched) residual, writes z back to TMEM and accumulates the row moments
-// sum(z), sum(z^2); pass 2 normalises, rounds to bf16 and TMA-stores.  16 epilogue warps
-// (4 per TMEM lane quarter, 128 columns each) combine their row partials through shared
-// memory under a 128-thread named barrier.  Pad slots (segment id < 0) are written as 0
-// (R12).
+// 512-column tile, i.e. complete rows: two M=256, N=256 accumulators fill all 512 TMEM
+// columns.  The MMAs of a tile run in two N-halves (all k-blocks of half 0, then of half 1),
+// each with its own TMEM full/empty barrier, so the epilogue overlaps the tensor cores:
+//   MMA(h0) | MMA(h1) || pass 1 on h0 | pass 1 on h1, row moments, pass 2 on h0 -> release
+//   h0 | MMA(next h0) || pass 2 on h1 -> release h1 | MMA(next h1) || pass 1 on next h0 ...
+// pass 1: z = acc + bias + residual (TMA-prefetched) -> TMEM, row moments sum z, sum z^2;
+// pass 2: (z - mean) * rstd * gamma + beta -> bf16 -> TMA store.  16 epilogue warps (4 per
+// TMEM lane quarter, 64 columns of each half) combine row partials through shared memory
+// under a 128-thread named barrier.  Pad slots (segment id < 0) are written as 0 (R12).
 constexpr int kLnN = 512;
 constexpr int kLnEpiWarps = 16;                                      // 4 per TMEM lane quarter
 constexpr int kLnThreads = (4 + kLnEpiWarps) * 32;
-constexpr int kLnChunks = kLnN / 4 / 32;                             // 32-col chunks per warp
-constexpr int kLnStageBytes = 3 * 128 * BK * 2;                     // A + 2 W halves: 48 KB
 constexpr int kLnEpiBytes = kLnEpiWarps * 2 * kStageBufBytes;        // 64 KB
-constexpr int kLnStages = (227 * 1024 - 1024 - kLnEpiBytes - 4096) / kLnStageBytes;  // 3
-constexpr int kLnSmemBytes = 1024 + kLnStages * kLnStageBytes + kLnEpiBytes +
-                             8 * (2 * kLnStages + 2 + 2 * kLnEpiWarps) + 16 + 2 * 4 * 128 * 4;
-static_assert(kLnSmemBytes <= 232448, "shared memory budget");
+// JOINT stages hold A + both W halves (48 KB, 3 stages; short split for long K); split stages
+// hold A + one W half (32 KB, 4 stages; every step is single-half, for short K).
+template <bool JOINT>
+struct LnCfg {
+  static constexpr int kStageBytes = (JOINT ? 3 : 2) * 128 * BK * 2;
+  static constexpr int kStages = (227 * 1024 - 1024 - kLnEpiBytes - 4096) / kStageBytes;
+  static constexpr int kSmemBytes = 1024 + kStages * kStageBytes + kLnEpiBytes +
+                                    8 * (2 * kStages + 4 + 2 * kLnEpiWarps) + 16 + 2 * 4 * 128 * 4;
+  static_assert(kSmemBytes <= 232448, "shared memory budget");
+};
 
 __device__ __forceinline__ void tmem_st32(uint32_t taddr, const float (&v)[32]) {
   asm volatile(
@@ -558,24 +563,45 @@ __device__ __forceinline__ void tmem_st32(uint32_t taddr, const float (&v)[32]) 
 __device__ __forceinline__ void named_bar(int id, int threads) {
   asm volatile("bar.sync %0, %1;" ::"r"(id), "r"(threads) : "memory");
 }
+__device__ __forceinline__ void tma_load_res(uint32_t dst, const CUtensorMap* map, uint64_t* bar,
+                                             int c0, int c1) {
+  asm volatile(
+      "cp.async.bulk.tensor.2d.shared::cluster.global.mbarrier::complete_tx::bytes"
+      " [%0], [%1, {%3, %4}], [%2];" ::"r"(dst),
+      "l"(reinterpret_cast<uint64_t>(map)), "r"(smem_u32(bar)), "r"(c0), "r"(c1)
+      : "memory");
+}
 
+// Step order of one tile: half 0 alone on k-blocks [0, j), both halves on [j, K/BK), then
+// half 1 alone on [0, j).  Accumulator 0 completes j steps before accumulator 1 (pass 1 of
+// its epilogue overlaps them), and the first j steps of the next tile need only accumulator
+// 0 (they overlap pass 2 of accumulator 1).  The price is re-reading A for j k-blocks.
+__device__ __forceinline__ void ln_step(int step, int nkb, int j, int& kb, int& mask) {
+  if (step < j) { kb = step; mask = 1; }
+  else if (step < nkb) { kb = step; mask = 3; }
+  else { kb = step - nkb; mask = 2; }
+}
+
+template <bool JOINT>
 __global__ void __launch_bounds__(kLnThreads, 1)
 linear_ln_kernel(const __grid_constant__ CUtensorMap tmA, const __grid_constant__ CUtensorMap tmW,
                  const __grid_constant__ CUtensorMap tmC, const __grid_constant__ CUtensorMap tmR,
                  int M, int K, const float* __restrict__ bias, const float* __restrict__ gamma,
-                 const float* __restrict__ beta, float eps, const int32_t* __restrict__ seg_ids) {
-  constexpr int S = kLnStages;
+                 const float* __restrict__ beta, float eps, const int32_t* __restrict__ seg_ids,
+                 int split_kb) {
+  constexpr int S = LnCfg<JOINT>::kStages;
+  constexpr int kLnStageBytes = LnCfg<JOINT>::kStageBytes;
   constexpr int kHalfBytes = 128 * BK * 2;
   extern __shared__ uint8_t smem_raw[];
   uint8_t* smem = reinterpret_cast<uint8_t*>((reinterpret_cast<uintptr_t>(smem_raw) + 1023) &
                                              ~static_cast<uintptr_t>(1023));
-  uint8_t* sStage = smem;                                   // S x {A, W half 0, W half 1}
+  uint8_t* sStage = smem;                                   // S x {A, W half}
   uint8_t* sEpi = smem + S * kLnStageBytes;                 // 16 warps x 2 x 2 KB
   uint64_t* full = reinterpret_cast<uint64_t*>(sEpi + kLnEpiBytes);
   uint64_t* empty = full + S;
-  uint64_t* tfull = empty + S;
-  uint64_t* tempty = tfull + 1;
-  uint64_t* rbar = tempty + 1;                              // [16 warps][2]
+  uint64_t* tfull = empty + S;                              // [2 halves]
+  uint64_t* tempty = tfull + 2;                             // [2 halves]
+  uint64_t* rbar = tempty + 2;                              // [16 warps][2]
   uint32_t* tmem_slot = reinterpret_cast<uint32_t*>(rbar + 2 * kLnEpiWarps);
   float* stats = reinterpret_cast<float*>(tmem_slot + 4);   // [4 parts][128 rows] x 2
 
@@ -584,13 +610,13 @@ linear_ln_kernel(const __grid_constant__ CUtensorMap tmA, const __grid_constant_
   const int cluster_id = blockIdx.x / 2, num_clusters = gridDim.x / 2;
   const int num_tiles = (M + 255) / 256;
   const int num_kb = K / BK;
+  const int num_steps = num_kb + split_kb;
 
   if (warp == 0 && lane == 0) {
     asm volatile("prefetch.tensormap [%0];" ::"l"(reinterpret_cast<uint64_t>(&tmA)) : "memory");
     asm volatile("prefetch.tensormap [%0];" ::"l"(reinterpret_cast<uint64_t>(&tmW)) : "memory");
     for (int i = 0; i < S; ++i) { mbar_init(&full[i], 1); mbar_init(&empty[i], 1); }
-    mbar_init(tfull, 1);
-    mbar_init(tempty, 2 * kLnEpiWarps);
+    for (int i = 0; i < 2; ++i) { mbar_init(&tfull[i], 1); mbar_init(&tempty[i], 2 * kLnEpiWarps); }
     for (int i = 0; i < 2 * kLnEpiWarps; ++i) mbar_init(&rbar[i], 1);
     asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
   }
@@ -605,80 +631,76 @@ linear_ln_kernel(const __grid_constant__ CUtensorMap tmA, const __grid_constant_
   const uint32_t tmem_base = *tmem_slot;
 
   if (warp == 0) {
-    // ===== TMA producer: A rows once, both W halves, per k-block =====
+    // ===== TMA producer: A rows + the W half (or both halves) each step needs =====
     if (lane == 0) {
       const uint32_t full0 = map_to_rank0(smem_u32(full));
       int stage = 0;
       uint32_t phase = 0;
       for (int tile = cluster_id; tile < num_tiles; tile += num_clusters) {
         const int a_row = tile * 256 + static_cast<int>(rank) * 128;
-        for (int kb = 0; kb < num_kb; ++kb) {
+        for (int step = 0; step < num_steps; ++step) {
+          int kb, mask;
+          ln_step(step, num_kb, split_kb, kb, mask);
           mbar_wait(&empty[stage], phase ^ 1);
-          if (rank == 0) mbar_expect_tx(&full[stage], 2 * kLnStageBytes);
+          if (rank == 0)
+            mbar_expect_tx(&full[stage], 2 * kHalfBytes * (1 + (mask & 1) + (mask >> 1)));
           const uint32_t fb = full0 + 8u * stage;
           uint8_t* st = sStage + stage * kLnStageBytes;
           tma_load_2d<2>(st, &tmA, fb, kb * BK, a_row);
-          tma_load_2d<2>(st + kHalfBytes, &tmW, fb, kb * BK, static_cast<int>(rank) * 128);
-          tma_load_2d<2>(st + 2 * kHalfBytes, &tmW, fb, kb * BK, 256 + static_cast<int>(rank) * 128);
+#pragma unroll
+          for (int h = 0; h < 2; ++h)
+            if (mask & (1 << h))
+              tma_load_2d<2>(st + (1 + (mask == 3 ? h : 0)) * kHalfBytes, &tmW, fb, kb * BK,
+                             h * 256 + static_cast<int>(rank) * 128);
           if (++stage == S) { stage = 0; phase ^= 1; }
         }
       }
     }
   } else if (warp == 1) {
-    // ===== MMA issuer (even CTA): two N=256 halves per k-step =====
+    // ===== MMA issuer (even CTA) =====
     if (rank == 0) {
       constexpr uint32_t idesc = idesc_bf16<2, 256>();
       int stage = 0;
       uint32_t phase = 0, tphase = 0;
-#ifdef TCB_GEMM_PROBE
-      long long t_start = clock64(), t_full = 0, t_empty = 0;
-#endif
       for (int tile = cluster_id; tile < num_tiles; tile += num_clusters) {
-#ifdef TCB_GEMM_PROBE
-        long long t0 = clock64();
-#endif
-        mbar_wait(tempty, tphase ^ 1);
-#ifdef TCB_GEMM_PROBE
-        t_empty += clock64() - t0;
-#endif
-        tc_fence_after();
-        for (int kb = 0; kb < num_kb; ++kb) {
-#ifdef TCB_GEMM_PROBE
-          long long t1 = clock64();
-#endif
+        int done[2] = {0, 0};                   // k-blocks accumulated per half
+        for (int step = 0; step < num_steps; ++step) {
+          int kb, mask;
+          ln_step(step, num_kb, split_kb, kb, mask);
+#pragma unroll
+          for (int h = 0; h < 2; ++h)
+            if ((mask & (1 << h)) && done[h] == 0) mbar_wait(&tempty[h], tphase ^ 1);
           mbar_wait(&full[stage], phase);
-#ifdef TCB_GEMM_PROBE
-          t_full += clock64() - t1;
-#endif
           tc_fence_after();
           if (lane == 0) {
             const uint32_t a0 = smem_u32(sStage + stage * kLnStageBytes);
-            const uint32_t b0 = a0 + kHalfBytes, b1 = a0 + 2 * kHalfBytes;
 #pragma unroll
-            for (int k = 0; k < BK / 16; ++k) {
-              const uint64_t ad = sdesc_sw128(a0 + k * 32);
-              tc_mma<2>(tmem_base, ad, sdesc_sw128(b0 + k * 32), idesc, (kb | k) != 0 ? 1u : 0u);
-              tc_mma<2>(tmem_base + 256, ad, sdesc_sw128(b1 + k * 32), idesc, (kb | k) != 0 ? 1u : 0u);
+            for (int h = 0; h < 2; ++h) {
+              if (!(mask & (1 << h))) continue;
+              const uint32_t b0 = a0 + (1 + (mask == 3 ? h : 0)) * kHalfBytes;
+#pragma unroll
+              for (int k = 0; k < BK / 16; ++k)
+                tc_mma<2>(tmem_base + h * 256, sdesc_sw128(a0 + k * 32), sdesc_sw128(b0 + k * 32),
+                          idesc, (done[h] | k) != 0 ? 1u : 0u);
             }
             tc_commit<2>(&empty[stage]);
-            if (kb == num_kb - 1) tc_commit<2>(tfull);
           }
+#pragma unroll
+          for (int h = 0; h < 2; ++h)
+            if (mask & (1 << h)) {
+              if (++done[h] == num_kb && lane == 0) tc_commit<2>(&tfull[h]);
+            }
           __syncwarp();
           if (++stage == S) { stage = 0; phase ^= 1; }
         }
         tphase ^= 1;
       }
-#ifdef TCB_GEMM_PROBE
-      if (lane == 0 && blockIdx.x < 4)
-        printf("lnprobe mma cta %d total %lld wait_full %lld wait_tempty %lld\n", blockIdx.x,
-               clock64() - t_start, t_full, t_empty);
-#endif
     }
   } else if (warp >= 4) {
     // ===== Epilogue: bias + residual + LayerNorm over complete 512-column rows =====
     const int ew = warp - 4;
     const int q = warp & 3;                       // TMEM lane quarter (rows 32q..32q+31)
-    const int part = ew >> 2;                     // 128-column quarter of the row
+    const int part = ew >> 2;                     // 64-column part of each 256-column half
     const uint32_t bufs = smem_u32(sEpi) + ew * 2 * kStageBufBytes;
     uint64_t* my_rbar = rbar + 2 * ew;
     uint32_t rph = 0;                             // bit b: phase of residual barrier b
@@ -687,45 +709,38 @@ linear_ln_kernel(const __grid_constant__ CUtensorMap tmA, const __grid_constant_
     float* stat2 = stats + 512;
     const int srow = q * 32 + lane;               // row within this CTA's 128
     uint32_t tphase = 0;
+    // chunk j (0..3): half j>>1, columns h*256 + part*64 + (j&1)*32
+    auto col_of = [&](int j) { return (j >> 1) * 256 + part * 64 + (j & 1) * 32; };
     for (int tile = cluster_id; tile < num_tiles; tile += num_clusters) {
       const int row0 = tile * 256 + static_cast<int>(rank) * 128 + q * 32;
       const int64_t grow = static_cast<int64_t>(row0) + lane;
       const bool pad = grow >= M || (seg_ids && __ldg(&seg_ids[grow]) < 0);
-      const int col0 = part * (kLnN / 4);
       if (lane == 0) bulk_wait_read<0>();         // previous tile's stores have read the buffers
       __syncwarp();
       if (lane == 0) {
 #pragma unroll
         for (int j = 0; j < 2; ++j) {
           mbar_expect_tx(&my_rbar[j], kStageBufBytes);
-          asm volatile(
-              "cp.async.bulk.tensor.2d.shared::cluster.global.mbarrier::complete_tx::bytes"
-              " [%0], [%1, {%3, %4}], [%2];" ::"r"(bufs + j * kStageBufBytes),
-              "l"(reinterpret_cast<uint64_t>(&tmR)), "r"(smem_u32(&my_rbar[j])),
-              "r"(col0 + 32 * j), "r"(row0)
-              : "memory");
+          tma_load_res(bufs + j * kStageBufBytes, &tmR, &my_rbar[j], col_of(j), row0);
         }
       }
-#ifdef TCB_GEMM_PROBE
-      long long e0 = clock64();
-#endif
-      mbar_wait(tfull, tphase);
-#ifdef TCB_GEMM_PROBE
-      long long e1 = clock64();
-#endif
-      tc_fence_after();
-      const uint32_t tbase = tmem_base + (static_cast<uint32_t>(q * 32) << 16) + col0;
-      // pass 1: z = acc + bias + residual -> TMEM; row moments sum(z), sum(z^2)
+      // pass 1 on half 0 (overlaps the MMAs of half 1), then on half 1
       float sum = 0.f, sumsq = 0.f;
 #pragma unroll 1
-      for (int j = 0; j < kLnChunks; ++j) {
+      for (int j = 0; j < 4; ++j) {
+        if ((j & 1) == 0) {
+          mbar_wait(&tfull[j >> 1], tphase);
+          tc_fence_after();
+        }
         const int b = j & 1;
         const uint32_t buf = bufs + b * kStageBufBytes;
+        const int gc0 = col_of(j);
+        const uint32_t taddr = tmem_base + (static_cast<uint32_t>(q * 32) << 16) + gc0;
         uint32_t r[32];
-        tmem_ld32_nowait(tbase + 32 * j, r);
+        tmem_ld32_nowait(taddr, r);
         tmem_wait_ld();
         float* v = reinterpret_cast<float*>(r);
-        const float4* b4 = reinterpret_cast<const float4*>(bias + col0 + 32 * j);
+        const float4* b4 = reinterpret_cast<const float4*>(bias + gc0);
 #pragma unroll
         for (int t = 0; t < 8; ++t) {
           const float4 bb = __ldg(b4 + t);
@@ -752,16 +767,11 @@ linear_ln_kernel(const __grid_constant__ CUtensorMap tmA, const __grid_constant_
           sum += v[t];
           sumsq = fmaf(v[t], v[t], sumsq);
         }
-        tmem_st32(tbase + 32 * j, *reinterpret_cast<float(*)[32]>(v));
+        tmem_st32(taddr, *reinterpret_cast<float(*)[32]>(v));
         __syncwarp();                             // every lane has read buffer b
-        if (j + 2 < kLnChunks && lane == 0) {
+        if (j + 2 < 4 && lane == 0) {
           mbar_expect_tx(&my_rbar[b], kStageBufBytes);
-          asm volatile(
-              "cp.async.bulk.tensor.2d.shared::cluster.global.mbarrier::complete_tx::bytes"
-              " [%0], [%1, {%3, %4}], [%2];" ::"r"(buf),
-              "l"(reinterpret_cast<uint64_t>(&tmR)), "r"(smem_u32(&my_rbar[b])),
-              "r"(col0 + 32 * (j + 2)), "r"(row0)
-              : "memory");
+          tma_load_res(buf, &tmR, &my_rbar[b], col_of(j + 2), row0);
         }
       }
       asm volatile("tcgen05.wait::st.sync.aligned;" ::: "memory");
@@ -775,17 +785,24 @@ linear_ln_kernel(const __grid_constant__ CUtensorMap tmA, const __grid_constant_
       const float ex2m = (stat2[srow] + stat2[128 + srow] + stat2[256 + srow] + stat2[384 + srow]) *
                          (1.f / kLnN);
       const float rstd = rsqrtf(fmaxf(ex2m - mean * mean, 0.f) + eps);
-      // pass 2: normalise, bf16, TMA store
+      // pass 2: normalise, bf16, TMA store; each half is released to the MMA as soon as its
+      // last read is done
 #pragma unroll 1
-      for (int j = 0; j < kLnChunks; ++j) {
+      for (int j = 0; j < 4; ++j) {
         const int b = j & 1;
         const uint32_t buf = bufs + b * kStageBufBytes;
+        const int gc0 = col_of(j);
         uint32_t r[32];
-        tmem_ld32_nowait(tbase + 32 * j, r);
+        tmem_ld32_nowait(tmem_base + (static_cast<uint32_t>(q * 32) << 16) + gc0, r);
         tmem_wait_ld();
+        if (j & 1) {                              // half j>>1 fully read by this warp
+          tc_fence_before();
+          __syncwarp();
+          if (lane == 0) mbar_arrive_remote(tempty0 + 8u * (j >> 1));
+        }
         float* y = reinterpret_cast<float*>(r);
-        const float4* g4 = reinterpret_cast<const float4*>(gamma + col0 + 32 * j);
-        const float4* e4 = reinterpret_cast<const float4*>(beta + col0 + 32 * j);
+        const float4* g4 = reinterpret_cast<const float4*>(gamma + gc0);
+        const float4* e4 = reinterpret_cast<const float4*>(beta + gc0);
 #pragma unroll
         for (int t = 0; t < 8; ++t) {
           const float4 gg = __ldg(g4 + t), ee = __ldg(e4 + t);
@@ -794,10 +811,8 @@ linear_ln_kernel(const __grid_constant__ CUtensorMap tmA, const __grid_constant_
           y[4 * t + 2] = pad ? 0.f : (y[4 * t + 2] - mean) * rstd * gg.z + ee.z;
           y[4 * t + 3] = pad ? 0.f : (y[4 * t + 3] - mean) * rstd * gg.w + ee.w;
         }
-        if (j >= 2) {
-          if (lane == 0) bulk_wait_read<1>();     // the store that last used `buf` read it
-          __syncwarp();
-        }
+        if (lane == 0) bulk_wait_read<1>();       // the store that last used `buf` has read it
+        __syncwarp();
 #pragma unroll
         for (int t = 0; t < 4; ++t) {
           uint4 x;
@@ -812,20 +827,13 @@ linear_ln_kernel(const __grid_constant__ CUtensorMap tmA, const __grid_constant_
         if (lane == 0) {
           asm volatile("cp.async.bulk.tensor.2d.global.shared::cta.bulk_group [%0, {%2, %3}], [%1];" ::"l"(
                            reinterpret_cast<uint64_t>(&tmC)),
-                       "r"(buf), "r"(col0 + 32 * j), "r"(row0)
+                       "r"(buf), "r"(gc0), "r"(row0)
                        : "memory");
           asm volatile("cp.async.bulk.commit_group;" ::: "memory");
         }
       }
       // the stats slots are rewritten next tile only after all 4 warps passed this barrier
       named_bar(1 + q, 128);
-      tc_fence_before();
-      __syncwarp();
-      if (lane == 0) mbar_arrive_remote(tempty0);
-#ifdef TCB_GEMM_PROBE
-      if (lane == 0 && blockIdx.x < 2 && warp == 4)
-        printf("lnprobe epi cta %d tile %d wait_tfull %lld epilogue %lld\n", blockIdx.x, tile, e1 - e0, clock64() - e1);
-#endif
       tphase ^= 1;
     }
     if (lane == 0) bulk_wait_all();
@@ -917,12 +925,22 @@ cudaError_t launch_linear_ln_bf16_tc(const GemmMaps& m, int64_t M, int N, int K,
                                      float eps, const int32_t* seg_ids, cudaStream_t s) {
   if (M == 0) return cudaSuccess;
   if (N != kLnN) return cudaErrorInvalidValue;
-  static bool attr_set = false;
-  if (!attr_set) {
-    cudaError_t e = cudaFuncSetAttribute(linear_ln_kernel,
-                                         cudaFuncAttributeMaxDynamicSharedMemorySize, kLnSmemBytes);
+  const int nkb = K / BK;
+  static const int split_env = [] {
+    const char* e = getenv("TCB_LN_SPLIT");             // tuning override (k-blocks)
+    return e ? atoi(e) : -1;
+  }();
+  // measured (scripts/ln_ab.py): K = 512 fastest fully split with 4 stages; K = 2048 fastest
+  // with 3 joint stages and a 2-block split (A re-reads cost more than the overlap there)
+  int split_kb = split_env >= 0 ? (split_env < nkb ? split_env : nkb) : (nkb <= 16 ? nkb : 2);
+  const bool joint = split_kb < nkb;
+  auto kern = joint ? linear_ln_kernel<true> : linear_ln_kernel<false>;
+  const int smem = joint ? LnCfg<true>::kSmemBytes : LnCfg<false>::kSmemBytes;
+  static bool attr_set[2] = {false, false};
+  if (!attr_set[joint]) {
+    cudaError_t e = cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, smem);
     if (e != cudaSuccess) return e;
-    attr_set = true;
+    attr_set[joint] = true;
   }
   const int tiles = static_cast<int>((M + 255) / 256);
   int clusters = num_sms() / 2;
@@ -930,7 +948,7 @@ cudaError_t launch_linear_ln_bf16_tc(const GemmMaps& m, int64_t M, int N, int K,
   cudaLaunchConfig_t cfg{};
   cfg.gridDim = dim3(clusters * 2);
   cfg.blockDim = dim3(kLnThreads);
-  cfg.dynamicSmemBytes = kLnSmemBytes;
+  cfg.dynamicSmemBytes = smem;
   cfg.stream = s;
   cudaLaunchAttribute attr[1];
   attr[0].id = cudaLaunchAttributeClusterDimension;
@@ -939,8 +957,8 @@ cudaError_t launch_linear_ln_bf16_tc(const GemmMaps& m, int64_t M, int N, int K,
   attr[0].val.clusterDim.z = 1;
   cfg.attrs = attr;
   cfg.numAttrs = 1;
-  return cudaLaunchKernelEx(&cfg, linear_ln_kernel, m.a, m.w, m.c, m.r, static_cast<int>(M), K,
-                            bias, gamma, beta, eps, seg_ids);
+  return cudaLaunchKernelEx(&cfg, kern, m.a, m.w, m.c, m.r, static_cast<int>(M), K, bias, gamma,
+                            beta, eps, seg_ids, split_kb);
 }
 
 bool make_tmap_bf16(CUtensorMap* map, const void* ptr, uint64_t rows, uint64_t cols,

@@ -51,7 +51,8 @@ def test_linear_bf16_tcgen05_vs_oracle(M, N, K, epi):
     assert np.all(err <= bound), float(np.max(err / bound))
 
 
-@pytest.mark.parametrize("M,K", [(1, 512), (300, 512), (4133, 512), (1000, 2048), (32768, 512)])
+@pytest.mark.parametrize("M,K", [(1, 512), (300, 512), (4133, 512), (1000, 1024), (1000, 2048),
+                                 (513, 4096), (32768, 512)])
 def test_linear_ln_fused_vs_oracle(M, K):
     """W_O / FFN2 + bias + residual + LayerNorm in one tcgen05 kernel (N = 512)."""
     N = 512
