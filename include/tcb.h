@@ -78,14 +78,31 @@ typedef struct tcb_plan tcb_plan;
  *              the scheduler defers them, Alg. 1 picks a subset).
  *   policy   : tcb_pack_policy
  *   out      : receives a new plan (tcb_plan_destroy).
- * Within a row, requests are laid out contiguously from column 0 in placement order.
+ * Within a row, requests are laid out contiguously from column 0 in placement order
+ * (slotted plans below leave gaps at slot tails: those slots are pad, like the row tail).
  * Segments (placed requests) are numbered globally in (row, column) order (R13). */
 tcb_status tcb_pack(const int32_t* lengths, int32_t n, int32_t row_len, int32_t max_rows,
                     int32_t policy, tcb_plan** out);
+
+/* Slotted ConcatBatching (§4.2; Eq. (8); Alg. 2 l.4-7; reading R26).
+ * Each row is divided into floor(row_len / z) slots of z words (the tail is unused); in
+ * input order each request goes to the first slot (rows in order, slots left to right) with
+ * room, opening a new row when none has room (up to max_rows, 0 = unbounded).  Requests
+ * never straddle a slot; inside a slot they are contiguous from the slot start.  A request
+ * longer than z, or one that finds no slot under the row cap, is left unplaced (req_row = -1,
+ * status OK: deferred, R26).  slot_len = 0 selects z = the largest length (Alg. 2 l.4);
+ * slot_len = row_len is tcb_pack(TCB_PACK_FIRST_FIT).  The plan is an ordinary plan: the
+ * kernels are unchanged, because attention already restricts every query to its own request
+ * (Eq. (8)'s per-slot softmax is the special case where a slot holds one request).
+ *   slot_len : z in [0, row_len]; tcb_plan_info.slot_len reports the z used.
+ * Errors as tcb_pack (a request longer than row_len is TCB_ERR_REQUEST_TOO_LONG). */
+tcb_status tcb_pack_slotted(const int32_t* lengths, int32_t n, int32_t row_len, int32_t max_rows,
+                            int32_t slot_len, tcb_plan** out);
 void tcb_plan_destroy(tcb_plan* plan);
 
 typedef struct {
-  int32_t num_requests, num_placed, num_rows, row_len, num_segments, reserved;
+  int32_t num_requests, num_placed, num_rows, row_len, num_segments;
+  int32_t slot_len;            /* slotted plans: slot size z; 0 for the other policies      */
   int64_t total_tokens;        /* sum of all lengths (token_ids / outputs are this long)   */
   int64_t placed_tokens;       /* T: non-pad tokens in the rows                            */
   int64_t num_slots;           /* M = num_rows * row_len                                  */

@@ -99,6 +99,24 @@ def pack(lengths: Sequence[int], row_len: int, max_rows: int = 0,
     return {"req_row": req_row[:n], "req_col": req_col[:n], "num_rows": int(rows.value)}
 
 
+def pack_slotted(lengths: Sequence[int], row_len: int, slot_len: int = 0,
+                 max_rows: int = 0) -> Dict[str, np.ndarray]:
+    """o1 slotted (§4.2, Alg. 2, R26): First-Fit of requests into slots of slot_len words
+    (0 = the largest length); requests never straddle a slot."""
+    lengths = _i32(lengths)
+    n = len(lengths)
+    req_row = np.zeros(max(n, 1), np.int32)
+    req_col = np.zeros(max(n, 1), np.int32)
+    rows = ctypes.c_int32(0)
+    z = ctypes.c_int32(0)
+    rc = lib().oracle_pack_slotted(_p(lengths), n, row_len, max_rows, slot_len, _p(req_row),
+                                   _p(req_col), ctypes.byref(rows), ctypes.byref(z))
+    if rc != 0:
+        raise OracleError(rc)
+    return {"req_row": req_row[:n], "req_col": req_col[:n], "num_rows": int(rows.value),
+            "slot_len": int(z.value)}
+
+
 def layout(lengths, req_row, req_col, num_rows: int, row_len: int,
            qtile: int = 128) -> Dict[str, np.ndarray]:
     """o1 (layout): segment_ids, positions, tok_index, seg_req, seg_start, cu_seqlens,
@@ -211,9 +229,13 @@ def unpack(x, tok_index, total_tokens: int) -> np.ndarray:
 
 
 def run(model, weights, names, lengths, ids, row_len: int, max_rows: int = 0,
-        policy: str = "first_fit") -> Dict[str, np.ndarray]:
-    """The whole path: pack -> layout -> encoder -> unpack (request order)."""
-    pk = pack(lengths, row_len, max_rows, policy)
+        policy: str = "first_fit", slot_len: int = 0) -> Dict[str, np.ndarray]:
+    """The whole path: pack -> layout -> encoder -> unpack (request order).  policy
+    "slotted" packs into slots of slot_len words (§4.2, R26)."""
+    if policy == "slotted":
+        pk = pack_slotted(lengths, row_len, slot_len, max_rows)
+    else:
+        pk = pack(lengths, row_len, max_rows, policy)
     lay = layout(lengths, pk["req_row"], pk["req_col"], pk["num_rows"], row_len)
     x = encoder_rows(model, weights, names, ids, lay, row_len)
     out = unpack(x, lay["tok_index"], int(np.sum(lengths)))

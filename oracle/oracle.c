@@ -91,6 +91,63 @@ int oracle_pack(const int32_t* lengths, int32_t n, int32_t row_len, int32_t max_
 }
 
 /* ------------------------------------------------------------------------------------ */
+/* o1 (slotted ConcatBatching, §4.2; Alg. 2; reading R26).         */
+/* Each row of L words is divided into floor(L / z) slots of z words ("Divide each row of */
+/* the batch into multiple slots based on the slot size z", Alg. 2 l.5); the tail        */
+/* L - floor(L/z)*z is unused.  Requests are put into slots greedily (Alg. 2 l.7): in    */
+/* input order, each request goes to the first slot (rows in order, slots left to right) */
+/* whose residual is >= its length; if none, a new row is opened (while rows < max_rows, */
+/* 0 = unbounded), else it is deferred (req_row = -1).  A request never straddles a slot */
+/* boundary; within a slot requests are contiguous from the slot start in placement      */
+/* order.  z = 0 selects z = the largest request length (Alg. 2 l.4 with H_U = all       */
+/* requests).  z == L is pure ConcatBatching First-Fit ("a special case whose slot size  */
+/* is equal to the batch length L").                                        */
+/* ------------------------------------------------------------------------------------ */
+int oracle_pack_slotted(const int32_t* lengths, int32_t n, int32_t row_len, int32_t max_rows,
+                        int32_t slot_len, int32_t* req_row, int32_t* req_col, int32_t* num_rows,
+                        int32_t* slot_len_used) {
+  if (n < 0 || row_len <= 0 || max_rows < 0 || slot_len < 0 || slot_len > row_len)
+    return ORACLE_ERR_INVALID;
+  if (n > 0 && (!lengths || !req_row || !req_col)) return ORACLE_ERR_INVALID;
+  if (!num_rows || !slot_len_used) return ORACLE_ERR_INVALID;
+  int32_t z = slot_len;
+  for (int32_t i = 0; i < n; ++i) {
+    if (lengths[i] <= 0) return ORACLE_ERR_INVALID;
+    if (lengths[i] > row_len) return ORACLE_ERR_TOO_LONG;
+  }
+  if (z == 0) {
+    for (int32_t i = 0; i < n; ++i) if (lengths[i] > z) z = lengths[i];
+    if (z == 0) z = row_len; /* no requests */
+  }
+  const int32_t per_row = row_len / z;
+  const int32_t cap = (max_rows == 0) ? n : max_rows;
+  /* fill[row * per_row + j] = words used in slot j of row */
+  int32_t* fill = (int32_t*)calloc((size_t)(n > 0 ? n : 1) * (size_t)per_row, sizeof(int32_t));
+  int32_t rows = 0;
+  for (int32_t r = 0; r < n; ++r) {
+    const int32_t l = lengths[r];
+    int32_t slot = -1;
+    if (l <= z) {
+      for (int32_t s = 0; s < rows * per_row; ++s)
+        if (z - fill[s] >= l) { slot = s; break; }
+      if (slot < 0 && rows < cap) { slot = rows * per_row; ++rows; }
+    }
+    if (slot >= 0) {
+      req_row[r] = slot / per_row;
+      req_col[r] = (slot % per_row) * z + fill[slot];
+      fill[slot] += l;
+    } else {
+      req_row[r] = -1; /* deferred (R26) */
+      req_col[r] = -1;
+    }
+  }
+  *num_rows = rows;
+  *slot_len_used = z;
+  free(fill);
+  return ORACLE_OK;
+}
+
+/* ------------------------------------------------------------------------------------ */
 /* o1 (layout): per-slot metadata of the packed rows.  Segments are numbered globally in  */
 /* (row, column) order (R13); pad slots have segment -1, position -1, tok_index -1 (R12). */
 /* Positions restart at 0 at each request's first token: separate PE, R2.     */

@@ -38,6 +38,10 @@ typedef struct {
 
 int oracle_pack(const int32_t* lengths, int32_t n, int32_t row_len, int32_t max_rows,
                 int32_t policy, int32_t* req_row, int32_t* req_col, int32_t* num_rows);
+/* o1, slotted ConcatBatching (§4.2, Alg. 2, R26): First-Fit over slots of z words. */
+int oracle_pack_slotted(const int32_t* lengths, int32_t n, int32_t row_len, int32_t max_rows,
+                        int32_t slot_len, int32_t* req_row, int32_t* req_col, int32_t* num_rows,
+                        int32_t* slot_len_used);
 
 int oracle_layout(const int32_t* lengths, int32_t n, const int32_t* req_row,
                   const int32_t* req_col, int32_t num_rows, int32_t row_len, int32_t qtile,

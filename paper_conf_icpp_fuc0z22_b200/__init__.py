@@ -19,7 +19,7 @@ import numpy as np
 from . import _lib
 from ._lib import KCLASSES, POLICIES, TcbError, check, lib
 
-__all__ = ["Plan", "Encoder", "tcb_pack", "op_linear", "op_linear_ln", "op_attention", "op_layernorm",
+__all__ = ["Plan", "Encoder", "tcb_pack", "tcb_pack_slotted", "op_linear", "op_linear_ln", "op_attention", "op_layernorm",
            "launch_count", "profile_enable", "profile_collect", "TcbError", "KCLASSES"]
 
 _DTYPES = {"fp32": 0, "bf16": 1}
@@ -102,6 +102,17 @@ def tcb_pack(lengths: Sequence[int], row_len: int, max_rows: int = 0,
     h = ctypes.c_void_p()
     check(lib().tcb_pack(_ptr(arr) if len(arr) else None, len(arr), int(row_len),
                          int(max_rows), POLICIES[policy], ctypes.byref(h)))
+    return Plan(h)
+
+
+def tcb_pack_slotted(lengths: Sequence[int], row_len: int, slot_len: int = 0,
+                     max_rows: int = 0) -> Plan:
+    """Slotted ConcatBatching (C++ packer): First-Fit into slots of slot_len words
+    (0 = the largest length).  See include/tcb.h tcb_pack_slotted."""
+    arr = np.ascontiguousarray(np.asarray(lengths, dtype=np.int32))
+    h = ctypes.c_void_p()
+    check(lib().tcb_pack_slotted(_ptr(arr) if len(arr) else None, len(arr), int(row_len),
+                                 int(max_rows), int(slot_len), ctypes.byref(h)))
     return Plan(h)
 
 
@@ -207,10 +218,14 @@ class Encoder:
         return out
 
     def run(self, lengths, token_ids, row_len: int, max_rows: int = 0,
-            policy: str = "first_fit"):
-        """Host arrays in, device outputs out: pack -> H2D -> forward -> unpack."""
+            policy: str = "first_fit", slot_len: int = 0):
+        """Host arrays in, device outputs out: pack -> H2D -> forward -> unpack.
+        policy "slotted" packs with tcb_pack_slotted(slot_len)."""
         import torch
-        plan = tcb_pack(lengths, row_len, max_rows, policy)
+        if policy == "slotted":
+            plan = tcb_pack_slotted(lengths, row_len, slot_len, max_rows)
+        else:
+            plan = tcb_pack(lengths, row_len, max_rows, policy)
         d_segtab = torch.from_numpy(plan.segtab()).to(self.device)
         d_ids = torch.from_numpy(np.ascontiguousarray(token_ids, dtype=np.int32)).to(self.device)
         rows = self.encoder_forward(plan, d_segtab, d_ids)

@@ -23,7 +23,7 @@ KCLASSES = ["embed", "gemm_qkv", "attention", "gemm_o", "layernorm", "gemm_ffn1"
             "unpack"]
 
 # Every symbol include/tcb.h and include/tcb_ops.h declare (checked by the CPU tests).
-EXPORTS = ["tcb_last_error", "tcb_version", "tcb_pack", "tcb_plan_destroy",
+EXPORTS = ["tcb_last_error", "tcb_version", "tcb_pack", "tcb_pack_slotted", "tcb_plan_destroy",
            "tcb_plan_info_get", "tcb_plan_copy", "tcb_plan_segtab_words",
            "tcb_plan_write_segtab", "tcb_weights_count", "tcb_weights_create",
            "tcb_weights_destroy", "tcb_workspace_size", "tcb_embed", "tcb_encoder_forward",
@@ -40,7 +40,7 @@ class TcbError(RuntimeError):
 class PlanInfo(ctypes.Structure):
     _fields_ = [("num_requests", ctypes.c_int32), ("num_placed", ctypes.c_int32),
                 ("num_rows", ctypes.c_int32), ("row_len", ctypes.c_int32),
-                ("num_segments", ctypes.c_int32), ("reserved", ctypes.c_int32),
+                ("num_segments", ctypes.c_int32), ("slot_len", ctypes.c_int32),
                 ("total_tokens", ctypes.c_int64), ("placed_tokens", ctypes.c_int64),
                 ("num_slots", ctypes.c_int64), ("qtiles", ctypes.c_int64),
                 ("kv_tiles_visited", ctypes.c_int64), ("kv_tiles_dense", ctypes.c_int64),
@@ -48,7 +48,7 @@ class PlanInfo(ctypes.Structure):
                 ("executed_score_elems", ctypes.c_int64)]
 
     def as_dict(self):
-        return {f: getattr(self, f) for f, _ in self._fields_ if f != "reserved"}
+        return {f: getattr(self, f) for f, _ in self._fields_}
 
 
 class ModelConfig(ctypes.Structure):
@@ -80,6 +80,7 @@ def lib() -> ctypes.CDLL:
         "tcb_last_error": (ctypes.c_char_p, []),
         "tcb_version": (ctypes.c_char_p, []),
         "tcb_pack": (I32, [P, I32, I32, I32, I32, ctypes.POINTER(P)]),
+        "tcb_pack_slotted": (I32, [P, I32, I32, I32, I32, ctypes.POINTER(P)]),
         "tcb_plan_destroy": (None, [P]),
         "tcb_plan_info_get": (I32, [P, ctypes.POINTER(PlanInfo)]),
         "tcb_plan_copy": (I32, [P] + [P] * 8),

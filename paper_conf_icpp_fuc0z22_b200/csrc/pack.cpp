@@ -8,6 +8,7 @@
 // residual capacity of all candidate rows finds the leftmost row with room; rows not yet
 // opened have residual L, so "leftmost row with room" also opens new rows in order.
 #include <algorithm>
+#include <cstdint>
 #include <cstring>
 #include <new>
 #include <numeric>
@@ -121,6 +122,58 @@ void compute_info(tcb_plan* p) {
   }
 }
 
+tcb_status validate_pack(const char* fn, const int32_t* lengths, int32_t n, int32_t row_len,
+                         int32_t max_rows, tcb_plan** out) {
+  const std::string f(fn);
+  if (!out) return fail(TCB_ERR_INVALID_ARGUMENT, f + ": out is NULL");
+  *out = nullptr;
+  if (n < 0) return fail(TCB_ERR_INVALID_ARGUMENT, f + ": n < 0");
+  if (n > 0 && !lengths) return fail(TCB_ERR_INVALID_ARGUMENT, f + ": lengths is NULL");
+  if (row_len <= 0 || row_len % 8 != 0)
+    return fail(TCB_ERR_INVALID_ARGUMENT, f + ": row_len must be a positive multiple of 8");
+  if (max_rows < 0) return fail(TCB_ERR_INVALID_ARGUMENT, f + ": max_rows < 0");
+  for (int32_t i = 0; i < n; ++i) {
+    if (lengths[i] <= 0)
+      return fail(TCB_ERR_INVALID_ARGUMENT, f + ": lengths[" + std::to_string(i) + "] <= 0");
+    if (lengths[i] > row_len)
+      return fail(TCB_ERR_REQUEST_TOO_LONG, f + ": request " + std::to_string(i) + " has " +
+                                                std::to_string(lengths[i]) + " tokens > row_len " +
+                                                std::to_string(row_len));
+  }
+  return TCB_OK;
+}
+
+void init_plan(tcb_plan* p, const int32_t* lengths, int32_t n, int32_t row_len, int32_t max_rows,
+               int32_t policy) {
+  p->n = n;
+  p->row_len = row_len;
+  p->max_rows = max_rows;
+  p->policy = policy;
+  p->lengths.assign(lengths, lengths + n);
+  p->req_row.assign(n, -1);
+  p->req_col.assign(n, -1);
+  p->tok_off.resize(static_cast<size_t>(n) + 1);
+  p->tok_off[0] = 0;
+  for (int32_t i = 0; i < n; ++i) p->tok_off[i + 1] = p->tok_off[i] + lengths[i];
+}
+
+// Segments in (row, column) order from req_row / req_col; then the counters.
+void finish_plan(tcb_plan* p) {
+  std::vector<std::vector<int32_t>> members(p->num_rows);
+  for (int32_t r = 0; r < p->n; ++r)
+    if (p->req_row[r] >= 0) members[p->req_row[r]].push_back(r);
+  for (int32_t k = 0; k < p->num_rows; ++k) {
+    std::sort(members[k].begin(), members[k].end(),
+              [&](int32_t a, int32_t b) { return p->req_col[a] < p->req_col[b]; });
+    for (int32_t r : members[k]) {
+      p->seg_req.push_back(r);
+      p->seg_start.push_back(k * p->row_len + p->req_col[r]);
+    }
+  }
+  compute_info(p);
+  p->info.slot_len = p->slot_len;
+}
+
 }  // namespace
 }  // namespace tcb
 
@@ -134,37 +187,14 @@ const char* tcb_version(void) { return "tcb-b200 0.1 (sm_100a)"; }
 tcb_status tcb_pack(const int32_t* lengths, int32_t n, int32_t row_len, int32_t max_rows,
                     int32_t policy, tcb_plan** out) {
   tcb::clear_error();
-  if (!out) return fail(TCB_ERR_INVALID_ARGUMENT, "tcb_pack: out is NULL");
-  *out = nullptr;
-  if (n < 0) return fail(TCB_ERR_INVALID_ARGUMENT, "tcb_pack: n < 0");
-  if (n > 0 && !lengths) return fail(TCB_ERR_INVALID_ARGUMENT, "tcb_pack: lengths is NULL");
-  if (row_len <= 0 || row_len % 8 != 0)
-    return fail(TCB_ERR_INVALID_ARGUMENT, "tcb_pack: row_len must be a positive multiple of 8");
-  if (max_rows < 0) return fail(TCB_ERR_INVALID_ARGUMENT, "tcb_pack: max_rows < 0");
+  tcb_status st = tcb::validate_pack("tcb_pack", lengths, n, row_len, max_rows, out);
+  if (st != TCB_OK) return st;
   if (policy < TCB_PACK_FIRST_FIT || policy > TCB_PACK_LENGTH_SORTED)
     return fail(TCB_ERR_INVALID_ARGUMENT, "tcb_pack: unknown policy");
-  for (int32_t i = 0; i < n; ++i) {
-    if (lengths[i] <= 0)
-      return fail(TCB_ERR_INVALID_ARGUMENT, "tcb_pack: lengths[" + std::to_string(i) + "] <= 0");
-    if (lengths[i] > row_len)
-      return fail(TCB_ERR_REQUEST_TOO_LONG, "tcb_pack: request " + std::to_string(i) + " has " +
-                                                std::to_string(lengths[i]) + " tokens > row_len " +
-                                                std::to_string(row_len));
-  }
   tcb_plan* p = new (std::nothrow) tcb_plan();
   if (!p) return fail(TCB_ERR_OUT_OF_MEMORY, "tcb_pack: out of host memory");
   try {
-    p->n = n;
-    p->row_len = row_len;
-    p->max_rows = max_rows;
-    p->policy = policy;
-    p->lengths.assign(lengths, lengths + n);
-    p->req_row.assign(n, -1);
-    p->req_col.assign(n, -1);
-    p->tok_off.resize(static_cast<size_t>(n) + 1);
-    p->tok_off[0] = 0;
-    for (int32_t i = 0; i < n; ++i) p->tok_off[i + 1] = p->tok_off[i] + lengths[i];
-
+    tcb::init_plan(p, lengths, n, row_len, max_rows, policy);
     std::vector<int32_t> order(n);
     std::iota(order.begin(), order.end(), 0);
     if (policy == TCB_PACK_FIRST_FIT_DECREASING)
@@ -175,17 +205,12 @@ tcb_status tcb_pack(const int32_t* lengths, int32_t n, int32_t row_len, int32_t 
                        [&](int32_t a, int32_t b) { return lengths[a] < lengths[b]; });
 
     const int32_t cap = max_rows > 0 ? max_rows : std::max<int32_t>(n, 1);
-    std::vector<std::vector<int32_t>> row_members;  // placement order within each row
     std::vector<int32_t> used;
     auto place = [&](int32_t r, int32_t row) {
-      if (row >= static_cast<int32_t>(row_members.size())) {
-        row_members.resize(row + 1);
-        used.resize(row + 1, 0);
-      }
+      if (row >= static_cast<int32_t>(used.size())) used.resize(row + 1, 0);
       p->req_row[r] = row;
       p->req_col[r] = used[row];
       used[row] += lengths[r];
-      row_members[row].push_back(r);
     };
     if (policy == TCB_PACK_FIRST_FIT || policy == TCB_PACK_FIRST_FIT_DECREASING) {
       tcb::ResidualTree tree(cap, row_len);
@@ -212,20 +237,60 @@ tcb_status tcb_pack(const int32_t* lengths, int32_t n, int32_t row_len, int32_t 
         place(r, next++);
       }
     }
-    p->num_rows = static_cast<int32_t>(row_members.size());
-    // Segments in (row, column) order == rows in order, placement order inside a row.
-    for (int32_t k = 0; k < p->num_rows; ++k)
-      for (int32_t r : row_members[k]) {
-        p->seg_req.push_back(r);
-        p->seg_start.push_back(k * row_len + p->req_col[r]);
-      }
-    tcb::compute_info(p);
+    p->num_rows = static_cast<int32_t>(used.size());
+    tcb::finish_plan(p);
   } catch (const std::bad_alloc&) {
     delete p;
     return fail(TCB_ERR_OUT_OF_MEMORY, "tcb_pack: out of host memory");
   } catch (...) {
     delete p;
     return fail(TCB_ERR_INVALID_ARGUMENT, "tcb_pack: internal error");
+  }
+  *out = p;
+  return TCB_OK;
+}
+
+tcb_status tcb_pack_slotted(const int32_t* lengths, int32_t n, int32_t row_len, int32_t max_rows,
+                            int32_t slot_len, tcb_plan** out) {
+  tcb::clear_error();
+  tcb_status st = tcb::validate_pack("tcb_pack_slotted", lengths, n, row_len, max_rows, out);
+  if (st != TCB_OK) return st;
+  if (slot_len < 0 || slot_len > row_len)
+    return fail(TCB_ERR_INVALID_ARGUMENT, "tcb_pack_slotted: slot_len must be in [0, row_len]");
+  tcb_plan* p = new (std::nothrow) tcb_plan();
+  if (!p) return fail(TCB_ERR_OUT_OF_MEMORY, "tcb_pack_slotted: out of host memory");
+  try {
+    tcb::init_plan(p, lengths, n, row_len, max_rows, TCB_PACK_FIRST_FIT);
+    int32_t z = slot_len;
+    if (z == 0) z = n > 0 ? *std::max_element(lengths, lengths + n) : row_len;  // Alg. 2 l.4
+    p->slot_len = z;
+    const int32_t per_row = row_len / z;
+    const int32_t cap = max_rows > 0 ? max_rows : std::max<int32_t>(n, 1);
+    // First-Fit over slots (row-major): the leftmost slot with residual >= l; slots of rows
+    // not yet opened have residual z, so "no open slot fits" opens the next row.
+    tcb::ResidualTree tree(static_cast<int32_t>(std::min<int64_t>(
+                               static_cast<int64_t>(cap) * per_row, INT32_MAX)), z);
+    std::vector<int32_t> fill;
+    int32_t rows = 0;
+    for (int32_t r = 0; r < n; ++r) {
+      if (lengths[r] > z) continue;  // longer than a slot: deferred (R26)
+      const int32_t slot = tree.leftmost_at_least(lengths[r]);
+      if (slot < 0) continue;        // row cap reached: deferred
+      if (slot >= static_cast<int32_t>(fill.size())) fill.resize(slot + 1, 0);
+      tree.sub(slot, lengths[r]);
+      p->req_row[r] = slot / per_row;
+      p->req_col[r] = (slot % per_row) * z + fill[slot];
+      fill[slot] += lengths[r];
+      rows = std::max(rows, slot / per_row + 1);
+    }
+    p->num_rows = rows;
+    tcb::finish_plan(p);
+  } catch (const std::bad_alloc&) {
+    delete p;
+    return fail(TCB_ERR_OUT_OF_MEMORY, "tcb_pack_slotted: out of host memory");
+  } catch (...) {
+    delete p;
+    return fail(TCB_ERR_INVALID_ARGUMENT, "tcb_pack_slotted: internal error");
   }
   *out = p;
   return TCB_OK;

@@ -31,6 +31,7 @@ struct SegRec {
 
 struct tcb_plan {
   int32_t n = 0, row_len = 0, num_rows = 0, max_rows = 0, policy = 0;
+  int32_t slot_len = 0;                  // slotted ConcatBatching slot size z, 0 = none
   std::vector<int32_t> lengths, req_row, req_col;
   std::vector<int64_t> tok_off;          // request-order offset of each request's tokens
   std::vector<int32_t> seg_req, seg_start;

@@ -21,8 +21,11 @@ def per_request_errors(gpu_rows, ref_rows, segment_ids, seg_bounds):
 
 
 def oracle_selected_rows(model, weights, names, lengths, ids, row_len, rows, max_rows=0,
-                         policy="first_fit"):
-    pk = oracle.pack(lengths, row_len, max_rows, policy)
+                         policy="first_fit", slot_len=0):
+    if policy == "slotted":
+        pk = oracle.pack_slotted(lengths, row_len, slot_len, max_rows)
+    else:
+        pk = oracle.pack(lengths, row_len, max_rows, policy)
     lay = oracle.layout(lengths, pk["req_row"], pk["req_col"], pk["num_rows"], row_len)
     x = oracle.encoder_rows(model, weights, names, ids, lay, row_len, rows)
     return pk, lay, x

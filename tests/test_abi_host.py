@@ -90,6 +90,74 @@ def test_pack_golden_f1(golden_dir):
     assert plan.info["placed_tokens"] == 58 and plan.info["num_slots"] == 64
 
 
+def _slotted_vs_oracle(lengths, L, z, max_rows):
+    plan = tcb.tcb_pack_slotted(lengths, L, z, max_rows)
+    pk = oracle.pack_slotted(lengths, L, z, max_rows)
+    lay = oracle.layout(lengths, pk["req_row"], pk["req_col"], pk["num_rows"], L, 128)
+    a = plan.arrays()
+    assert plan.info["slot_len"] == pk["slot_len"]
+    assert plan.info["num_rows"] == pk["num_rows"]
+    assert a["req_row"].tolist() == pk["req_row"].tolist()
+    assert a["req_col"].tolist() == pk["req_col"].tolist()
+    for k in ("seg_req", "seg_start", "cu_seqlens", "segment_ids", "positions"):
+        assert a[k].tolist() == lay[k].tolist(), k
+    assert a["qtile_kv"].tolist() == lay["qtile_kv"].tolist()
+    return plan
+
+
+@pytest.mark.parametrize("seed", range(16))
+def test_pack_slotted_bit_exact_vs_oracle_random(seed):
+    rng = np.random.default_rng(900 + seed)
+    L = int(rng.choice([8, 32, 64, 128, 256]))
+    n = int(rng.integers(0, 200))
+    lengths = rng.integers(1, L + 1, size=n).astype(np.int32)
+    max_rows = int(rng.choice([0, 0, 3, 20]))
+    for z in (0, int(rng.integers(1, L + 1)), L):
+        _slotted_vs_oracle(lengths, L, z, max_rows)
+
+
+@pytest.mark.parametrize("dist,L,slots", [("paracrawl", 128, (2, 4)), ("dia", 512, (2, 4, 7)),
+                                          ("paper_normal_20", 128, (2, 3, 6))])
+def test_pack_slotted_bit_exact_vs_oracle_workloads(dist, L, slots):
+    lengths = np.minimum(wl.draw_lengths(dist, 800, 78), L).astype(np.int32)
+    for s in slots:
+        _slotted_vs_oracle(lengths, L, L // s, 64)
+
+
+def test_pack_slotted_golden_f1s(golden_dir):
+    f = json.load(open(os.path.join(golden_dir, "f1s_slotted.json")))
+    for c in f["cases"]:
+        plan = tcb.tcb_pack_slotted(f["lengths"], f["row_len"], c["slot_len_arg"])
+        a = plan.arrays()
+        assert plan.info["slot_len"] == c["slot_len"]
+        assert a["req_row"].tolist() == c["req_row"]
+        assert a["req_col"].tolist() == c["req_col"]
+        assert a["seg_req"].tolist() == c["seg_req"]
+        assert a["seg_start"].tolist() == c["seg_start"]
+        assert a["cu_seqlens"].tolist() == c["cu_seqlens"]
+        assert a["qtile_kv"].tolist() == c["qtile_kv_128"]
+        st = plan.segtab()
+        S = len(c["seg_req"])
+        recs = st[4:4 + 4 * S].reshape(-1, 4)
+        assert recs[:, 0].tolist() == c["seg_start"]
+        assert recs[:, 3].tolist() == c["seg_req"]
+
+
+def test_pack_slotted_errors():
+    with pytest.raises(tcb.TcbError) as e:
+        tcb.tcb_pack_slotted([3, 40], 32, 8)
+    assert e.value.status == -2
+    with pytest.raises(tcb.TcbError) as e:
+        tcb.tcb_pack_slotted([3], 32, 33)
+    assert e.value.status == -1
+    with pytest.raises(tcb.TcbError) as e:
+        tcb.tcb_pack_slotted([3], 32, -1)
+    assert e.value.status == -1
+    p = tcb.tcb_pack_slotted([9, 4], 32, 8)          # 9 > z: deferred, not an error
+    assert p.arrays()["req_row"].tolist() == [-1, 0]
+    assert tcb.tcb_pack([3], 32).info["slot_len"] == 0
+
+
 def test_pack_errors():
     with pytest.raises(tcb.TcbError) as e:
         tcb.tcb_pack([3, 40], 32)

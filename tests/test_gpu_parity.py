@@ -19,8 +19,8 @@ import paper_conf_icpp_fuc0z22_b200 as tcb  # noqa: E402
 from _helpers import TOL, oracle_selected_rows, per_request_errors, segments_in_rows  # noqa: E402
 
 
-def _gpu_rows(enc, lengths, ids, L, max_rows=0, policy="first_fit"):
-    plan, rows, out = enc.run(lengths, ids, L, max_rows, policy)
+def _gpu_rows(enc, lengths, ids, L, max_rows=0, policy="first_fit", slot_len=0):
+    plan, rows, out = enc.run(lengths, ids, L, max_rows, policy, slot_len)
     torch.cuda.synchronize()
     return plan, rows.float().cpu().numpy(), out.float().cpu().numpy()
 
@@ -102,6 +102,53 @@ def test_gpu_concat_equals_naive_and_alone(key):
         for other in (naive[sl], srt[sl], alone):
             e = np.max(np.abs(concat[sl] - other)) / np.max(np.abs(other))
             assert e <= TOL["bf16"], (r, e)
+
+
+@pytest.mark.parametrize("z", [0, 16, 20])
+def test_c1_slotted_fp32_full_oracle(z):
+    """§8(f) f1: slotted ConcatBatching plans (gaps at slot tails) through the same kernels."""
+    lengths, ids, w = wl.workload_inputs("c1")
+    model = wl.MODELS["toy"]
+    names = wl.weight_names(model)
+    enc = tcb.Encoder(model, w, names)
+    plan, rows, out = _gpu_rows(enc, lengths, ids, 32, 0, "slotted", z)
+    ref = oracle.run(model, w, names, lengths, ids, 32, policy="slotted", slot_len=z)
+    assert plan.info["num_rows"] == ref["pack"]["num_rows"]
+    cu = np.concatenate([[0], np.cumsum(lengths)])
+    for r in range(len(lengths)):
+        o, g = ref["out"][cu[r]:cu[r + 1]], out[cu[r]:cu[r + 1]]
+        assert np.max(np.abs(g - o)) / np.max(np.abs(o)) <= TOL["fp32"], r
+    seg = ref["layout"]["segment_ids"]
+    assert np.all(rows[seg < 0] == 0)
+
+
+@pytest.mark.parametrize("key,slots,sel", [("c2", 4, [0, 20, -1]), ("c3", 3, [1])])
+def test_slotted_bf16_sampled_rows_and_equal_to_concat(key, slots, sel):
+    """Slotted plans at the workloads' shapes: sampled rows vs the oracle, and every
+    request's output equal to its pure-ConcatBatching output within the bf16 bar."""
+    wlc = wl.WORKLOADS[key]
+    model = wlc.model
+    L = wlc.row_len
+    nrows = 64 if key == "c2" else 8
+    lengths, ids, w = wl.workload_inputs(key, rows=nrows)
+    lengths = np.minimum(lengths, L // slots).astype(np.int32)   # every request fits a slot
+    ids = ids[:int(lengths.sum())]
+    names = wl.weight_names(model)
+    enc = tcb.Encoder(model, w, names)
+    plan, rows, out = _gpu_rows(enc, lengths, ids, L, 0, "slotted", L // slots)
+    assert plan.info["num_placed"] == len(lengths)
+    sel = [r if r >= 0 else plan.info["num_rows"] + r for r in sel]
+    pk, lay, x = oracle_selected_rows(model, w, names, lengths, ids, L, sel, 0, "slotted",
+                                      L // slots)
+    g = np.concatenate([rows[r * L:(r + 1) * L] for r in sel])
+    errs = per_request_errors(g, x, None, segments_in_rows(lay, L, sel))
+    assert max(errs.values()) <= TOL["bf16"], max(errs.values())
+    _, _, concat = _gpu_rows(enc, lengths, ids, L)
+    cu = np.concatenate([[0], np.cumsum(lengths)])
+    for r in range(len(lengths)):
+        sl = slice(cu[r], cu[r + 1])
+        e = np.max(np.abs(concat[sl] - out[sl])) / np.max(np.abs(concat[sl]))
+        assert e <= TOL["bf16"], (r, e)
 
 
 def test_forward_deterministic_and_graph_replay():
