@@ -236,6 +236,78 @@ enum {
 tcb_status tcb_profile_enable(int32_t on);
 tcb_status tcb_profile_collect(double* ms, int64_t* launches);
 
+/* ======================================================================================
+ * 5. Online request scheduling (host; §5; §8(f) row f2).
+ *    Request n has arrival a_n, deadline d_n and length l_n; one batch of
+ *    B rows x L words runs per time slot; utility v_n = 1/l_n counts only if n
+ *    is scheduled inside [a_n, d_n] (Eq. (9)-(13)).  Per time slot the waiting
+ *    set N_t (arrived, not yet scheduled, deadline not passed) is turned into
+ *    one batch by:
+ *      TCB_SCHED_DAS  Alg. 1 (§5.2): per row a utility-dominant
+ *                     set N_U (the first p = max(1, floor(eta * s)) requests by utility,
+ *                     s = how many of them fit the row), then the deadline-aware set N_D
+ *                     (v >= q * mean v(N_U)) in deadline order, then the rest by utility,
+ *                     each placed only if it fits; if everything left fits, it all goes
+ *                     in (l.4-5).  eta + q = 1 gives the eta*q/(eta*q+1) competitive ratio
+ *                     of Theorem 5.1 (1/5 at eta = q = 1/2).  Readings R27.
+ *      TCB_SCHED_FCFS / _SJF / _DEF  the baselines of §6.2.4: arrival /
+ *                     length / deadline order (ties: arrival, then id), First-Fit into
+ *                     the B rows.
+ *    Within a row, requests occupy consecutive columns from 0 in the order they are put in.
+ * ==================================================================================== */
+typedef enum {
+  TCB_SCHED_DAS = 0,
+  TCB_SCHED_FCFS = 1,
+  TCB_SCHED_SJF = 2,
+  TCB_SCHED_DEF = 3
+} tcb_sched_policy;
+
+/* One batch from a given waiting set (stateless).
+ *   lengths/arrival/deadline/ids : [n] host arrays describing N_t (ids unique; they only
+ *                                  break ties); every length in [1, L]
+ *   B, L                         : batch rows and row length
+ *   eta, q                       : DAS parameters in (0, 1] (ignored by the baselines)
+ *   row, col                     : [n] outputs, -1 when the request is not in the batch
+ * Errors: TCB_ERR_INVALID_ARGUMENT (bad sizes / NULL / policy / eta, q),
+ *         TCB_ERR_REQUEST_TOO_LONG (a length > L). */
+tcb_status tcb_sched_batch(int32_t policy, const int32_t* lengths, const double* arrival,
+                           const double* deadline, const int64_t* ids, int32_t n, int32_t B,
+                           int32_t L, double eta, double q, int32_t* row, int32_t* col);
+
+/* Stateful online scheduler: a queue of submitted requests, one batch per time slot. */
+typedef struct tcb_scheduler tcb_scheduler;
+typedef struct {
+  int64_t submitted;   /* requests ever submitted                                        */
+  int64_t waiting;     /* in the queue now (arrived or not)                               */
+  int64_t scheduled;   /* put into some batch (a response is produced)      */
+  int64_t expired;     /* dropped at a slot start after their deadline (utility 0)       */
+  int64_t batches;     /* tcb_sched_next_batch calls that succeeded                      */
+  double utility;      /* sum of 1/l over scheduled requests: the objective (9)          */
+} tcb_sched_stats;
+
+/* batch_rows = B > 0, row_len = L > 0 and a multiple of 8; library-owned (destroy). */
+tcb_status tcb_sched_create(int32_t policy, int32_t batch_rows, int32_t row_len, double eta,
+                            double q, tcb_scheduler** out);
+void tcb_sched_destroy(tcb_scheduler* sched);
+/* Enqueue n requests (copied).  A length > row_len is TCB_ERR_REQUEST_TOO_LONG (nothing is
+ * enqueued); deadline < arrival is TCB_ERR_INVALID_ARGUMENT. */
+tcb_status tcb_sched_submit(tcb_scheduler* sched, int32_t n, const int64_t* ids,
+                            const int32_t* lengths, const double* arrival,
+                            const double* deadline);
+/* The time slot starting at `now`: requests with deadline < now are dropped (expired);
+ * N_t = queued requests with arrival <= now; the policy picks the batch, which leaves the
+ * queue.  Outputs: ids_out / lengths_out [capacity] = the chosen requests in (row, column)
+ * order, *n_out = their count; if plan_out != NULL, *plan_out = a new plan of exactly B rows
+ * whose request order is that output order (gather the token ids in that order; empty rows
+ * are all pad), ready for tcb_plan_write_segtab / tcb_encoder_forward (a fixed B x L shape,
+ * so a captured CUDA graph can be replayed with each slot's segment table).  If capacity is
+ * smaller than the batch, nothing is scheduled (expired requests are still dropped), *n_out =
+ * the size needed and the status is TCB_ERR_INVALID_ARGUMENT. */
+tcb_status tcb_sched_next_batch(tcb_scheduler* sched, double now, int64_t* ids_out,
+                                int32_t* lengths_out, int32_t capacity, int32_t* n_out,
+                                tcb_plan** plan_out);
+tcb_status tcb_sched_stats_get(const tcb_scheduler* sched, tcb_sched_stats* out);
+
 #ifdef __cplusplus
 }
 #endif

@@ -117,6 +117,54 @@ def pack_slotted(lengths: Sequence[int], row_len: int, slot_len: int = 0,
             "slot_len": int(z.value)}
 
 
+SCHED_POLICIES = {"das": 0, "fcfs": 1, "sjf": 2, "def": 3}
+
+
+def sched_batch(policy: str, lengths, arrival, deadline, ids, B: int, L: int,
+                eta: float = 0.5, q: float = 0.5):
+    """f2: one time slot's batch from the waiting set (Alg. 1 / baselines, R27).
+    Returns (row, col) per waiting request, -1 = not chosen."""
+    lengths = _i32(lengths)
+    n = len(lengths)
+    arrival = _f64(arrival)
+    deadline = _f64(deadline)
+    ids = np.ascontiguousarray(np.asarray(ids, dtype=np.int64))
+    row = np.zeros(max(n, 1), np.int32)
+    col = np.zeros(max(n, 1), np.int32)
+    rc = lib().oracle_sched_batch(SCHED_POLICIES[policy], _p(lengths), _p(arrival),
+                                  _p(deadline), _p(ids), n, B, L, ctypes.c_double(eta),
+                                  ctypes.c_double(q), _p(row), _p(col))
+    if rc != 0:
+        raise OracleError(rc)
+    return row[:n], col[:n]
+
+
+def sched_simulate(policy: str, lengths, arrival, deadline, B: int, L: int, slot_time: float,
+                   num_slots: int, eta: float = 0.5, q: float = 0.5):
+    """The online setting of §5.1: time slot t starts at t * slot_time; the
+    waiting set N_t holds requests with arrival <= t*slot_time <= deadline not scheduled
+    yet (constraint (12)); each slot schedules one batch.  Returns per request
+    (slot, row, col) (-1 if never scheduled) and the total utility sum 1/l (Eq. (9))."""
+    lengths = _i32(lengths)
+    n = len(lengths)
+    arrival, deadline = _f64(arrival), _f64(deadline)
+    slot = np.full(n, -1, np.int64)
+    row = np.full(n, -1, np.int32)
+    col = np.full(n, -1, np.int32)
+    for t in range(num_slots):
+        now = t * slot_time
+        wait = [i for i in range(n) if slot[i] < 0 and arrival[i] <= now <= deadline[i]]
+        if not wait:
+            continue
+        w = np.array(wait, np.int64)
+        r, c = sched_batch(policy, lengths[w], arrival[w], deadline[w], w, B, L, eta, q)
+        for j, i in enumerate(wait):
+            if r[j] >= 0:
+                slot[i], row[i], col[i] = t, r[j], c[j]
+    utility = float(sum(1.0 / lengths[i] for i in range(n) if slot[i] >= 0))
+    return {"slot": slot, "row": row, "col": col, "utility": utility}
+
+
 def layout(lengths, req_row, req_col, num_rows: int, row_len: int,
            qtile: int = 128) -> Dict[str, np.ndarray]:
     """o1 (layout): segment_ids, positions, tok_index, seg_req, seg_start, cu_seqlens,

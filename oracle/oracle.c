@@ -148,6 +148,135 @@ int oracle_pack_slotted(const int32_t* lengths, int32_t n, int32_t row_len, int3
 }
 
 /* ------------------------------------------------------------------------------------ */
+/* §8(f) f2: request scheduling (§5).  One time slot's batch H_t of B rows chosen from the  */
+/* waiting set N_t (requests arrived, not yet scheduled, deadline not passed; the caller    */
+/* passes exactly that set).  Utility v_n = 1 / l_n.              */
+/* ORACLE_SCHED_DAS follows Alg. 1 (§5.2) line by line, with the   */
+/* readings R27 of DESIGN.md:                                                              */
+/*   - rows k = 0..B-1 in order; a request placed in a row leaves N_t (constraint (10));   */
+/*   - l.4-5: if the remaining requests fit the row, all of them go in, in N_t order      */
+/*     (arrival, then id);                                                                 */
+/*   - l.7: utility order = v non-increasing = length ascending, ties by arrival then id; */
+/*   - l.8: s = the largest prefix count of that order whose lengths sum to <= L;        */
+/*   - l.9: p = max(1, floor(eta * s)) (p_tk = eta s_tk, and p >= 1);       */
+/*   - l.11: N_D = requests after the first p whose v >= q * mean(v over N_U) ("no less   */
+/*     than"), evaluated in double as 1.0/l >= q * (sum(1.0/l) / p), the sum */
+/*     in utility order;                                                                   */
+/*   - l.12: N_D in deadline order (ties arrival, id), each placed if it still fits;     */
+/*   - l.13-14: then the rest (utility order), each placed if it still fits.             */
+/* Within a row, requests occupy columns in the order they are put in.  The baselines of */
+/* §6.2.4 put requests in their priority order into the first row with room */
+/* (First-Fit): FCFS = arrival order, SJF = length ascending, DEF = deadline ascending     */
+/* (ties: arrival, then id).                                                               */
+/* ------------------------------------------------------------------------------------ */
+typedef struct {
+  const int32_t* len;
+  const double* arr;
+  const double* dl;
+  const int64_t* id;
+  int key; /* 0 = arrival, 1 = length (utility), 2 = deadline */
+} sched_ctx;
+
+static int sched_before(const sched_ctx* c, int32_t a, int32_t b) {
+  if (c->key == 1 && c->len[a] != c->len[b]) return c->len[a] < c->len[b];
+  if (c->key == 2 && c->dl[a] != c->dl[b]) return c->dl[a] < c->dl[b];
+  if (c->arr[a] != c->arr[b]) return c->arr[a] < c->arr[b];
+  return c->id[a] < c->id[b];
+}
+
+/* plain insertion sort of idx[0..m) by the context key (stable, obviously correct) */
+static void sched_sort(const sched_ctx* c, int32_t* idx, int32_t m) {
+  for (int32_t i = 1; i < m; ++i) {
+    int32_t v = idx[i], j = i - 1;
+    while (j >= 0 && sched_before(c, v, idx[j])) { idx[j + 1] = idx[j]; --j; }
+    idx[j + 1] = v;
+  }
+}
+
+int oracle_sched_batch(int32_t policy, const int32_t* lengths, const double* arrival,
+                       const double* deadline, const int64_t* ids, int32_t n, int32_t B,
+                       int32_t L, double eta, double q, int32_t* row, int32_t* col) {
+  if (n < 0 || B < 0 || L <= 0 || policy < 0 || policy > 3) return ORACLE_ERR_INVALID;
+  if (n > 0 && (!lengths || !arrival || !deadline || !ids || !row || !col)) return ORACLE_ERR_INVALID;
+  for (int32_t i = 0; i < n; ++i) {
+    if (lengths[i] <= 0) return ORACLE_ERR_INVALID;
+    if (lengths[i] > L) return ORACLE_ERR_TOO_LONG;
+    row[i] = -1;
+    col[i] = -1;
+  }
+  sched_ctx c = {lengths, arrival, deadline, ids, 0};
+  int32_t* idx = (int32_t*)malloc(sizeof(int32_t) * (size_t)(n > 0 ? n : 1));
+  if (policy != ORACLE_SCHED_DAS) {
+    int32_t* used = (int32_t*)calloc((size_t)(B > 0 ? B : 1), sizeof(int32_t));
+    for (int32_t i = 0; i < n; ++i) idx[i] = i;
+    c.key = policy == ORACLE_SCHED_FCFS ? 0 : (policy == ORACLE_SCHED_SJF ? 1 : 2);
+    sched_sort(&c, idx, n);
+    for (int32_t t = 0; t < n; ++t) {
+      const int32_t r = idx[t];
+      for (int32_t k = 0; k < B; ++k)
+        if (used[k] + lengths[r] <= L) {
+          row[r] = k; col[r] = used[k]; used[k] += lengths[r];
+          break;
+        }
+    }
+    free(used);
+    free(idx);
+    return ORACLE_OK;
+  }
+  for (int32_t k = 0; k < B; ++k) {
+    /* N_t: the requests not placed yet */
+    int32_t m = 0;
+    int64_t total = 0;
+    for (int32_t i = 0; i < n; ++i)
+      if (row[i] < 0) { idx[m++] = i; total += lengths[i]; }
+    if (m == 0) break;
+    int32_t used = 0;
+    if (total <= L) {                               /* l.4-5 */
+      c.key = 0;
+      sched_sort(&c, idx, m);
+      for (int32_t t = 0; t < m; ++t) {
+        row[idx[t]] = k; col[idx[t]] = used; used += lengths[idx[t]];
+      }
+      continue;
+    }
+    c.key = 1;                                      /* l.7: utility order */
+    sched_sort(&c, idx, m);
+    int32_t s = 0;                                  /* l.8 */
+    int64_t pre = 0;
+    while (s < m && pre + lengths[idx[s]] <= L) { pre += lengths[idx[s]]; ++s; }
+    int32_t p = (int32_t)floor(eta * (double)s);    /* l.9 */
+    if (p < 1) p = 1;
+    double vsum = 0.0;
+    for (int32_t t = 0; t < p; ++t) {               /* l.10: N_U into the row */
+      const int32_t r = idx[t];
+      row[r] = k; col[r] = used; used += lengths[r];
+      vsum += 1.0 / (double)lengths[r];
+    }
+    const double thr = q * (vsum / (double)p);
+    int32_t* nd = (int32_t*)malloc(sizeof(int32_t) * (size_t)m);
+    int32_t nnd = 0;
+    for (int32_t t = p; t < m; ++t)                 /* l.11: N_D */
+      if (1.0 / (double)lengths[idx[t]] >= thr) nd[nnd++] = idx[t];
+    c.key = 2;                                      /* l.12: deadline order, greedy */
+    sched_sort(&c, nd, nnd);
+    for (int32_t t = 0; t < nnd; ++t) {
+      const int32_t r = nd[t];
+      if (used + lengths[r] <= L) { row[r] = k; col[r] = used; used += lengths[r]; }
+    }
+    for (int32_t t = p; t < m; ++t) {               /* l.13-14: the rest, utility order */
+      const int32_t r = idx[t];
+      int in_nd = 0;
+      for (int32_t u = 0; u < nnd; ++u) if (nd[u] == r) in_nd = 1;
+      if (in_nd || row[r] >= 0) continue;
+      if (used + lengths[r] <= L) { row[r] = k; col[r] = used; used += lengths[r]; }
+    }
+    free(nd);
+  }
+  free(idx);
+  return ORACLE_OK;
+}
+
+/* ------------------------------------------------------------------------------------ */
 /* o1 (layout): per-slot metadata of the packed rows.  Segments are numbered globally in  */
 /* (row, column) order (R13); pad slots have segment -1, position -1, tok_index -1 (R12). */
 /* Positions restart at 0 at each request's first token: separate PE, R2.     */

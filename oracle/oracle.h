@@ -27,6 +27,11 @@ extern "C" {
 #define ORACLE_NAIVE 3
 #define ORACLE_LENGTH_SORTED 4
 
+#define ORACLE_SCHED_DAS 0
+#define ORACLE_SCHED_FCFS 1
+#define ORACLE_SCHED_SJF 2
+#define ORACLE_SCHED_DEF 3
+
 typedef struct {
   int32_t num_layers, d_model, num_heads, d_ff;
   int32_t act;          /* 0 gelu (erf), 1 relu                          (R9)  */
@@ -42,6 +47,11 @@ int oracle_pack(const int32_t* lengths, int32_t n, int32_t row_len, int32_t max_
 int oracle_pack_slotted(const int32_t* lengths, int32_t n, int32_t row_len, int32_t max_rows,
                         int32_t slot_len, int32_t* req_row, int32_t* req_col, int32_t* num_rows,
                         int32_t* slot_len_used);
+/* f2 (§5, Alg. 1, R27): one time slot's batch of B rows from the waiting set; row/col per
+ * waiting request (-1 = not chosen).  policy: DAS 0, FCFS 1, SJF 2, DEF 3. */
+int oracle_sched_batch(int32_t policy, const int32_t* lengths, const double* arrival,
+                       const double* deadline, const int64_t* ids, int32_t n, int32_t B,
+                       int32_t L, double eta, double q, int32_t* row, int32_t* col);
 
 int oracle_layout(const int32_t* lengths, int32_t n, const int32_t* req_row,
                   const int32_t* req_col, int32_t num_rows, int32_t row_len, int32_t qtile,

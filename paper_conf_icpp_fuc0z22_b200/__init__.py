@@ -19,7 +19,7 @@ import numpy as np
 from . import _lib
 from ._lib import KCLASSES, POLICIES, TcbError, check, lib
 
-__all__ = ["Plan", "Encoder", "tcb_pack", "tcb_pack_slotted", "op_linear", "op_linear_ln", "op_attention", "op_layernorm",
+__all__ = ["Plan", "Encoder", "Scheduler", "sched_batch", "tcb_pack", "tcb_pack_slotted", "op_linear", "op_linear_ln", "op_attention", "op_layernorm",
            "launch_count", "profile_enable", "profile_collect", "TcbError", "KCLASSES"]
 
 _DTYPES = {"fp32": 0, "bf16": 1}
@@ -114,6 +114,69 @@ def tcb_pack_slotted(lengths: Sequence[int], row_len: int, slot_len: int = 0,
     check(lib().tcb_pack_slotted(_ptr(arr) if len(arr) else None, len(arr), int(row_len),
                                  int(max_rows), int(slot_len), ctypes.byref(h)))
     return Plan(h)
+
+
+def sched_batch(policy: str, lengths, arrival, deadline, ids, B: int, L: int,
+                eta: float = 0.5, q: float = 0.5):
+    """One time slot's batch from a waiting set (C++ scheduler, include/tcb.h §5).
+    Returns (row, col) per request (-1 = not in the batch)."""
+    lengths = np.ascontiguousarray(np.asarray(lengths, dtype=np.int32))
+    n = len(lengths)
+    arrival = np.ascontiguousarray(np.asarray(arrival, dtype=np.float64))
+    deadline = np.ascontiguousarray(np.asarray(deadline, dtype=np.float64))
+    ids = np.ascontiguousarray(np.asarray(ids, dtype=np.int64))
+    row = np.zeros(max(n, 1), np.int32)
+    col = np.zeros(max(n, 1), np.int32)
+    check(lib().tcb_sched_batch(_lib.SCHED_POLICIES[policy], _ptr(lengths), _ptr(arrival),
+                                _ptr(deadline), _ptr(ids), n, int(B), int(L), float(eta),
+                                float(q), _ptr(row), _ptr(col)))
+    return row[:n], col[:n]
+
+
+class Scheduler:
+    """Online request scheduler (DAS / FCFS / SJF / DEF) over B x L batches; wraps
+    tcb_scheduler*.  next_batch(now) returns (ids, lengths, Plan of exactly B rows)."""
+
+    def __init__(self, policy: str, batch_rows: int, row_len: int, eta: float = 0.5,
+                 q: float = 0.5):
+        h = ctypes.c_void_p()
+        check(lib().tcb_sched_create(_lib.SCHED_POLICIES[policy], int(batch_rows),
+                                     int(row_len), float(eta), float(q), ctypes.byref(h)))
+        self._h = h
+        self.B, self.L = int(batch_rows), int(row_len)
+        self._cap = 1024
+
+    def __del__(self):
+        h, self._h = getattr(self, "_h", None), None
+        try:
+            if h and _lib._lib is not None:
+                _lib._lib.tcb_sched_destroy(h)
+        except Exception:  # interpreter shutdown
+            pass
+
+    def submit(self, ids, lengths, arrival, deadline) -> None:
+        ids = np.ascontiguousarray(np.asarray(ids, dtype=np.int64))
+        lengths = np.ascontiguousarray(np.asarray(lengths, dtype=np.int32))
+        arrival = np.ascontiguousarray(np.asarray(arrival, dtype=np.float64))
+        deadline = np.ascontiguousarray(np.asarray(deadline, dtype=np.float64))
+        check(lib().tcb_sched_submit(self._h, len(ids), _ptr(ids), _ptr(lengths),
+                                     _ptr(arrival), _ptr(deadline)))
+
+    def next_batch(self, now: float, with_plan: bool = True):
+        cap = max(self._cap, self.B * self.L)          # a batch holds at most B*L requests
+        ids = np.zeros(cap, np.int64)
+        lens = np.zeros(cap, np.int32)
+        n = ctypes.c_int32(0)
+        h = ctypes.c_void_p()
+        check(lib().tcb_sched_next_batch(self._h, float(now), _ptr(ids), _ptr(lens), cap,
+                                         ctypes.byref(n), ctypes.byref(h) if with_plan else None))
+        k = int(n.value)
+        return ids[:k], lens[:k], (Plan(h) if with_plan else None)
+
+    def stats(self) -> Dict[str, float]:
+        st = _lib.SchedStats()
+        check(lib().tcb_sched_stats_get(self._h, ctypes.byref(st)))
+        return st.as_dict()
 
 
 def launch_count() -> int:

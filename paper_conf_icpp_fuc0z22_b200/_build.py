@@ -14,7 +14,7 @@ NVCC = os.environ.get("NVCC", "/usr/local/cuda/bin/nvcc")
 ARCH = ["-gencode", "arch=compute_100a,code=sm_100a"]
 FLAGS = ["-O3", "-std=c++17", "-lineinfo", "-Xcompiler", "-fPIC,-Wall", "--expt-relaxed-constexpr",
          "-Xptxas", "-warn-spills"]
-SOURCES = ["pack.cpp", "api.cu", "elementwise.cu", "linear_f32.cu", "linear_tc.cu",
+SOURCES = ["pack.cpp", "sched.cpp", "api.cu", "elementwise.cu", "linear_f32.cu", "linear_tc.cu",
            "attention.cu", "attention_tc.cu"]
 
 

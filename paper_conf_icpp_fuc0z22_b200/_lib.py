@@ -28,7 +28,10 @@ EXPORTS = ["tcb_last_error", "tcb_version", "tcb_pack", "tcb_pack_slotted", "tcb
            "tcb_plan_write_segtab", "tcb_weights_count", "tcb_weights_create",
            "tcb_weights_destroy", "tcb_workspace_size", "tcb_embed", "tcb_encoder_forward",
            "tcb_unpack", "tcb_launch_count", "tcb_profile_enable", "tcb_profile_collect",
-           "tcb_op_linear", "tcb_op_linear_ln", "tcb_op_attention", "tcb_op_layernorm"]
+           "tcb_op_linear", "tcb_op_linear_ln", "tcb_op_attention", "tcb_op_layernorm",
+           "tcb_sched_batch", "tcb_sched_create", "tcb_sched_destroy", "tcb_sched_submit",
+           "tcb_sched_next_batch", "tcb_sched_stats_get"]
+SCHED_POLICIES = {"das": 0, "fcfs": 1, "sjf": 2, "def": 3}
 
 
 class TcbError(RuntimeError):
@@ -46,6 +49,15 @@ class PlanInfo(ctypes.Structure):
                 ("kv_tiles_visited", ctypes.c_int64), ("kv_tiles_dense", ctypes.c_int64),
                 ("useful_score_elems", ctypes.c_int64),
                 ("executed_score_elems", ctypes.c_int64)]
+
+    def as_dict(self):
+        return {f: getattr(self, f) for f, _ in self._fields_}
+
+
+class SchedStats(ctypes.Structure):
+    _fields_ = [("submitted", ctypes.c_int64), ("waiting", ctypes.c_int64),
+                ("scheduled", ctypes.c_int64), ("expired", ctypes.c_int64),
+                ("batches", ctypes.c_int64), ("utility", ctypes.c_double)]
 
     def as_dict(self):
         return {f: getattr(self, f) for f, _ in self._fields_}
@@ -101,6 +113,15 @@ def lib() -> ctypes.CDLL:
         "tcb_op_linear_ln": (I32, [I64, I32, I32, P, P, P, P, P, P, ctypes.c_float, P, P, P]),
         "tcb_op_attention": (I32, [I32, I64, I32, I32, P, P, P, P, P]),
         "tcb_op_layernorm": (I32, [I32, I64, I32, P, P, P, ctypes.c_float, P, P, P]),
+        "tcb_sched_batch": (I32, [I32, P, P, P, P, I32, I32, I32, ctypes.c_double,
+                                  ctypes.c_double, P, P]),
+        "tcb_sched_create": (I32, [I32, I32, I32, ctypes.c_double, ctypes.c_double,
+                                   ctypes.POINTER(P)]),
+        "tcb_sched_destroy": (None, [P]),
+        "tcb_sched_submit": (I32, [P, I32, P, P, P, P]),
+        "tcb_sched_next_batch": (I32, [P, ctypes.c_double, P, P, I32, ctypes.POINTER(I32),
+                                       ctypes.POINTER(P)]),
+        "tcb_sched_stats_get": (I32, [P, ctypes.POINTER(SchedStats)]),
     }
     for name, (res, args) in sig.items():
         fn = getattr(L, name)

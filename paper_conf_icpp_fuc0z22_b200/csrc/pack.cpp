@@ -143,6 +143,8 @@ tcb_status validate_pack(const char* fn, const int32_t* lengths, int32_t n, int3
   return TCB_OK;
 }
 
+}  // namespace
+
 void init_plan(tcb_plan* p, const int32_t* lengths, int32_t n, int32_t row_len, int32_t max_rows,
                int32_t policy) {
   p->n = n;
@@ -174,7 +176,6 @@ void finish_plan(tcb_plan* p) {
   p->info.slot_len = p->slot_len;
 }
 
-}  // namespace
 }  // namespace tcb
 
 using tcb::fail;

@@ -15,12 +15,21 @@ constexpr int kAttnQBlock = 128;   // query slots per CTA (8 warps x 16 rows)
 constexpr int kAttnWarpRows = 16;  // query rows per warp (one m16 MMA tile)
 constexpr int kAttnKSub = 16;      // keys per skip decision (one k16 MMA step of P.V)
 
+struct tcb_plan;
+
 namespace tcb {
 
 // Error reporting -------------------------------------------------------------------------
 void set_error(const std::string& msg);
 void clear_error();
 tcb_status fail(tcb_status st, const std::string& msg);
+
+// Plan construction (pack.cpp): init_plan sets the request arrays (all unplaced);
+// finish_plan derives the segments in (row, column) order from req_row / req_col and the
+// counters.  Every plan producer (tcb_pack, tcb_pack_slotted, the scheduler) uses them.
+void init_plan(tcb_plan* p, const int32_t* lengths, int32_t n, int32_t row_len, int32_t max_rows,
+               int32_t policy);
+void finish_plan(tcb_plan* p);
 
 // Segment-table record (16 bytes), see tcb.h "device form of a plan".
 struct SegRec {
