@@ -281,33 +281,43 @@ attn_tc_kernel(const __grid_constant__ CUtensorMap tmQKV, const int32_t* __restr
     }
   } else if (warp == 1) {
     // ================= MMA issuer =================
-    int qs = 0, ks = 0, ks_prev = 0;
+    // Flat software pipeline over all chunks of all items: S = Q K^T of chunk g is issued
+    // before P V of chunk g-1 waits for its P, also across item boundaries, so the softmax
+    // warps find the next S ready when they finish a chunk.
+    int qs = 0, ks = 0;
     uint32_t qph = 0, kph = 0;
     uint32_t gc = 0;            // global chunk counter (S / P double buffers)
-    uint32_t it = 0;            // items with at least one chunk (O reuse)
+    uint32_t it = 0;            // items with at least one chunk (O double buffer)
+    struct Pend {
+      uint32_t gc, it;
+      int stage;
+      bool first, last, valid;
+    } pend{0, 0, 0, false, false, false};
+    auto issue_pv = [&](const Pend& pp) {
+      const uint32_t b = pp.gc & 1, u = pp.gc >> 1;
+      mbar_wait(p_full + 8 * b, u & 1);
+      if (pp.first) mbar_wait(o_empty + 8 * (pp.it & 1), ((pp.it >> 1) & 1) ^ 1);
+      tc_fence_after();
+      if (lane == 0) {
+        const uint32_t pa = sP + b * kPBytes, va = sV + pp.stage * kTileBytes;
+#pragma unroll
+        for (int k = 0; k < TK / 16; ++k) {
+          const uint32_t a_addr = pa + (k >> 2) * kTileBytes + (k & 3) * 32;
+          tc_mma(tmem + 256 + (pp.it & 1) * 64, desc_kmajor(a_addr), desc_mnmajor(va + k * 2048),
+                 kIdescPV, (!pp.first || k > 0) ? 1u : 0u);
+        }
+        tc_commit(p_empty + 8 * b);
+        tc_commit(kv_empty + 8 * pp.stage);
+        if (pp.last) tc_commit(o_full + 8 * (pp.it & 1));
+      }
+      __syncwarp();
+    };
     for (int item = blockIdx.x; item < num_items; item += gridDim.x) {
       mbar_wait(q_full + 8 * qs, qph);
       const int nch = infos[qs].nch;
       const uint32_t qaddr = sQ + qs * kTileBytes;
       tc_fence_after();
-      auto pv = [&](uint32_t c_glob, int stage, bool first) {
-        const uint32_t b = c_glob & 1, u = c_glob >> 1;
-        mbar_wait(p_full + 8 * b, u & 1);
-        if (first) mbar_wait(o_empty + 8 * (it & 1), ((it >> 1) & 1) ^ 1);
-        tc_fence_after();
-        if (lane == 0) {
-          const uint32_t pa = sP + b * kPBytes, va = sV + stage * kTileBytes;
-#pragma unroll
-          for (int k = 0; k < TK / 16; ++k) {
-            const uint32_t a_addr = pa + (k >> 2) * kTileBytes + (k & 3) * 32;
-            tc_mma(tmem + 256 + (it & 1) * 64, desc_kmajor(a_addr), desc_mnmajor(va + k * 2048), kIdescPV,
-                   (!first || k > 0) ? 1u : 0u);
-          }
-          tc_commit(p_empty + 8 * b);
-          tc_commit(kv_empty + 8 * stage);
-        }
-        __syncwarp();
-      };
+      if (nch == 0 && lane == 0) mbar_arrive(q_empty + 8 * qs);
       for (int c = 0; c < nch; ++c) {
         const uint32_t b = gc & 1, u = gc >> 1;
         mbar_wait(kv_full + 8 * ks, kph);
@@ -323,21 +333,15 @@ attn_tc_kernel(const __grid_constant__ CUtensorMap tmQKV, const int32_t* __restr
           if (c == nch - 1) tc_commit(q_empty + 8 * qs);
         }
         __syncwarp();
-        if (c > 0) pv(gc - 1, ks_prev, c == 1);
-        ks_prev = ks;
+        if (pend.valid) issue_pv(pend);
+        pend = Pend{gc, it, ks, c == 0, c == nch - 1, true};
         if (++ks == kKVStages) { ks = 0; kph ^= 1; }
         ++gc;
       }
-      if (nch > 0) {
-        pv(gc - 1, ks_prev, nch == 1);
-        if (lane == 0) tc_commit(o_full + 8 * (it & 1));
-        __syncwarp();
-        ++it;
-      } else if (lane == 0) {
-        mbar_arrive(q_empty + 8 * qs);
-      }
+      if (nch > 0) ++it;
       if (++qs == kQStages) { qs = 0; qph ^= 1; }
     }
+    if (pend.valid) issue_pv(pend);
   } else if (warp >= 4) {
     // ================= softmax + epilogue =================
     const int sw = warp - 4;
