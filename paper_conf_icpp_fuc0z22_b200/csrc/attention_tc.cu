@@ -317,7 +317,16 @@ attn_tc_kernel(const __grid_constant__ CUtensorMap tmQKV, const int32_t* __restr
       const int nch = infos[qs].nch;
       const uint32_t qaddr = sQ + qs * kTileBytes;
       tc_fence_after();
-      if (nch == 0 && lane == 0) mbar_arrive(q_empty + 8 * qs);
+      if (nch == 0) {
+        // An empty item must not hold back the pending P V: the softmax warps are waiting
+        // for it (deferred epilogue of the previous item) and would stop releasing Q slots,
+        // so a run of more than kQStages empty items would deadlock the Q ring.
+        if (pend.valid) {
+          issue_pv(pend);
+          pend.valid = false;
+        }
+        if (lane == 0) mbar_arrive(q_empty + 8 * qs);
+      }
       for (int c = 0; c < nch; ++c) {
         const uint32_t b = gc & 1, u = gc >> 1;
         mbar_wait(kv_full + 8 * ks, kph);

@@ -175,6 +175,46 @@ def test_attention_bf16_running_max_rescale():
         assert e <= 2e-2, (s_, e)
 
 
+def test_attention_bf16_long_runs_of_empty_query_blocks():
+    """NaiveBatching layout (R17) with one 512-token request: every other row is a short
+    request followed by ~490 pad slots, so most 128-slot query blocks are empty and each
+    persistent CTA meets long runs of empty items between items with work (regression: the
+    MMA issuer held the previous item's last P V back across them and deadlocked the Q ring).
+    Per-request outputs vs the oracle on the First-Fit layout of the same requests (P4)."""
+    rng = np.random.default_rng(23)
+    n, d, h = 300, 256, 4
+    lengths = np.concatenate([[512], rng.integers(3, 41, n - 1)]).astype(np.int32)
+    T = int(lengths.sum())
+    cu = np.concatenate([[0], np.cumsum(lengths)])
+    tok = _bf16(rng.normal(size=(T, 3 * d)).astype(np.float32))
+
+    def scatter(plan):
+        a = plan.arrays()
+        L = plan.info["row_len"]
+        x = np.zeros((plan.num_slots, 3 * d), np.float32)
+        for r in range(n):
+            s0 = a["req_row"][r] * L + a["req_col"][r]
+            x[s0:s0 + lengths[r]] = tok[cu[r]:cu[r + 1]]
+        return a, x
+
+    naive = tcb.tcb_pack(lengths, 512, 0, "naive")
+    a_n, x_n = scatter(naive)
+    out = tcb.op_attention(_dev(x_n, torch.bfloat16), _dev(a_n["segment_ids"]),
+                           _dev(naive.segtab()), h)
+    torch.cuda.synchronize()
+    got = out.float().cpu().numpy()
+    ff = tcb.tcb_pack(lengths, 512, 0)
+    a_f, x_f = scatter(ff)
+    ref = oracle.attention(x_f, a_f["segment_ids"], ff.info["num_rows"], 512, d, h)
+    for r in range(n):
+        g0 = a_n["req_row"][r] * 512 + a_n["req_col"][r]
+        f0 = a_f["req_row"][r] * 512 + a_f["req_col"][r]
+        g, o = got[g0:g0 + lengths[r]], ref[f0:f0 + lengths[r]]
+        e = np.max(np.abs(g - o)) / np.max(np.abs(o))
+        assert e <= 1.5e-2, (r, e)
+    assert np.all(got[a_n["segment_ids"] < 0] == 0)
+
+
 def test_attention_f32_vs_oracle():
     lengths = wl.draw_lengths("uniform_3_16", 8, 0)
     got, ref, seg = _attn_case(lengths, 32, 64, 2, "fp32", 2)
