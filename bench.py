@@ -16,8 +16,10 @@ value: device time (CUDA events on the launching stream), inputs resident in HBM
 e2e:   the same metric through the public API from host memory: per step tcb_pack (C++),
        H2D of the segment table + token ids from pinned memory, forward, unpack, D2H of the
        per-request outputs [T, d] into pinned memory; host wall clock, synchronised.
-roofline: the dominant kernel (the tcgen05 GEMM class) measured live with CUDA events
-       around each launch (tcb_profile_*), algorithmic flops = 24 d^2 S T per forward.
+roofline: the dominant kernel class (largest device time per step) measured live with CUDA
+       events around each launch (tcb_profile_*); algorithmic flops / bytes per class in
+       DESIGN.md section 7 (GEMMs: 2 T d_in d_out per layer over non-pad tokens T); every
+       class is listed under roofline.classes.
 cpu_baseline / --impl reference: the float64 oracle (oracle/, test infrastructure) on a
        bounded sample of the same workload, on this host's cores.
 """
@@ -51,29 +53,64 @@ def _peaks():
 
 
 class ClockSampler:
-    """nvidia-smi clocks / throttle reasons sampled during the timed region."""
+    """SM clocks / throttle reasons sampled DURING the timed region: NVML every 2 ms
+    (nvidia_ml_py), else nvidia-smi every 0.2 s."""
 
     Q = ("index,clocks.sm,clocks.max.sm,power.draw,clocks_event_reasons.active,"
          "clocks_event_reasons.hw_slowdown,clocks_event_reasons.hw_thermal_slowdown,"
          "clocks_event_reasons.sw_thermal_slowdown,clocks_event_reasons.sw_power_cap")
+    NAMES = ["hw_slowdown", "hw_thermal_slowdown", "sw_thermal_slowdown", "sw_power_cap"]
 
     def __init__(self, gpu: int):
         self.gpu = gpu
-        self.rows = []
+        self.rows = []          # (sm_mhz, max_mhz, power_w, set(reasons))
+        self.source = None
         self._stop = threading.Event()
         self._t = None
+        self._nvml = None
+        try:
+            import pynvml
+            pynvml.nvmlInit()
+            self._nvml = pynvml
+            self._h = pynvml.nvmlDeviceGetHandleByIndex(gpu)
+            self._max = pynvml.nvmlDeviceGetMaxClockInfo(self._h, pynvml.NVML_CLOCK_SM)
+            self.source = "nvml"
+        except Exception:
+            self._nvml = None
+
+    def _sample_nvml(self):
+        nv = self._nvml
+        sm = nv.nvmlDeviceGetClockInfo(self._h, nv.NVML_CLOCK_SM)
+        try:
+            pw = nv.nvmlDeviceGetPowerUsage(self._h) / 1000.0
+        except Exception:
+            pw = None
+        bits = nv.nvmlDeviceGetCurrentClocksEventReasons(self._h)
+        masks = [0x8, 0x40, 0x20, 0x4]   # hw_slowdown, hw_thermal, sw_thermal, sw_power_cap
+        reasons = {n for n, m in zip(self.NAMES, masks) if bits & m}
+        self.rows.append((float(sm), float(self._max), pw, reasons))
+
+    def _sample_smi(self):
+        out = subprocess.run(["nvidia-smi", "-i", str(self.gpu), f"--query-gpu={self.Q}",
+                              "--format=csv,noheader,nounits"],
+                             capture_output=True, text=True, timeout=5).stdout
+        for line in out.strip().splitlines():
+            r = [x.strip() for x in line.split(",")]
+            num = lambda x: float(x) if x.replace(".", "").isdigit() else None  # noqa: E731
+            reasons = {self.NAMES[i] for i in range(4) if len(r) > 5 + i and r[5 + i].lower() == "active"}
+            self.rows.append((num(r[1]), num(r[2]), num(r[3]), reasons))
+        self.source = "nvidia-smi"
 
     def _run(self):
         while not self._stop.is_set():
             try:
-                out = subprocess.run(["nvidia-smi", "-i", str(self.gpu),
-                                      f"--query-gpu={self.Q}", "--format=csv,noheader,nounits"],
-                                     capture_output=True, text=True, timeout=5).stdout
-                for line in out.strip().splitlines():
-                    self.rows.append([x.strip() for x in line.split(",")])
+                if self._nvml is not None:
+                    self._sample_nvml()
+                else:
+                    self._sample_smi()
             except Exception:
                 pass
-            self._stop.wait(0.2)
+            self._stop.wait(0.002 if self._nvml is not None else 0.2)
 
     def __enter__(self):
         self._t = threading.Thread(target=self._run, daemon=True)
@@ -87,17 +124,16 @@ class ClockSampler:
 
     def summary(self):
         if not self.rows:
-            return {"sm_mhz": None, "sm_max_mhz": None, "reasons": ["nvidia-smi unavailable"],
+            return {"sm_mhz": None, "sm_max_mhz": None, "reasons": ["clock sampling unavailable"],
                     "samples": 0}
-        sm = [float(r[1]) for r in self.rows if r[1].replace(".", "").isdigit()]
-        mx = [float(r[2]) for r in self.rows if r[2].replace(".", "").isdigit()]
-        names = ["hw_slowdown", "hw_thermal_slowdown", "sw_thermal_slowdown", "sw_power_cap"]
-        reasons = sorted({names[i] for r in self.rows for i in range(4)
-                          if len(r) > 5 + i and r[5 + i].lower() == "active"})
-        pw = [float(r[3]) for r in self.rows if r[3].replace(".", "").isdigit()]
+        sm = [r[0] for r in self.rows if r[0] is not None]
+        mx = [r[1] for r in self.rows if r[1] is not None]
+        pw = [r[2] for r in self.rows if r[2] is not None]
+        reasons = sorted(set().union(*[r[3] for r in self.rows]))
         return {"sm_mhz": float(np.median(sm)) if sm else None,
                 "sm_max_mhz": max(mx) if mx else None, "reasons": reasons,
-                "power_w_max": max(pw) if pw else None, "samples": len(self.rows)}
+                "power_w_max": max(pw) if pw else None, "samples": len(self.rows),
+                "source": self.source}
 
 
 def make_batches(key: str, rank: int, nbatches: int):
@@ -181,7 +217,7 @@ def run_reference(args):
 def main():
     ap = argparse.ArgumentParser()
     ap.add_argument("--gpus", type=int, default=1)
-    ap.add_argument("--steps", type=int, default=20)
+    ap.add_argument("--steps", type=int, default=50)
     ap.add_argument("--warmup", type=int, default=5)
     ap.add_argument("--impl", default="ours", choices=["ours", "reference"])
     ap.add_argument("--workload", default="c2", choices=sorted(wl.WORKLOADS))
@@ -297,30 +333,65 @@ def main():
     prof = tcb.profile_collect()
     tcb.profile_enable(False)
     peaks, peak_src = _peaks()
-    d, S = model.d_model, model.num_layers
+    d, S, f = model.d_model, model.num_layers, model.d_ff
+    T = tokens_rank
     gemm_cls = ["gemm_qkv", "gemm_o", "gemm_ffn1", "gemm_ffn2"]
-    gemm_ms = sum(prof[c][0] for c in gemm_cls) / args.steps
-    gemm_launches = sum(prof[c][1] for c in gemm_cls) / args.steps
-    total_prof_ms = sum(v[0] for v in prof.values()) / args.steps
-    gemm_flops = 2.0 * tokens_rank * S * (3 * d * d + d * d + 2 * d * model.d_ff)
+    gemm_flops = 2.0 * T * S * (3 * d * d + d * d + 2 * d * f)
     attn_flops = 4.0 * d * S * info["useful_score_elems"]
-    achieved_tf = gemm_flops / (gemm_ms / 1e3) / 1e12
-    peak_tf = peaks.get("bf16_tflops_sustained", peaks["bf16_tflops"])
+    tc_peak = peaks.get("bf16_tflops_sustained", peaks["bf16_tflops"])
+    hbm_peak = peaks["hbm_gbs"]
+    esz = 2 if model.dtype == "bf16" else 4
+    fused_ln = d == 512 and model.dtype == "bf16"
+    # algorithmic work per forward of each kernel class: flops for the
+    # contractions (non-pad tokens only), bytes for the HBM-bound kernels
+    work = {
+        "gemm_qkv": ("tensor", 2.0 * T * S * 3 * d * d),
+        "gemm_o": ("tensor", 2.0 * T * S * d * d),
+        "gemm_ffn1": ("tensor", 2.0 * T * S * d * f),
+        "gemm_ffn2": ("tensor", 2.0 * T * S * d * f),
+        "attention": ("tensor", attn_flops),
+        "embed": ("hbm", T * (4 + 2 * d * esz + 8)),
+        "layernorm": ("hbm", 0.0 if fused_ln else 2.0 * S * T * 2 * d * esz),
+        "unpack": ("hbm", T * 2 * d * esz),
+    }
+    names = {"gemm_qkv": "linear_tc_kernel<2,256,EPI_BIAS> (QKV)",
+             "gemm_o": "linear_ln_kernel (W_O + residual + LN1)" if fused_ln else "linear_tc_kernel (W_O + residual)",
+             "gemm_ffn1": "linear_tc_kernel<2,256,EPI_ACT> (FFN1 + act)",
+             "gemm_ffn2": "linear_ln_kernel (FFN2 + residual + LN2)" if fused_ln else "linear_tc_kernel (FFN2 + residual)",
+             "attention": "attn_tc_kernel (segment-masked attention, useful flops)",
+             "embed": "pack_embed_kernel", "layernorm": "layernorm_kernel", "unpack": "unpack_kernel"}
+    classes = {}
+    for c, (bound, w) in work.items():
+        ms_c, n_c = prof.get(c, (0.0, 0))
+        if n_c == 0 or ms_c <= 0 or w <= 0:
+            continue
+        w_all = w * args.steps                      # prof times cover args.steps forwards
+        if bound == "tensor":
+            ach, pk, unit = w_all / (ms_c / 1e3) / 1e12, tc_peak, "TFLOP/s"
+        else:
+            ach, pk, unit = w_all / (ms_c / 1e3) / 1e9, hbm_peak, "GB/s"
+        classes[c] = {"kernel": names[c], "bound": bound, "achieved": ach, "peak": pk, "unit": unit,
+                      "frac": ach / pk, "launches_per_step": n_c / args.steps,
+                      "ms_per_step": ms_c / args.steps,
+                      "us_per_launch": 1e3 * ms_c / n_c}
+    dom = max(classes, key=lambda c: classes[c]["ms_per_step"])
     traffic = None
     tpath = os.path.join(ROOT, "profiles", "traffic.json")
     if os.path.exists(tpath):
         try:
-            traffic = json.load(open(tpath)).get(key, {}).get("gemm_dram_bytes_per_launch")
+            traffic = json.load(open(tpath)).get(key, {}).get(dom)
         except Exception:
             traffic = None
-    roofline = {"bound": "tensor", "kernel": "linear_tc_kernel (tcgen05 GEMMs: QKV, W_O, FFN1, FFN2)",
-                "achieved": achieved_tf, "peak": peak_tf, "unit": "TFLOP/s",
-                "frac": achieved_tf / peak_tf, "traffic": traffic,
-                "peak_source": f"{peak_src} bf16_tflops_sustained (kernel timed inside a long step)",
-                "frac_of_burst_peak": achieved_tf / peaks["bf16_tflops"],
-                "gemm_share_of_step": gemm_ms / total_prof_ms if total_prof_ms else None,
-                "launches_per_step": gemm_launches,
-                "per_class_ms_per_step": {k: v[0] / args.steps for k, v in prof.items()}}
+    total_prof_ms = sum(v[0] for v in prof.values()) / args.steps
+    dc = classes[dom]
+    roofline = {"bound": dc["bound"], "kernel": dc["kernel"], "class": dom,
+                "achieved": dc["achieved"], "peak": dc["peak"], "unit": dc["unit"],
+                "frac": dc["frac"], "traffic": traffic,
+                "peak_source": f"{peak_src} " + ("bf16_tflops_sustained (kernel timed inside a long step)"
+                                                 if dc["bound"] == "tensor" else "hbm_gbs"),
+                "share_of_step": dc["ms_per_step"] / total_prof_ms if total_prof_ms else None,
+                "gemm_class_frac": (gemm_flops / (sum(prof[c][0] for c in gemm_cls) / args.steps / 1e3) / 1e12) / tc_peak,
+                "classes": classes}
     whole_tc = (gemm_flops + attn_flops) / (ms_per_step / 1e3) / 1e12
 
     # ---- e2e: public API from host memory, every step -------------------------------------

@@ -235,6 +235,8 @@ attn_tc_kernel(const __grid_constant__ CUtensorMap tmQKV, const int32_t* __restr
   __syncthreads();
   tc_fence_after();
   const uint32_t tmem = *tmem_slot;           // S0: +0, S1: +128, O: +256
+  pdl_wait();                                 // QKV / segment ids come from earlier kernels
+  pdl_trigger();
 
   if (warp == 0) {
     // ================= item metadata + Q tile =================
@@ -624,10 +626,9 @@ cudaError_t launch_attention_bf16_tc(int64_t num_slots, int d_model, int num_hea
   const int items = static_cast<int>(qblocks * num_heads);
   const unsigned grid = static_cast<unsigned>(items < sms ? items : sms);
   const float scale_log2 = 1.4426950408889634f / sqrtf(static_cast<float>(DH));
-  attn_tc_kernel<<<grid, kThreads, kSmemBytes, s>>>(map, seg_ids, segtab,
-                                                    static_cast<__nv_bfloat16*>(O), num_slots,
-                                                    d_model, num_heads, items, scale_log2);
-  return cudaGetLastError();
+  return launch_ex(attn_tc_kernel, dim3(grid), dim3(kThreads), kSmemBytes, s, 1, map, seg_ids,
+                   segtab, static_cast<__nv_bfloat16*>(O), num_slots, d_model, num_heads, items,
+                   scale_log2);
 }
 
 }  // namespace k

@@ -67,6 +67,8 @@ __global__ void __launch_bounds__(kWarpsPerBlock * 32) pack_embed_kernel(EmbedAr
   extern __shared__ int4 row_recs[];
   const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
   const int row = blockIdx.x;
+  pdl_wait();
+  pdl_trigger();
   const int S = a.segtab[0].x;
   const int* row_first = reinterpret_cast<const int*>(a.segtab + 1 + S);
   const int f = __ldg(&row_first[row]);
@@ -192,6 +194,8 @@ layernorm_kernel(int64_t rows, int d, const T* __restrict__ Z, const float* __re
   const int lane = threadIdx.x & 31;
   const int64_t row0 =
       (static_cast<int64_t>(blockIdx.x) * kWarpsPerBlock + (threadIdx.x >> 5)) * kLnRows;
+  pdl_wait();
+  pdl_trigger();
   if (row0 >= rows) return;
   const int nvec = d / V;
   float v[kLnRows][NV][V];
@@ -260,6 +264,8 @@ __global__ void __launch_bounds__(kWarpsPerBlock * 32)
 unpack_kernel(const int4* __restrict__ segtab, int row_len, int row_bytes_per_slot,
               const uint8_t* __restrict__ rows, uint8_t* __restrict__ out) {
   const int row = blockIdx.x;
+  pdl_wait();
+  pdl_trigger();
   const int S = segtab[0].x;
   const int* row_first = reinterpret_cast<const int*>(segtab + 1 + S);
   const int f = __ldg(&row_first[row]), e = __ldg(&row_first[row + 1]);
@@ -327,24 +333,25 @@ cudaError_t launch_embed(int dtype, const EmbedArgs& a, cudaStream_t s) {
   // <= row_len segment records + type embedding, LN gamma, LN beta (fp32, d each)
   const size_t smem = static_cast<size_t>(a.row_len) * sizeof(int4) + 3 * sizeof(float) * a.d;
   const int nv = (a.d / (dtype == 0 ? 4 : 8) + 31) / 32;
-  cudaError_t attr_err = cudaSuccess;
+  cudaError_t attr_err = cudaSuccess, launch_err = cudaSuccess;
   auto go = [&](auto tag) {
     constexpr int NV = decltype(tag)::value;
     if (dtype == 0) {
       if (smem > 48 * 1024)
         attr_err = cudaFuncSetAttribute(pack_embed_kernel<float, NV>,
                                         cudaFuncAttributeMaxDynamicSharedMemorySize, static_cast<int>(smem));
-      pack_embed_kernel<float, NV><<<grid, kWarpsPerBlock * 32, smem, s>>>(a);
+      launch_err = launch_ex(pack_embed_kernel<float, NV>, grid, dim3(kWarpsPerBlock * 32), smem, s, 1, a);
     } else {
       if (smem > 48 * 1024)
         attr_err = cudaFuncSetAttribute(pack_embed_kernel<__nv_bfloat16, NV>,
                                         cudaFuncAttributeMaxDynamicSharedMemorySize, static_cast<int>(smem));
-      pack_embed_kernel<__nv_bfloat16, NV><<<grid, kWarpsPerBlock * 32, smem, s>>>(a);
+      launch_err = launch_ex(pack_embed_kernel<__nv_bfloat16, NV>, grid, dim3(kWarpsPerBlock * 32), smem, s,
+                             1, a);
     }
   };
   if (!dispatch_nv(nv, go)) return cudaErrorInvalidValue;
   if (attr_err != cudaSuccess) return attr_err;
-  return cudaGetLastError();
+  return launch_err;
 }
 
 cudaError_t launch_layernorm(int dtype, int64_t rows, int d, const void* Z, const float* g,
@@ -354,18 +361,20 @@ cudaError_t launch_layernorm(int dtype, int64_t rows, int d, const void* Z, cons
   const int64_t per_block = static_cast<int64_t>(kWarpsPerBlock) * kLnRows;
   const unsigned grid = static_cast<unsigned>((rows + per_block - 1) / per_block);
   const int nv = (d / (dtype == 0 ? 4 : 8) + 31) / 32;
+  cudaError_t err = cudaSuccess;
   auto go = [&](auto tag) {
     constexpr int NV = decltype(tag)::value;
     if (dtype == 0)
-      layernorm_kernel<float, NV><<<grid, kWarpsPerBlock * 32, 0, s>>>(
-          rows, d, static_cast<const float*>(Z), g, b, eps, seg_ids, static_cast<float*>(Y));
+      err = launch_ex(layernorm_kernel<float, NV>, dim3(grid), dim3(kWarpsPerBlock * 32), 0, s, 1,
+                      rows, d, static_cast<const float*>(Z), g, b, eps, seg_ids,
+                      static_cast<float*>(Y));
     else
-      layernorm_kernel<__nv_bfloat16, NV><<<grid, kWarpsPerBlock * 32, 0, s>>>(
-          rows, d, static_cast<const __nv_bfloat16*>(Z), g, b, eps, seg_ids,
-          static_cast<__nv_bfloat16*>(Y));
+      err = launch_ex(layernorm_kernel<__nv_bfloat16, NV>, dim3(grid), dim3(kWarpsPerBlock * 32), 0,
+                      s, 1, rows, d, static_cast<const __nv_bfloat16*>(Z), g, b, eps, seg_ids,
+                      static_cast<__nv_bfloat16*>(Y));
   };
   if (!dispatch_nv(nv, go)) return cudaErrorInvalidValue;
-  return cudaGetLastError();
+  return err;
 }
 
 cudaError_t launch_unpack(int dtype, const int4* segtab, int num_rows, int row_len, int d,
@@ -373,9 +382,8 @@ cudaError_t launch_unpack(int dtype, const int4* segtab, int num_rows, int row_l
   if (num_rows == 0) return cudaSuccess;
   const int bytes_per_slot = d * (dtype == 0 ? 4 : 2);
   const dim3 grid(static_cast<unsigned>(num_rows), static_cast<unsigned>((row_len + kRowChunk - 1) / kRowChunk));
-  unpack_kernel<<<grid, kWarpsPerBlock * 32, 0, s>>>(
-      segtab, row_len, bytes_per_slot, static_cast<const uint8_t*>(rows), static_cast<uint8_t*>(out));
-  return cudaGetLastError();
+  return launch_ex(unpack_kernel, grid, dim3(kWarpsPerBlock * 32), 0, s, 1, segtab, row_len,
+                   bytes_per_slot, static_cast<const uint8_t*>(rows), static_cast<uint8_t*>(out));
 }
 
 cudaError_t launch_pe_table(float* table, int max_pos, int d, int variant, cudaStream_t s) {

@@ -4,9 +4,53 @@
 #include <cuda.h>
 #include <cuda_runtime.h>
 #include <cstdint>
+#include <utility>
 
 namespace tcb {
 namespace k {
+
+// Programmatic dependent launch (PDL).  Every kernel of the forward is launched with
+// programmaticStreamSerialization, so its CTAs can be scheduled (and run their prologue:
+// mbarrier init, TMEM allocation, tensor-map prefetch) as the previous kernel's CTAs retire.
+// Device side, pdl_wait() precedes the first global-memory access (read OR write: the
+// previous kernel may still read a buffer this one overwrites), and pdl_trigger() lets the
+// next kernel launch early.  Without the launch attribute both are no-ops.
+#ifdef __CUDACC__
+__device__ __forceinline__ void pdl_wait() { asm volatile("griddepcontrol.wait;" ::: "memory"); }
+__device__ __forceinline__ void pdl_trigger() {
+  asm volatile("griddepcontrol.launch_dependents;" ::: "memory");
+}
+#endif
+// Host: whether launches carry the PDL attribute (TCB_NO_PDL=1 turns it off), and the
+// attribute itself.
+bool pdl_enabled();
+inline void pdl_attr(cudaLaunchAttribute& a) {
+  a.id = cudaLaunchAttributeProgrammaticStreamSerialization;
+  a.val.programmaticStreamSerializationAllowed = 1;
+}
+// cudaLaunchKernelEx with an optional cluster size and the PDL attribute.
+template <typename... KArgs, typename... Args>
+cudaError_t launch_ex(void (*kern)(KArgs...), dim3 grid, dim3 block, size_t smem,
+                      cudaStream_t s, int cluster, Args&&... args) {
+  cudaLaunchConfig_t cfg{};
+  cfg.gridDim = grid;
+  cfg.blockDim = block;
+  cfg.dynamicSmemBytes = smem;
+  cfg.stream = s;
+  cudaLaunchAttribute attr[2];
+  int n = 0;
+  if (cluster > 1) {
+    attr[n].id = cudaLaunchAttributeClusterDimension;
+    attr[n].val.clusterDim.x = cluster;
+    attr[n].val.clusterDim.y = 1;
+    attr[n].val.clusterDim.z = 1;
+    ++n;
+  }
+  if (pdl_enabled()) pdl_attr(attr[n++]);
+  cfg.attrs = attr;
+  cfg.numAttrs = n;
+  return cudaLaunchKernelEx(&cfg, kern, std::forward<Args>(args)...);
+}
 
 // Embedding / metadata / elementwise (elementwise.cu) -------------------------------------
 struct EmbedArgs {

@@ -317,6 +317,8 @@ linear_tc_kernel(const __grid_constant__ CUtensorMap tmA, const __grid_constant_
   if constexpr (CG == 2) cluster_sync(); else __syncthreads();
   tc_fence_after();
   const uint32_t tmem_base = *tmem_slot;
+  pdl_wait();                 // A / residual come from the previous kernel; C may still be read
+  pdl_trigger();
 
   if (warp == 0) {
     // ===== TMA producer (both CTAs of a pair load their own halves) =====
@@ -629,6 +631,8 @@ linear_ln_kernel(const __grid_constant__ CUtensorMap tmA, const __grid_constant_
   cluster_sync();
   tc_fence_after();
   const uint32_t tmem_base = *tmem_slot;
+  pdl_wait();
+  pdl_trigger();
 
   if (warp == 0) {
     // ===== TMA producer: A rows + the W half (or both halves) each step needs =====
@@ -893,13 +897,14 @@ cudaError_t launch_tc(const GemmMaps& m, int M, int N, int K, const float* bias,
   cfg.blockDim = dim3(kThreads);
   cfg.dynamicSmemBytes = Cfg::kSmemBytes;
   cfg.stream = s;
-  cudaLaunchAttribute attr[1];
+  cudaLaunchAttribute attr[2];
   attr[0].id = cudaLaunchAttributeClusterDimension;
   attr[0].val.clusterDim.x = CG;
   attr[0].val.clusterDim.y = 1;
   attr[0].val.clusterDim.z = 1;
   cfg.attrs = attr;
   cfg.numAttrs = 1;
+  if (pdl_enabled()) pdl_attr(attr[cfg.numAttrs++]);
   static const int raster = std::getenv("TCB_GEMM_RASTER") ? std::atoi(std::getenv("TCB_GEMM_RASTER")) : 8;
   return cudaLaunchKernelEx(&cfg, kern, m.a, m.w, m.c, m.r, M, N, K, bias, raster);
 }
@@ -919,6 +924,14 @@ cudaError_t dispatch_epi(const GemmMaps& m, int M, int N, int K, const float* bi
 }  // namespace
 
 bool linear_ln_supported(int N) { return N == kLnN; }
+
+bool pdl_enabled() {
+  static const bool on = [] {
+    const char* e = std::getenv("TCB_NO_PDL");
+    return !(e && e[0] == '1');
+  }();
+  return on;
+}
 
 cudaError_t launch_linear_ln_bf16_tc(const GemmMaps& m, int64_t M, int N, int K,
                                      const float* bias, const float* gamma, const float* beta,
@@ -950,13 +963,14 @@ cudaError_t launch_linear_ln_bf16_tc(const GemmMaps& m, int64_t M, int N, int K,
   cfg.blockDim = dim3(kLnThreads);
   cfg.dynamicSmemBytes = smem;
   cfg.stream = s;
-  cudaLaunchAttribute attr[1];
+  cudaLaunchAttribute attr[2];
   attr[0].id = cudaLaunchAttributeClusterDimension;
   attr[0].val.clusterDim.x = 2;
   attr[0].val.clusterDim.y = 1;
   attr[0].val.clusterDim.z = 1;
   cfg.attrs = attr;
   cfg.numAttrs = 1;
+  if (pdl_enabled()) pdl_attr(attr[cfg.numAttrs++]);
   return cudaLaunchKernelEx(&cfg, kern, m.a, m.w, m.c, m.r, static_cast<int>(M), K, bias, gamma,
                             beta, eps, seg_ids, split_kb);
 }
