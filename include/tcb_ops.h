@@ -26,7 +26,8 @@ tcb_status tcb_op_linear(int32_t dtype, int64_t M, int32_t N, int32_t K, const v
 /* Fused post-LN residual block (R10): C = LN(A W^T + bias + R) * gamma + beta, row-wise
  * over the N output columns (biased variance, two-pass, fp32) -- tcb_op_linear with
  * TCB_EPI_BIAS_RESIDUAL followed by tcb_op_layernorm in one tcgen05 kernel.  bf16 only and
- * N == 512 (a 2-CTA pair keeps complete 512-column rows in TMEM); K % 64 == 0.  Rows whose
+ * N in {512, 768, 1024} (a cluster of N / 256 CTA pairs owns complete rows, each pair 256
+ * columns in TMEM, row statistics exchanged over DSMEM); K % 64 == 0.  Rows whose
  * d_segment_ids entry is < 0 (pad slots) are written as 0; d_segment_ids may be NULL.
  * Returns TCB_ERR_UNSUPPORTED for other shapes. */
 tcb_status tcb_op_linear_ln(int64_t M, int32_t N, int32_t K, const void* A, const void* W,

@@ -374,8 +374,9 @@ tcb_status tcb_encoder_forward(const tcb_weights* wc, const tcb_plan* plan,
         w->c_M = M;
       }
     }
-    // bias + residual + LayerNorm fused into the W_O / FFN2 GEMMs when a 2-CTA pair can hold
-    // complete rows in TMEM (d == 512); TCB_NO_LN_FUSION=1 forces the unfused kernels.
+    // bias + residual + LayerNorm fused into the W_O / FFN2 GEMMs (d = 512, 768, 1024: a
+    // cluster of d / 256 CTA pairs owns complete rows); TCB_NO_LN_FUSION=1 forces the unfused
+    // kernels.
     static const bool no_fusion = std::getenv("TCB_NO_LN_FUSION") != nullptr;
     const bool fuse_ln = !no_fusion && tcb::k::linear_ln_supported(d);
     for (int l = 0; l < c.num_layers; ++l) {
@@ -503,7 +504,7 @@ tcb_status tcb_op_linear_ln(int64_t M, int32_t N, int32_t K, const void* A, cons
   if (!A || !W || !bias || !R || !gamma || !beta || !C)
     return fail(TCB_ERR_INVALID_ARGUMENT, "tcb_op_linear_ln: NULL pointer");
   if (!tcb::k::linear_ln_supported(N) || K % 64 != 0 || M > INT32_MAX)
-    return fail(TCB_ERR_UNSUPPORTED, "tcb_op_linear_ln: needs N == 512 and K % 64 == 0");
+    return fail(TCB_ERR_UNSUPPORTED, "tcb_op_linear_ln: needs N in {512, 768, 1024} and K % 64 == 0");
   if (tcb_status st = check_device()) return st;
   cudaStream_t s = reinterpret_cast<cudaStream_t>(stream);
   tcb::k::GemmMaps maps;

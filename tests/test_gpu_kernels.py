@@ -51,12 +51,15 @@ def test_linear_bf16_tcgen05_vs_oracle(M, N, K, epi):
     assert np.all(err <= bound), float(np.max(err / bound))
 
 
-@pytest.mark.parametrize("M,K", [(1, 512), (300, 512), (4133, 512), (1000, 1024), (1000, 2048),
-                                 (513, 4096), (32768, 512)])
-def test_linear_ln_fused_vs_oracle(M, K):
-    """W_O / FFN2 + bias + residual + LayerNorm in one tcgen05 kernel (N = 512)."""
-    N = 512
-    rng = np.random.default_rng(M + K)
+@pytest.mark.parametrize("M,K,N", [(1, 512, 512), (300, 512, 512), (4133, 512, 512),
+                                   (1000, 1024, 512), (1000, 2048, 512), (513, 4096, 512),
+                                   (32768, 512, 512), (1, 768, 768), (777, 768, 768),
+                                   (3001, 3072, 768), (300, 1024, 1024), (2049, 4096, 1024),
+                                   (32768, 1024, 1024)])
+def test_linear_ln_fused_vs_oracle(M, K, N):
+    """W_O / FFN2 + bias + residual + LayerNorm in one tcgen05 kernel (N = 512, 768, 1024:
+    clusters of N / 256 CTA pairs exchanging the row statistics over DSMEM)."""
+    rng = np.random.default_rng(M + K + N)
     A = _bf16(rng.normal(size=(M, K)))
     W = _bf16(rng.uniform(-1, 1, size=(N, K)) * np.sqrt(3.0 / K))
     b = _bf16(rng.normal(0, 0.1, size=N))
@@ -76,6 +79,18 @@ def test_linear_ln_fused_vs_oracle(M, K):
     err = np.abs(got[real] - ref[real])
     assert np.all(err <= 2.0 ** -8 * np.abs(ref[real]) + 2e-2), float(err.max())
     assert np.all(got[~real] == 0)
+
+
+def test_linear_ln_cluster_kernel_at_d512():
+    """The cluster kernel also serves N = 512 (TCB_LN_KERNEL=cluster, read once per process):
+    checked in a subprocess so the default (single-pair) choice of this process stays."""
+    import subprocess, sys, os
+    code = ("import sys; sys.path.insert(0, 'tests'); import test_gpu_kernels as t; "
+            "t.test_linear_ln_fused_vs_oracle(4133, 1024, 512); t.test_linear_ln_fused_vs_oracle(1, 512, 512)")
+    env = dict(os.environ, TCB_LN_KERNEL="cluster")
+    r = subprocess.run([sys.executable, "-c", code], env=env, capture_output=True, text=True,
+                       cwd=os.path.dirname(os.path.dirname(os.path.abspath(__file__))), timeout=300)
+    assert r.returncode == 0, r.stderr[-2000:]
 
 
 @pytest.mark.parametrize("M,N,K", [(64, 192, 64), (130, 256, 64), (37, 64, 256)])
