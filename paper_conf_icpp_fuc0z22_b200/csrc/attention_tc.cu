@@ -33,7 +33,8 @@ constexpr int TQ = 128;                 // query slots per item (TMEM lanes)
 constexpr int TK = 128;                 // keys per chunk
 constexpr int DH = 64;                  // head dim
 constexpr int kSmWarps = 8;             // softmax warps (2 per TMEM lane quarter)
-constexpr int kThreads = (4 + kSmWarps) * 32;
+constexpr int kEpWarps = 4;             // output epilogue warps (one per TMEM lane quarter)
+constexpr int kThreads = (4 + kSmWarps + kEpWarps) * 32;
 constexpr int kQStages = 3, kKVStages = 3;
 constexpr int kTileBytes = 128 * DH * 2;            // 16 KB: Q, K or V tile (128 rows x 128 B)
 constexpr int kPBytes = TQ * TK * 2;                // 32 KB: P tile (two 64-key K blocks)
@@ -45,7 +46,7 @@ struct ItemInfo {
 };
 
 constexpr int kSmemBytes = 1024 + kQStages * kTileBytes + 2 * kKVStages * kTileBytes +
-                           2 * kPBytes + kQStages * static_cast<int>(sizeof(ItemInfo)) + 4096;
+                           2 * kPBytes + kQStages * static_cast<int>(sizeof(ItemInfo)) + 6144;
 
 __device__ __forceinline__ uint32_t smem_u32(const void* p) {
   return static_cast<uint32_t>(__cvta_generic_to_shared(p));
@@ -112,6 +113,46 @@ __device__ __forceinline__ void tmem_ld32(uint32_t taddr, uint32_t (&r)[32]) {
       : "r"(taddr)
       : "memory");
 }
+// Two 32-column loads AND the wait in one asm statement: the compiler must not touch the
+// destination registers (e.g. spill them) before tcgen05.wait::ld has completed.
+__device__ __forceinline__ void tmem_ld64_sync(uint32_t taddr, uint32_t (&r)[64]) {
+  asm volatile(
+      "tcgen05.ld.sync.aligned.32x32b.x32.b32 "
+      "{%0,%1,%2,%3,%4,%5,%6,%7,%8,%9,%10,%11,%12,%13,%14,%15,"
+      "%16,%17,%18,%19,%20,%21,%22,%23,%24,%25,%26,%27,%28,%29,%30,%31}, [%64];\n\t"
+      "tcgen05.ld.sync.aligned.32x32b.x32.b32 "
+      "{%32,%33,%34,%35,%36,%37,%38,%39,%40,%41,%42,%43,%44,%45,%46,%47,"
+      "%48,%49,%50,%51,%52,%53,%54,%55,%56,%57,%58,%59,%60,%61,%62,%63}, [%65];\n\t"
+      "tcgen05.wait::ld.sync.aligned;"
+      : "=r"(r[0]), "=r"(r[1]), "=r"(r[2]), "=r"(r[3]), "=r"(r[4]), "=r"(r[5]), "=r"(r[6]),
+        "=r"(r[7]), "=r"(r[8]), "=r"(r[9]), "=r"(r[10]), "=r"(r[11]), "=r"(r[12]),
+        "=r"(r[13]), "=r"(r[14]), "=r"(r[15]), "=r"(r[16]), "=r"(r[17]), "=r"(r[18]),
+        "=r"(r[19]), "=r"(r[20]), "=r"(r[21]), "=r"(r[22]), "=r"(r[23]), "=r"(r[24]),
+        "=r"(r[25]), "=r"(r[26]), "=r"(r[27]), "=r"(r[28]), "=r"(r[29]), "=r"(r[30]),
+        "=r"(r[31]), "=r"(r[32]), "=r"(r[33]), "=r"(r[34]), "=r"(r[35]), "=r"(r[36]),
+        "=r"(r[37]), "=r"(r[38]), "=r"(r[39]), "=r"(r[40]), "=r"(r[41]), "=r"(r[42]),
+        "=r"(r[43]), "=r"(r[44]), "=r"(r[45]), "=r"(r[46]), "=r"(r[47]), "=r"(r[48]),
+        "=r"(r[49]), "=r"(r[50]), "=r"(r[51]), "=r"(r[52]), "=r"(r[53]), "=r"(r[54]),
+        "=r"(r[55]), "=r"(r[56]), "=r"(r[57]), "=r"(r[58]), "=r"(r[59]), "=r"(r[60]),
+        "=r"(r[61]), "=r"(r[62]), "=r"(r[63])
+      : "r"(taddr), "r"(taddr + 32)
+      : "memory");
+}
+__device__ __forceinline__ void tmem_ld32_sync(uint32_t taddr, uint32_t (&r)[32]) {
+  asm volatile(
+      "tcgen05.ld.sync.aligned.32x32b.x32.b32 "
+      "{%0,%1,%2,%3,%4,%5,%6,%7,%8,%9,%10,%11,%12,%13,%14,%15,"
+      "%16,%17,%18,%19,%20,%21,%22,%23,%24,%25,%26,%27,%28,%29,%30,%31}, [%32];\n\t"
+      "tcgen05.wait::ld.sync.aligned;"
+      : "=r"(r[0]), "=r"(r[1]), "=r"(r[2]), "=r"(r[3]), "=r"(r[4]), "=r"(r[5]), "=r"(r[6]),
+        "=r"(r[7]), "=r"(r[8]), "=r"(r[9]), "=r"(r[10]), "=r"(r[11]), "=r"(r[12]),
+        "=r"(r[13]), "=r"(r[14]), "=r"(r[15]), "=r"(r[16]), "=r"(r[17]), "=r"(r[18]),
+        "=r"(r[19]), "=r"(r[20]), "=r"(r[21]), "=r"(r[22]), "=r"(r[23]), "=r"(r[24]),
+        "=r"(r[25]), "=r"(r[26]), "=r"(r[27]), "=r"(r[28]), "=r"(r[29]), "=r"(r[30]),
+        "=r"(r[31])
+      : "r"(taddr)
+      : "memory");
+}
 __device__ __forceinline__ void tmem_wait_ld() { asm volatile("tcgen05.wait::ld.sync.aligned;" ::: "memory"); }
 __device__ __forceinline__ void tmem_st32(uint32_t taddr, const uint32_t (&v)[32]) {
   asm volatile(
@@ -127,6 +168,11 @@ __device__ __forceinline__ void tmem_st32(uint32_t taddr, const uint32_t (&v)[32
 }
 __device__ __forceinline__ void named_bar(int id, int threads) {
   asm volatile("bar.sync %0, %1;" ::"r"(id), "r"(threads) : "memory");
+}
+__device__ __forceinline__ float fmax3(float a, float b, float c) {
+  float d;
+  asm("max.f32 %0, %1, %2, %3;" : "=f"(d) : "f"(a), "f"(b), "f"(c));
+  return d;
 }
 __device__ __forceinline__ float ex2(float x) {
   float y;
@@ -199,8 +245,10 @@ attn_tc_kernel(const __grid_constant__ CUtensorMap tmQKV, const int32_t* __restr
   const uint32_t sP = sV + kKVStages * kTileBytes;             // [2][2 blocks][128 x 64]
   uint8_t* gen = smem_raw + (sP + 2 * kPBytes - raw);
   ItemInfo* infos = reinterpret_cast<ItemInfo*>(gen);          // [3]
-  float* xch = reinterpret_cast<float*>(gen + kQStages * sizeof(ItemInfo));   // [2][128]
-  uint32_t* tmem_slot = reinterpret_cast<uint32_t*>(xch + 6 * TQ);   // [2 bufs][2][128] + l[2][128]
+  float* xch = reinterpret_cast<float*>(gen + kQStages * sizeof(ItemInfo));   // max: [2 bufs][2][128]
+  float* lbuf = xch + 4 * TQ;                                  // row sums: [2 items][2 halves][128]
+  int* meta = reinterpret_cast<int*>(lbuf + 4 * TQ);           // [2 items]: item has an O
+  uint32_t* tmem_slot = reinterpret_cast<uint32_t*>(meta + 4);
   const uint32_t bars = (smem_u32(tmem_slot + 4) + 7) & ~7u;
   const uint32_t q_full = bars, q_empty = q_full + 8 * kQStages;
   const uint32_t kv_full = q_empty + 8 * kQStages, kv_empty = kv_full + 8 * kKVStages;
@@ -208,6 +256,7 @@ attn_tc_kernel(const __grid_constant__ CUtensorMap tmQKV, const int32_t* __restr
   const uint32_t p_full = s_empty + 16, p_empty = p_full + 16;
   const uint32_t o_full = p_empty + 16, o_empty = o_full + 16;   // [2] each (O double buffer)
   const uint32_t info_full = o_empty + 16;                     // [3]
+  const uint32_t l_full = info_full + 8 * kQStages, l_empty = l_full + 16;   // [2] each
 
   const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
   if (threadIdx.x == 0) {
@@ -223,7 +272,12 @@ attn_tc_kernel(const __grid_constant__ CUtensorMap tmQKV, const int32_t* __restr
       mbar_init(p_full + 8 * i, kSmWarps);
       mbar_init(p_empty + 8 * i, 1);
     }
-    for (int i = 0; i < 2; ++i) { mbar_init(o_full + 8 * i, 1); mbar_init(o_empty + 8 * i, kSmWarps); }
+    for (int i = 0; i < 2; ++i) {
+      mbar_init(o_full + 8 * i, 1);
+      mbar_init(o_empty + 8 * i, kEpWarps);
+      mbar_init(l_full + 8 * i, kSmWarps);
+      mbar_init(l_empty + 8 * i, kEpWarps);
+    }
     asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
   }
   if (warp == 2) {
@@ -353,47 +407,41 @@ attn_tc_kernel(const __grid_constant__ CUtensorMap tmQKV, const int32_t* __restr
       if (++qs == kQStages) { qs = 0; qph ^= 1; }
     }
     if (pend.valid) issue_pv(pend);
-  } else if (warp >= 4) {
-    // ================= softmax + epilogue =================
-    const int sw = warp - 4;
-    const int q = warp & 3;                 // TMEM lane quarter
-    const int half = sw >> 2;               // key columns [64*half, 64*half+64) of a chunk
+  } else if (warp >= 4 + kSmWarps) {
+    // ================= output epilogue: O / l -> bf16 -> global =================
+    // Per item (in order): the softmax warps hand over the row sums (and whether the item
+    // had any chunk); O comes from TMEM (double-buffered); pad / empty rows are written 0.
+    const int q = warp & 3;
     const int row = q * 32 + lane;
     const uint32_t lane_off = static_cast<uint32_t>(q * 32) << 16;
-    int qs = 0;
-    uint32_t qph = 0, gc = 0, it = 0;
-#ifdef TCB_ATTN_PROBE
-    long long p_start = clock64(), p_sfull = 0, p_ld = 0, p_max = 0, p_pempty = 0, p_exp = 0, p_q = 0, p_fin = 0;
-#endif
-    // deferred epilogue state (previous item)
-    bool have_prev = false, p_real = false;
-    int p_qb = 0, p_h = 0, p_nch = 0;
-    float p_l = 0.f;
-    uint32_t p_it = 0;
-    auto finish = [&]() {
-      // ---- epilogue: O / l -> bf16 -> global (pad / empty rows -> 0) ----
-      const int64_t grow = static_cast<int64_t>(p_qb) * TQ + row;
-      float* xl = xch + 4 * TQ;              // separate from the per-chunk max exchange
-      xl[half * TQ + row] = p_l;
-      named_bar(1 + q, 64);
-      const float lt = xl[row] + xl[TQ + row];
-      named_bar(1 + q, 64);
-      uint32_t o[32];
-      if (p_nch > 0) {
-        const uint32_t os = p_it & 1;
-        mbar_wait(o_full + 8 * os, (p_it >> 1) & 1);
+    uint32_t oit = 0;
+    int k = 0;
+    for (int item = blockIdx.x; item < num_items; item += gridDim.x, ++k) {
+      const int qb = item / num_heads, h = item % num_heads;
+      const int lb = k & 1;
+      mbar_wait(l_full + 8 * lb, (k >> 1) & 1);
+      const bool has_o = meta[lb] != 0;
+      const float lt = lbuf[(lb * 2) * TQ + row] + lbuf[(lb * 2 + 1) * TQ + row];
+      uint32_t o[64];
+      if (has_o) {
+        const uint32_t os = oit & 1;
+        mbar_wait(o_full + 8 * os, (oit >> 1) & 1);
         tc_fence_after();
-        tmem_ld32(tmem + lane_off + 256 + os * 64 + half * 32, o);
-        tmem_wait_ld();
+        tmem_ld64_sync(tmem + lane_off + 256 + os * 64, o);
         tc_fence_before();
-        __syncwarp();
-        if (lane == 0) mbar_arrive(o_empty + 8 * os);
+        ++oit;
       }
-      const float inv = (p_nch > 0 && p_real && lt > 0.f) ? 1.f / lt : 0.f;
+      __syncwarp();
+      if (lane == 0) {
+        if (has_o) mbar_arrive(o_empty + 8 * (oit - 1 & 1));
+        mbar_arrive(l_empty + 8 * lb);
+      }
+      const float inv = (has_o && lt > 0.f) ? 1.f / lt : 0.f;
+      const int64_t grow = static_cast<int64_t>(qb) * TQ + row;
       if (grow < num_slots) {
-        uint4* dst = reinterpret_cast<uint4*>(O + grow * d_model + p_h * DH + half * 32);
+        uint4* dst = reinterpret_cast<uint4*>(O + grow * d_model + h * DH);
 #pragma unroll
-        for (int t = 0; t < 4; ++t) {
+        for (int t = 0; t < 8; ++t) {
           uint4 x;
           uint32_t* xp = reinterpret_cast<uint32_t*>(&x);
 #pragma unroll
@@ -407,7 +455,20 @@ attn_tc_kernel(const __grid_constant__ CUtensorMap tmQKV, const int32_t* __restr
           dst[t] = x;
         }
       }
-    };
+    }
+  } else if (warp >= 4) {
+    // ================= softmax =================
+    const int sw = warp - 4;
+    const int q = warp & 3;                 // TMEM lane quarter
+    const int half = sw >> 2;               // key columns [64*half, 64*half+64) of a chunk
+    const int row = q * 32 + lane;
+    const uint32_t lane_off = static_cast<uint32_t>(q * 32) << 16;
+    int qs = 0;
+    uint32_t qph = 0, gc = 0, it = 0;
+#ifdef TCB_ATTN_PROBE
+    long long p_start = clock64(), p_sfull = 0, p_ld = 0, p_max = 0, p_pempty = 0, p_exp = 0, p_q = 0, p_fin = 0;
+#endif
+    int ic = 0;                             // items processed (row-sum hand-over buffers)
     for (int item = blockIdx.x; item < num_items; item += gridDim.x) {
       const int qb = item / num_heads, h = item % num_heads;
 #ifdef TCB_ATTN_PROBE
@@ -448,9 +509,7 @@ attn_tc_kernel(const __grid_constant__ CUtensorMap tmQKV, const int32_t* __restr
 #endif
         tc_fence_after();
         uint32_t sr[64];
-        tmem_ld32(tmem + lane_off + b * 128 + half * 64, *reinterpret_cast<uint32_t(*)[32]>(&sr[0]));
-        tmem_ld32(tmem + lane_off + b * 128 + half * 64 + 32, *reinterpret_cast<uint32_t(*)[32]>(&sr[32]));
-        tmem_wait_ld();
+        tmem_ld64_sync(tmem + lane_off + b * 128 + half * 64, sr);
         tc_fence_before();
         __syncwarp();
         if (lane == 0) mbar_arrive(s_empty + 8 * b);
@@ -479,7 +538,8 @@ attn_tc_kernel(const __grid_constant__ CUtensorMap tmQKV, const int32_t* __restr
           if (!live[gi]) continue;
           if (inner[gi]) {
 #pragma unroll
-            for (int j = 32 * gi; j < 32 * gi + 32; ++j) mxp[j & 7] = fmaxf(mxp[j & 7], __uint_as_float(sr[j]));
+            for (int j = 32 * gi; j < 32 * gi + 32; j += 2)
+              mxp[(j >> 1) & 7] = fmax3(mxp[(j >> 1) & 7], __uint_as_float(sr[j]), __uint_as_float(sr[j + 1]));
           } else {
 #pragma unroll
             for (int j = 32 * gi; j < 32 * gi + 32; ++j) {
@@ -516,8 +576,7 @@ attn_tc_kernel(const __grid_constant__ CUtensorMap tmQKV, const int32_t* __restr
           const float f = grow ? ex2((m_used - rmax) * scale_log2) : 1.f;
           uint32_t o[32];
           const uint32_t oaddr = tmem + lane_off + 256 + (it & 1) * 64 + half * 32;
-          tmem_ld32(oaddr, o);
-          tmem_wait_ld();
+          tmem_ld32_sync(oaddr, o);
 #pragma unroll
           for (int t = 0; t < 32; ++t) o[t] = __float_as_uint(__uint_as_float(o[t]) * f);
           tmem_st32(oaddr, o);
@@ -569,25 +628,18 @@ attn_tc_kernel(const __grid_constant__ CUtensorMap tmQKV, const int32_t* __restr
         if (lane == 0) mbar_arrive(p_full + 8 * b);
         ++gc;
       }
-      // the epilogue of the PREVIOUS item runs now, while the MMAs of this item's last chunk
-      // (and the next item's first) proceed -- O is double-buffered in TMEM
-#ifdef TCB_ATTN_PROBE
-      long long tf0 = clock64();
-#endif
-      if (have_prev) finish();
-#ifdef TCB_ATTN_PROBE
-      p_fin += clock64() - tf0;
-#endif
-      have_prev = true;
-      p_qb = qb;
-      p_h = h;
-      p_nch = nch;
-      p_real = rr.y > rr.x;
-      p_l = l;
-      p_it = it;
+      // hand the row sums to the epilogue warps (buffer ic & 1, free once they read item ic-2)
+      {
+        const int lb = ic & 1;
+        if (ic >= 2) mbar_wait(l_empty + 8 * lb, ((ic >> 1) & 1) ^ 1);
+        lbuf[(lb * 2 + half) * TQ + row] = l;
+        if (sw == 0 && lane == 0) meta[lb] = nch > 0 ? 1 : 0;
+        __syncwarp();
+        if (lane == 0) mbar_arrive(l_full + 8 * lb);
+        ++ic;
+      }
       if (nch > 0) ++it;
     }
-    if (have_prev) finish();
 #ifdef TCB_ATTN_PROBE
     if (lane == 0 && blockIdx.x == 0 && (sw == 0 || sw == 5))
       printf("tcprobe warp %d total %lld wait_q %lld wait_s %lld tmem_ld %lld max %lld wait_p %lld exp %lld finish %lld chunks %u\n",
