@@ -288,3 +288,40 @@ def run(model, weights, names, lengths, ids, row_len: int, max_rows: int = 0,
     x = encoder_rows(model, weights, names, ids, lay, row_len)
     out = unpack(x, lay["tok_index"], int(np.sum(lengths)))
     return {"pack": pk, "layout": lay, "rows": x, "out": out}
+
+
+# ---------------------------------------------------------------------------------------
+# f4: decoder (§4.2.2; readings R30-R33).  Plain definition, one request alone.
+# ---------------------------------------------------------------------------------------
+def decoder_stack(model, dec_weights: Dict[str, np.ndarray], dec_names, x, mem) -> np.ndarray:
+    """S decoder layers over one request's embedded target prefix x [t, d] with its encoder
+    output mem [l, d]: causal self-attention, cross-attention, FFN, post-LN each."""
+    cfg = make_cfg(model)
+    arrs, ptrs = _weight_ptrs([dec_weights[n] for n in dec_names])
+    x = _f64(x).copy()
+    mem = _f64(mem)
+    rc = lib().oracle_decoder_stack(ctypes.byref(cfg), ptrs, len(arrs), x.shape[0], mem.shape[0],
+                                    _p(x), _p(mem))
+    if rc != 0:
+        raise OracleError(rc)
+    return x
+
+
+def decode_greedy(model, weights, names, dec_weights, dec_names, src_ids, t_max: int,
+                  bos: int = 1, eos: int = 2, with_logits: bool = False):
+    """Greedy decode of one request alone: tokens y_1.. (stops after EOS or t_max) and,
+    optionally, the logits of every step [n_out, vocab]."""
+    cfg = make_cfg(model)
+    ea, ep = _weight_ptrs([weights[n] for n in names])
+    da, dp = _weight_ptrs([dec_weights[n] for n in dec_names])
+    src = _i32(src_ids)
+    toks = np.zeros(t_max, np.int32)
+    n = ctypes.c_int32(0)
+    lg = np.zeros((t_max, model.vocab), np.float64) if with_logits else None
+    rc = lib().oracle_decode_greedy(ctypes.byref(cfg), ep, len(ea), dp, len(da), model.vocab,
+                                    _p(src), len(src), t_max, bos, eos, _p(toks), ctypes.byref(n),
+                                    _p(lg) if lg is not None else None)
+    if rc != 0:
+        raise OracleError(rc)
+    k = int(n.value)
+    return (toks[:k], lg[:k]) if with_logits else toks[:k]

@@ -528,3 +528,137 @@ void oracle_unpack(const double* x, int32_t num_slots, int32_t d, const int32_t*
     memcpy(out + (int64_t)tok_index[s] * d, x + (int64_t)s * d, sizeof(double) * (size_t)d);
   }
 }
+
+/* ---------------------------------------------------------------------------------------
+ * f4: the decoder of the paper's Seq2Seq setting.  "These embeddings are sent
+ * to the encoder and decoder, each of which contains S layers ... Decoder outputs go
+ * through a final linear layer and activation function to generate final results"
+ * (P:340-351); the decoder "is an auto-regressive model" (§4.2.2).  Readings
+ * R30-R33: standard post-LN decoder layer of [32] (causal self-attention,
+ * cross-attention over the request's OWN encoder output -- the segment-aware form --, FFN),
+ * target tokens embedded like the source (tied E_tok, separate PE restarting at 0 per
+ * request), output projection tied to E_tok without bias, greedy argmax (lowest index on
+ * ties), BOS = 1, EOS = 2, at most t_max generated tokens.
+ * Plain definition: every step recomputes the whole target prefix (no KV cache).
+ * ------------------------------------------------------------------------------------- */
+
+/* softmax(Q K^T / sqrt(dh)) V per head for tq queries over tk keys; causal: query i sees
+ * keys j <= i + causal_off only (masked terms are -inf -> exp = 0 exactly, R11). */
+static void attend(const double* q, int64_t ldq, const double* k, const double* v, int64_t ldkv,
+                   int32_t tq, int32_t tk, int32_t d_model, int32_t num_heads, int32_t causal,
+                   double* o) {
+  const int32_t dh = d_model / num_heads;
+  const double scale = sqrt((double)dh);
+  double* s = (double*)malloc(sizeof(double) * (size_t)(tk > 0 ? tk : 1));
+  for (int32_t h = 0; h < num_heads; ++h) {
+    for (int32_t i = 0; i < tq; ++i) {
+      double m = -INFINITY;
+      for (int32_t j = 0; j < tk; ++j) {
+        if (causal && j > i) { s[j] = -INFINITY; continue; }
+        double dot = 0.0;
+        for (int32_t c = 0; c < dh; ++c)
+          dot += q[(int64_t)i * ldq + (int64_t)h * dh + c] * k[(int64_t)j * ldkv + (int64_t)h * dh + c];
+        s[j] = dot / scale;
+        if (s[j] > m) m = s[j];
+      }
+      double den = 0.0;
+      for (int32_t j = 0; j < tk; ++j) {
+        s[j] = exp(s[j] - m);
+        den += s[j];
+      }
+      for (int32_t c = 0; c < dh; ++c) {
+        double acc = 0.0;
+        for (int32_t j = 0; j < tk; ++j)
+          acc += (s[j] / den) * v[(int64_t)j * ldkv + (int64_t)h * dh + c];
+        o[(int64_t)i * d_model + (int64_t)h * dh + c] = acc;
+      }
+    }
+  }
+  free(s);
+}
+
+int oracle_decoder_stack(const oracle_cfg* cfg, const double* const* w, int32_t num_w,
+                         int32_t t, int32_t l, double* x, const double* mem) {
+  if (num_w != 20 * cfg->num_layers || t <= 0 || l <= 0) return ORACLE_ERR_INVALID;
+  const int32_t d = cfg->d_model, f = cfg->d_ff;
+  double* qkv = (double*)malloc(sizeof(double) * (size_t)t * 3 * d);
+  double* qc = (double*)malloc(sizeof(double) * (size_t)t * d);
+  double* kv = (double*)malloc(sizeof(double) * (size_t)l * 2 * d);
+  double* att = (double*)malloc(sizeof(double) * (size_t)t * d);
+  double* z = (double*)malloc(sizeof(double) * (size_t)t * d);
+  double* x1 = (double*)malloc(sizeof(double) * (size_t)t * d);
+  double* x2 = (double*)malloc(sizeof(double) * (size_t)t * d);
+  double* h = (double*)malloc(sizeof(double) * (size_t)t * f);
+  const int32_t act = cfg->act == 0 ? 1 : 2;
+  for (int32_t layer = 0; layer < cfg->num_layers; ++layer) {
+    const double* const* W = w + 20 * layer;
+    /* causal self-attention over the request's own target prefix */
+    oracle_linear(x, W[0], W[1], NULL, t, 3 * d, d, 0, qkv);
+    attend(qkv, 3 * (int64_t)d, qkv + d, qkv + 2 * d, 3 * (int64_t)d, t, t, d, cfg->num_heads, 1, att);
+    oracle_linear(att, W[2], W[3], x, t, d, d, 0, z);
+    oracle_layernorm(z, W[4], W[5], t, d, cfg->ln_eps, x1);
+    /* cross-attention over the request's own encoder output (segment-aware) */
+    oracle_linear(x1, W[6], W[7], NULL, t, d, d, 0, qc);
+    oracle_linear(mem, W[8], W[9], NULL, l, 2 * d, d, 0, kv);
+    attend(qc, d, kv, kv + d, 2 * (int64_t)d, t, l, d, cfg->num_heads, 0, att);
+    oracle_linear(att, W[10], W[11], x1, t, d, d, 0, z);
+    oracle_layernorm(z, W[12], W[13], t, d, cfg->ln_eps, x2);
+    /* FFN */
+    oracle_linear(x2, W[14], W[15], NULL, t, f, d, act, h);
+    oracle_linear(h, W[16], W[17], x2, t, d, f, 0, z);
+    oracle_layernorm(z, W[18], W[19], t, d, cfg->ln_eps, x);
+  }
+  free(qkv); free(qc); free(kv); free(att); free(z); free(x1); free(x2); free(h);
+  return ORACLE_OK;
+}
+
+/* Greedy decode of ONE request run alone (no padding, no other request): encoder over its
+ * l source tokens, then up to t_max steps of the decoder on the full prefix BOS y_1..y_k;
+ * y_{k+1} = argmax over the vocabulary of x_last . E_tok^T (lowest index on ties); stops
+ * after EOS.  tokens[0..n_out) = y_1..; logits (nullable) [t_max, vocab] per step. */
+int oracle_decode_greedy(const oracle_cfg* cfg, const double* const* enc_w, int32_t n_enc_w,
+                         const double* const* dec_w, int32_t n_dec_w, int32_t vocab,
+                         const int32_t* src, int32_t l, int32_t t_max, int32_t bos, int32_t eos,
+                         int32_t* tokens, int32_t* n_out, double* logits) {
+  if (l <= 0 || t_max <= 0 || vocab <= 0) return ORACLE_ERR_INVALID;
+  const int32_t d = cfg->d_model;
+  int32_t* seg = (int32_t*)malloc(sizeof(int32_t) * (size_t)l);
+  int32_t* pos = (int32_t*)malloc(sizeof(int32_t) * (size_t)l);
+  int32_t* tok = (int32_t*)malloc(sizeof(int32_t) * (size_t)l);
+  for (int32_t i = 0; i < l; ++i) { seg[i] = 0; pos[i] = i; tok[i] = i; }
+  double* mem = (double*)malloc(sizeof(double) * (size_t)l * d);
+  int rc = oracle_encoder(cfg, enc_w, n_enc_w, src, 1, l, seg, pos, tok, mem);
+  int32_t* y = (int32_t*)malloc(sizeof(int32_t) * (size_t)(t_max + 1));
+  double* x = (double*)malloc(sizeof(double) * (size_t)(t_max + 1) * d);
+  double* lg = (double*)malloc(sizeof(double) * (size_t)vocab);
+  const double* E = enc_w[0];
+  y[0] = bos;
+  int32_t k = 0;
+  while (rc == ORACLE_OK && k < t_max) {
+    const int32_t t = k + 1;                               /* prefix length incl. BOS */
+    for (int32_t i = 0; i < t; ++i)                        /* embed: E[y_i] * scale + PE(i) */
+      for (int32_t c = 0; c < d; ++c) {
+        const double pe = cfg->pe == 2 ? enc_w[1][(int64_t)i * d + c] : oracle_pe(i, c, d, cfg->pe);
+        x[(int64_t)i * d + c] = E[(int64_t)y[i] * d + c] * cfg->emb_scale + pe;
+      }
+    rc = oracle_decoder_stack(cfg, dec_w, n_dec_w, t, l, x, mem);
+    if (rc != ORACLE_OK) break;
+    const double* xl = x + (int64_t)(t - 1) * d;
+    int32_t best = 0;
+    for (int32_t v = 0; v < vocab; ++v) {
+      double acc = 0.0;
+      for (int32_t c = 0; c < d; ++c) acc += xl[c] * E[(int64_t)v * d + c];
+      lg[v] = acc;
+      if (acc > lg[best]) best = v;
+    }
+    if (logits)
+      for (int32_t v = 0; v < vocab; ++v) logits[(int64_t)k * vocab + v] = lg[v];
+    y[t] = best;
+    tokens[k] = best;
+    ++k;
+    if (best == eos) break;
+  }
+  *n_out = k;
+  free(seg); free(pos); free(tok); free(mem); free(y); free(x); free(lg);
+  return rc;
+}

@@ -83,6 +83,16 @@ int oracle_encoder(const oracle_cfg* cfg, const double* const* weights, int32_t 
 void oracle_unpack(const double* x, int32_t num_slots, int32_t d, const int32_t* tok_index,
                    double* out);
 
+/* f4 decoder (§4.2.2; readings R30-R33).  dec weights: 20 per layer in the order
+ * w_qkv b_qkv w_o b_o ln1_g ln1_b w_q b_q w_kv b_kv w_co b_co ln2_g ln2_b w_1 b_1 w_2 b_2
+ * ln3_g ln3_b.  x [t, d] (embedded target prefix) is updated in place; mem [l, d]. */
+int oracle_decoder_stack(const oracle_cfg* cfg, const double* const* w, int32_t num_w,
+                         int32_t t, int32_t l, double* x, const double* mem);
+int oracle_decode_greedy(const oracle_cfg* cfg, const double* const* enc_w, int32_t n_enc_w,
+                         const double* const* dec_w, int32_t n_dec_w, int32_t vocab,
+                         const int32_t* src, int32_t l, int32_t t_max, int32_t bos, int32_t eos,
+                         int32_t* tokens, int32_t* n_out, double* logits);
+
 #ifdef __cplusplus
 }
 #endif

@@ -233,3 +233,55 @@ def workload_inputs(key: str, rows: int | None = None, fill: float = 0.995):
     ids = draw_token_ids(int(lengths.sum()), wl.model.vocab, wl.seeds[1])
     weights = draw_weights(wl.model, wl.seeds[2])
     return lengths, ids, weights
+
+
+# ----------------------------------------------------------------------------------------
+# f4: the decoder of the Seq2Seq setting (readings R30-R33 in DESIGN.md)
+# ----------------------------------------------------------------------------------------
+BOS, EOS = 1, 2                      # reading R31
+DEC_LAYER_WEIGHT_NAMES = ["w_qkv", "b_qkv", "w_o", "b_o", "ln1_g", "ln1_b",
+                          "w_q", "b_q", "w_kv", "b_kv", "w_co", "b_co", "ln2_g", "ln2_b",
+                          "w_1", "b_1", "w_2", "b_2", "ln3_g", "ln3_b"]
+
+
+def dec_weight_names(cfg: ModelConfig) -> List[str]:
+    return [f"dec.l{layer}.{n}" for layer in range(cfg.num_layers) for n in DEC_LAYER_WEIGHT_NAMES]
+
+
+def max_target_len(l_src: int, cfg: ModelConfig) -> int:
+    """Reading R32: a request may generate up to as many tokens as its source has (a
+    translation-like budget), capped so every target position has a PE row."""
+    return int(min(l_src, cfg.max_pos - 1))
+
+
+def draw_dec_weights(cfg: ModelConfig, seed: int) -> Dict[str, np.ndarray]:
+    """Random-init decoder weights with the encoder's recipe (Xavier linears, N(0, .02^2)
+    biases, LN gamma 1 + N(0, .1^2), beta N(0, .1^2)); rounded to bf16 for bf16 models."""
+    rng = np.random.default_rng(seed)
+    d, f = cfg.d_model, cfg.d_ff
+    shapes = {"w_qkv": (3 * d, d), "b_qkv": (3 * d,), "w_o": (d, d), "b_o": (d,),
+              "ln1_g": (d,), "ln1_b": (d,), "w_q": (d, d), "b_q": (d,), "w_kv": (2 * d, d),
+              "b_kv": (2 * d,), "w_co": (d, d), "b_co": (d,), "ln2_g": (d,), "ln2_b": (d,),
+              "w_1": (f, d), "b_1": (f,), "w_2": (d, f), "b_2": (d,), "ln3_g": (d,),
+              "ln3_b": (d,)}
+    out: Dict[str, np.ndarray] = {}
+    for name in dec_weight_names(cfg):
+        base = name.split(".")[-1]
+        shp = shapes[base]
+        if base.startswith("w_"):
+            fan_out, fan_in = shp
+            if base in ("w_qkv", "w_kv"):
+                fan_out = d           # per projection, as torch's in_proj
+            a = np.sqrt(6.0 / (fan_in + fan_out))
+            w = rng.uniform(-a, a, size=shp)
+        elif base.startswith("b_"):
+            w = rng.normal(0.0, 0.02, size=shp)
+        elif base.endswith("_g"):
+            w = 1.0 + rng.normal(0.0, 0.1, size=shp)
+        else:
+            w = rng.normal(0.0, 0.1, size=shp)
+        w = w.astype(np.float32)
+        if cfg.dtype == "bf16":
+            w = round_to_bf16(w)
+        out[name] = np.ascontiguousarray(w)
+    return out
