@@ -19,7 +19,7 @@ import numpy as np
 from . import _lib
 from ._lib import KCLASSES, POLICIES, TcbError, check, lib
 
-__all__ = ["Plan", "Encoder", "Scheduler", "sched_batch", "tcb_pack", "tcb_pack_slotted", "op_linear", "op_linear_ln", "op_attention", "op_layernorm",
+__all__ = ["Plan", "Encoder", "Decoder", "Scheduler", "sched_batch", "tcb_pack", "tcb_pack_slotted", "op_linear", "op_linear_ln", "op_attention", "op_layernorm",
            "launch_count", "profile_enable", "profile_collect", "TcbError", "KCLASSES"]
 
 _DTYPES = {"fp32": 0, "bf16": 1}
@@ -342,3 +342,65 @@ def op_layernorm(Z, g, b, eps: float, seg_ids=None, out=None, stream=None):
     check(lib().tcb_op_layernorm(dt, rows, d, _ptr(Z), _ptr(g), _ptr(b), float(eps),
                                  _ptr(seg_ids), _ptr(out), _stream_ptr(stream)))
     return out
+
+
+class Decoder:
+    """Greedy auto-regressive decoder of the Seq2Seq setting (include/tcb_decoder.h, f4) over
+    an Encoder's weights: tied E_tok, causal self-attention with a KV cache per request,
+    cross-attention over the request's own segment of the packed encoder rows, early memory
+    cleaning (finished requests leave the active set).  Argument marshalling only."""
+
+    def __init__(self, encoder: "Encoder", dec_weights: Dict[str, np.ndarray],
+                 dec_names: Sequence[str], max_requests: int, max_slots: int, max_target: int):
+        import torch
+        self.encoder = encoder
+        self.max_target = int(max_target)
+        dev = encoder.device
+        self.tensors = []
+        for n in dec_names:
+            base = n.split(".")[-1]
+            dt = torch.float32 if (base.startswith("b_") or base.startswith("ln")) else encoder.dtype
+            self.tensors.append(torch.from_numpy(np.ascontiguousarray(dec_weights[n]))
+                                .to(device=dev, dtype=dt).contiguous())
+        ptrs = (ctypes.c_void_p * len(self.tensors))(*[t.data_ptr() for t in self.tensors])
+        h = ctypes.c_void_p()
+        check(lib().tcb_decoder_create(encoder._h, ptrs, len(self.tensors), int(max_requests),
+                                       int(max_slots), int(max_target), ctypes.byref(h)))
+        self._h = h
+
+    def __del__(self):
+        h, self._h = getattr(self, "_h", None), None
+        try:
+            if h and _lib._lib is not None:
+                _lib._lib.tcb_decoder_destroy(h)
+        except Exception:  # interpreter shutdown
+            pass
+
+    def decode(self, plan: "Plan", enc_rows, early_clean: bool = True, tokens=None, stream=None):
+        """Returns (device tokens [n, max_target] int32 with -1 past the end, host lengths)."""
+        import torch
+        n = plan.info["num_requests"]
+        if tokens is None:
+            tokens = torch.empty((max(n, 1), self.max_target), dtype=torch.int32,
+                                 device=self.encoder.device)
+        lens = np.zeros(max(n, 1), np.int32)
+        check(lib().tcb_decode_greedy(self._h, plan.handle, _ptr(enc_rows), int(bool(early_clean)),
+                                      _ptr(tokens), lens.ctypes.data_as(ctypes.c_void_p),
+                                      _stream_ptr(stream)))
+        return tokens, lens[:n]
+
+    def stats(self) -> Dict[str, float]:
+        st = _lib.DecodeStats()
+        check(lib().tcb_decoder_stats(self._h, ctypes.byref(st)))
+        return st.as_dict()
+
+    def last_logits(self) -> np.ndarray:
+        """bf16 logits of the last step as float32 [rows, vocab]."""
+        import torch
+        V = self.encoder.model.vocab
+        cap = self.encoder.model.vocab * max(1, 4096)
+        buf = torch.empty(cap, dtype=torch.bfloat16)
+        rows = ctypes.c_int32(0)
+        check(lib().tcb_decoder_last_logits(self._h, ctypes.c_void_p(buf.data_ptr()), cap,
+                                            ctypes.byref(rows)))
+        return buf[:rows.value * V].float().numpy().reshape(rows.value, V)

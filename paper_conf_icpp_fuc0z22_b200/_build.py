@@ -15,7 +15,7 @@ ARCH = ["-gencode", "arch=compute_100a,code=sm_100a"]
 FLAGS = ["-O3", "-std=c++17", "-lineinfo", "-Xcompiler", "-fPIC,-Wall", "--expt-relaxed-constexpr",
          "-Xptxas", "-warn-spills"] + os.environ.get("TCB_EXTRA_NVCC_FLAGS", "").split()
 SOURCES = ["pack.cpp", "sched.cpp", "api.cu", "elementwise.cu", "linear_f32.cu", "linear_tc.cu",
-           "attention.cu", "attention_tc.cu"]
+           "attention.cu", "attention_tc.cu", "decoder.cu"]
 
 
 def _newest_dep() -> float:

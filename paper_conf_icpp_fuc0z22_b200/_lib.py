@@ -30,7 +30,9 @@ EXPORTS = ["tcb_last_error", "tcb_version", "tcb_pack", "tcb_pack_slotted", "tcb
            "tcb_unpack", "tcb_launch_count", "tcb_profile_enable", "tcb_profile_collect",
            "tcb_op_linear", "tcb_op_linear_ln", "tcb_op_attention", "tcb_op_layernorm",
            "tcb_sched_batch", "tcb_sched_create", "tcb_sched_destroy", "tcb_sched_submit",
-           "tcb_sched_next_batch", "tcb_sched_stats_get"]
+           "tcb_sched_next_batch", "tcb_sched_stats_get",
+           "tcb_decoder_weights_count", "tcb_decoder_create", "tcb_decoder_destroy",
+           "tcb_decode_greedy", "tcb_decoder_stats", "tcb_decoder_last_logits"]
 SCHED_POLICIES = {"das": 0, "fcfs": 1, "sjf": 2, "def": 3}
 
 
@@ -58,6 +60,15 @@ class SchedStats(ctypes.Structure):
     _fields_ = [("submitted", ctypes.c_int64), ("waiting", ctypes.c_int64),
                 ("scheduled", ctypes.c_int64), ("expired", ctypes.c_int64),
                 ("batches", ctypes.c_int64), ("utility", ctypes.c_double)]
+
+    def as_dict(self):
+        return {f: getattr(self, f) for f, _ in self._fields_}
+
+
+class DecodeStats(ctypes.Structure):
+    _fields_ = [("steps", ctypes.c_int32), ("rows_computed", ctypes.c_int64),
+                ("tokens_generated", ctypes.c_int64), ("kv_bytes_peak", ctypes.c_int64),
+                ("kv_bytes_avg", ctypes.c_double), ("ms_total", ctypes.c_double)]
 
     def as_dict(self):
         return {f: getattr(self, f) for f, _ in self._fields_}
@@ -122,6 +133,12 @@ def lib() -> ctypes.CDLL:
         "tcb_sched_next_batch": (I32, [P, ctypes.c_double, P, P, I32, ctypes.POINTER(I32),
                                        ctypes.POINTER(P)]),
         "tcb_sched_stats_get": (I32, [P, ctypes.POINTER(SchedStats)]),
+        "tcb_decoder_weights_count": (I32, [ctypes.POINTER(ModelConfig)]),
+        "tcb_decoder_create": (I32, [P, P, I32, I32, I64, I32, ctypes.POINTER(P)]),
+        "tcb_decoder_destroy": (None, [P]),
+        "tcb_decode_greedy": (I32, [P, P, P, I32, P, P, P]),
+        "tcb_decoder_stats": (I32, [P, ctypes.POINTER(DecodeStats)]),
+        "tcb_decoder_last_logits": (I32, [P, P, I64, ctypes.POINTER(I32)]),
     }
     for name, (res, args) in sig.items():
         fn = getattr(L, name)

@@ -7,6 +7,7 @@
 #include <cuda.h>
 #include <cuda_runtime.h>
 
+#include <algorithm>
 #include <atomic>
 #include <cstdlib>
 #include <cstring>
@@ -553,6 +554,327 @@ tcb_status tcb_op_layernorm(int32_t dtype, int64_t rows, int32_t d, const void* 
   if (tcb_status st = check_device()) return st;
   cudaStream_t s = reinterpret_cast<cudaStream_t>(stream);
   TCB_LAUNCH(TCB_K_LN, s, tcb::k::launch_layernorm(dtype, rows, d, Z, g, b, eps, d_seg, Y, s));
+  return TCB_OK;
+}
+
+}  // extern "C"
+
+// ============================================================================================
+// f4: auto-regressive decoder with early memory cleaning (include/tcb_decoder.h)
+// ============================================================================================
+#include <chrono>
+
+#include "../../include/tcb_decoder.h"
+
+struct tcb_decoder {
+  const tcb_weights* enc = nullptr;
+  std::vector<const void*> t;            // 20 per layer (tcb_decoder.h order)
+  int32_t R = 0, T = 0;                  // max requests, max target tokens (= KV positions)
+  int64_t max_slots = 0;
+  std::vector<void*> bufs;               // every owned device allocation
+  uint8_t* memkv = nullptr;              // S x [max_slots, 2d]  encoder memory K | V
+  uint8_t* cache = nullptr;              // S x [R * T, 2d]      self-attention K | V
+  void *x = nullptr, *qkv = nullptr, *att = nullptr, *x1 = nullptr, *qc = nullptr,
+       *x2 = nullptr, *h = nullptr, *logits = nullptr;
+  float* zero_bias = nullptr;            // [vocab] (the tied output projection has no bias)
+  int32_t *act = nullptr, *out_len = nullptr, *done = nullptr, *flag = nullptr,
+          *tmax = nullptr, *mem_start = nullptr, *mem_len = nullptr;
+  struct LayerMaps {
+    CUtensorMap qkv, o, q, kv, co, w1, w2, memkv_c;
+  };
+  std::vector<LayerMaps> wm;
+  CUtensorMap w_logits{};
+  CUtensorMap aX{}, aAtt{}, aX1{}, aX2{}, aH{};
+  CUtensorMap cQkv{}, cX{}, cX1{}, cX2{}, cQc{}, cH{}, cLogits{};
+  tcb_decode_stats stats{};
+  int32_t last_rows = 0;
+  const void* L(int layer, int i) const { return t[20 * layer + i]; }
+  const float* Lf(int layer, int i) const { return static_cast<const float*>(L(layer, i)); }
+};
+
+namespace {
+enum { D_W_QKV = 0, D_B_QKV, D_W_O, D_B_O, D_LN1_G, D_LN1_B, D_W_Q, D_B_Q, D_W_KV, D_B_KV,
+       D_W_CO, D_B_CO, D_LN2_G, D_LN2_B, D_W_1, D_B_1, D_W_2, D_B_2, D_LN3_G, D_LN3_B };
+
+void free_decoder(tcb_decoder* dec) {
+  for (void* p : dec->bufs) cudaFree(p);
+  delete dec;
+}
+
+template <typename T>
+bool dalloc(tcb_decoder* dec, T** p, size_t bytes) {
+  void* v = nullptr;
+  if (cudaMalloc(&v, bytes ? bytes : 16) != cudaSuccess) {
+    cudaGetLastError();
+    return false;
+  }
+  dec->bufs.push_back(v);
+  *p = static_cast<T*>(v);
+  return true;
+}
+}  // namespace
+
+extern "C" {
+
+int32_t tcb_decoder_weights_count(const tcb_model_config* cfg) { return cfg ? 20 * cfg->num_layers : -1; }
+
+tcb_status tcb_decoder_create(const tcb_weights* enc, const void* const* tensors,
+                              int32_t num_tensors, int32_t max_requests, int64_t max_slots,
+                              int32_t max_target, tcb_decoder** out) {
+  tcb::clear_error();
+  if (!out) return fail(TCB_ERR_INVALID_ARGUMENT, "tcb_decoder_create: out is NULL");
+  *out = nullptr;
+  if (!enc) return fail(TCB_ERR_INVALID_ARGUMENT, "tcb_decoder_create: enc is NULL");
+  const tcb_model_config& c = enc->cfg;
+  if (c.dtype != 1 || c.pe == 2 || c.emb_ln || c.use_type_emb)
+    return fail(TCB_ERR_UNSUPPORTED, "tcb_decoder_create: bf16 Transformer-family models only "
+                                     "(sinusoidal PE, no embedding LN / type embedding)");
+  if (c.d_model / c.num_heads != 64 || !tcb::k::linear_ln_supported(c.d_model) || c.vocab % 64)
+    return fail(TCB_ERR_UNSUPPORTED, "tcb_decoder_create: needs d_head 64, d_model in "
+                                     "{512, 768, 1024}, vocab % 64 == 0");
+  if (!tensors || num_tensors != tcb_decoder_weights_count(&c))
+    return fail(TCB_ERR_INVALID_ARGUMENT, "tcb_decoder_create: expected " +
+                                              std::to_string(tcb_decoder_weights_count(&c)) + " tensors");
+  for (int i = 0; i < num_tensors; ++i)
+    if (!tensors[i] || (reinterpret_cast<uintptr_t>(tensors[i]) & 15))
+      return fail(TCB_ERR_INVALID_ARGUMENT, "tcb_decoder_create: tensor " + std::to_string(i) +
+                                                " is NULL or not 16-byte aligned");
+  if (max_requests <= 0 || max_slots <= 0 || max_target <= 0 || max_target >= c.max_pos ||
+      max_target > tcb::k::dec_max_keys() || max_slots > INT32_MAX)
+    return fail(TCB_ERR_INVALID_ARGUMENT, "tcb_decoder_create: bad capacities");
+  if (tcb_status st = check_device()) return st;
+  tcb_decoder* dec = new (std::nothrow) tcb_decoder();
+  if (!dec) return fail(TCB_ERR_OUT_OF_MEMORY, "tcb_decoder_create");
+  dec->enc = enc;
+  dec->t.assign(tensors, tensors + num_tensors);
+  dec->R = max_requests;
+  dec->T = max_target;
+  dec->max_slots = max_slots;
+  const int64_t d = c.d_model, f = c.d_ff, V = c.vocab, R = max_requests, S = c.num_layers;
+  bool ok = dalloc(dec, &dec->memkv, sizeof(uint16_t) * S * max_slots * 2 * d) &&
+            dalloc(dec, &dec->cache, sizeof(uint16_t) * S * R * max_target * 2 * d) &&
+            dalloc(dec, &dec->x, 2 * R * d) && dalloc(dec, &dec->qkv, 2 * R * 3 * d) &&
+            dalloc(dec, &dec->att, 2 * R * d) && dalloc(dec, &dec->x1, 2 * R * d) &&
+            dalloc(dec, &dec->qc, 2 * R * d) && dalloc(dec, &dec->x2, 2 * R * d) &&
+            dalloc(dec, &dec->h, 2 * R * f) && dalloc(dec, &dec->logits, 2 * R * V) &&
+            dalloc(dec, &dec->zero_bias, sizeof(float) * V) &&
+            dalloc(dec, &dec->act, 4 * R) && dalloc(dec, &dec->out_len, 4 * R) &&
+            dalloc(dec, &dec->done, 4 * R) && dalloc(dec, &dec->flag, 4 * R) &&
+            dalloc(dec, &dec->tmax, 4 * R) && dalloc(dec, &dec->mem_start, 4 * R) &&
+            dalloc(dec, &dec->mem_len, 4 * R);
+  if (!ok) {
+    free_decoder(dec);
+    return fail(TCB_ERR_OUT_OF_MEMORY, "tcb_decoder_create: device buffers");
+  }
+  if (cudaMemset(dec->zero_bias, 0, sizeof(float) * V) != cudaSuccess) {
+    free_decoder(dec);
+    return cuda_fail(cudaGetLastError(), "tcb_decoder_create: memset");
+  }
+  using namespace tcb::k;
+  dec->wm.resize(S);
+  for (int l = 0; l < S && ok; ++l) {
+    auto& m = dec->wm[l];
+    ok = make_gemm_w_map(&m.qkv, dec->L(l, D_W_QKV), 3 * d, d) &&
+         make_gemm_w_map(&m.o, dec->L(l, D_W_O), d, d) &&
+         make_gemm_w_map(&m.q, dec->L(l, D_W_Q), d, d) &&
+         make_gemm_w_map(&m.kv, dec->L(l, D_W_KV), 2 * d, d) &&
+         make_gemm_w_map(&m.co, dec->L(l, D_W_CO), d, d) &&
+         make_gemm_w_map(&m.w1, dec->L(l, D_W_1), f, d) &&
+         make_gemm_w_map(&m.w2, dec->L(l, D_W_2), d, f) &&
+         make_gemm_c_map(&m.memkv_c, dec->memkv + sizeof(uint16_t) * l * max_slots * 2 * d,
+                         max_slots, 2 * d);
+  }
+  ok = ok && make_gemm_w_map(&dec->w_logits, enc->tok_emb(), V, d) &&
+       make_gemm_a_map(&dec->aX, dec->x, R, d) && make_gemm_a_map(&dec->aAtt, dec->att, R, d) &&
+       make_gemm_a_map(&dec->aX1, dec->x1, R, d) && make_gemm_a_map(&dec->aX2, dec->x2, R, d) &&
+       make_gemm_a_map(&dec->aH, dec->h, R, f) && make_gemm_c_map(&dec->cQkv, dec->qkv, R, 3 * d) &&
+       make_gemm_c_map(&dec->cX, dec->x, R, d) && make_gemm_c_map(&dec->cX1, dec->x1, R, d) &&
+       make_gemm_c_map(&dec->cX2, dec->x2, R, d) && make_gemm_c_map(&dec->cQc, dec->qc, R, d) &&
+       make_gemm_c_map(&dec->cH, dec->h, R, f) && make_gemm_c_map(&dec->cLogits, dec->logits, R, V);
+  if (!ok) {
+    free_decoder(dec);
+    return fail(TCB_ERR_CUDA, "tcb_decoder_create: cuTensorMapEncodeTiled failed");
+  }
+  *out = dec;
+  return TCB_OK;
+}
+
+void tcb_decoder_destroy(tcb_decoder* dec) {
+  if (dec) free_decoder(dec);
+}
+
+tcb_status tcb_decode_greedy(tcb_decoder* dec, const tcb_plan* plan, const void* d_enc_rows,
+                             int32_t early_clean, int32_t* d_tokens, int32_t* h_lengths,
+                             tcb_stream_t stream) {
+  tcb::clear_error();
+  const auto t0 = std::chrono::steady_clock::now();
+  if (!dec || !plan || !h_lengths) return fail(TCB_ERR_INVALID_ARGUMENT, "tcb_decode_greedy: NULL");
+  const tcb_model_config& c = dec->enc->cfg;
+  const int32_t n = plan->n;
+  if (n > dec->R) return fail(TCB_ERR_INVALID_ARGUMENT, "tcb_decode_greedy: more requests than max_requests");
+  if (plan->info.num_slots > dec->max_slots)
+    return fail(TCB_ERR_INVALID_ARGUMENT, "tcb_decode_greedy: plan larger than max_slots");
+  if (tcb_status st = validate_plan_for(dec->enc, plan)) return st;
+  for (int32_t r = 0; r < n; ++r) h_lengths[r] = 0;
+  dec->stats = tcb_decode_stats{};
+  if (n == 0) return TCB_OK;
+  if (!d_enc_rows || !d_tokens) return fail(TCB_ERR_INVALID_ARGUMENT, "tcb_decode_greedy: NULL device pointer");
+  cudaStream_t s = reinterpret_cast<cudaStream_t>(stream);
+  const int d = c.d_model, f = c.d_ff, V = c.vocab, S = c.num_layers, T = dec->T;
+  const int act_epi = c.act == 0 ? TCB_EPI_BIAS_GELU : TCB_EPI_BIAS_RELU;
+  const int64_t M = plan->info.num_slots;
+  // per-request host metadata: memory segment in the packed rows, generation budget (R32)
+  std::vector<int32_t> act_h, tmax_h(n, 0), ms_h(n, 0), ml_h(n, 0);
+  int32_t max_steps = 0;
+  for (int32_t r = 0; r < n; ++r) {
+    if (plan->req_row[r] < 0) continue;
+    ms_h[r] = plan->req_row[r] * plan->row_len + plan->req_col[r];
+    ml_h[r] = plan->lengths[r];
+    tmax_h[r] = std::min(plan->lengths[r], T);
+    max_steps = std::max(max_steps, tmax_h[r]);
+    act_h.push_back(r);
+  }
+  cudaError_t e = cudaMemcpyAsync(dec->tmax, tmax_h.data(), 4 * n, cudaMemcpyHostToDevice, s);
+  if (e == cudaSuccess) e = cudaMemcpyAsync(dec->mem_start, ms_h.data(), 4 * n, cudaMemcpyHostToDevice, s);
+  if (e == cudaSuccess) e = cudaMemcpyAsync(dec->mem_len, ml_h.data(), 4 * n, cudaMemcpyHostToDevice, s);
+  if (e == cudaSuccess) e = cudaMemsetAsync(dec->done, 0, 4 * n, s);
+  if (e == cudaSuccess) e = cudaMemsetAsync(dec->out_len, 0, 4 * n, s);
+  if (e == cudaSuccess) e = cudaMemsetAsync(d_tokens, 0xff, sizeof(int32_t) * n * T, s);
+  if (e != cudaSuccess) return cuda_fail(e, "tcb_decode_greedy: metadata upload");
+  using namespace tcb::k;
+  // encoder memory K | V of every layer over the packed rows (the request's segment is its
+  // memory, R30): one GEMM per layer, M = num_slots
+  {
+    CUtensorMap aEnc;
+    if (!make_gemm_a_map(&aEnc, d_enc_rows, M, d))
+      return fail(TCB_ERR_CUDA, "tcb_decode_greedy: encoder-rows tensor map");
+    for (int l = 0; l < S; ++l) {
+      const GemmMaps g{aEnc, dec->wm[l].kv, dec->wm[l].memkv_c, dec->wm[l].memkv_c};
+      TCB_LAUNCH(TCB_K_GEMM_QKV, s, launch_linear_bf16_tc(g, M, 2 * d, d, dec->Lf(l, D_B_KV), TCB_EPI_BIAS, s));
+    }
+  }
+  const float scale = 1.f / 8.f;                          // 1 / sqrt(d_head = 64)
+  std::vector<int32_t> flag_h(act_h.size());
+  const int64_t kv_per_pos = 2LL * d * 2 * S;             // bytes of K|V per position, all layers
+  double kv_sum = 0.0;
+  int32_t t = 0;
+  bool act_dirty = true;
+  for (; t < max_steps && !act_h.empty(); ++t) {
+    const int A = static_cast<int>(act_h.size());
+    if (act_dirty) {
+      e = cudaMemcpyAsync(dec->act, act_h.data(), 4 * A, cudaMemcpyHostToDevice, s);
+      if (e != cudaSuccess) return cuda_fail(e, "tcb_decode_greedy: active set upload");
+      act_dirty = false;
+    }
+    DecEmbedArgs ea{dec->act, d_tokens, T, t, 1, 2, d, A,
+                    static_cast<const __nv_bfloat16*>(dec->enc->tok_emb()), dec->enc->pe_table,
+                    c.emb_scale, static_cast<__nv_bfloat16*>(dec->x)};
+    TCB_LAUNCH(TCB_K_EMBED, s, launch_dec_embed(ea, s));
+    for (int l = 0; l < S; ++l) {
+      const auto& m = dec->wm[l];
+      TCB_LAUNCH(TCB_K_GEMM_QKV, s, launch_linear_bf16_tc(GemmMaps{dec->aX, m.qkv, dec->cQkv, dec->cQkv},
+                                                          A, 3 * d, d, dec->Lf(l, D_B_QKV), TCB_EPI_BIAS, s));
+      DecAttnArgs sa{};
+      sa.act = dec->act;
+      sa.q = static_cast<const __nv_bfloat16*>(dec->qkv);
+      sa.ldq = 3 * d;
+      sa.qoff = 0;
+      sa.kv = reinterpret_cast<__nv_bfloat16*>(dec->cache + sizeof(uint16_t) * l * dec->R * T * 2 * d);
+      sa.ld_kv = 2 * d;
+      sa.voff = d;
+      sa.self = 1;
+      sa.t = t;
+      sa.t_cap = T;
+      sa.d = d;
+      sa.heads = c.num_heads;
+      sa.rows = A;
+      sa.scale = scale;
+      sa.out = static_cast<__nv_bfloat16*>(dec->att);
+      TCB_LAUNCH(TCB_K_ATTN, s, launch_dec_attn(sa, s));
+      TCB_LAUNCH(TCB_K_GEMM_O, s, launch_linear_ln_bf16_tc(GemmMaps{dec->aAtt, m.o, dec->cX1, dec->cX},
+                                                           A, d, d, dec->Lf(l, D_B_O), dec->Lf(l, D_LN1_G),
+                                                           dec->Lf(l, D_LN1_B), c.ln_eps, nullptr, s));
+      TCB_LAUNCH(TCB_K_GEMM_QKV, s, launch_linear_bf16_tc(GemmMaps{dec->aX1, m.q, dec->cQc, dec->cQc},
+                                                          A, d, d, dec->Lf(l, D_B_Q), TCB_EPI_BIAS, s));
+      DecAttnArgs ca = sa;
+      ca.q = static_cast<const __nv_bfloat16*>(dec->qc);
+      ca.ldq = d;
+      ca.kv = reinterpret_cast<__nv_bfloat16*>(dec->memkv + sizeof(uint16_t) * l * dec->max_slots * 2 * d);
+      ca.self = 0;
+      ca.mem_start = dec->mem_start;
+      ca.mem_len = dec->mem_len;
+      TCB_LAUNCH(TCB_K_ATTN, s, launch_dec_attn(ca, s));
+      TCB_LAUNCH(TCB_K_GEMM_O, s, launch_linear_ln_bf16_tc(GemmMaps{dec->aAtt, m.co, dec->cX2, dec->cX1},
+                                                           A, d, d, dec->Lf(l, D_B_CO), dec->Lf(l, D_LN2_G),
+                                                           dec->Lf(l, D_LN2_B), c.ln_eps, nullptr, s));
+      TCB_LAUNCH(TCB_K_GEMM_FFN1, s, launch_linear_bf16_tc(GemmMaps{dec->aX2, m.w1, dec->cH, dec->cH},
+                                                           A, f, d, dec->Lf(l, D_B_1), act_epi, s));
+      TCB_LAUNCH(TCB_K_GEMM_FFN2, s, launch_linear_ln_bf16_tc(GemmMaps{dec->aH, m.w2, dec->cX, dec->cX2},
+                                                              A, d, f, dec->Lf(l, D_B_2), dec->Lf(l, D_LN3_G),
+                                                              dec->Lf(l, D_LN3_B), c.ln_eps, nullptr, s));
+    }
+    // tied output projection (R31) and greedy argmax
+    TCB_LAUNCH(TCB_K_GEMM_QKV, s, launch_linear_bf16_tc(GemmMaps{dec->aX, dec->w_logits, dec->cLogits, dec->cLogits},
+                                                        A, V, d, dec->zero_bias, TCB_EPI_BIAS, s));
+    DecArgmaxArgs ga{static_cast<const __nv_bfloat16*>(dec->logits), V, A, t, 2, T, dec->act,
+                     dec->tmax, d_tokens, dec->out_len, dec->done, dec->flag};
+    TCB_LAUNCH(TCB_K_UNPACK, s, launch_dec_argmax(ga, s));
+    e = cudaMemcpyAsync(flag_h.data(), dec->flag, 4 * A, cudaMemcpyDeviceToHost, s);
+    if (e == cudaSuccess) e = cudaStreamSynchronize(s);
+    if (e != cudaSuccess) return cuda_fail(e, "tcb_decode_greedy: step");
+    dec->last_rows = A;
+    dec->stats.rows_computed += A;
+    const int64_t kv_live = static_cast<int64_t>(A) * (t + 1) * kv_per_pos;
+    kv_sum += static_cast<double>(kv_live);
+    dec->stats.kv_bytes_peak = std::max(dec->stats.kv_bytes_peak, kv_live);
+    // early memory cleaning (R33): finished requests leave the active set
+    bool all_done = true;
+    std::vector<int32_t> next;
+    next.reserve(A);
+    for (int i = 0; i < A; ++i) {
+      if (!flag_h[i]) {
+        all_done = false;
+        next.push_back(act_h[i]);
+      }
+    }
+    if (all_done) { ++t; break; }
+    if (early_clean && static_cast<int>(next.size()) != A) {
+      act_h.swap(next);
+      act_dirty = true;
+    }
+  }
+  std::vector<int32_t> len_h(n);
+  e = cudaMemcpyAsync(len_h.data(), dec->out_len, 4 * n, cudaMemcpyDeviceToHost, s);
+  if (e == cudaSuccess) e = cudaStreamSynchronize(s);
+  if (e != cudaSuccess) return cuda_fail(e, "tcb_decode_greedy: lengths");
+  for (int32_t r = 0; r < n; ++r) {
+    h_lengths[r] = len_h[r];
+    dec->stats.tokens_generated += len_h[r];
+  }
+  dec->stats.steps = t;
+  dec->stats.kv_bytes_avg = t > 0 ? kv_sum / t : 0.0;
+  dec->stats.ms_total =
+      std::chrono::duration<double, std::milli>(std::chrono::steady_clock::now() - t0).count();
+  return TCB_OK;
+}
+
+tcb_status tcb_decoder_stats(const tcb_decoder* dec, tcb_decode_stats* out) {
+  tcb::clear_error();
+  if (!dec || !out) return fail(TCB_ERR_INVALID_ARGUMENT, "tcb_decoder_stats: NULL");
+  *out = dec->stats;
+  return TCB_OK;
+}
+
+tcb_status tcb_decoder_last_logits(const tcb_decoder* dec, void* h_logits, int64_t capacity_elems,
+                                   int32_t* rows) {
+  tcb::clear_error();
+  if (!dec || !h_logits || !rows) return fail(TCB_ERR_INVALID_ARGUMENT, "tcb_decoder_last_logits: NULL");
+  const int64_t need = static_cast<int64_t>(dec->last_rows) * dec->enc->cfg.vocab;
+  if (capacity_elems < need) return fail(TCB_ERR_INVALID_ARGUMENT, "tcb_decoder_last_logits: buffer too small");
+  *rows = dec->last_rows;
+  if (need == 0) return TCB_OK;
+  cudaError_t e = cudaMemcpy(h_logits, dec->logits, 2 * need, cudaMemcpyDeviceToHost);
+  if (e != cudaSuccess) return cuda_fail(e, "tcb_decoder_last_logits");
   return TCB_OK;
 }
 

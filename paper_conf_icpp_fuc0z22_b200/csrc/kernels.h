@@ -3,6 +3,7 @@
 
 #include <cuda.h>
 #include <cuda_runtime.h>
+#include <cuda_bf16.h>
 #include <cstdint>
 #include <utility>
 
@@ -120,6 +121,45 @@ cudaError_t launch_attention_bf16_tc(int64_t num_slots, int d_model, int num_hea
 cudaError_t launch_attention_f32(int64_t num_slots, int d_model, int num_heads,
                                  const float* qkv, const int32_t* seg_ids, const int4* segtab,
                                  float* O, cudaStream_t s);
+
+// Decoder (decoder.cu, f4) ------------------------------------------------------------------
+struct DecEmbedArgs {
+  const int32_t* act;          // [rows] request index of each active row
+  const int32_t* out_tok;      // [R, ld_out] generated tokens
+  int32_t ld_out, t, bos, eos, d, rows;
+  const __nv_bfloat16* tok_emb;  // [vocab, d]
+  const float* pe;             // [max_pos, d] fp32 sinusoidal table
+  float emb_scale;
+  __nv_bfloat16* x;            // out [rows, d]
+};
+struct DecAttnArgs {
+  const int32_t* act;
+  const __nv_bfloat16* q;      // [rows, ldq]; the query of head h at column qoff + 64h
+  int32_t ldq, qoff;
+  __nv_bfloat16* kv;           // keys at column 64h, values at column voff + 64h
+  int64_t ld_kv;
+  int32_t voff;
+  int32_t self, t, t_cap;      // self: cache of request r = rows [r t_cap, r t_cap + t]
+  const int32_t* mem_start;    // cross: keys [mem_start[r], + mem_len[r])
+  const int32_t* mem_len;
+  int32_t d, heads, rows;
+  float scale;
+  __nv_bfloat16* out;          // [rows, d]
+};
+struct DecArgmaxArgs {
+  const __nv_bfloat16* logits; // [rows, vocab]
+  int32_t vocab, rows, t, eos, ld_out;
+  const int32_t* act;
+  const int32_t* t_max;        // [R]
+  int32_t* out_tok;            // [R, ld_out]
+  int32_t* out_len;            // [R]
+  int32_t* done;               // [R]
+  int32_t* flag;               // [rows] finished after this step
+};
+cudaError_t launch_dec_embed(const DecEmbedArgs& a, cudaStream_t s);
+cudaError_t launch_dec_attn(const DecAttnArgs& a, cudaStream_t s);
+cudaError_t launch_dec_argmax(const DecArgmaxArgs& a, cudaStream_t s);
+int dec_max_keys();
 
 }  // namespace k
 }  // namespace tcb

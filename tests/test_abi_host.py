@@ -20,7 +20,7 @@ ROOT = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
 
 def _declared_symbols():
     names = set()
-    for h in ("tcb.h", "tcb_ops.h"):
+    for h in ("tcb.h", "tcb_ops.h", "tcb_decoder.h"):
         src = open(os.path.join(ROOT, "include", h)).read()
         src = re.sub(r"/\*.*?\*/", "", src, flags=re.S)
         names |= set(re.findall(r"\b(tcb_[a-z_0-9]+)\s*\(", src))
@@ -232,3 +232,20 @@ def test_device_calls_fail_loudly_without_gpu():
     assert b"no CPU fallback" in _lib.lib().tcb_last_error()
     st = _lib.lib().tcb_op_linear(1, 128, 64, 64, 4096, 4096, 4096, None, 0, 4096, None)
     assert st == -7
+
+
+def test_decoder_abi_validates_without_a_gpu():
+    """f4 ABI (include/tcb_decoder.h): weight count, NULL checks, no CPU fallback."""
+    import ctypes
+    import tcb_workload as wl
+    m = wl.MODELS["transformer-base"]
+    cfg = _lib.ModelConfig(m.num_layers, m.d_model, m.num_heads, m.d_ff, m.vocab, m.max_pos, 1,
+                           1, 0, 0, 0, m.ln_eps, m.emb_ln_eps, m.emb_scale)
+    L = _lib.lib()
+    assert L.tcb_decoder_weights_count(ctypes.byref(cfg)) == 20 * m.num_layers
+    h = ctypes.c_void_p()
+    assert L.tcb_decoder_create(None, None, 0, 1, 1, 1, ctypes.byref(h)) == -1
+    assert L.tcb_decode_greedy(None, None, None, 1, None, None, None) == -1
+    st = _lib.DecodeStats()
+    assert L.tcb_decoder_stats(None, ctypes.byref(st)) == -1
+    assert len(wl.dec_weight_names(m)) == 20 * m.num_layers
