@@ -203,21 +203,19 @@ __device__ __forceinline__ constexpr uint32_t idesc_bf16() {
 }
 
 // GELU, erf form (R9): x * Phi(x) = x * (x >= 0 ? 1 - h : h) with h = Phi(-|x|) =
-// 0.5 erfc(|x| / sqrt 2) evaluated as 2^P(|x|), P a degree-8 Chebyshev fit of log2 Phi(-a) on
-// [0, 5.75] (|x| clamped there).  Max |error| vs the erf form 4.8e-7 (relative 3e-6), far
-// below the bf16 rounding of the output, with ONE MUFU op per element -- the FFN1 epilogue
-// is issue/MUFU-bound, and libdevice erff (+ reciprocal forms) cost 2-3x more.
+// 0.5 erfc(|x| / sqrt 2) evaluated as 2^P(|x|), P a degree-6 Chebyshev fit of log2 Phi(-a) on
+// [0, 5.75] (|x| clamped there).  Max |error| vs the erf form 4.6e-6 (relative 7e-5 where
+// |GELU| > 1e-3), far below the bf16 rounding of the output (2^-9), with ONE MUFU op per
+// element -- the FFN1 epilogue is issue-bound, and libdevice erff costs 2-3x more.
 __device__ __forceinline__ float gelu_erf(float x) {
   const float a = fminf(fabsf(x), 5.75f);
-  float p = -4.726407710e-08f;
-  p = fmaf(p, a, -8.334873201e-07f);
-  p = fmaf(p, a, 5.311644418e-05f);
-  p = fmaf(p, a, -8.938793326e-04f);
-  p = fmaf(p, a, 8.422582410e-03f);
-  p = fmaf(p, a, -5.385634303e-02f);
-  p = fmaf(p, a, -4.585228264e-01f);
-  p = fmaf(p, a, -1.151239634e+00f);
-  p = fmaf(p, a, -9.999955893e-01f);
+  float p = 2.468310274e-05f;
+  p = fmaf(p, a, -6.366563243e-04f);
+  p = fmaf(p, a, 7.334408915e-03f);
+  p = fmaf(p, a, -5.150612900e-02f);
+  p = fmaf(p, a, -4.610041018e-01f);
+  p = fmaf(p, a, -1.150170450e+00f);
+  p = fmaf(p, a, -1.000105574e+00f);
   float h;
   asm("ex2.approx.ftz.f32 %0, %1;" : "=f"(h) : "f"(p));
   return x * (x >= 0.f ? 1.f - h : h);
@@ -1325,7 +1323,9 @@ cudaError_t launch_linear_ln_bf16_tc(const GemmMaps& m, int64_t M, int N, int K,
   if (N == 768) return launch_lnc<3>(m, Mi, K, bias, gamma, beta, eps, seg_ids, s);
   if (N == 1024) return launch_lnc<4>(m, Mi, K, bias, gamma, beta, eps, seg_ids, s);
   if (N != kLnN) return cudaErrorInvalidValue;
-  if (!pair_512) return launch_lnc<2>(m, Mi, K, bias, gamma, beta, eps, seg_ids, s);
+  // K >= 1024 (FFN2): the cluster kernel measured faster (64.1 vs 66.6 us at K = 2048);
+  // K = 512 (W_O): the single pair (32.3 vs 34.9 us)
+  if (!pair_512 || K >= 1024) return launch_lnc<2>(m, Mi, K, bias, gamma, beta, eps, seg_ids, s);
   const int nkb = K / BK;
   static const int split_env = [] {
     const char* e = getenv("TCB_LN_SPLIT");             // tuning override (k-blocks)
