@@ -913,20 +913,6 @@ __device__ __forceinline__ void tc_commit_mask(uint64_t* bar, uint16_t mask) {
       "h"(mask)
       : "memory");
 }
-__device__ __forceinline__ void mbar_wait_cluster(uint64_t* bar, uint32_t parity) {
-  const uint32_t addr = smem_u32(bar);
-  uint32_t done = 0;
-  do {
-    asm volatile(
-        "{\n\t.reg .pred p;\n\t"
-        "mbarrier.try_wait.parity.acquire.cluster.shared::cta.b64 p, [%1], %2;\n\t"
-        "selp.u32 %0, 1, 0, p;\n\t}"
-        : "=r"(done)
-        : "r"(addr), "r"(parity)
-        : "memory");
-  } while (!done);
-}
-
 template <int P>
 __global__ void __launch_bounds__(kThreads, 1)
 linear_lnc_kernel(const __grid_constant__ CUtensorMap tmA, const __grid_constant__ CUtensorMap tmW,
@@ -968,7 +954,7 @@ linear_lnc_kernel(const __grid_constant__ CUtensorMap tmA, const __grid_constant
     for (int i = 0; i < 2; ++i) {
       mbar_init(&tfull[i], 1);
       mbar_init(&tempty[i], 2 * kLncEpiWarps);
-      mbar_init(&sfull[i], P * kLncEpiWarps * 32);             // every lane of every writer
+      mbar_init(&sfull[i], 1);       // local arrive.expect_tx; the partials land via st.async
     }
     for (int i = 0; i < kLncEpiWarps * kLncChunks; ++i) mbar_init(&rbar[i], 1);
     asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
@@ -1051,6 +1037,9 @@ linear_lnc_kernel(const __grid_constant__ CUtensorMap tmA, const __grid_constant
       const int col0 = static_cast<int>(p) * 256 + half * 128;
       const int64_t grow = static_cast<int64_t>(row0) + lane;
       const bool pad = grow >= M || (seg_ids && __ldg(&seg_ids[grow]) < 0);
+      // this tile's phase of the statistics barrier completes once all 2P x 128 partials
+      // (8 B each, from this CTA and its P-1 peers) have landed
+      if (ew == 0 && lane == 0) mbar_expect_tx(&sfull[acc], 2 * P * 128 * 8);
       // the previous tile's stores have read the staging buffers: prefetch this tile's
       // residual chunks into them while the MMAs run
       if (lane == 0) bulk_wait_read<0>();
@@ -1105,22 +1094,23 @@ linear_lnc_kernel(const __grid_constant__ CUtensorMap tmA, const __grid_constant
       }
       rphase ^= 1;
       asm volatile("tcgen05.wait::st.sync.aligned;" ::: "memory");
-      // row statistics to the P CTAs holding these rows (ranks 2pp + r), this one included
+      // row statistics to the P CTAs holding these rows (ranks 2pp + r), this one included:
+      // st.async with complete_tx on the receiver's mbarrier -- no release fence per store
+      // (a release.cluster arrive per partial cost ~1/3 of the epilogue's issue samples)
       {
         const uint32_t slot = smem_u32(&stats[(acc * 2 * P + wid) * 128 + srow]);
         const uint32_t bar = smem_u32(&sfull[acc]);
 #pragma unroll
         for (int pp = 0; pp < P; ++pp) {
           const uint32_t rank = 2u * pp + r;
-          asm volatile("st.shared::cluster.v2.f32 [%0], {%1, %2};" ::"r"(mapa_rank(slot, rank)),
-                       "f"(sum), "f"(sumsq)
-                       : "memory");
-          asm volatile("mbarrier.arrive.release.cluster.shared::cluster.b64 _, [%0];" ::"r"(
-                           mapa_rank(bar, rank))
-                       : "memory");
+          asm volatile(
+              "st.async.shared::cluster.mbarrier::complete_tx::bytes.v2.f32 [%0], {%1, %2}, [%3];" ::"r"(
+                  mapa_rank(slot, rank)),
+              "f"(sum), "f"(sumsq), "r"(mapa_rank(bar, rank))
+              : "memory");
         }
       }
-      mbar_wait_cluster(&sfull[acc], acc_phase);
+      mbar_wait(&sfull[acc], acc_phase);
       float s1 = 0.f, s2 = 0.f;
 #pragma unroll
       for (int k = 0; k < 2 * P; ++k) {
