@@ -7,11 +7,14 @@
 // requests) are never loaded or computed.  Per chunk:
 //   S = Q K^T       tcgen05.mma M=128 N=128 K=64 (Q, K K-major in smem) -> TMEM (fp32)
 //   softmax         8 warps: thread = one query row (its TMEM lane) x 64 of the 128 key
-//                   columns; mask = key outside the row's own request -> p = 0 exactly;
-//                   online max with lazy rescaling (O is only rescaled when the running
-//                   max grows by more than 2^8); p = 2^(s*log2e/sqrt(d) - m) in fp32, row
-//                   sum in fp32, P rounded to bf16 into smem (K-major, 128B swizzle)
-//   O += P V        tcgen05.mma M=128 N=64 K=128 (P K-major, V MN-major in smem) -> TMEM
+//                   columns (key half h); mask = key outside the row's own request -> p = 0
+//                   exactly; each key half keeps its OWN running max m_h and sum l_h (lazy
+//                   rescaling: O_h is only rescaled when m_h grows by more than 2^8), so the
+//                   two warps of a row never synchronise; p = 2^(s*log2e/sqrt(d) - m_h) in
+//                   fp32, row sum in fp32, P rounded to bf16 into smem (K-major, 128B swizzle)
+//   O_h += P_h V_h  tcgen05.mma M=128 N=64 K=64 per key half (P K-major, V MN-major in smem)
+//                   into two TMEM accumulators; the epilogue merges them:
+//                   O = (2^(m_0-m) O_0 + 2^(m_1-m) O_1) / (2^(m_0-m) l_0 + 2^(m_1-m) l_1)
 // Roles (one CTA per SM, persistent over items): warp 0 = item metadata + Q TMA, warp 1 =
 // MMA issuer (one thread), warp 2 = TMEM allocator, then K/V TMA producer, warps 4..11 =
 // softmax/epilogue.  Q/K/V rings and S/P double buffers are mbarrier-guarded, so loads,
@@ -166,9 +169,6 @@ __device__ __forceinline__ void tmem_st32(uint32_t taddr, const uint32_t (&v)[32
       "r"(v[29]), "r"(v[30]), "r"(v[31])
       : "memory");
 }
-__device__ __forceinline__ void named_bar(int id, int threads) {
-  asm volatile("bar.sync %0, %1;" ::"r"(id), "r"(threads) : "memory");
-}
 __device__ __forceinline__ float fmax3(float a, float b, float c) {
   float d;
   asm("max.f32 %0, %1, %2, %3;" : "=f"(d) : "f"(a), "f"(b), "f"(c));
@@ -245,8 +245,8 @@ attn_tc_kernel(const __grid_constant__ CUtensorMap tmQKV, const int32_t* __restr
   const uint32_t sP = sV + kKVStages * kTileBytes;             // [2][2 blocks][128 x 64]
   uint8_t* gen = smem_raw + (sP + 2 * kPBytes - raw);
   ItemInfo* infos = reinterpret_cast<ItemInfo*>(gen);          // [3]
-  float* xch = reinterpret_cast<float*>(gen + kQStages * sizeof(ItemInfo));   // max: [2 bufs][2][128]
-  float* lbuf = xch + 4 * TQ;                                  // row sums: [2 items][2 halves][128]
+  float* mbuf = reinterpret_cast<float*>(gen + kQStages * sizeof(ItemInfo));  // row maxima: [2 items][2 halves][128]
+  float* lbuf = mbuf + 4 * TQ;                                 // row sums: [2 items][2 halves][128]
   int* meta = reinterpret_cast<int*>(lbuf + 4 * TQ);           // [2 items]: item has an O
   uint32_t* tmem_slot = reinterpret_cast<uint32_t*>(meta + 4);
   const uint32_t bars = (smem_u32(tmem_slot + 4) + 7) & ~7u;
@@ -288,7 +288,7 @@ attn_tc_kernel(const __grid_constant__ CUtensorMap tmQKV, const int32_t* __restr
   tc_fence_before();
   __syncthreads();
   tc_fence_after();
-  const uint32_t tmem = *tmem_slot;           // S0: +0, S1: +128, O: +256
+  const uint32_t tmem = *tmem_slot;           // S0: +0, S1: +128, O[item & 1][half]: +256 + 128 (item & 1) + 64 half
   pdl_wait();                                 // QKV / segment ids come from earlier kernels
   pdl_trigger();
 
@@ -359,8 +359,8 @@ attn_tc_kernel(const __grid_constant__ CUtensorMap tmQKV, const int32_t* __restr
 #pragma unroll
         for (int k = 0; k < TK / 16; ++k) {
           const uint32_t a_addr = pa + (k >> 2) * kTileBytes + (k & 3) * 32;
-          tc_mma(tmem + 256 + (pp.it & 1) * 64, desc_kmajor(a_addr), desc_mnmajor(va + k * 2048),
-                 kIdescPV, (!pp.first || k > 0) ? 1u : 0u);
+          tc_mma(tmem + 256 + (pp.it & 1) * 128 + (k >> 2) * 64, desc_kmajor(a_addr),
+                 desc_mnmajor(va + k * 2048), kIdescPV, (!pp.first || (k & 3) > 0) ? 1u : 0u);
         }
         tc_commit(p_empty + 8 * b);
         tc_commit(kv_empty + 8 * pp.stage);
@@ -421,40 +421,77 @@ attn_tc_kernel(const __grid_constant__ CUtensorMap tmQKV, const int32_t* __restr
       const int lb = k & 1;
       mbar_wait(l_full + 8 * lb, (k >> 1) & 1);
       const bool has_o = meta[lb] != 0;
-      const float lt = lbuf[(lb * 2) * TQ + row] + lbuf[(lb * 2 + 1) * TQ + row];
-      uint32_t o[64];
+      // merge the two key halves: weights 2^(m_h - m) (0 for a half that saw no key)
+      const float m0 = mbuf[(lb * 2) * TQ + row], m1 = mbuf[(lb * 2 + 1) * TQ + row];
+      const float l0 = lbuf[(lb * 2) * TQ + row], l1 = lbuf[(lb * 2 + 1) * TQ + row];
+      const float mm = fmaxf(m0, m1);
+      const float w0 = m0 == -INFINITY ? 0.f : ex2((m0 - mm) * scale_log2);
+      const float w1 = m1 == -INFINITY ? 0.f : ex2((m1 - mm) * scale_log2);
+      const float den = w0 * l0 + w1 * l1;
+      const float inv = (has_o && den > 0.f) ? 1.f / den : 0.f;
+      const float a0 = w0 * inv, a1 = w1 * inv;
+      const int64_t grow = static_cast<int64_t>(qb) * TQ + row;
+      uint4* dst = reinterpret_cast<uint4*>(O + grow * d_model + h * DH);
+      const uint32_t os = oit & 1;
       if (has_o) {
-        const uint32_t os = oit & 1;
         mbar_wait(o_full + 8 * os, (oit >> 1) & 1);
         tc_fence_after();
-        tmem_ld64_sync(tmem + lane_off + 256 + os * 64, o);
-        tc_fence_before();
-        ++oit;
       }
-      __syncwarp();
-      if (lane == 0) {
-        if (has_o) mbar_arrive(o_empty + 8 * (oit - 1 & 1));
-        mbar_arrive(l_empty + 8 * lb);
-      }
-      const float inv = (has_o && lt > 0.f) ? 1.f / lt : 0.f;
-      const int64_t grow = static_cast<int64_t>(qb) * TQ + row;
-      if (grow < num_slots) {
-        uint4* dst = reinterpret_cast<uint4*>(O + grow * d_model + h * DH);
-#pragma unroll
-        for (int t = 0; t < 8; ++t) {
-          uint4 x;
-          uint32_t* xp = reinterpret_cast<uint32_t*>(&x);
-#pragma unroll
-          for (int e = 0; e < 4; ++e) {
-            const int j = 8 * t + 2 * e;
-            const float a = inv == 0.f ? 0.f : __uint_as_float(o[j]) * inv;
-            const float bq = inv == 0.f ? 0.f : __uint_as_float(o[j + 1]) * inv;
-            __nv_bfloat162 hv = __floats2bfloat162_rn(a, bq);
-            xp[e] = *reinterpret_cast<uint32_t*>(&hv);
+#pragma unroll 1
+      for (int cq = 0; cq < 2; ++cq) {          // 32 output columns at a time
+        uint32_t o[64];
+        if (has_o) {
+          const uint32_t ob = tmem + lane_off + 256 + os * 128 + cq * 32;
+          asm volatile(
+              "tcgen05.ld.sync.aligned.32x32b.x32.b32 "
+              "{%0,%1,%2,%3,%4,%5,%6,%7,%8,%9,%10,%11,%12,%13,%14,%15,"
+              "%16,%17,%18,%19,%20,%21,%22,%23,%24,%25,%26,%27,%28,%29,%30,%31}, [%64];\n\t"
+              "tcgen05.ld.sync.aligned.32x32b.x32.b32 "
+              "{%32,%33,%34,%35,%36,%37,%38,%39,%40,%41,%42,%43,%44,%45,%46,%47,"
+              "%48,%49,%50,%51,%52,%53,%54,%55,%56,%57,%58,%59,%60,%61,%62,%63}, [%65];\n\t"
+              "tcgen05.wait::ld.sync.aligned;"
+              : "=r"(o[0]), "=r"(o[1]), "=r"(o[2]), "=r"(o[3]), "=r"(o[4]), "=r"(o[5]), "=r"(o[6]),
+                "=r"(o[7]), "=r"(o[8]), "=r"(o[9]), "=r"(o[10]), "=r"(o[11]), "=r"(o[12]),
+                "=r"(o[13]), "=r"(o[14]), "=r"(o[15]), "=r"(o[16]), "=r"(o[17]), "=r"(o[18]),
+                "=r"(o[19]), "=r"(o[20]), "=r"(o[21]), "=r"(o[22]), "=r"(o[23]), "=r"(o[24]),
+                "=r"(o[25]), "=r"(o[26]), "=r"(o[27]), "=r"(o[28]), "=r"(o[29]), "=r"(o[30]),
+                "=r"(o[31]), "=r"(o[32]), "=r"(o[33]), "=r"(o[34]), "=r"(o[35]), "=r"(o[36]),
+                "=r"(o[37]), "=r"(o[38]), "=r"(o[39]), "=r"(o[40]), "=r"(o[41]), "=r"(o[42]),
+                "=r"(o[43]), "=r"(o[44]), "=r"(o[45]), "=r"(o[46]), "=r"(o[47]), "=r"(o[48]),
+                "=r"(o[49]), "=r"(o[50]), "=r"(o[51]), "=r"(o[52]), "=r"(o[53]), "=r"(o[54]),
+                "=r"(o[55]), "=r"(o[56]), "=r"(o[57]), "=r"(o[58]), "=r"(o[59]), "=r"(o[60]),
+                "=r"(o[61]), "=r"(o[62]), "=r"(o[63])
+              : "r"(ob), "r"(ob + 64)
+              : "memory");
+        }
+        if (cq == 1) {                          // O and the row statistics are consumed
+          tc_fence_before();
+          __syncwarp();
+          if (lane == 0) {
+            if (has_o) mbar_arrive(o_empty + 8 * os);
+            mbar_arrive(l_empty + 8 * lb);
           }
-          dst[t] = x;
+        }
+        if (grow < num_slots) {
+#pragma unroll
+          for (int t = 0; t < 4; ++t) {
+            uint4 x;
+            uint32_t* xp = reinterpret_cast<uint32_t*>(&x);
+#pragma unroll
+            for (int e = 0; e < 4; ++e) {
+              const int j = 8 * t + 2 * e;
+              const float a = inv == 0.f ? 0.f
+                                         : fmaf(__uint_as_float(o[j]), a0, __uint_as_float(o[32 + j]) * a1);
+              const float bq = inv == 0.f ? 0.f
+                                          : fmaf(__uint_as_float(o[j + 1]), a0, __uint_as_float(o[33 + j]) * a1);
+              __nv_bfloat162 hv = __floats2bfloat162_rn(a, bq);
+              xp[e] = *reinterpret_cast<uint32_t*>(&hv);
+            }
+            dst[cq * 4 + t] = x;
+          }
         }
       }
+      if (has_o) ++oit;
     }
   } else if (warp >= 4) {
     // ================= softmax =================
@@ -549,13 +586,9 @@ attn_tc_kernel(const __grid_constant__ CUtensorMap tmQKV, const int32_t* __restr
             }
           }
         }
-        const float mx = fmaxf(fmaxf(fmaxf(mxp[0], mxp[1]), fmaxf(mxp[2], mxp[3])),
-                               fmaxf(fmaxf(mxp[4], mxp[5]), fmaxf(mxp[6], mxp[7])));
-        // row max across the two column halves (double-buffered exchange: one barrier)
-        float* xb = xch + (gc & 1) * 2 * TQ;
-        xb[half * TQ + row] = mx;
-        named_bar(1 + q, 64);
-        const float rmax = fmaxf(xb[row], xb[TQ + row]);
+        // this key half's row max (the other half keeps its own; merged in the epilogue)
+        const float rmax = fmaxf(fmaxf(fmaxf(mxp[0], mxp[1]), fmaxf(mxp[2], mxp[3])),
+                                 fmaxf(fmaxf(mxp[4], mxp[5]), fmaxf(mxp[6], mxp[7])));
 #ifdef TCB_ATTN_PROBE
         long long t3 = clock64();
         p_max += t3 - t2;
@@ -574,12 +607,15 @@ attn_tc_kernel(const __grid_constant__ CUtensorMap tmQKV, const int32_t* __restr
           mbar_wait(p_empty + 8 * pb, pu & 1);
           tc_fence_after();
           const float f = grow ? ex2((m_used - rmax) * scale_log2) : 1.f;
-          uint32_t o[32];
-          const uint32_t oaddr = tmem + lane_off + 256 + (it & 1) * 64 + half * 32;
-          tmem_ld32_sync(oaddr, o);
+          const uint32_t oaddr = tmem + lane_off + 256 + (it & 1) * 128 + half * 64;
+#pragma unroll 1
+          for (int cq = 0; cq < 2; ++cq) {
+            uint32_t o[32];
+            tmem_ld32_sync(oaddr + 32 * cq, o);
 #pragma unroll
-          for (int t = 0; t < 32; ++t) o[t] = __float_as_uint(__uint_as_float(o[t]) * f);
-          tmem_st32(oaddr, o);
+            for (int t = 0; t < 32; ++t) o[t] = __float_as_uint(__uint_as_float(o[t]) * f);
+            tmem_st32(oaddr + 32 * cq, o);
+          }
           asm volatile("tcgen05.wait::st.sync.aligned;" ::: "memory");
           if (grow) {
             l *= f;
@@ -633,6 +669,7 @@ attn_tc_kernel(const __grid_constant__ CUtensorMap tmQKV, const int32_t* __restr
         const int lb = ic & 1;
         if (ic >= 2) mbar_wait(l_empty + 8 * lb, ((ic >> 1) & 1) ^ 1);
         lbuf[(lb * 2 + half) * TQ + row] = l;
+        mbuf[(lb * 2 + half) * TQ + row] = m_used;
         if (sw == 0 && lane == 0) meta[lb] = nch > 0 ? 1 : 0;
         __syncwarp();
         if (lane == 0) mbar_arrive(l_full + 8 * lb);
