@@ -38,8 +38,20 @@ def _compile(src: str, verbose: bool) -> str:
     return obj
 
 
+STAMP = SO + ".flags"   # nvcc flags of the current libtcb.so (a stale
+                        # instrumented build must not be reused; ships with the .so)
+
+
+def _stamp_ok() -> bool:
+    try:
+        return open(STAMP).read() == " ".join(ARCH + FLAGS)
+    except OSError:
+        return False
+
+
 def build(force: bool = False, verbose: bool = False) -> str:
-    if not force and os.path.exists(SO) and os.path.getmtime(SO) >= _newest_dep():
+    if (not force and os.path.exists(SO) and os.path.getmtime(SO) >= _newest_dep()
+            and _stamp_ok()):
         return SO
     os.makedirs(BUILD, exist_ok=True)
     with cf.ThreadPoolExecutor(max_workers=len(SOURCES)) as ex:
@@ -50,6 +62,8 @@ def build(force: bool = False, verbose: bool = False) -> str:
     if r.returncode != 0:
         raise RuntimeError(f"link failed:\n{r.stdout}\n{r.stderr}")
     os.replace(tmp, SO)
+    with open(STAMP, "w") as f:
+        f.write(" ".join(ARCH + FLAGS))
     return SO
 
 

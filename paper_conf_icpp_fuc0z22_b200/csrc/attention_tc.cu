@@ -503,7 +503,7 @@ attn_tc_kernel(const __grid_constant__ CUtensorMap tmQKV, const int32_t* __restr
     int qs = 0;
     uint32_t qph = 0, gc = 0, it = 0;
 #ifdef TCB_ATTN_PROBE
-    long long p_start = clock64(), p_sfull = 0, p_ld = 0, p_max = 0, p_pempty = 0, p_exp = 0, p_q = 0, p_fin = 0;
+    long long p_start = clock64(), p_sfull = 0, p_ld = 0, p_max = 0, p_pempty = 0, p_exp = 0, p_q = 0, p_fin = 0, p_resc = 0;
 #endif
     int ic = 0;                             // items processed (row-sum hand-over buffers)
     for (int item = blockIdx.x; item < num_items; item += gridDim.x) {
@@ -625,6 +625,7 @@ attn_tc_kernel(const __grid_constant__ CUtensorMap tmQKV, const int32_t* __restr
         const float off = m_used == -INFINITY ? 0.f : -m_used * scale_log2;
 #ifdef TCB_ATTN_PROBE
         long long t4 = clock64();
+        p_resc += t4 - t3;
 #endif
         // P buffer b is free once P V of chunk gc-2 is done
         if (gc >= 2) mbar_wait(p_empty + 8 * b, (u & 1) ^ 1);
@@ -665,6 +666,9 @@ attn_tc_kernel(const __grid_constant__ CUtensorMap tmQKV, const int32_t* __restr
         ++gc;
       }
       // hand the row sums to the epilogue warps (buffer ic & 1, free once they read item ic-2)
+#ifdef TCB_ATTN_PROBE
+      long long tf = clock64();
+#endif
       {
         const int lb = ic & 1;
         if (ic >= 2) mbar_wait(l_empty + 8 * lb, ((ic >> 1) & 1) ^ 1);
@@ -675,12 +679,15 @@ attn_tc_kernel(const __grid_constant__ CUtensorMap tmQKV, const int32_t* __restr
         if (lane == 0) mbar_arrive(l_full + 8 * lb);
         ++ic;
       }
+#ifdef TCB_ATTN_PROBE
+      p_fin += clock64() - tf;
+#endif
       if (nch > 0) ++it;
     }
 #ifdef TCB_ATTN_PROBE
     if (lane == 0 && blockIdx.x == 0 && (sw == 0 || sw == 5))
-      printf("tcprobe warp %d total %lld wait_q %lld wait_s %lld tmem_ld %lld max %lld wait_p %lld exp %lld finish %lld chunks %u\n",
-             warp, clock64() - p_start, p_q, p_sfull, p_ld, p_max, p_pempty, p_exp, p_fin, gc);
+      printf("tcprobe warp %d total %lld wait_q %lld wait_s %lld tmem_ld %lld max %lld rescale %lld wait_p %lld exp %lld finish %lld chunks %u\n",
+             warp, clock64() - p_start, p_q, p_sfull, p_ld, p_max, p_resc, p_pempty, p_exp, p_fin, gc);
 #endif
   }
   __syncwarp();
