@@ -886,13 +886,22 @@ __device__ __forceinline__ void tmem_ld2x32_sync(uint32_t taddr, uint32_t (&a)[3
 // the statistics slots of the P CTAs holding the same 128 rows (itself included) with
 // st.shared::cluster and arrives on their mbarrier (release.cluster); pass 2 normalises once
 // all 2P partials of its rows are in.  Pad slots (segment id < 0) are written as 0 (R12).
-constexpr int kLncEpiWarps = 8;
-constexpr int kLncChunks = 4;                                         // 32-col chunks per warp
+// Epilogue warps: 4 per TMEM lane quarter x kLncColGroups column groups of the pair's 256
+// columns.  8 warps (128 columns each) is the default: 16 warps (64 columns each, 96
+// registers) measured 2% faster for C3's W_O but 6-8% slower for C4/C5's W_O and FFN2.
+#ifndef TCB_LNC_EPI_WARPS
+#define TCB_LNC_EPI_WARPS 8
+#endif
+constexpr int kLncEpiWarps = TCB_LNC_EPI_WARPS;
+constexpr int kLncColGroups = kLncEpiWarps / 4;                       // per pair, per lane quarter
+constexpr int kLncChunks = 256 / kLncColGroups / 32;                  // 32-col chunks per warp
+constexpr int kLncThreads = (4 + kLncEpiWarps) * 32;
 template <int P>
 struct LncCfg {
   static constexpr int kStageBytes = 2 * 128 * BK * 2;               // A 128 rows + W 128 rows
   static constexpr int kEpiBytes = kLncEpiWarps * kLncChunks * kStageBufBytes;   // 64 KB
-  static constexpr int kStatBytes = 2 * 2 * P * 128 * 8;             // [acc][2P][128] float2
+  static constexpr int kContrib = P * kLncColGroups;                 // partials per row
+  static constexpr int kStatBytes = 2 * kContrib * 128 * 8;           // [acc][contrib][128] float2
   static constexpr int kStages =
       (227 * 1024 - 1024 - kEpiBytes - kStatBytes - 1024) / kStageBytes;
   static constexpr int kSmemBytes =
@@ -914,7 +923,7 @@ __device__ __forceinline__ void tc_commit_mask(uint64_t* bar, uint16_t mask) {
       : "memory");
 }
 template <int P>
-__global__ void __launch_bounds__(kThreads, 1)
+__global__ void __launch_bounds__(kLncThreads, 1)
 linear_lnc_kernel(const __grid_constant__ CUtensorMap tmA, const __grid_constant__ CUtensorMap tmW,
                   const __grid_constant__ CUtensorMap tmC, const __grid_constant__ CUtensorMap tmR,
                   int M, int K, const float* __restrict__ bias, const float* __restrict__ gamma,
@@ -1024,8 +1033,8 @@ linear_lnc_kernel(const __grid_constant__ CUtensorMap tmA, const __grid_constant
     // ===== Epilogue: bias + residual, DSMEM row statistics, LayerNorm, TMA store =====
     const int ew = warp - 4;
     const int q = warp & 3;                       // TMEM lane quarter
-    const int half = ew >> 2;                     // 128-column half of the pair's 256
-    const int wid = static_cast<int>(p) * 2 + half;   // this warp's contribution slot (0..2P-1)
+    const int cg = ew >> 2;                       // column group of the pair's 256
+    const int wid = static_cast<int>(p) * kLncColGroups + cg;   // contribution slot of this warp
     const int srow = q * 32 + lane;               // row within this CTA's 128
     const uint32_t bufs = smem_u32(sEpi) + ew * kLncChunks * kStageBufBytes;
     uint64_t* my_rbar = rbar + kLncChunks * ew;
@@ -1034,12 +1043,12 @@ linear_lnc_kernel(const __grid_constant__ CUtensorMap tmA, const __grid_constant
     uint32_t acc_phase = 0, rphase = 0;
     for (int tile = cluster_id; tile < num_tiles; tile += num_clusters) {
       const int row0 = tile * 256 + static_cast<int>(r) * 128 + q * 32;
-      const int col0 = static_cast<int>(p) * 256 + half * 128;
+      const int col0 = static_cast<int>(p) * 256 + cg * (32 * kLncChunks);
       const int64_t grow = static_cast<int64_t>(row0) + lane;
       const bool pad = grow >= M || (seg_ids && __ldg(&seg_ids[grow]) < 0);
       // this tile's phase of the statistics barrier completes once all 2P x 128 partials
       // (8 B each, from this CTA and its P-1 peers) have landed
-      if (ew == 0 && lane == 0) mbar_expect_tx(&sfull[acc], 2 * P * 128 * 8);
+      if (ew == 0 && lane == 0) mbar_expect_tx(&sfull[acc], Cfg::kContrib * 128 * 8);
       // the previous tile's stores have read the staging buffers: prefetch this tile's
       // residual chunks into them while the MMAs run
       if (lane == 0) bulk_wait_read<0>();
@@ -1054,7 +1063,7 @@ linear_lnc_kernel(const __grid_constant__ CUtensorMap tmA, const __grid_constant
       mbar_wait(&tfull[acc], acc_phase);
       tc_fence_after();
       const uint32_t tbase = tmem_base + (static_cast<uint32_t>(q * 32) << 16) +
-                             static_cast<uint32_t>(acc * 256 + half * 128);
+                             static_cast<uint32_t>(acc * 256 + cg * (32 * kLncChunks));
       // pass 1: z = acc + bias + residual -> TMEM; row partial moments
       float sum = 0.f, sumsq = 0.f;
 #pragma unroll 1
@@ -1098,7 +1107,7 @@ linear_lnc_kernel(const __grid_constant__ CUtensorMap tmA, const __grid_constant
       // st.async with complete_tx on the receiver's mbarrier -- no release fence per store
       // (a release.cluster arrive per partial cost ~1/3 of the epilogue's issue samples)
       {
-        const uint32_t slot = smem_u32(&stats[(acc * 2 * P + wid) * 128 + srow]);
+        const uint32_t slot = smem_u32(&stats[(acc * Cfg::kContrib + wid) * 128 + srow]);
         const uint32_t bar = smem_u32(&sfull[acc]);
 #pragma unroll
         for (int pp = 0; pp < P; ++pp) {
@@ -1113,8 +1122,8 @@ linear_lnc_kernel(const __grid_constant__ CUtensorMap tmA, const __grid_constant
       mbar_wait(&sfull[acc], acc_phase);
       float s1 = 0.f, s2 = 0.f;
 #pragma unroll
-      for (int k = 0; k < 2 * P; ++k) {
-        const float2 st = stats[(acc * 2 * P + k) * 128 + srow];
+      for (int k = 0; k < Cfg::kContrib; ++k) {
+        const float2 st = stats[(acc * Cfg::kContrib + k) * 128 + srow];
         s1 += st.x;
         s2 += st.y;
       }
@@ -1261,7 +1270,7 @@ cudaError_t launch_lnc(const GemmMaps& m, int M, int K, const float* bias, const
   auto kern = linear_lnc_kernel<P>;
   static int max_clusters = 0;
   cudaLaunchConfig_t cfg{};
-  cfg.blockDim = dim3(kThreads);
+  cfg.blockDim = dim3(kLncThreads);
   cfg.dynamicSmemBytes = Cfg::kSmemBytes;
   cfg.stream = s;
   cudaLaunchAttribute attr[2];
