@@ -97,7 +97,7 @@ tcb_status check_device() {
 constexpr size_t align256(size_t x) { return (x + 255) & ~static_cast<size_t>(255); }
 
 struct WsLayout {
-  size_t seg, qkv, att, z, x1, h, total;
+  size_t seg, qkv, att, z, x1, h, lnst, lncnt, lncnt_per_launch, total;
 };
 WsLayout ws_layout(const tcb_model_config& c, int64_t M) {
   const size_t es = c.dtype == 0 ? 4 : 2;
@@ -109,6 +109,17 @@ WsLayout ws_layout(const tcb_model_config& c, int64_t M) {
   L.z = off;   off += align256(es * static_cast<size_t>(M) * c.d_model);
   L.x1 = off;  off += align256(es * static_cast<size_t>(M) * c.d_model);
   L.h = off;   off += align256(es * static_cast<size_t>(M) * c.d_ff);
+  // row-statistics scratch of the L2-exchange LayerNorm GEMM (bf16, d = 768 / 1024): partials
+  // per 256-row tile, and one zeroed counter region per fused launch (2 per layer)
+  L.lnst = off;
+  L.lncnt = off;
+  L.lncnt_per_launch = 0;
+  if (c.dtype == 1 && (c.d_model == 768 || c.d_model == 1024)) {
+    off += align256(tcb::k::linear_ln_scratch_stats_bytes(M, c.d_model));
+    L.lncnt = off;
+    L.lncnt_per_launch = align256(tcb::k::linear_ln_scratch_cnt_bytes(M));
+    off += L.lncnt_per_launch * 2 * static_cast<size_t>(c.num_layers);
+  }
   L.total = off;
   return L;
 }
@@ -380,6 +391,14 @@ tcb_status tcb_encoder_forward(const tcb_weights* wc, const tcb_plan* plan,
     // kernels.
     static const bool no_fusion = std::getenv("TCB_NO_LN_FUSION") != nullptr;
     const bool fuse_ln = !no_fusion && tcb::k::linear_ln_supported(d);
+    float2* lnst = L.lncnt_per_launch ? reinterpret_cast<float2*>(ws + L.lnst) : nullptr;
+    auto lncnt = [&](int launch) -> int* {
+      return L.lncnt_per_launch ? reinterpret_cast<int*>(ws + L.lncnt + L.lncnt_per_launch * launch)
+                                : nullptr;
+    };
+    if (fuse_ln && L.lncnt_per_launch &&
+        cudaMemsetAsync(ws + L.lncnt, 0, L.lncnt_per_launch * 2 * c.num_layers, s) != cudaSuccess)
+      return fail(TCB_ERR_CUDA, "tcb_encoder_forward: counter reset failed");
     for (int l = 0; l < c.num_layers; ++l) {
       const auto& mp = w->maps[l];
       const tcb::k::GemmMaps g_qkv{w->aX, mp.qkv, w->cQkv, w->cQkv};
@@ -393,7 +412,7 @@ tcb_status tcb_encoder_forward(const tcb_weights* wc, const tcb_plan* plan,
         const tcb::k::GemmMaps g_o_ln{w->aAtt, mp.o, w->cX1, w->cX};
         TCB_LAUNCH(TCB_K_GEMM_O, s, tcb::k::launch_linear_ln_bf16_tc(
                                         g_o_ln, M, d, d, w->Lf(l, B_O), w->Lf(l, LN1_G),
-                                        w->Lf(l, LN1_B), c.ln_eps, seg, s));
+                                        w->Lf(l, LN1_B), c.ln_eps, seg, s, lnst, lncnt(2 * l)));
       } else {
         TCB_LAUNCH(TCB_K_GEMM_O, s, tcb::k::launch_linear_bf16_tc(g_o, M, d, d, w->Lf(l, B_O),
                                                                   TCB_EPI_BIAS_RESIDUAL, s));
@@ -406,7 +425,7 @@ tcb_status tcb_encoder_forward(const tcb_weights* wc, const tcb_plan* plan,
         const tcb::k::GemmMaps g_2_ln{w->aH, mp.w2, w->cX, w->cX1};
         TCB_LAUNCH(TCB_K_GEMM_FFN2, s, tcb::k::launch_linear_ln_bf16_tc(
                                            g_2_ln, M, d, f, w->Lf(l, B_2), w->Lf(l, LN2_G),
-                                           w->Lf(l, LN2_B), c.ln_eps, seg, s));
+                                           w->Lf(l, LN2_B), c.ln_eps, seg, s, lnst, lncnt(2 * l + 1)));
       } else {
         TCB_LAUNCH(TCB_K_GEMM_FFN2, s, tcb::k::launch_linear_bf16_tc(g_2, M, d, f, w->Lf(l, B_2),
                                                                      TCB_EPI_BIAS_RESIDUAL, s));
@@ -512,8 +531,32 @@ tcb_status tcb_op_linear_ln(int64_t M, int32_t N, int32_t K, const void* A, cons
   if (!tcb::k::make_gemm_a_map(&maps.a, A, M, K) || !tcb::k::make_gemm_w_map(&maps.w, W, N, K) ||
       !tcb::k::make_gemm_c_map(&maps.c, C, M, N) || !tcb::k::make_gemm_c_map(&maps.r, R, M, N))
     return fail(TCB_ERR_CUDA, "tcb_op_linear_ln: cuTensorMapEncodeTiled failed (alignment?)");
+  // d >= 768: the row-statistics scratch of the L2-exchange kernel, library-owned for this op
+  // (grown on demand; the encoder forward uses its workspace instead)
+  float2* st = nullptr;
+  int* cnt = nullptr;
+  if (N >= 768) {
+    static std::mutex mu;
+    static void* buf = nullptr;
+    static size_t cap = 0;
+    const size_t sb = (tcb::k::linear_ln_scratch_stats_bytes(M, N) + 255) & ~size_t(255);
+    const size_t need = sb + tcb::k::linear_ln_scratch_cnt_bytes(M);
+    std::lock_guard<std::mutex> g(mu);
+    if (need > cap) {
+      if (buf) cudaFree(buf);
+      buf = nullptr;
+      cap = 0;
+      if (cudaMalloc(&buf, need) != cudaSuccess)
+        return fail(TCB_ERR_OUT_OF_MEMORY, "tcb_op_linear_ln: scratch allocation failed");
+      cap = need;
+    }
+    st = static_cast<float2*>(buf);
+    cnt = reinterpret_cast<int*>(static_cast<uint8_t*>(buf) + sb);
+    if (cudaMemsetAsync(cnt, 0, tcb::k::linear_ln_scratch_cnt_bytes(M), s) != cudaSuccess)
+      return fail(TCB_ERR_CUDA, "tcb_op_linear_ln: counter reset failed");
+  }
   TCB_LAUNCH(TCB_K_GEMM_O, s, tcb::k::launch_linear_ln_bf16_tc(maps, M, N, K, bias, gamma, beta,
-                                                               eps, d_seg, s));
+                                                               eps, d_seg, s, st, cnt));
   return TCB_OK;
 }
 

@@ -106,9 +106,14 @@ cudaError_t launch_linear_bf16_tc(const GemmMaps& maps, int64_t M, int N, int K,
                                   const float* bias, int epi, cudaStream_t s);
 // C = LayerNorm(A W^T + bias + R) * gamma + beta over rows of N = 512 columns (pad rows 0).
 bool linear_ln_supported(int N);
+// lng_stats / lng_cnt (optional scratch, sizes below; cnt zeroed before the launch) select the
+// L2-exchange kernel for N = 1024.
 cudaError_t launch_linear_ln_bf16_tc(const GemmMaps& maps, int64_t M, int N, int K,
                                      const float* bias, const float* gamma, const float* beta,
-                                     float eps, const int32_t* seg_ids, cudaStream_t s);
+                                     float eps, const int32_t* seg_ids, cudaStream_t s,
+                                     float2* lng_stats = nullptr, int* lng_cnt = nullptr);
+size_t linear_ln_scratch_stats_bytes(int64_t M, int N);
+size_t linear_ln_scratch_cnt_bytes(int64_t M);
 
 // Attention ------------------------------------------------------------------------------
 cudaError_t launch_attention_bf16(int64_t num_slots, int d_model, int num_heads,

@@ -1187,6 +1187,274 @@ linear_lnc_kernel(const __grid_constant__ CUtensorMap tmA, const __grid_constant
                  "r"(512) : "memory");
 }
 
+// ---- GEMM + bias + residual + LayerNorm, row statistics exchanged through L2 --------------
+// Same math and per-pair work as linear_lnc_kernel, but with clusters of ONE pair: the P
+// column blocks of a 256-row tile are independent work units u = P t + p, spread round-robin
+// over every CTA pair of the GPU (all 74 pairs -- an 8-CTA cluster fits only 15 times, i.e.
+// on 120 of the 148 SMs), and each unit's row partials (sum z, sum z^2) go through global
+// memory: st.global, then one release add on a per-(tile, CTA rank, lane quarter) counter;
+// the epilogue warps of the other units of the tile acquire-spin on it until all 2P partials
+// are in.  Deadlock-free because every CTA of the grid is resident (grid = max co-resident
+// pairs, one CTA per SM) and a unit only waits for units of its own tile, each of which
+// depends only on work of lower index (its pair's previous units).  The counters of a launch
+// are zeroed by the caller (one memset per forward, a distinct region per launch).
+template <int P>
+__global__ void __launch_bounds__(kLncThreads, 1)
+linear_lng_kernel(const __grid_constant__ CUtensorMap tmA, const __grid_constant__ CUtensorMap tmW,
+                  const __grid_constant__ CUtensorMap tmC, const __grid_constant__ CUtensorMap tmR,
+                  int M, int K, const float* __restrict__ bias, const float* __restrict__ gamma,
+                  const float* __restrict__ beta, float eps, const int32_t* __restrict__ seg_ids,
+                  float2* __restrict__ gstats, int* __restrict__ gcnt) {
+  constexpr int kStageBytes = 2 * 128 * BK * 2;
+  constexpr int kEpiBytes = kLncEpiWarps * kLncChunks * kStageBufBytes;
+  constexpr int S = (227 * 1024 - 1024 - kEpiBytes - 1024) / kStageBytes;
+  constexpr int kABytes = 128 * BK * 2;
+  constexpr int kContrib = P * kLncColGroups;
+  constexpr float kInvN = 1.f / (P * 256);
+  extern __shared__ uint8_t smem_raw[];
+  uint8_t* smem = reinterpret_cast<uint8_t*>((reinterpret_cast<uintptr_t>(smem_raw) + 1023) &
+                                             ~static_cast<uintptr_t>(1023));
+  uint8_t* sA = smem;
+  uint8_t* sB = smem + S * kABytes;
+  uint8_t* sEpi = smem + S * kStageBytes;
+  uint64_t* full = reinterpret_cast<uint64_t*>(sEpi + kEpiBytes);
+  uint64_t* empty = full + S;
+  uint64_t* tfull = empty + S;                               // [2]
+  uint64_t* tempty = tfull + 2;                              // [2] (pair leader)
+  uint64_t* rbar = tempty + 2;                               // [warps][chunks] residual loads
+  uint32_t* tmem_slot = reinterpret_cast<uint32_t*>(rbar + kLncEpiWarps * kLncChunks);
+
+  const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
+  const uint32_t r = cluster_rank() & 1u;
+  const int pair = blockIdx.x >> 1, num_pairs = gridDim.x >> 1;
+  const int num_units = ((M + 255) / 256) * P;
+  const int num_kb = K / BK;
+
+  if (warp == 0 && lane == 0) {
+    asm volatile("prefetch.tensormap [%0];" ::"l"(reinterpret_cast<uint64_t>(&tmA)) : "memory");
+    asm volatile("prefetch.tensormap [%0];" ::"l"(reinterpret_cast<uint64_t>(&tmW)) : "memory");
+    asm volatile("prefetch.tensormap [%0];" ::"l"(reinterpret_cast<uint64_t>(&tmC)) : "memory");
+    for (int i = 0; i < S; ++i) { mbar_init(&full[i], 1); mbar_init(&empty[i], 1); }
+    for (int i = 0; i < 2; ++i) { mbar_init(&tfull[i], 1); mbar_init(&tempty[i], 2 * kLncEpiWarps); }
+    for (int i = 0; i < kLncEpiWarps * kLncChunks; ++i) mbar_init(&rbar[i], 1);
+    asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
+  }
+  if (warp == 2) {
+    asm volatile("tcgen05.alloc.cta_group::2.sync.aligned.shared::cta.b32 [%0], %1;" ::"r"(
+                     smem_u32(tmem_slot)), "r"(512) : "memory");
+    asm volatile("tcgen05.relinquish_alloc_permit.cta_group::2.sync.aligned;" ::: "memory");
+  }
+  tc_fence_before();
+  cluster_sync();
+  tc_fence_after();
+  const uint32_t tmem_base = *tmem_slot;
+  pdl_wait();
+  pdl_trigger();
+
+  if (warp == 0) {
+    // ===== TMA producer: this CTA's 128 A rows and 128 W rows of the unit's column block =====
+    if (lane == 0) {
+      const uint32_t full0 = mapa_rank(smem_u32(full), 0);
+      int stage = 0;
+      uint32_t phase = 0;
+      for (int u = pair; u < num_units; u += num_pairs) {
+        const int t = u / P, p = u % P;
+        const int a_row = t * 256 + static_cast<int>(r) * 128;
+        const int b_row = p * 256 + static_cast<int>(r) * 128;
+        for (int kb = 0; kb < num_kb; ++kb) {
+          mbar_wait(&empty[stage], phase ^ 1);
+          if (r == 0) mbar_expect_tx(&full[stage], 2 * kStageBytes);
+          const uint32_t fb = full0 + 8u * stage;
+          tma_load_2d<2>(sA + stage * kABytes, &tmA, fb, kb * BK, a_row);
+          tma_load_2d<2>(sB + stage * kABytes, &tmW, fb, kb * BK, b_row);
+          if (++stage == S) { stage = 0; phase ^= 1; }
+        }
+      }
+    }
+  } else if (warp == 1) {
+    // ===== MMA issuer: the pair leader drives M=256 x N=256 into accumulator acc =====
+    if (r == 0) {
+      constexpr uint32_t idesc = idesc_bf16<2, 256>();
+      int stage = 0, acc = 0;
+      uint32_t phase = 0, acc_phase = 0;
+      for (int u = pair; u < num_units; u += num_pairs) {
+        mbar_wait(&tempty[acc], acc_phase ^ 1);
+        tc_fence_after();
+        const uint32_t d_tmem = tmem_base + static_cast<uint32_t>(acc * 256);
+        for (int kb = 0; kb < num_kb; ++kb) {
+          mbar_wait(&full[stage], phase);
+          tc_fence_after();
+          if (lane == 0) {
+            const uint32_t a0 = smem_u32(sA + stage * kABytes);
+            const uint32_t b0 = smem_u32(sB + stage * kABytes);
+#pragma unroll
+            for (int k = 0; k < BK / 16; ++k)
+              tc_mma<2>(d_tmem, sdesc_sw128(a0 + k * 32), sdesc_sw128(b0 + k * 32), idesc,
+                        (kb | k) != 0 ? 1u : 0u);
+            tc_commit_mask(&empty[stage], 0x3);
+            if (kb == num_kb - 1) tc_commit_mask(&tfull[acc], 0x3);
+          }
+          __syncwarp();
+          if (++stage == S) { stage = 0; phase ^= 1; }
+        }
+        acc ^= 1;
+        if (acc == 0) acc_phase ^= 1;
+      }
+    }
+  } else if (warp >= 4) {
+    // ===== Epilogue: bias + residual, row statistics through L2, LayerNorm, TMA store =====
+    const int ew = warp - 4;
+    const int q = warp & 3;                       // TMEM lane quarter
+    const int cg = ew >> 2;                       // column group of the unit's 256 columns
+    const int srow = q * 32 + lane;               // row within this CTA's 128
+    const uint32_t bufs = smem_u32(sEpi) + ew * kLncChunks * kStageBufBytes;
+    uint64_t* my_rbar = rbar + kLncChunks * ew;
+    const uint32_t tempty0 = mapa_rank(smem_u32(tempty), 0);
+    int acc = 0;
+    uint32_t acc_phase = 0, rphase = 0;
+    for (int u = pair; u < num_units; u += num_pairs) {
+      const int t = u / P, p = u % P;
+      const int wid = p * kLncColGroups + cg;     // contribution slot of this warp
+      const int row0 = t * 256 + static_cast<int>(r) * 128 + q * 32;
+      const int col0 = p * 256 + cg * (32 * kLncChunks);
+      const int64_t grow = static_cast<int64_t>(row0) + lane;
+      const bool pad = grow >= M || (seg_ids && __ldg(&seg_ids[grow]) < 0);
+      if (lane == 0) bulk_wait_read<0>();
+      __syncwarp();
+      if (lane == 0) {
+#pragma unroll
+        for (int j = 0; j < kLncChunks; ++j) {
+          mbar_expect_tx(&my_rbar[j], kStageBufBytes);
+          tma_load_res(bufs + j * kStageBufBytes, &tmR, &my_rbar[j], col0 + 32 * j, row0);
+        }
+      }
+      mbar_wait(&tfull[acc], acc_phase);
+      tc_fence_after();
+      const uint32_t tbase = tmem_base + (static_cast<uint32_t>(q * 32) << 16) +
+                             static_cast<uint32_t>(acc * 256 + cg * (32 * kLncChunks));
+      // pass 1: z = acc + bias + residual -> TMEM; row partial moments
+      float sum = 0.f, sumsq = 0.f;
+#pragma unroll 1
+      for (int j = 0; j < kLncChunks; ++j) {
+        uint32_t rr[32];
+        tmem_ld32_nowait(tbase + 32 * j, rr);
+        tmem_wait_ld();
+        float* v = reinterpret_cast<float*>(rr);
+        const float4* b4 = reinterpret_cast<const float4*>(bias + col0 + 32 * j);
+#pragma unroll
+        for (int tt = 0; tt < 8; ++tt) {
+          const float4 bb = __ldg(b4 + tt);
+          v[4 * tt + 0] += bb.x;
+          v[4 * tt + 1] += bb.y;
+          v[4 * tt + 2] += bb.z;
+          v[4 * tt + 3] += bb.w;
+        }
+        mbar_wait(&my_rbar[j], rphase);
+        const uint32_t buf = bufs + j * kStageBufBytes;
+#pragma unroll
+        for (int tt = 0; tt < 4; ++tt) {
+          const uint4 x = ld_shared_v4(buf + sw64(lane, tt));
+          const __nv_bfloat162* hh = reinterpret_cast<const __nv_bfloat162*>(&x);
+#pragma unroll
+          for (int e = 0; e < 4; ++e) {
+            const float2 f = __bfloat1622float2(hh[e]);
+            v[8 * tt + 2 * e] += f.x;
+            v[8 * tt + 2 * e + 1] += f.y;
+          }
+        }
+#pragma unroll
+        for (int tt = 0; tt < 32; ++tt) {
+          sum += v[tt];
+          sumsq = fmaf(v[tt], v[tt], sumsq);
+        }
+        tmem_st32(tbase + 32 * j, *reinterpret_cast<float(*)[32]>(v));
+      }
+      rphase ^= 1;
+      asm volatile("tcgen05.wait::st.sync.aligned;" ::: "memory");
+      // publish this warp's partials of its 32 rows, then wait for all kContrib of them
+      float2* tst = gstats + static_cast<size_t>(t) * kContrib * 256 + static_cast<int>(r) * 128 + srow;
+      tst[wid * 256] = make_float2(sum, sumsq);
+      int* cnt = gcnt + t * 8 + static_cast<int>(r) * 4 + q;
+      __syncwarp();
+      if (lane == 0) {
+        asm volatile("fence.acq_rel.gpu;\n\tred.relaxed.gpu.global.add.s32 [%0], 1;" ::"l"(cnt)
+                     : "memory");
+        int seen = 0;
+        do {
+          asm volatile("ld.acquire.gpu.global.s32 %0, [%1];" : "=r"(seen) : "l"(cnt) : "memory");
+        } while (seen < kContrib);
+      }
+      __syncwarp();
+      float s1 = 0.f, s2 = 0.f;
+#pragma unroll
+      for (int k = 0; k < kContrib; ++k) {
+        float2 st;
+        asm volatile("ld.relaxed.gpu.global.v2.f32 {%0, %1}, [%2];"
+                     : "=f"(st.x), "=f"(st.y)
+                     : "l"(tst + k * 256)
+                     : "memory");
+        s1 += st.x;
+        s2 += st.y;
+      }
+      const float mean = s1 * kInvN;
+      const float rstd = rsqrtf(fmaxf(s2 * kInvN - mean * mean, 0.f) + eps);
+      // pass 2: normalise -> bf16 -> staging -> TMA store
+#pragma unroll 1
+      for (int j = 0; j < kLncChunks; ++j) {
+        uint32_t rr[32];
+        tmem_ld32_nowait(tbase + 32 * j, rr);
+        tmem_wait_ld();
+        if (j == kLncChunks - 1) {
+          tc_fence_before();
+          __syncwarp();
+          if (lane == 0) mbar_arrive_remote(tempty0 + 8u * acc);
+        }
+        float* y = reinterpret_cast<float*>(rr);
+        const int gc = col0 + 32 * j;
+        const float4* g4 = reinterpret_cast<const float4*>(gamma + gc);
+        const float4* e4 = reinterpret_cast<const float4*>(beta + gc);
+#pragma unroll
+        for (int tt = 0; tt < 8; ++tt) {
+          const float4 gg = __ldg(g4 + tt), ee = __ldg(e4 + tt);
+          y[4 * tt + 0] = pad ? 0.f : (y[4 * tt + 0] - mean) * rstd * gg.x + ee.x;
+          y[4 * tt + 1] = pad ? 0.f : (y[4 * tt + 1] - mean) * rstd * gg.y + ee.y;
+          y[4 * tt + 2] = pad ? 0.f : (y[4 * tt + 2] - mean) * rstd * gg.z + ee.z;
+          y[4 * tt + 3] = pad ? 0.f : (y[4 * tt + 3] - mean) * rstd * gg.w + ee.w;
+        }
+        const uint32_t buf = bufs + j * kStageBufBytes;
+#pragma unroll
+        for (int tt = 0; tt < 4; ++tt) {
+          uint4 x;
+          __nv_bfloat162* hh = reinterpret_cast<__nv_bfloat162*>(&x);
+#pragma unroll
+          for (int e = 0; e < 4; ++e)
+            hh[e] = __floats2bfloat162_rn(y[8 * tt + 2 * e], y[8 * tt + 2 * e + 1]);
+          st_shared_v4(buf + sw64(lane, tt), x);
+        }
+        fence_async_smem();
+        __syncwarp();
+        if (lane == 0) {
+          asm volatile("cp.async.bulk.tensor.2d.global.shared::cta.bulk_group [%0, {%2, %3}], [%1];" ::"l"(
+                           reinterpret_cast<uint64_t>(&tmC)),
+                       "r"(buf), "r"(gc), "r"(row0)
+                       : "memory");
+          asm volatile("cp.async.bulk.commit_group;" ::: "memory");
+        }
+      }
+      acc ^= 1;
+      if (acc == 0) acc_phase ^= 1;
+    }
+    if (lane == 0) bulk_wait_all();
+  }
+  __syncwarp();
+  tc_fence_before();
+  cluster_sync();
+  tc_fence_after();
+  if (warp == 2)
+    asm volatile("tcgen05.dealloc.cta_group::2.sync.aligned.b32 %0, %1;" ::"r"(tmem_base),
+                 "r"(512) : "memory");
+}
+
 // ---- host side ---------------------------------------------------------------------------
 PFN_cuTensorMapEncodeTiled_v12000 g_encode = nullptr;
 std::once_flag g_encode_once;
@@ -1300,6 +1568,57 @@ cudaError_t launch_lnc(const GemmMaps& m, int M, int K, const float* bias, const
   return cudaLaunchKernelEx(&cfg, kern, m.a, m.w, m.c, m.r, M, K, bias, gamma, beta, eps, seg_ids);
 }
 
+// The L2-exchange kernel (clusters of one pair, every pair of the GPU).  `stats` holds
+// ceil(M/256) * 2P * 256 float2, `cnt` ceil(M/256) * 8 int32 zeroed before the launch.
+template <int P>
+cudaError_t launch_lng(const GemmMaps& m, int M, int K, const float* bias, const float* gamma,
+                       const float* beta, float eps, const int32_t* seg_ids, float2* stats,
+                       int* cnt, cudaStream_t s) {
+  constexpr int kStageBytes = 2 * 128 * BK * 2;
+  constexpr int kEpiBytes = kLncEpiWarps * kLncChunks * kStageBufBytes;
+  constexpr int S = (227 * 1024 - 1024 - kEpiBytes - 1024) / kStageBytes;
+  constexpr int kSmem = 1024 + S * kStageBytes + kEpiBytes + 1024;
+  static_assert(kSmem <= 232448, "shared memory budget");
+  auto kern = linear_lng_kernel<P>;
+  static int max_pairs = 0;
+  cudaLaunchConfig_t cfg{};
+  cfg.blockDim = dim3(kLncThreads);
+  cfg.dynamicSmemBytes = kSmem;
+  cfg.stream = s;
+  cudaLaunchAttribute attr[2];
+  attr[0].id = cudaLaunchAttributeClusterDimension;
+  attr[0].val.clusterDim.x = 2;
+  attr[0].val.clusterDim.y = 1;
+  attr[0].val.clusterDim.z = 1;
+  cfg.attrs = attr;
+  cfg.numAttrs = 1;
+  if (max_pairs == 0) {
+    cudaError_t e = cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, kSmem);
+    if (e != cudaSuccess) return e;
+    cfg.gridDim = dim3(2 * (num_sms() / 2));
+    int n = 0;
+    e = cudaOccupancyMaxActiveClusters(&n, kern, &cfg);
+    if (e != cudaSuccess || n <= 0) {
+      cudaGetLastError();
+      n = num_sms() / 2;
+    }
+    max_pairs = n;               // every CTA of the grid must be co-resident (see the kernel)
+  }
+  const int units = ((M + 255) / 256) * P;
+  const int pairs = units < max_pairs ? units : max_pairs;
+  cfg.gridDim = dim3(2 * pairs);
+  if (pdl_enabled()) pdl_attr(attr[cfg.numAttrs++]);
+  return cudaLaunchKernelEx(&cfg, kern, m.a, m.w, m.c, m.r, M, K, bias, gamma, beta, eps, seg_ids,
+                            stats, cnt);
+}
+
+size_t linear_ln_scratch_stats_bytes(int64_t M, int N) {
+  return static_cast<size_t>((M + 255) / 256) * (N / 256) * kLncColGroups * 256 * sizeof(float2);
+}
+size_t linear_ln_scratch_cnt_bytes(int64_t M) {
+  return static_cast<size_t>((M + 255) / 256) * 8 * sizeof(int);
+}
+
 bool pdl_enabled() {
   static const bool on = [] {
     const char* e = std::getenv("TCB_NO_PDL");
@@ -1310,8 +1629,27 @@ bool pdl_enabled() {
 
 cudaError_t launch_linear_ln_bf16_tc(const GemmMaps& m, int64_t M, int N, int K,
                                      const float* bias, const float* gamma, const float* beta,
-                                     float eps, const int32_t* seg_ids, cudaStream_t s) {
+                                     float eps, const int32_t* seg_ids, cudaStream_t s,
+                                     float2* lng_stats, int* lng_cnt) {
   if (M == 0) return cudaSuccess;
+  // d = 1024, K >= 2d (FFN2) with scratch: the L2-exchange kernel on all 74 pairs (the 8-CTA
+  // cluster kernel fits on 120 SMs only): C4/C5 FFN2 262 -> 218 us.  At K = d (W_O) the
+  // epilogue bounds the kernel and the L2 round trip of the statistics costs more than the
+  // extra SMs give (89 -> 99 us), likewise for d = 768 (57 -> 70 us).  TCB_LN_KERNEL=cluster
+  // forces the cluster kernel, =global the L2-exchange kernel wherever scratch is given.
+  static const int ln_env = [] {
+    const char* e = std::getenv("TCB_LN_KERNEL");
+    if (!e) return 0;
+    return std::string(e) == "cluster" ? 1 : std::string(e) == "global" ? 2 : 0;
+  }();
+  if (lng_stats && lng_cnt && ln_env != 1) {
+    if (N == 1024 && (K >= 2 * N || ln_env == 2))
+      return launch_lng<4>(m, static_cast<int>(M), K, bias, gamma, beta, eps, seg_ids, lng_stats,
+                           lng_cnt, s);
+    if (N == 768 && ln_env == 2)
+      return launch_lng<3>(m, static_cast<int>(M), K, bias, gamma, beta, eps, seg_ids, lng_stats,
+                           lng_cnt, s);
+  }
   // d = 512: the single-pair kernel measured 2% faster per forward (C2) than the 4-CTA
   // cluster kernel; TCB_LN_KERNEL=cluster selects the cluster kernel there too (A/B)
   static const bool pair_512 = [] {

@@ -55,10 +55,12 @@ def test_linear_bf16_tcgen05_vs_oracle(M, N, K, epi):
                                    (1000, 1024, 512), (1000, 2048, 512), (513, 4096, 512),
                                    (32768, 512, 512), (1, 768, 768), (777, 768, 768),
                                    (3001, 3072, 768), (300, 1024, 1024), (2049, 4096, 1024),
-                                   (32768, 1024, 1024)])
+                                   (1, 4096, 1024), (300, 2048, 1024), (32768, 1024, 1024),
+                                   (32768, 4096, 1024)])
 def test_linear_ln_fused_vs_oracle(M, K, N):
     """W_O / FFN2 + bias + residual + LayerNorm in one tcgen05 kernel (N = 512, 768, 1024:
-    clusters of N / 256 CTA pairs exchanging the row statistics over DSMEM)."""
+    clusters of N / 256 CTA pairs exchanging the row statistics over DSMEM; N = 1024 with
+    K >= 2048: single pairs exchanging them through L2)."""
     rng = np.random.default_rng(M + K + N)
     A = _bf16(rng.normal(size=(M, K)))
     W = _bf16(rng.uniform(-1, 1, size=(N, K)) * np.sqrt(3.0 / K))
@@ -88,6 +90,19 @@ def test_linear_ln_cluster_kernel_at_d512():
     code = ("import sys; sys.path.insert(0, 'tests'); import test_gpu_kernels as t; "
             "t.test_linear_ln_fused_vs_oracle(4133, 1024, 512); t.test_linear_ln_fused_vs_oracle(1, 512, 512)")
     env = dict(os.environ, TCB_LN_KERNEL="cluster")
+    r = subprocess.run([sys.executable, "-c", code], env=env, capture_output=True, text=True,
+                       cwd=os.path.dirname(os.path.dirname(os.path.abspath(__file__))), timeout=300)
+    assert r.returncode == 0, r.stderr[-2000:]
+
+
+def test_linear_ln_l2_exchange_kernel_everywhere():
+    """TCB_LN_KERNEL=global runs the L2-exchange kernel for every N = 768 / 1024 shape
+    (the default keeps the cluster kernel there): subprocess, the choice is read once."""
+    import subprocess, sys, os
+    code = ("import sys; sys.path.insert(0, 'tests'); import test_gpu_kernels as t; "
+            "t.test_linear_ln_fused_vs_oracle(777, 768, 768); t.test_linear_ln_fused_vs_oracle(1, 768, 768); "
+            "t.test_linear_ln_fused_vs_oracle(3001, 3072, 768); t.test_linear_ln_fused_vs_oracle(300, 1024, 1024)")
+    env = dict(os.environ, TCB_LN_KERNEL="global")
     r = subprocess.run([sys.executable, "-c", code], env=env, capture_output=True, text=True,
                        cwd=os.path.dirname(os.path.dirname(os.path.abspath(__file__))), timeout=300)
     assert r.returncode == 0, r.stderr[-2000:]
