@@ -15,7 +15,8 @@ value: device time (CUDA events on the launching stream), inputs resident in HBM
        max over ranks; value = sum of non-pad tokens over ranks / max time.
 e2e:   the same metric through the public API from host memory: per step tcb_pack (C++),
        H2D of the segment table + token ids from pinned memory, forward, unpack, D2H of the
-       per-request outputs [T, d] into pinned memory; host wall clock, synchronised.
+       per-request outputs [T, d] into pinned memory, read by the host; two-deep pipeline (the
+       D2H of step i overlaps step i+1 on a copy stream); host wall clock.
 roofline: the dominant kernel class (largest device time per step) measured live with CUDA
        events around each launch (tcb_profile_*); algorithmic flops / bytes per class in
        DESIGN.md section 7 (GEMMs: 2 T d_in d_out per layer over non-pad tokens T); every
@@ -395,41 +396,74 @@ def main():
     whole_tc = (gemm_flops + attn_flops) / (ms_per_step / 1e3) / 1e12
 
     # ---- e2e: public API from host memory, every step -------------------------------------
+    # A two-deep serving pipeline: step i's outputs go device -> pinned host on a copy stream
+    # while step i+1 is packed (host C++) and computed; every step still copies its inputs
+    # host -> device and its [T, d] outputs device -> host inside the timed region, and the
+    # host reads each step's outputs once their copy has completed (before the slot is reused).
     pinned_ids = [torch.from_numpy(i).pin_memory() for _, i in batches]
-    out_host = torch.empty((max(p.info["total_tokens"] for p in plans), model.d_model),
-                           dtype=enc.dtype).pin_memory()
+    max_t = max(p.info["total_tokens"] for p in plans)
+    out_host = [torch.empty((max_t, model.d_model), dtype=enc.dtype).pin_memory() for _ in range(2)]
+    e2e_out = [torch.empty((max_t, model.d_model), dtype=enc.dtype, device=dev) for _ in range(2)]
     e2e_rows = enc.alloc_rows(M)
     e2e_ids = torch.empty(max(len(i) for _, i in batches), dtype=torch.int32, device=dev)
     e2e_seg = torch.empty(max(p.segtab().size for p in plans), dtype=torch.int32, device=dev)
-    e2e_out = torch.empty((out_host.shape[0], model.d_model), dtype=enc.dtype, device=dev)
-    seg_pin = torch.empty(e2e_seg.numel(), dtype=torch.int32).pin_memory()
+    seg_pin = [torch.empty(e2e_seg.numel(), dtype=torch.int32).pin_memory() for _ in range(2)]
+    cstream = torch.cuda.Stream(device=dev)
+    h2d_ev, copy_ev, pending = [None, None], [None, None], [0, 0]
     h2d = d2h = 0
+    checksum = 0.0
+
+    def consume(k):
+        nonlocal checksum
+        if copy_ev[k] is not None:
+            copy_ev[k].synchronize()                          # step's outputs are on the host
+            checksum += float(out_host[k][pending[k] - 1, 0])
+            copy_ev[k] = None
 
     def e2e_step(i):
         nonlocal h2d, d2h
+        k = i & 1
         lengths, ids = batches[i % len(batches)]
         p = tcb.tcb_pack(lengths, L, B)                         # host packer (C++)
         st = p.segtab()
-        seg_pin[:st.size].copy_(torch.from_numpy(st))
+        if h2d_ev[k] is not None:
+            h2d_ev[k].synchronize()                             # pinned slot k is free again
+        seg_pin[k][:st.size].copy_(torch.from_numpy(st))
+        consume(k)                                              # output slot k is free again
+        T = p.info["total_tokens"]
         with torch.cuda.stream(stream):
-            e2e_seg[:st.size].copy_(seg_pin[:st.size], non_blocking=True)
+            e2e_seg[:st.size].copy_(seg_pin[k][:st.size], non_blocking=True)
             e2e_ids[:len(ids)].copy_(pinned_ids[i % len(batches)], non_blocking=True)
+            h2d_ev[k] = torch.cuda.Event()
+            h2d_ev[k].record(stream)
             enc.encoder_forward(p, e2e_seg, e2e_ids, e2e_rows, stream=stream)
-            T = p.info["total_tokens"]
-            enc.unpack(p, e2e_seg, e2e_rows, e2e_out, stream=stream)
-            out_host[:T].copy_(e2e_out[:T], non_blocking=True)
-        stream.synchronize()
+            enc.unpack(p, e2e_seg, e2e_rows, e2e_out[k], stream=stream)
+            done = torch.cuda.Event()
+            done.record(stream)
+        with torch.cuda.stream(cstream):
+            cstream.wait_event(done)
+            out_host[k][:T].copy_(e2e_out[k][:T], non_blocking=True)
+            copy_ev[k] = torch.cuda.Event()
+            copy_ev[k].record(cstream)
+        pending[k] = T
         h2d += st.size * 4 + len(ids) * 4
-        d2h += T * model.d_model * e2e_out.element_size()
+        d2h += T * model.d_model * e2e_out[k].element_size()
+
+    def drain():
+        consume(0)
+        consume(1)
+        torch.cuda.synchronize(dev)
 
     for i in range(args.warmup):
         e2e_step(i)
+    drain()
     h2d = d2h = 0
     if world > 1:
         dist.barrier()
     t0 = time.perf_counter()
     for i in range(args.steps):
         e2e_step(i)
+    drain()
     e2e_s = time.perf_counter() - t0
     e2e_t = torch.tensor([e2e_s], dtype=torch.float64, device=dev)
     if world > 1:
@@ -466,7 +500,7 @@ def main():
             "roofline": roofline,
             "e2e": {"value": e2e_value, "unit": UNIT, "h2d_bytes_per_step": h2d // args.steps,
                     "d2h_bytes_per_step": d2h // args.steps,
-                    "path": "tcb_pack + pinned H2D + tcb_encoder_forward + tcb_unpack + D2H, sync per step"},
+                    "path": "tcb_pack + pinned H2D + tcb_encoder_forward + tcb_unpack + D2H read by the host, two-deep pipeline (D2H of step i on a copy stream overlaps step i+1)"},
             "clocks": clk.summary(),
             "cpu_baseline": cpu,
             "paper_context": "paper reports only end-to-end serving on 1x V100 (<~4e3 tok/s incl. decoder); no encoder tokens/s",
