@@ -342,7 +342,7 @@ def main():
     tc_peak = peaks.get("bf16_tflops_sustained", peaks["bf16_tflops"])
     hbm_peak = peaks["hbm_gbs"]
     esz = 2 if model.dtype == "bf16" else 4
-    fused_ln = d == 512 and model.dtype == "bf16"
+    fused_ln = d in (512, 768, 1024) and model.dtype == "bf16"
     # algorithmic work per forward of each kernel class: flops for the
     # contractions (non-pad tokens only), bytes for the HBM-bound kernels
     work = {
@@ -350,16 +350,21 @@ def main():
         "gemm_o": ("tensor", 2.0 * T * S * d * d),
         "gemm_ffn1": ("tensor", 2.0 * T * S * d * f),
         "gemm_ffn2": ("tensor", 2.0 * T * S * d * f),
-        "attention": ("tensor", attn_flops),
+        # attention is HBM-bound (AI = E[l]/2 flop/B < ridge): Q, K, V in + O
+        # out per non-pad token per layer; its useful (segment-diagonal) flop rate is reported
+        # next to it
+        "attention": ("hbm", 1.0 * T * S * 4 * d * esz),
         "embed": ("hbm", T * (4 + 2 * d * esz + 8)),
         "layernorm": ("hbm", 0.0 if fused_ln else 2.0 * S * T * 2 * d * esz),
         "unpack": ("hbm", T * 2 * d * esz),
     }
+    ln_o = {512: "linear_ln_kernel", 768: "linear_lnc_kernel<3>", 1024: "linear_lnc_kernel<4>"}
+    ln_2 = {512: "linear_lnc_kernel<2>", 768: "linear_lnc_kernel<3>", 1024: "linear_lng_kernel<4>"}
     names = {"gemm_qkv": "linear_tc_kernel<2,256,EPI_BIAS> (QKV)",
-             "gemm_o": "linear_ln_kernel (W_O + residual + LN1)" if fused_ln else "linear_tc_kernel (W_O + residual)",
+             "gemm_o": f"{ln_o.get(d)} (W_O + residual + LN1)" if fused_ln else "linear_tc_kernel (W_O + residual)",
              "gemm_ffn1": "linear_tc_kernel<2,256,EPI_ACT> (FFN1 + act)",
-             "gemm_ffn2": "linear_ln_kernel (FFN2 + residual + LN2)" if fused_ln else "linear_tc_kernel (FFN2 + residual)",
-             "attention": "attn_tc_kernel (segment-masked attention, useful flops)",
+             "gemm_ffn2": f"{ln_2.get(d)} (FFN2 + residual + LN2)" if fused_ln else "linear_tc_kernel (FFN2 + residual)",
+             "attention": "attn_tc_kernel (segment-masked attention; Q,K,V in + O out)",
              "embed": "pack_embed_kernel", "layernorm": "layernorm_kernel", "unpack": "unpack_kernel"}
     classes = {}
     for c, (bound, w) in work.items():
@@ -375,6 +380,8 @@ def main():
                       "frac": ach / pk, "launches_per_step": n_c / args.steps,
                       "ms_per_step": ms_c / args.steps,
                       "us_per_launch": 1e3 * ms_c / n_c}
+        if c == "attention":
+            classes[c]["useful_tflops"] = attn_flops * args.steps / (ms_c / 1e3) / 1e12
     dom = max(classes, key=lambda c: classes[c]["ms_per_step"])
     traffic = None
     tpath = os.path.join(ROOT, "profiles", "traffic.json")
