@@ -109,12 +109,12 @@ WsLayout ws_layout(const tcb_model_config& c, int64_t M) {
   L.z = off;   off += align256(es * static_cast<size_t>(M) * c.d_model);
   L.x1 = off;  off += align256(es * static_cast<size_t>(M) * c.d_model);
   L.h = off;   off += align256(es * static_cast<size_t>(M) * c.d_ff);
-  // row-statistics scratch of the L2-exchange LayerNorm GEMM (bf16, d = 768 / 1024): partials
+  // row-statistics scratch of the L2-exchange LayerNorm GEMM (bf16, d = 512 / 768 / 1024): partials
   // per 256-row tile, and one zeroed counter region per fused launch (2 per layer)
   L.lnst = off;
   L.lncnt = off;
   L.lncnt_per_launch = 0;
-  if (c.dtype == 1 && (c.d_model == 768 || c.d_model == 1024)) {
+  if (c.dtype == 1 && (c.d_model == 512 || c.d_model == 768 || c.d_model == 1024)) {
     off += align256(tcb::k::linear_ln_scratch_stats_bytes(M, c.d_model));
     L.lncnt = off;
     L.lncnt_per_launch = align256(tcb::k::linear_ln_scratch_cnt_bytes(M));

@@ -1632,8 +1632,8 @@ cudaError_t launch_linear_ln_bf16_tc(const GemmMaps& m, int64_t M, int N, int K,
                                      float eps, const int32_t* seg_ids, cudaStream_t s,
                                      float2* lng_stats, int* lng_cnt) {
   if (M == 0) return cudaSuccess;
-  // d = 1024, K >= 2d (FFN2) with scratch: the L2-exchange kernel on all 74 pairs (the 8-CTA
-  // cluster kernel fits on 120 SMs only): C4/C5 FFN2 262 -> 218 us.  At K = d (W_O) the
+  // d = 512 / 1024, K >= 2d (FFN2) with scratch: the L2-exchange kernel on all 74 pairs (the
+  // 4- / 8-CTA cluster kernel fits on 132 / 120 SMs only): C4/C5 FFN2 262 -> 218 us.  At K = d (W_O) the
   // epilogue bounds the kernel and the L2 round trip of the statistics costs more than the
   // extra SMs give (89 -> 99 us), likewise for d = 768 (57 -> 70 us).  TCB_LN_KERNEL=cluster
   // forces the cluster kernel, =global the L2-exchange kernel wherever scratch is given.
@@ -1645,6 +1645,9 @@ cudaError_t launch_linear_ln_bf16_tc(const GemmMaps& m, int64_t M, int N, int K,
   if (lng_stats && lng_cnt && ln_env != 1) {
     if (N == 1024 && (K >= 2 * N || ln_env == 2))
       return launch_lng<4>(m, static_cast<int>(M), K, bias, gamma, beta, eps, seg_ids, lng_stats,
+                           lng_cnt, s);
+    if (N == 512 && K >= 2 * N)             // C2 FFN2: 73.4 -> 71.0 us (148 vs 132 SMs)
+      return launch_lng<2>(m, static_cast<int>(M), K, bias, gamma, beta, eps, seg_ids, lng_stats,
                            lng_cnt, s);
     if (N == 768 && ln_env == 2)
       return launch_lng<3>(m, static_cast<int>(M), K, bias, gamma, beta, eps, seg_ids, lng_stats,
