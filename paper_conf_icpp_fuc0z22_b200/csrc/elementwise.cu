@@ -60,7 +60,10 @@ __device__ __forceinline__ float warp_sum(float v) {
 // One CTA per (batch row, 64-slot chunk of it).  The row's segment records (row_first[] of
 // the device segment table gives them in O(1)) are staged in shared memory; each warp then
 // owns slots j = chunk*64 + warp, +8, ... and finds its segment by a binary search in smem.
-constexpr int kRowChunk = 64;
+#ifndef TCB_ROW_CHUNK
+#define TCB_ROW_CHUNK 16
+#endif
+constexpr int kRowChunk = TCB_ROW_CHUNK;   // slots per CTA (64 measured slower: fewer CTAs in flight)
 template <typename T, int NV>
 __global__ void __launch_bounds__(kWarpsPerBlock * 32) pack_embed_kernel(EmbedArgs a) {
   constexpr int V = Vec<T>::N;
