@@ -631,6 +631,8 @@ struct tcb_decoder {
   CUtensorMap cQkv{}, cX{}, cX1{}, cX2{}, cQc{}, cH{}, cLogits{};
   tcb_decode_stats stats{};
   int32_t last_rows = 0;
+  int32_t* pin = nullptr;                // pinned host: active list [2][R], done flags [2][R]
+  cudaEvent_t ev[2] = {nullptr, nullptr};  // done flags of a step on the host
   const void* L(int layer, int i) const { return t[20 * layer + i]; }
   const float* Lf(int layer, int i) const { return static_cast<const float*>(L(layer, i)); }
 };
@@ -641,6 +643,9 @@ enum { D_W_QKV = 0, D_B_QKV, D_W_O, D_B_O, D_LN1_G, D_LN1_B, D_W_Q, D_B_Q, D_W_K
 
 void free_decoder(tcb_decoder* dec) {
   for (void* p : dec->bufs) cudaFree(p);
+  if (dec->pin) cudaFreeHost(dec->pin);
+  for (cudaEvent_t e : dec->ev)
+    if (e) cudaEventDestroy(e);
   delete dec;
 }
 
@@ -705,9 +710,13 @@ tcb_status tcb_decoder_create(const tcb_weights* enc, const void* const* tensors
             dalloc(dec, &dec->done, 4 * R) && dalloc(dec, &dec->flag, 4 * R) &&
             dalloc(dec, &dec->tmax, 4 * R) && dalloc(dec, &dec->mem_start, 4 * R) &&
             dalloc(dec, &dec->mem_len, 4 * R);
+  ok = ok && cudaMallocHost(reinterpret_cast<void**>(&dec->pin), 16 * R) == cudaSuccess &&
+       cudaEventCreateWithFlags(&dec->ev[0], cudaEventDisableTiming) == cudaSuccess &&
+       cudaEventCreateWithFlags(&dec->ev[1], cudaEventDisableTiming) == cudaSuccess;
   if (!ok) {
+    cudaGetLastError();
     free_decoder(dec);
-    return fail(TCB_ERR_OUT_OF_MEMORY, "tcb_decoder_create: device buffers");
+    return fail(TCB_ERR_OUT_OF_MEMORY, "tcb_decoder_create: device / pinned buffers");
   }
   if (cudaMemset(dec->zero_bias, 0, sizeof(float) * V) != cudaSuccess) {
     free_decoder(dec);
@@ -797,15 +806,24 @@ tcb_status tcb_decode_greedy(tcb_decoder* dec, const tcb_plan* plan, const void*
     }
   }
   const float scale = 1.f / 8.f;                          // 1 / sqrt(d_head = 64)
-  std::vector<int32_t> flag_h(act_h.size());
   const int64_t kv_per_pos = 2LL * d * 2 * S;             // bytes of K|V per position, all layers
   double kv_sum = 0.0;
   int32_t t = 0;
   bool act_dirty = true;
+  // The host never waits for the step it has just enqueued: after enqueuing step t it reads
+  // the done flags of step t-1 (pinned, double-buffered) while step t runs, and drops the
+  // requests finished by then from the active set of step t+1 (early memory cleaning, R33,
+  // one step late).  A request finished at step t is thus recomputed once more at step t+1;
+  // the argmax kernel ignores it (its done flag is set) and no other row depends on it, so
+  // the generated tokens are those of the synchronous loop.
+  int32_t* act_pin[2] = {dec->pin, dec->pin + dec->R};
+  int32_t* done_pin[2] = {dec->pin + 2 * dec->R, dec->pin + 3 * dec->R};
   for (; t < max_steps && !act_h.empty(); ++t) {
     const int A = static_cast<int>(act_h.size());
-    if (act_dirty) {
-      e = cudaMemcpyAsync(dec->act, act_h.data(), 4 * A, cudaMemcpyHostToDevice, s);
+    const int sl = t & 1;
+    if (act_dirty) {   // act_pin[sl]'s previous upload (step t-2) completed: ev of t-2 was waited
+      std::memcpy(act_pin[sl], act_h.data(), 4 * static_cast<size_t>(A));
+      e = cudaMemcpyAsync(dec->act, act_pin[sl], 4 * A, cudaMemcpyHostToDevice, s);
       if (e != cudaSuccess) return cuda_fail(e, "tcb_decode_greedy: active set upload");
       act_dirty = false;
     }
@@ -862,25 +880,24 @@ tcb_status tcb_decode_greedy(tcb_decoder* dec, const tcb_plan* plan, const void*
     DecArgmaxArgs ga{static_cast<const __nv_bfloat16*>(dec->logits), V, A, t, 2, T, dec->act,
                      dec->tmax, d_tokens, dec->out_len, dec->done, dec->flag};
     TCB_LAUNCH(TCB_K_UNPACK, s, launch_dec_argmax(ga, s));
-    e = cudaMemcpyAsync(flag_h.data(), dec->flag, 4 * A, cudaMemcpyDeviceToHost, s);
-    if (e == cudaSuccess) e = cudaStreamSynchronize(s);
+    e = cudaMemcpyAsync(done_pin[sl], dec->done, 4 * n, cudaMemcpyDeviceToHost, s);
+    if (e == cudaSuccess) e = cudaEventRecord(dec->ev[sl], s);
     if (e != cudaSuccess) return cuda_fail(e, "tcb_decode_greedy: step");
     dec->last_rows = A;
     dec->stats.rows_computed += A;
     const int64_t kv_live = static_cast<int64_t>(A) * (t + 1) * kv_per_pos;
     kv_sum += static_cast<double>(kv_live);
     dec->stats.kv_bytes_peak = std::max(dec->stats.kv_bytes_peak, kv_live);
-    // early memory cleaning (R33): finished requests leave the active set
-    bool all_done = true;
+    if (t == 0) continue;
+    // early memory cleaning (R33): requests finished by step t-1 leave the active set
+    e = cudaEventSynchronize(dec->ev[sl ^ 1]);
+    if (e != cudaSuccess) return cuda_fail(e, "tcb_decode_greedy: step");
+    const int32_t* dn = done_pin[sl ^ 1];
     std::vector<int32_t> next;
     next.reserve(A);
-    for (int i = 0; i < A; ++i) {
-      if (!flag_h[i]) {
-        all_done = false;
-        next.push_back(act_h[i]);
-      }
-    }
-    if (all_done) { ++t; break; }
+    for (int i = 0; i < A; ++i)
+      if (!dn[act_h[i]]) next.push_back(act_h[i]);
+    if (next.empty()) { ++t; break; }   // step t only recomputed finished requests
     if (early_clean && static_cast<int>(next.size()) != A) {
       act_h.swap(next);
       act_dirty = true;

@@ -76,7 +76,9 @@ def test_decoder_tokens_valid_under_oracle_and_early_clean_bitwise():
     tok_c, tok_n = tok_c.cpu().numpy(), tok_n.cpu().numpy()
     assert np.array_equal(tok_c, tok_n) and np.array_equal(len_c, len_n)
     assert st_c["tokens_generated"] == int(len_c.sum()) == st_n["tokens_generated"]
-    assert st_c["rows_computed"] == int(len_c.sum())           # every active row yields a token
+    # every active row yields a token, except that a finished request is dropped one step
+    # late (the host reads step t-1's done flags while step t runs): at most one extra row each
+    assert int(len_c.sum()) <= st_c["rows_computed"] <= int(len_c.sum()) + len(LENGTHS)
     assert st_n["rows_computed"] == len(LENGTHS) * st_n["steps"]
     assert st_c["rows_computed"] < st_n["rows_computed"]
     assert st_c["kv_bytes_avg"] < st_n["kv_bytes_avg"]
