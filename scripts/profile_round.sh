@@ -17,8 +17,9 @@ ${LIST:-c2 linear_tc_kernel.*256, .int.0
 c2 attn_tc_kernel
 c2 linear_ln_kernel<.bool.0>
 c2 linear_tc_kernel.*256, .int.2
-c2 linear_lnc_kernel<.int.2>
+c2 linear_lng_kernel<.int.2>
 c2 pack_embed
 c2 unpack_kernel
-c4 linear_lnc_kernel<.int.4>}
+c4 linear_lnc_kernel<.int.4>
+c4 linear_lng_kernel<.int.4>}
 LIST
