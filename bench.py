@@ -502,6 +502,7 @@ def main():
                        "l2": "flushed (256 MiB write) between timed steps",
                        "cuda_graph": graph is not None},
             "tc_frac_whole_step": whole_tc / peaks["bf16_tflops"],
+            "tc_frac_whole_step_vs_sustained": whole_tc / tc_peak,
             "tc_whole_step_tflops": whole_tc,
             "gpu_launches": int(launches_per_step * args.steps),
             "roofline": roofline,
