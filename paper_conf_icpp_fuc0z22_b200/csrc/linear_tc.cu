@@ -542,9 +542,10 @@ constexpr int kLnEpiBytes = kLnEpiWarps * 2 * kStageBufBytes;        // 64 KB
 template <bool JOINT>
 struct LnCfg {
   static constexpr int kStageBytes = (JOINT ? 3 : 2) * 128 * BK * 2;
-  static constexpr int kStages = (227 * 1024 - 1024 - kLnEpiBytes - 4096) / kStageBytes;
+  static constexpr int kStages = (227 * 1024 - 1024 - kLnEpiBytes - 4096 - 6144) / kStageBytes;
   static constexpr int kSmemBytes = 1024 + kStages * kStageBytes + kLnEpiBytes +
-                                    8 * (2 * kStages + 4 + 2 * kLnEpiWarps) + 16 + 2 * 4 * 128 * 4;
+                                    8 * (2 * kStages + 4 + 2 * kLnEpiWarps) + 16 + 2 * 4 * 128 * 4 +
+                                    3 * kLnN * 4;
   static_assert(kSmemBytes <= 232448, "shared memory budget");
 };
 
@@ -604,6 +605,9 @@ linear_ln_kernel(const __grid_constant__ CUtensorMap tmA, const __grid_constant_
   uint64_t* rbar = tempty + 2;                              // [16 warps][2]
   uint32_t* tmem_slot = reinterpret_cast<uint32_t*>(rbar + 2 * kLnEpiWarps);
   float* stats = reinterpret_cast<float*>(tmem_slot + 4);   // [4 parts][128 rows] x 2
+  float* s_bias = stats + 2 * 4 * 128;                      // bias, gamma, beta [512] each
+  float* s_gamma = s_bias + kLnN;
+  float* s_beta = s_gamma + kLnN;
 
   const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
   const uint32_t rank = cluster_rank();
@@ -611,6 +615,12 @@ linear_ln_kernel(const __grid_constant__ CUtensorMap tmA, const __grid_constant_
   const int num_tiles = (M + 255) / 256;
   const int num_kb = K / BK;
   const int num_steps = num_kb + split_kb;
+  // per-column constants (weights, not produced by the previous kernel) -> shared memory
+  for (int i = threadIdx.x; i < kLnN; i += blockDim.x) {
+    s_bias[i] = __ldg(&bias[i]);
+    s_gamma[i] = __ldg(&gamma[i]);
+    s_beta[i] = __ldg(&beta[i]);
+  }
 
   if (warp == 0 && lane == 0) {
     asm volatile("prefetch.tensormap [%0];" ::"l"(reinterpret_cast<uint64_t>(&tmA)) : "memory");
@@ -664,15 +674,28 @@ linear_ln_kernel(const __grid_constant__ CUtensorMap tmA, const __grid_constant_
       constexpr uint32_t idesc = idesc_bf16<2, 256>();
       int stage = 0;
       uint32_t phase = 0, tphase = 0;
+#ifdef TCB_LN_PROBE
+      long long p0 = clock64(), pt = 0, pf = 0;
+#endif
       for (int tile = cluster_id; tile < num_tiles; tile += num_clusters) {
         int done[2] = {0, 0};                   // k-blocks accumulated per half
         for (int step = 0; step < num_steps; ++step) {
           int kb, mask;
           ln_step(step, num_kb, split_kb, kb, mask);
+#ifdef TCB_LN_PROBE
+          long long q0 = clock64();
+#endif
 #pragma unroll
           for (int h = 0; h < 2; ++h)
             if ((mask & (1 << h)) && done[h] == 0) mbar_wait(&tempty[h], tphase ^ 1);
+#ifdef TCB_LN_PROBE
+          long long q1 = clock64();
+          pt += q1 - q0;
+#endif
           mbar_wait(&full[stage], phase);
+#ifdef TCB_LN_PROBE
+          pf += clock64() - q1;
+#endif
           tc_fence_after();
           if (lane == 0) {
             const uint32_t a0 = smem_u32(sStage + stage * kLnStageBytes);
@@ -697,6 +720,11 @@ linear_ln_kernel(const __grid_constant__ CUtensorMap tmA, const __grid_constant_
         }
         tphase ^= 1;
       }
+#ifdef TCB_LN_PROBE
+      if (lane == 0 && blockIdx.x < 6)
+        printf("lnprobe mma cta %d total %lld wait_tempty %lld wait_full %lld\n", blockIdx.x,
+               clock64() - p0, pt, pf);
+#endif
     }
   } else if (warp >= 4) {
     // ===== Epilogue: bias + residual + LayerNorm over complete 512-column rows =====
@@ -713,7 +741,13 @@ linear_ln_kernel(const __grid_constant__ CUtensorMap tmA, const __grid_constant_
     uint32_t tphase = 0;
     // chunk j (0..3): half j>>1, columns h*256 + part*64 + (j&1)*32
     auto col_of = [&](int j) { return (j >> 1) * 256 + part * 64 + (j & 1) * 32; };
+#ifdef TCB_LN_PROBE
+    long long e0 = clock64(), e_tfull = 0, e_res = 0, e_p1 = 0, e_bar = 0, e_p2 = 0, e_st = 0;
+#endif
     for (int tile = cluster_id; tile < num_tiles; tile += num_clusters) {
+#ifdef TCB_LN_PROBE
+      long long ta = clock64();
+#endif
       const int row0 = tile * 256 + static_cast<int>(rank) * 128 + q * 32;
       const int64_t grow = static_cast<int64_t>(row0) + lane;
       const bool pad = grow >= M || (seg_ids && __ldg(&seg_ids[grow]) < 0);
@@ -731,8 +765,14 @@ linear_ln_kernel(const __grid_constant__ CUtensorMap tmA, const __grid_constant_
 #pragma unroll 1
       for (int j = 0; j < 4; ++j) {
         if ((j & 1) == 0) {
+#ifdef TCB_LN_PROBE
+          long long tw = clock64();
+#endif
           mbar_wait(&tfull[j >> 1], tphase);
           tc_fence_after();
+#ifdef TCB_LN_PROBE
+          e_tfull += clock64() - tw;
+#endif
         }
         const int b = j & 1;
         const uint32_t buf = bufs + b * kStageBufBytes;
@@ -742,16 +782,22 @@ linear_ln_kernel(const __grid_constant__ CUtensorMap tmA, const __grid_constant_
         tmem_ld32_nowait(taddr, r);
         tmem_wait_ld();
         float* v = reinterpret_cast<float*>(r);
-        const float4* b4 = reinterpret_cast<const float4*>(bias + gc0);
+        const float4* b4 = reinterpret_cast<const float4*>(s_bias + gc0);
 #pragma unroll
         for (int t = 0; t < 8; ++t) {
-          const float4 bb = __ldg(b4 + t);
+          const float4 bb = b4[t];
           v[4 * t + 0] += bb.x;
           v[4 * t + 1] += bb.y;
           v[4 * t + 2] += bb.z;
           v[4 * t + 3] += bb.w;
         }
+#ifdef TCB_LN_PROBE
+        long long tr = clock64();
+#endif
         mbar_wait(&my_rbar[b], (rph >> b) & 1);
+#ifdef TCB_LN_PROBE
+        e_res += clock64() - tr;
+#endif
         rph ^= 1u << b;
 #pragma unroll
         for (int t = 0; t < 4; ++t) {
@@ -764,11 +810,14 @@ linear_ln_kernel(const __grid_constant__ CUtensorMap tmA, const __grid_constant_
             v[8 * t + 2 * e + 1] += f.y;
           }
         }
+        float ps[4] = {0.f, 0.f, 0.f, 0.f}, pq[4] = {0.f, 0.f, 0.f, 0.f};   // short chains
 #pragma unroll
         for (int t = 0; t < 32; ++t) {
-          sum += v[t];
-          sumsq = fmaf(v[t], v[t], sumsq);
+          ps[t & 3] += v[t];
+          pq[t & 3] = fmaf(v[t], v[t], pq[t & 3]);
         }
+        sum += (ps[0] + ps[1]) + (ps[2] + ps[3]);
+        sumsq += (pq[0] + pq[1]) + (pq[2] + pq[3]);
         tmem_st32(taddr, *reinterpret_cast<float(*)[32]>(v));
         __syncwarp();                             // every lane has read buffer b
         if (j + 2 < 4 && lane == 0) {
@@ -777,9 +826,17 @@ linear_ln_kernel(const __grid_constant__ CUtensorMap tmA, const __grid_constant_
         }
       }
       asm volatile("tcgen05.wait::st.sync.aligned;" ::: "memory");
+#ifdef TCB_LN_PROBE
+      long long tb = clock64();
+      e_p1 += tb - ta;
+#endif
       stat1[part * 128 + srow] = sum;
       stat2[part * 128 + srow] = sumsq;
       named_bar(1 + q, 128);
+#ifdef TCB_LN_PROBE
+      long long tc2 = clock64();
+      e_bar += tc2 - tb;
+#endif
       // single-pass moments in fp32: |mean| is O(std) for these residual streams, so
       // E[z^2] - mean^2 loses nothing material at the bf16 output precision
       const float mean = (stat1[srow] + stat1[128 + srow] + stat1[256 + srow] + stat1[384 + srow]) *
@@ -787,6 +844,7 @@ linear_ln_kernel(const __grid_constant__ CUtensorMap tmA, const __grid_constant_
       const float ex2m = (stat2[srow] + stat2[128 + srow] + stat2[256 + srow] + stat2[384 + srow]) *
                          (1.f / kLnN);
       const float rstd = rsqrtf(fmaxf(ex2m - mean * mean, 0.f) + eps);
+      const float nmr = -mean * rstd;             // (z - mean) rstd = fma(z, rstd, nmr)
       // pass 2: normalise, bf16, TMA store; each half is released to the MMA as soon as its
       // last read is done
 #pragma unroll 1
@@ -803,15 +861,15 @@ linear_ln_kernel(const __grid_constant__ CUtensorMap tmA, const __grid_constant_
           if (lane == 0) mbar_arrive_remote(tempty0 + 8u * (j >> 1));
         }
         float* y = reinterpret_cast<float*>(r);
-        const float4* g4 = reinterpret_cast<const float4*>(gamma + gc0);
-        const float4* e4 = reinterpret_cast<const float4*>(beta + gc0);
+        const float4* g4 = reinterpret_cast<const float4*>(s_gamma + gc0);
+        const float4* e4 = reinterpret_cast<const float4*>(s_beta + gc0);
 #pragma unroll
         for (int t = 0; t < 8; ++t) {
-          const float4 gg = __ldg(g4 + t), ee = __ldg(e4 + t);
-          y[4 * t + 0] = pad ? 0.f : (y[4 * t + 0] - mean) * rstd * gg.x + ee.x;
-          y[4 * t + 1] = pad ? 0.f : (y[4 * t + 1] - mean) * rstd * gg.y + ee.y;
-          y[4 * t + 2] = pad ? 0.f : (y[4 * t + 2] - mean) * rstd * gg.z + ee.z;
-          y[4 * t + 3] = pad ? 0.f : (y[4 * t + 3] - mean) * rstd * gg.w + ee.w;
+          const float4 gg = g4[t], ee = e4[t];
+          y[4 * t + 0] = pad ? 0.f : fmaf(fmaf(y[4 * t + 0], rstd, nmr), gg.x, ee.x);
+          y[4 * t + 1] = pad ? 0.f : fmaf(fmaf(y[4 * t + 1], rstd, nmr), gg.y, ee.y);
+          y[4 * t + 2] = pad ? 0.f : fmaf(fmaf(y[4 * t + 2], rstd, nmr), gg.z, ee.z);
+          y[4 * t + 3] = pad ? 0.f : fmaf(fmaf(y[4 * t + 3], rstd, nmr), gg.w, ee.w);
         }
         if (lane == 0) bulk_wait_read<1>();       // the store that last used `buf` has read it
         __syncwarp();
@@ -835,10 +893,23 @@ linear_ln_kernel(const __grid_constant__ CUtensorMap tmA, const __grid_constant_
         }
       }
       // the stats slots are rewritten next tile only after all 4 warps passed this barrier
+#ifdef TCB_LN_PROBE
+      long long td = clock64();
+      e_p2 += td - tc2;
+#endif
       named_bar(1 + q, 128);
+#ifdef TCB_LN_PROBE
+      e_bar += clock64() - td;
+#endif
       tphase ^= 1;
     }
     if (lane == 0) bulk_wait_all();
+#ifdef TCB_LN_PROBE
+    if (lane == 0 && ew == 0 && blockIdx.x < 6)
+      printf("lnprobe epi cta %d total %lld pass1 %lld (wait_tfull %lld wait_res %lld) bar %lld pass2 %lld tiles %d\n",
+             blockIdx.x, clock64() - e0, e_p1, e_tfull, e_res, e_bar, e_p2,
+             (num_tiles - cluster_id + num_clusters - 1) / num_clusters);
+#endif
   }
   __syncwarp();
   tc_fence_before();
@@ -1094,11 +1165,14 @@ linear_lnc_kernel(const __grid_constant__ CUtensorMap tmA, const __grid_constant
             v[8 * t + 2 * e + 1] += f.y;
           }
         }
+        float ps[4] = {0.f, 0.f, 0.f, 0.f}, pq[4] = {0.f, 0.f, 0.f, 0.f};   // short chains
 #pragma unroll
         for (int t = 0; t < 32; ++t) {
-          sum += v[t];
-          sumsq = fmaf(v[t], v[t], sumsq);
+          ps[t & 3] += v[t];
+          pq[t & 3] = fmaf(v[t], v[t], pq[t & 3]);
         }
+        sum += (ps[0] + ps[1]) + (ps[2] + ps[3]);
+        sumsq += (pq[0] + pq[1]) + (pq[2] + pq[3]);
         tmem_st32(tbase + 32 * j, *reinterpret_cast<float(*)[32]>(v));
       }
       rphase ^= 1;
@@ -1130,6 +1204,7 @@ linear_lnc_kernel(const __grid_constant__ CUtensorMap tmA, const __grid_constant
       // single-pass moments in fp32 (as the 512-column kernel): |mean| = O(std) here
       const float mean = s1 * kInvN;
       const float rstd = rsqrtf(fmaxf(s2 * kInvN - mean * mean, 0.f) + eps);
+      const float nmr = -mean * rstd;             // (z - mean) rstd = fma(z, rstd, nmr)
       // pass 2: normalise -> bf16 -> staging (the residual chunks are consumed) -> TMA store
 #pragma unroll 1
       for (int j = 0; j < kLncChunks; ++j) {
@@ -1148,10 +1223,10 @@ linear_lnc_kernel(const __grid_constant__ CUtensorMap tmA, const __grid_constant
 #pragma unroll
         for (int t = 0; t < 8; ++t) {
           const float4 gg = __ldg(g4 + t), ee = __ldg(e4 + t);
-          y[4 * t + 0] = pad ? 0.f : (y[4 * t + 0] - mean) * rstd * gg.x + ee.x;
-          y[4 * t + 1] = pad ? 0.f : (y[4 * t + 1] - mean) * rstd * gg.y + ee.y;
-          y[4 * t + 2] = pad ? 0.f : (y[4 * t + 2] - mean) * rstd * gg.z + ee.z;
-          y[4 * t + 3] = pad ? 0.f : (y[4 * t + 3] - mean) * rstd * gg.w + ee.w;
+          y[4 * t + 0] = pad ? 0.f : fmaf(fmaf(y[4 * t + 0], rstd, nmr), gg.x, ee.x);
+          y[4 * t + 1] = pad ? 0.f : fmaf(fmaf(y[4 * t + 1], rstd, nmr), gg.y, ee.y);
+          y[4 * t + 2] = pad ? 0.f : fmaf(fmaf(y[4 * t + 2], rstd, nmr), gg.z, ee.z);
+          y[4 * t + 3] = pad ? 0.f : fmaf(fmaf(y[4 * t + 3], rstd, nmr), gg.w, ee.w);
         }
         const uint32_t buf = bufs + j * kStageBufBytes;
 #pragma unroll
@@ -1362,11 +1437,14 @@ linear_lng_kernel(const __grid_constant__ CUtensorMap tmA, const __grid_constant
             v[8 * tt + 2 * e + 1] += f.y;
           }
         }
+        float ps[4] = {0.f, 0.f, 0.f, 0.f}, pq[4] = {0.f, 0.f, 0.f, 0.f};   // short chains
 #pragma unroll
         for (int tt = 0; tt < 32; ++tt) {
-          sum += v[tt];
-          sumsq = fmaf(v[tt], v[tt], sumsq);
+          ps[tt & 3] += v[tt];
+          pq[tt & 3] = fmaf(v[tt], v[tt], pq[tt & 3]);
         }
+        sum += (ps[0] + ps[1]) + (ps[2] + ps[3]);
+        sumsq += (pq[0] + pq[1]) + (pq[2] + pq[3]);
         tmem_st32(tbase + 32 * j, *reinterpret_cast<float(*)[32]>(v));
       }
       rphase ^= 1;
@@ -1398,6 +1476,7 @@ linear_lng_kernel(const __grid_constant__ CUtensorMap tmA, const __grid_constant
       }
       const float mean = s1 * kInvN;
       const float rstd = rsqrtf(fmaxf(s2 * kInvN - mean * mean, 0.f) + eps);
+      const float nmr = -mean * rstd;             // (z - mean) rstd = fma(z, rstd, nmr)
       // pass 2: normalise -> bf16 -> staging -> TMA store
 #pragma unroll 1
       for (int j = 0; j < kLncChunks; ++j) {
@@ -1416,10 +1495,10 @@ linear_lng_kernel(const __grid_constant__ CUtensorMap tmA, const __grid_constant
 #pragma unroll
         for (int tt = 0; tt < 8; ++tt) {
           const float4 gg = __ldg(g4 + tt), ee = __ldg(e4 + tt);
-          y[4 * tt + 0] = pad ? 0.f : (y[4 * tt + 0] - mean) * rstd * gg.x + ee.x;
-          y[4 * tt + 1] = pad ? 0.f : (y[4 * tt + 1] - mean) * rstd * gg.y + ee.y;
-          y[4 * tt + 2] = pad ? 0.f : (y[4 * tt + 2] - mean) * rstd * gg.z + ee.z;
-          y[4 * tt + 3] = pad ? 0.f : (y[4 * tt + 3] - mean) * rstd * gg.w + ee.w;
+          y[4 * tt + 0] = pad ? 0.f : fmaf(fmaf(y[4 * tt + 0], rstd, nmr), gg.x, ee.x);
+          y[4 * tt + 1] = pad ? 0.f : fmaf(fmaf(y[4 * tt + 1], rstd, nmr), gg.y, ee.y);
+          y[4 * tt + 2] = pad ? 0.f : fmaf(fmaf(y[4 * tt + 2], rstd, nmr), gg.z, ee.z);
+          y[4 * tt + 3] = pad ? 0.f : fmaf(fmaf(y[4 * tt + 3], rstd, nmr), gg.w, ee.w);
         }
         const uint32_t buf = bufs + j * kStageBufBytes;
 #pragma unroll
