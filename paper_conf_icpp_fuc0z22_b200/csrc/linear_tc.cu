@@ -315,29 +315,50 @@ linear_tc_kernel(const __grid_constant__ CUtensorMap tmA, const __grid_constant_
   if constexpr (CG == 2) cluster_sync(); else __syncthreads();
   tc_fence_after();
   const uint32_t tmem_base = *tmem_slot;
-  pdl_wait();                 // A / residual come from the previous kernel; C may still be read
+  // A / residual come from the previous kernel and C may still be read by it: everything but
+  // the producer waits for it here (PDL).  The weights are constant, so the producer issues the
+  // W halves of the first S stages BEFORE its wait -- their latency hides in that kernel's tail.
+  if (warp != 0) pdl_wait();
   pdl_trigger();
 
   if (warp == 0) {
     // ===== TMA producer (both CTAs of a pair load their own halves) =====
     if (lane == 0) {
       const uint32_t full0 = CG == 2 ? map_to_rank0(smem_u32(full)) : smem_u32(full);
-      int stage = 0;
+      int npre = 0;                           // leading steps whose W is already in flight
+      {
+        int stage = 0;
+        for (int tile = cluster_id; tile < num_tiles && npre < S; tile += num_clusters) {
+          int m_blk, n_blk;
+          tile_coords(tile, m_blocks, n_blocks, raster, m_blk, n_blk);
+          const int b_row = n_blk * BN + static_cast<int>(rank) * Cfg::kBRows;
+          for (int kb = 0; kb < num_kb && npre < S; ++kb, ++npre, ++stage) {
+            if (rank == 0) mbar_expect_tx(&full[stage], CG * Cfg::kStageBytes);
+            tma_load_2d<CG>(sB + stage * Cfg::kBBytes, &tmW, full0 + 8u * stage, kb * BK, b_row);
+          }
+        }
+      }
+      pdl_wait();
+      int stage = 0, step = 0;
       uint32_t phase = 0;
       for (int tile = cluster_id; tile < num_tiles; tile += num_clusters) {
         int m_blk, n_blk;
         tile_coords(tile, m_blocks, n_blocks, raster, m_blk, n_blk);
         const int a_row = m_blk * TILE_M + static_cast<int>(rank) * 128;
         const int b_row = n_blk * BN + static_cast<int>(rank) * Cfg::kBRows;
-        for (int kb = 0; kb < num_kb; ++kb) {
-          mbar_wait(&empty[stage], phase ^ 1);
-          if (rank == 0) mbar_expect_tx(&full[stage], CG * Cfg::kStageBytes);
+        for (int kb = 0; kb < num_kb; ++kb, ++step) {
           const uint32_t fb = full0 + 8u * stage;
+          if (step >= npre) {
+            mbar_wait(&empty[stage], phase ^ 1);
+            if (rank == 0) mbar_expect_tx(&full[stage], CG * Cfg::kStageBytes);
+            tma_load_2d<CG>(sB + stage * Cfg::kBBytes, &tmW, fb, kb * BK, b_row);
+          }
           tma_load_2d<CG>(sA + stage * Cfg::kABytes, &tmA, fb, kb * BK, a_row);
-          tma_load_2d<CG>(sB + stage * Cfg::kBBytes, &tmW, fb, kb * BK, b_row);
           if (++stage == S) { stage = 0; phase ^= 1; }
         }
       }
+    } else {
+      pdl_wait();
     }
   } else if (warp == 1) {
     // ===== MMA issuer: one thread of the even CTA drives the pair =====
