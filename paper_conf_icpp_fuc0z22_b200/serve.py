@@ -14,6 +14,13 @@ The batch runs through the ConcatBatching encoder and its responses are returned
   batch's device time (CUDA events around H2D + graph), so utility and throughput are those
   of a serial scheduler + GPU pipeline on this hardware.  When no request is waiting, the
   clock jumps to the next arrival.
+* ``overlap=True``: a two-deep pipeline.  Right after batch k is enqueued (slot start S_k),
+  the host schedules batch k+1 from the requests that arrived by S_k, with deadlines checked
+  against its predicted start S_k + (mean device time so far), and enqueues it behind batch k
+  (double-buffered device segment table / ids / responses, one captured graph per buffer).
+  Batch k+1 starts at S_{k+1} = S_k + max(device time of k, scheduling time of k+1): the
+  scheduler's host time hides behind the GPU (the paper's overhead argument, P:1805-1811,
+  without the serial sum), at the price of not seeing arrivals during batch k until slot k+2.
 
 All compute runs in libtcb's kernels; this module only moves buffers and keeps time.
 """
@@ -29,8 +36,9 @@ from . import Encoder, Scheduler
 
 class Server:
     def __init__(self, encoder: Encoder, policy: str, batch_rows: int, row_len: int,
-                 eta: float = 0.5, q: float = 0.5):
+                 eta: float = 0.5, q: float = 0.5, overlap: bool = False):
         import torch
+        self.overlap = bool(overlap)
         self.enc = encoder
         self.B, self.L = int(batch_rows), int(row_len)
         self.policy, self.eta, self.q = policy, eta, q
@@ -48,6 +56,14 @@ class Server:
         self.stream = torch.cuda.Stream()
         self.graph = None
         self.last_batch = None
+        self.last_out = self.out
+        if self.overlap:   # second set of per-batch buffers (slot 1; slot 0 is the above)
+            self.bufs = [(self.d_segtab, self.d_ids, self.out, self.h_segtab, self.h_ids),
+                         (torch.zeros_like(self.d_segtab), torch.zeros_like(self.d_ids),
+                          torch.zeros_like(self.out),
+                          torch.zeros(self.seg_words, dtype=torch.int32).pin_memory(),
+                          torch.zeros(M, dtype=torch.int32).pin_memory())]
+            self.graphs = [None, None]
 
     def _capture(self, plan) -> None:
         import torch
@@ -63,11 +79,116 @@ class Server:
             self.enc.encoder_forward(plan, self.d_segtab, self.d_ids, self.rows, stream=s)
             self.enc.unpack(plan, self.d_segtab, self.rows, self.out, stream=s)
 
+    def _capture_slot(self, k, plan) -> None:
+        import torch
+        d_seg, d_ids, out = self.bufs[k][:3]
+        s = self.stream
+        s.wait_stream(torch.cuda.current_stream())
+        with torch.cuda.stream(s):
+            for _ in range(2):
+                self.enc.encoder_forward(plan, d_seg, d_ids, self.rows, stream=s)
+                self.enc.unpack(plan, d_seg, self.rows, out, stream=s)
+        s.synchronize()
+        g = torch.cuda.CUDAGraph()
+        with torch.cuda.graph(g, stream=s):
+            self.enc.encoder_forward(plan, d_seg, d_ids, self.rows, stream=s)
+            self.enc.unpack(plan, d_seg, self.rows, out, stream=s)
+        self.graphs[k] = g
+
+    def _run_overlap(self, lengths, arrival, deadline, token_ids, tok_offsets, horizon):
+        import torch
+        n = len(lengths)
+        sched = Scheduler(self.policy, self.B, self.L, self.eta, self.q)
+        order = np.argsort(arrival, kind="stable")
+        arr_sorted = arrival[order]
+        nxt = 0
+        ev = [(torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True))
+              for _ in range(2)]
+        batches, gpu_ms, sched_ms, tokens = 0, 0.0, 0.0, 0
+        now = 0.0                 # start of the batch in flight (or the host clock when idle)
+        inflight = None           # (slot, ids, lens)
+        k = 0                     # buffer slot of the next batch
+
+        def finish(slot_ids_lens):
+            nonlocal gpu_ms, batches, tokens
+            kp, ids_p, lens_p = slot_ids_lens
+            ev[kp][1].synchronize()
+            g = ev[kp][0].elapsed_time(ev[kp][1])
+            gpu_ms += g
+            batches += 1
+            tokens += int(lens_p.sum())
+            self.last_batch, self.last_out = (ids_p, lens_p), self.bufs[kp][2]
+            return g / 1e3
+
+        while now <= horizon:
+            end = int(np.searchsorted(arr_sorted, now, side="right"))
+            if end > nxt:                          # arrivals up to the current slot start
+                sel = order[nxt:end]
+                sched.submit(sel, lengths[sel], arrival[sel], deadline[sel])
+                nxt = end
+            est = (gpu_ms / batches / 1e3) if batches else 0.0
+            t0 = time.perf_counter()
+            ids, lens, plan = sched.next_batch(now + (est if inflight is not None else 0.0))
+            t_sched = time.perf_counter() - t0
+            sched_ms += t_sched * 1e3
+            if len(ids) > 0:
+                d_seg, d_ids, out, h_seg, h_ids = self.bufs[k]
+                words = plan.segtab()
+                h_seg[:len(words)].copy_(torch.from_numpy(words))
+                tok = np.concatenate([token_ids[tok_offsets[i]:tok_offsets[i] + lengths[i]]
+                                      for i in ids])
+                h_ids[:len(tok)].copy_(torch.from_numpy(tok))
+                if self.graphs[k] is None:         # first use of this buffer slot
+                    self.stream.synchronize()
+                    d_seg.copy_(h_seg)
+                    self._capture_slot(k, plan)
+                with torch.cuda.stream(self.stream):
+                    ev[k][0].record(self.stream)
+                    d_seg.copy_(h_seg, non_blocking=True)
+                    d_ids[:len(tok)].copy_(h_ids[:len(tok)], non_blocking=True)
+                    self.graphs[k].replay()
+                    ev[k][1].record(self.stream)
+            # the batch in flight completes; the new one starts once both it and the new
+            # one's scheduling are done
+            if inflight is not None:
+                now += max(finish(inflight), t_sched)
+            else:
+                now += t_sched
+            if len(ids) > 0:
+                inflight = (k, ids, lens)
+                k ^= 1
+            else:
+                inflight = None
+                if sched.stats()["waiting"] == 0:
+                    if nxt >= n:
+                        break
+                    now = max(now, float(arr_sorted[nxt]))
+        if inflight is not None:
+            now += finish(inflight)
+        return self._result(sched, n, now, tokens, batches, gpu_ms, sched_ms)
+
+    def _result(self, sched, n, now, tokens, batches, gpu_ms, sched_ms):
+        st = sched.stats()
+        elapsed = max(now, 1e-12)
+        return {"policy": self.policy, "B": self.B, "L": self.L, "requests": n,
+                "overlap": self.overlap,
+                "scheduled": st["scheduled"], "expired": st["expired"],
+                "utility": st["utility"], "sim_seconds": elapsed,
+                "responses_per_s": st["scheduled"] / elapsed,
+                "tokens_per_s": tokens / elapsed, "batches": batches,
+                "batch_ms": gpu_ms / max(batches, 1),
+                "sched_ms": sched_ms / max(st["batches"], 1),
+                "sched_over_batch": (sched_ms / max(st["batches"], 1)) /
+                                    max(gpu_ms / max(batches, 1), 1e-12)}
+
     def run(self, lengths, arrival, deadline, token_ids, tok_offsets,
             horizon: float) -> Dict[str, float]:
         """Serve the stream until the clock passes ``horizon`` seconds (or the stream is
         exhausted).  Returns utility / throughput / timing statistics."""
         import torch
+        if self.overlap:
+            return self._run_overlap(lengths, arrival, deadline, token_ids, tok_offsets, horizon)
+
         n = len(lengths)
         sched = Scheduler(self.policy, self.B, self.L, self.eta, self.q)
         order = np.argsort(arrival, kind="stable")
@@ -107,18 +228,9 @@ class Server:
             self.stream.synchronize()
             g = ev0.elapsed_time(ev1)
             self.last_batch = (ids, lens)        # its responses are in self.out[:sum(lens)]
+            self.last_out = self.out
             gpu_ms += g
             batches += 1
             tokens += int(lens.sum())
             now += t_sched + g / 1e3
-        st = sched.stats()
-        elapsed = max(now, 1e-12)
-        return {"policy": self.policy, "B": self.B, "L": self.L, "requests": n,
-                "scheduled": st["scheduled"], "expired": st["expired"],
-                "utility": st["utility"], "sim_seconds": elapsed,
-                "responses_per_s": st["scheduled"] / elapsed,
-                "tokens_per_s": tokens / elapsed, "batches": batches,
-                "batch_ms": gpu_ms / max(batches, 1),
-                "sched_ms": sched_ms / max(st["batches"], 1),
-                "sched_over_batch": (sched_ms / max(st["batches"], 1)) /
-                                    max(gpu_ms / max(batches, 1), 1e-12)}
+        return self._result(sched, n, now, tokens, batches, gpu_ms, sched_ms)

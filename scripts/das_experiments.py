@@ -59,7 +59,7 @@ def full_batch_ms(enc, lengths, B, L):
     return a.elapsed_time(b) / 10, per_batch
 
 
-def run(enc, model, policy, B, L, rate_mult, var, slots, seed, dist=None):
+def run(enc, model, policy, B, L, rate_mult, var, slots, seed, dist=None, overlap=False):
     probe = lengths_normal(20000, var, seed + 7) if dist is None else \
         np.minimum(wl.draw_lengths(dist, 20000, seed + 7), L).astype(np.int32)
     tau_ms, per_batch = full_batch_ms(enc, probe, B, L)
@@ -74,7 +74,7 @@ def run(enc, model, policy, B, L, rate_mult, var, slots, seed, dist=None):
     deadline = arrival + rng.uniform(1.0, 10.0, size=n) * (tau_ms / 1e3)
     offs = np.concatenate([[0], np.cumsum(lengths)])[:-1].astype(np.int64)
     ids = wl.draw_token_ids(int(lengths.sum()), model.vocab, seed + 2)
-    srv = Server(enc, policy, B, L)
+    srv = Server(enc, policy, B, L, overlap=overlap)
     res = srv.run(lengths, arrival, deadline, ids, offs, horizon)
     res.update({"model": model.name, "rate_x_capacity": rate_mult, "rate_req_s": rate,
                 "capacity_req_s": cap, "full_batch_ms": tau_ms, "length_var": var,
@@ -102,6 +102,11 @@ def main():
         for L in (104, 200, 304):
             for pol in POLICIES:
                 run(enc, base, pol, 16, L, 2.0, 20, slots, 400)
+    if what == "overlap":              # serial vs pipelined scheduler + GPU (Server overlap)
+        for rm in (0.5, 1.0, 2.0, 3.0):
+            for pol in ("das", "fcfs"):
+                for ov in (False, True):
+                    run(enc, base, pol, 64, 128, rm, 20, slots, 100, overlap=ov)
     if what in ("c5", "all"):          # C5: Transformer-big encoder, WMT-like, 128 x 256
         big = wl.MODELS["transformer-big"]
         enc_big = tcb.Encoder(big, wl.draw_weights(big, 42), wl.weight_names(big))

@@ -15,8 +15,9 @@ from paper_conf_icpp_fuc0z22_b200.serve import Server  # noqa: E402
 from _helpers import TOL  # noqa: E402
 
 
-@pytest.mark.parametrize("policy", ["das", "fcfs"])
-def test_server_responses_match_oracle(policy):
+@pytest.mark.parametrize("policy,overlap", [("das", False), ("fcfs", False), ("das", True),
+                                            ("fcfs", True)])
+def test_server_responses_match_oracle(policy, overlap):
     model = wl.MODELS["toy"]
     w = wl.draw_weights(model, 3)
     names = wl.weight_names(model)
@@ -28,11 +29,11 @@ def test_server_responses_match_oracle(policy):
     deadline = arrival + 1.0
     offs = np.concatenate([[0], np.cumsum(lengths)])[:-1].astype(np.int64)
     ids = wl.draw_token_ids(int(lengths.sum()), model.vocab, 6)
-    srv = Server(enc, policy, 2, 32)
+    srv = Server(enc, policy, 2, 32, overlap=overlap)
     res = srv.run(lengths, arrival, deadline, ids, offs, horizon=10.0)
     assert res["scheduled"] == n and res["expired"] == 0 and res["batches"] >= n * 9 // 64
     got_ids, got_lens = srv.last_batch
-    out = srv.out[:int(got_lens.sum())].float().cpu().numpy()
+    out = srv.last_out[:int(got_lens.sum())].float().cpu().numpy()
     base = 0
     for i, l in zip(got_ids.tolist(), got_lens.tolist()):
         tok = ids[offs[i]:offs[i] + l]
