@@ -4,6 +4,7 @@ share nothing; the question is whether one half's kernels fill the other's tails
 Run with TCB_LN_KERNEL=cluster (the L2-exchange LN kernel assumes a co-resident grid and must
 not run concurrently with itself)."""
 import json, os, sys
+os.environ.setdefault("TCB_LN_KERNEL", "cluster")   # never two L2-exchange kernels at once
 sys.path.insert(0, os.path.dirname(os.path.dirname(os.path.abspath(__file__))))
 import numpy as np, torch
 import tcb_workload as wl
