@@ -1707,9 +1707,32 @@ cudaError_t launch_lng(const GemmMaps& m, int M, int K, const float* bias, const
   const int units = ((M + 255) / 256) * P;
   const int pairs = units < max_pairs ? units : max_pairs;
   cfg.gridDim = dim3(2 * pairs);
-  if (pdl_enabled()) pdl_attr(attr[cfg.numAttrs++]);
-  return cudaLaunchKernelEx(&cfg, kern, m.a, m.w, m.c, m.r, M, K, bias, gamma, beta, eps, seg_ids,
-                            stats, cnt);
+  // cooperative: the runtime guarantees every CTA of the grid is co-resident (the kernel's
+  // cross-CTA waits rely on it), also when another launch on another stream holds SMs
+  static int coop = -1;     // -1 untried, 1 accepted with clusters + PDL, 0 rejected
+  cudaLaunchAttribute attr3[3] = {attr[0], attr[1], attr[1]};
+  cfg.attrs = attr3;
+  if (pdl_enabled()) pdl_attr(attr3[cfg.numAttrs++]);
+  if (coop != 0) {
+    attr3[cfg.numAttrs].id = cudaLaunchAttributeCooperative;
+    attr3[cfg.numAttrs].val.cooperative = 1;
+    ++cfg.numAttrs;
+  }
+  cudaError_t e = cudaLaunchKernelEx(&cfg, kern, m.a, m.w, m.c, m.r, M, K, bias, gamma, beta, eps,
+                                     seg_ids, stats, cnt);
+  if (coop == -1) {
+    coop = e == cudaSuccess ? 1 : 0;
+    if (std::getenv("TCB_VERBOSE"))
+      std::fprintf(stderr, "tcb: L2-exchange LN kernel cooperative launch %s\n",
+                   coop ? "accepted" : "rejected, plain launch");
+    if (e != cudaSuccess) {       // not supported with these attributes: plain launch
+      cudaGetLastError();
+      --cfg.numAttrs;
+      e = cudaLaunchKernelEx(&cfg, kern, m.a, m.w, m.c, m.r, M, K, bias, gamma, beta, eps, seg_ids,
+                             stats, cnt);
+    }
+  }
+  return e;
 }
 
 size_t linear_ln_scratch_stats_bytes(int64_t M, int N) {
