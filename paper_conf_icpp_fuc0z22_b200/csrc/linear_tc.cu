@@ -1709,7 +1709,9 @@ cudaError_t launch_lng(const GemmMaps& m, int M, int K, const float* bias, const
   cfg.gridDim = dim3(2 * pairs);
   // cooperative: the runtime guarantees every CTA of the grid is co-resident (the kernel's
   // cross-CTA waits rely on it), also when another launch on another stream holds SMs
-  static int coop = -1;     // -1 untried, 1 accepted with clusters + PDL, 0 rejected
+  // (off under a profiler's injection library -- ncu's kernel replay rejects cooperative
+  // cluster launches -- and with TCB_NO_COOP=1)
+  static int coop = (std::getenv("TCB_NO_COOP") || std::getenv("CUDA_INJECTION64_PATH")) ? 0 : -1;
   cudaLaunchAttribute attr3[3] = {attr[0], attr[1], attr[1]};
   cfg.attrs = attr3;
   if (pdl_enabled()) pdl_attr(attr3[cfg.numAttrs++]);
