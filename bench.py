@@ -311,7 +311,8 @@ def main():
         torch.cuda.synchronize()
     if world > 1:
         dist.barrier()
-    ms = sum(a.elapsed_time(b) for a, b in ev)
+    step_ms = [a.elapsed_time(b) for a, b in ev]
+    ms = sum(step_ms)
     t_local = torch.tensor([ms, float(tokens_rank)], dtype=torch.float64, device=dev)
     if world > 1:
         tmax = t_local.clone()
@@ -501,6 +502,7 @@ def main():
                        "parallelism": f"dp{world} (rows sharded, weights broadcast once)",
                        "l2": "flushed (256 MiB write) between timed steps",
                        "cuda_graph": graph is not None},
+            "ms_per_step_p10_p50_p90": [float(np.percentile(step_ms, q)) for q in (10, 50, 90)],
             "tc_frac_whole_step": whole_tc / peaks["bf16_tflops"],
             "tc_frac_whole_step_vs_sustained": whole_tc / tc_peak,
             "tc_whole_step_tflops": whole_tc,
