@@ -158,9 +158,21 @@ struct tcb_weights {
   // activation TMA descriptors, rebuilt when the (rows, workspace) pointers change:
   // A-role (GEMM input) and C-role (GEMM output / residual input) views of each buffer
   std::mutex mu;
+  std::mutex graph_mu;                    // fwd_graphs
   const void* c_rows = nullptr;
   const void* c_ws = nullptr;
   int64_t c_M = -1;
+  // tcb_encoder_forward's instantiated CUDA graphs, keyed on the launch geometry and buffers
+  // (the kernels read everything plan-specific from the device segment table)
+  struct FwdGraph {
+    int64_t M;
+    int32_t rows, row_len;
+    const void *segtab, *ids, *drows, *ws;
+    cudaGraphExec_t exec;
+    uint64_t launches, last_use;
+  };
+  std::vector<FwdGraph> fwd_graphs;
+  uint64_t fwd_tick = 0;
   CUtensorMap aX{}, aAtt{}, aX1{}, aH{};
   CUtensorMap cQkv{}, cZ{}, cH{}, cX{}, cX1{};
 
@@ -320,6 +332,7 @@ tcb_status tcb_weights_create(const tcb_model_config* cfg, const void* const* te
 
 void tcb_weights_destroy(tcb_weights* w) {
   if (!w) return;
+  for (auto& g : w->fwd_graphs) cudaGraphExecDestroy(g.exec);
   if (w->pe_table) cudaFree(w->pe_table);
   delete w;
 }
@@ -337,10 +350,95 @@ tcb_status tcb_embed(const tcb_weights* w, const tcb_plan* plan, const int32_t* 
                     reinterpret_cast<cudaStream_t>(stream));
 }
 
+namespace {
+tcb_status forward_impl(const tcb_weights* wc, const tcb_plan* plan, const int32_t* d_segtab,
+                        const int32_t* d_token_ids, void* d_rows, void* d_ws, size_t ws_bytes,
+                        tcb_stream_t stream);
+}  // namespace
+
+// The public forward replays a CUDA graph of its own launch sequence when it can: on a
+// non-default stream that is not being captured by the caller, with profiling off, and
+// TCB_NO_FWD_GRAPH unset.  The graph is captured on the first call with a given geometry and
+// set of buffers (LRU of 4 per weights handle) and replayed for any later plan of the same
+// B x L (every plan-specific value is read from the device segment table); otherwise the
+// kernels are launched directly.  Either way the work is the same.
 tcb_status tcb_encoder_forward(const tcb_weights* wc, const tcb_plan* plan,
                                const int32_t* d_segtab, const int32_t* d_token_ids,
                                void* d_rows, void* d_ws, size_t ws_bytes, tcb_stream_t stream) {
   tcb::clear_error();
+  static const bool no_graph =
+      std::getenv("TCB_NO_FWD_GRAPH") != nullptr || std::getenv("TCB_DEBUG_SYNC") != nullptr;
+  cudaStream_t s = reinterpret_cast<cudaStream_t>(stream);
+  bool use_graph = !no_graph && s != nullptr && wc && plan && plan->info.num_slots > 0 &&
+                   d_segtab && d_rows && d_ws;
+  if (use_graph) {
+    std::lock_guard<std::mutex> g(g_prof_mu);
+    use_graph = !g_prof_on;
+  }
+  if (use_graph) {
+    cudaStreamCaptureStatus cs = cudaStreamCaptureStatusNone;
+    if (cudaStreamIsCapturing(s, &cs) != cudaSuccess || cs != cudaStreamCaptureStatusNone) {
+      cudaGetLastError();
+      use_graph = false;
+    }
+  }
+  if (!use_graph)
+    return forward_impl(wc, plan, d_segtab, d_token_ids, d_rows, d_ws, ws_bytes, stream);
+  if (tcb_status st = validate_plan_for(wc, plan)) return st;
+  tcb_weights* w = const_cast<tcb_weights*>(wc);
+  const int64_t M = plan->info.num_slots;
+  std::lock_guard<std::mutex> gl(w->graph_mu);
+  for (auto& e : w->fwd_graphs) {
+    if (e.M == M && e.rows == plan->num_rows && e.row_len == plan->row_len &&
+        e.segtab == d_segtab && e.ids == d_token_ids && e.drows == d_rows && e.ws == d_ws) {
+      if (ws_bytes < ws_layout(w->cfg, M).total)
+        break;                                   // let forward_impl report it
+      e.last_use = ++w->fwd_tick;
+      cudaError_t err = cudaGraphLaunch(e.exec, s);
+      if (err != cudaSuccess) return cuda_fail(err, "tcb_encoder_forward: graph launch");
+      g_launches.fetch_add(e.launches, std::memory_order_relaxed);
+      return TCB_OK;
+    }
+  }
+  // miss: capture this call's launches, instantiate, run the graph
+  if (cudaStreamBeginCapture(s, cudaStreamCaptureModeThreadLocal) != cudaSuccess) {
+    cudaGetLastError();
+    return forward_impl(wc, plan, d_segtab, d_token_ids, d_rows, d_ws, ws_bytes, stream);
+  }
+  const uint64_t c0 = g_launches.load();
+  const tcb_status st = forward_impl(wc, plan, d_segtab, d_token_ids, d_rows, d_ws, ws_bytes, stream);
+  cudaGraph_t graph = nullptr;
+  const cudaError_t ce = cudaStreamEndCapture(s, &graph);
+  if (st != TCB_OK || ce != cudaSuccess || !graph) {
+    if (graph) cudaGraphDestroy(graph);
+    cudaGetLastError();
+    if (st != TCB_OK) return st;
+    return forward_impl(wc, plan, d_segtab, d_token_ids, d_rows, d_ws, ws_bytes, stream);
+  }
+  cudaGraphExec_t exec = nullptr;
+  const cudaError_t ie = cudaGraphInstantiate(&exec, graph, 0);
+  cudaGraphDestroy(graph);
+  if (ie != cudaSuccess) {
+    cudaGetLastError();
+    return forward_impl(wc, plan, d_segtab, d_token_ids, d_rows, d_ws, ws_bytes, stream);
+  }
+  if (w->fwd_graphs.size() >= 4) {               // evict the least recently used
+    auto lru = std::min_element(w->fwd_graphs.begin(), w->fwd_graphs.end(),
+                                [](const auto& a, const auto& b) { return a.last_use < b.last_use; });
+    cudaGraphExecDestroy(lru->exec);
+    w->fwd_graphs.erase(lru);
+  }
+  w->fwd_graphs.push_back({M, plan->num_rows, plan->row_len, d_segtab, d_token_ids, d_rows, d_ws,
+                           exec, g_launches.load() - c0, ++w->fwd_tick});
+  const cudaError_t le = cudaGraphLaunch(exec, s);
+  if (le != cudaSuccess) return cuda_fail(le, "tcb_encoder_forward: graph launch");
+  return TCB_OK;
+}
+
+namespace {
+tcb_status forward_impl(const tcb_weights* wc, const tcb_plan* plan, const int32_t* d_segtab,
+                        const int32_t* d_token_ids, void* d_rows, void* d_ws, size_t ws_bytes,
+                        tcb_stream_t stream) {
   if (tcb_status st = validate_plan_for(wc, plan)) return st;
   tcb_weights* w = const_cast<tcb_weights*>(wc);
   const tcb_model_config& c = w->cfg;
@@ -468,6 +566,7 @@ tcb_status tcb_encoder_forward(const tcb_weights* wc, const tcb_plan* plan,
   }
   return TCB_OK;
 }
+}  // namespace
 
 tcb_status tcb_unpack(const tcb_weights* w, const tcb_plan* plan, const int32_t* d_segtab,
                       const void* d_rows, void* d_out, tcb_stream_t stream) {
