@@ -173,6 +173,7 @@ struct tcb_weights {
   };
   std::vector<FwdGraph> fwd_graphs;
   uint64_t fwd_tick = 0;
+  cudaStream_t cap_stream = nullptr;      // private stream the graphs are captured on
   CUtensorMap aX{}, aAtt{}, aX1{}, aH{};
   CUtensorMap cQkv{}, cZ{}, cH{}, cX{}, cX1{};
 
@@ -333,6 +334,7 @@ tcb_status tcb_weights_create(const tcb_model_config* cfg, const void* const* te
 void tcb_weights_destroy(tcb_weights* w) {
   if (!w) return;
   for (auto& g : w->fwd_graphs) cudaGraphExecDestroy(g.exec);
+  if (w->cap_stream) cudaStreamDestroy(w->cap_stream);
   if (w->pe_table) cudaFree(w->pe_table);
   delete w;
 }
@@ -369,13 +371,13 @@ tcb_status tcb_encoder_forward(const tcb_weights* wc, const tcb_plan* plan,
   static const bool no_graph =
       std::getenv("TCB_NO_FWD_GRAPH") != nullptr || std::getenv("TCB_DEBUG_SYNC") != nullptr;
   cudaStream_t s = reinterpret_cast<cudaStream_t>(stream);
-  bool use_graph = !no_graph && s != nullptr && wc && plan && plan->info.num_slots > 0 &&
-                   d_segtab && d_rows && d_ws;
+  bool use_graph = !no_graph && wc && plan && plan->info.num_slots > 0 && d_segtab && d_rows &&
+                   d_ws;
   if (use_graph) {
     std::lock_guard<std::mutex> g(g_prof_mu);
     use_graph = !g_prof_on;
   }
-  if (use_graph) {
+  if (use_graph && s != nullptr) {
     cudaStreamCaptureStatus cs = cudaStreamCaptureStatusNone;
     if (cudaStreamIsCapturing(s, &cs) != cudaSuccess || cs != cudaStreamCaptureStatusNone) {
       cudaGetLastError();
@@ -400,15 +402,22 @@ tcb_status tcb_encoder_forward(const tcb_weights* wc, const tcb_plan* plan,
       return TCB_OK;
     }
   }
-  // miss: capture this call's launches, instantiate, run the graph
-  if (cudaStreamBeginCapture(s, cudaStreamCaptureModeThreadLocal) != cudaSuccess) {
+  // miss: capture this call's launches on the private stream, instantiate, run the graph on s
+  if (!w->cap_stream && cudaStreamCreateWithFlags(&w->cap_stream, cudaStreamNonBlocking) != cudaSuccess) {
+    cudaGetLastError();
+    w->cap_stream = nullptr;
+    return forward_impl(wc, plan, d_segtab, d_token_ids, d_rows, d_ws, ws_bytes, stream);
+  }
+  cudaStream_t cap = w->cap_stream;
+  if (cudaStreamBeginCapture(cap, cudaStreamCaptureModeThreadLocal) != cudaSuccess) {
     cudaGetLastError();
     return forward_impl(wc, plan, d_segtab, d_token_ids, d_rows, d_ws, ws_bytes, stream);
   }
   const uint64_t c0 = g_launches.load();
-  const tcb_status st = forward_impl(wc, plan, d_segtab, d_token_ids, d_rows, d_ws, ws_bytes, stream);
+  const tcb_status st = forward_impl(wc, plan, d_segtab, d_token_ids, d_rows, d_ws, ws_bytes,
+                                     reinterpret_cast<tcb_stream_t>(cap));
   cudaGraph_t graph = nullptr;
-  const cudaError_t ce = cudaStreamEndCapture(s, &graph);
+  const cudaError_t ce = cudaStreamEndCapture(cap, &graph);
   if (st != TCB_OK || ce != cudaSuccess || !graph) {
     if (graph) cudaGraphDestroy(graph);
     cudaGetLastError();
@@ -731,6 +740,15 @@ struct tcb_decoder {
   tcb_decode_stats stats{};
   int32_t last_rows = 0;
   int32_t* pin = nullptr;                // pinned host: active list [2][R], done flags [2][R]
+  int32_t* tstep = nullptr;              // device step index read by the graphs' kernels
+  struct StepGraph {                     // one decode step captured for a bucket of rows
+    int32_t rows;
+    const int32_t* tokens;
+    cudaGraphExec_t exec;
+    uint64_t launches;
+  };
+  std::vector<StepGraph> graphs;
+  cudaStream_t cap_stream = nullptr;     // private stream the step graphs are captured on
   cudaEvent_t ev[2] = {nullptr, nullptr};  // done flags of a step on the host
   const void* L(int layer, int i) const { return t[20 * layer + i]; }
   const float* Lf(int layer, int i) const { return static_cast<const float*>(L(layer, i)); }
@@ -741,6 +759,8 @@ enum { D_W_QKV = 0, D_B_QKV, D_W_O, D_B_O, D_LN1_G, D_LN1_B, D_W_Q, D_B_Q, D_W_K
        D_W_CO, D_B_CO, D_LN2_G, D_LN2_B, D_W_1, D_B_1, D_W_2, D_B_2, D_LN3_G, D_LN3_B };
 
 void free_decoder(tcb_decoder* dec) {
+  for (auto& g : dec->graphs) cudaGraphExecDestroy(g.exec);
+  if (dec->cap_stream) cudaStreamDestroy(dec->cap_stream);
   for (void* p : dec->bufs) cudaFree(p);
   if (dec->pin) cudaFreeHost(dec->pin);
   for (cudaEvent_t e : dec->ev)
@@ -808,10 +828,11 @@ tcb_status tcb_decoder_create(const tcb_weights* enc, const void* const* tensors
             dalloc(dec, &dec->act, 4 * R) && dalloc(dec, &dec->out_len, 4 * R) &&
             dalloc(dec, &dec->done, 4 * R) && dalloc(dec, &dec->flag, 4 * R) &&
             dalloc(dec, &dec->tmax, 4 * R) && dalloc(dec, &dec->mem_start, 4 * R) &&
-            dalloc(dec, &dec->mem_len, 4 * R);
+            dalloc(dec, &dec->mem_len, 4 * R) && dalloc(dec, &dec->tstep, 16);
   ok = ok && cudaMallocHost(reinterpret_cast<void**>(&dec->pin), 16 * R) == cudaSuccess &&
        cudaEventCreateWithFlags(&dec->ev[0], cudaEventDisableTiming) == cudaSuccess &&
-       cudaEventCreateWithFlags(&dec->ev[1], cudaEventDisableTiming) == cudaSuccess;
+       cudaEventCreateWithFlags(&dec->ev[1], cudaEventDisableTiming) == cudaSuccess &&
+       cudaStreamCreateWithFlags(&dec->cap_stream, cudaStreamNonBlocking) == cudaSuccess;
   if (!ok) {
     cudaGetLastError();
     free_decoder(dec);
@@ -917,18 +938,11 @@ tcb_status tcb_decode_greedy(tcb_decoder* dec, const tcb_plan* plan, const void*
   // the generated tokens are those of the synchronous loop.
   int32_t* act_pin[2] = {dec->pin, dec->pin + dec->R};
   int32_t* done_pin[2] = {dec->pin + 2 * dec->R, dec->pin + 3 * dec->R};
-  for (; t < max_steps && !act_h.empty(); ++t) {
-    const int A = static_cast<int>(act_h.size());
-    const int sl = t & 1;
-    if (act_dirty) {   // act_pin[sl]'s previous upload (step t-2) completed: ev of t-2 was waited
-      std::memcpy(act_pin[sl], act_h.data(), 4 * static_cast<size_t>(A));
-      e = cudaMemcpyAsync(dec->act, act_pin[sl], 4 * A, cudaMemcpyHostToDevice, s);
-      if (e != cudaSuccess) return cuda_fail(e, "tcb_decode_greedy: active set upload");
-      act_dirty = false;
-    }
+  // one decode step's kernels over `A` rows (step index t, or *d_t when d_t is set)
+  auto enqueue_step = [&](int A, int t, const int32_t* d_t, cudaStream_t s) -> tcb_status {
     DecEmbedArgs ea{dec->act, d_tokens, T, t, 1, 2, d, A,
                     static_cast<const __nv_bfloat16*>(dec->enc->tok_emb()), dec->enc->pe_table,
-                    c.emb_scale, static_cast<__nv_bfloat16*>(dec->x)};
+                    c.emb_scale, static_cast<__nv_bfloat16*>(dec->x), d_t};
     TCB_LAUNCH(TCB_K_EMBED, s, launch_dec_embed(ea, s));
     for (int l = 0; l < S; ++l) {
       const auto& m = dec->wm[l];
@@ -950,6 +964,7 @@ tcb_status tcb_decode_greedy(tcb_decoder* dec, const tcb_plan* plan, const void*
       sa.rows = A;
       sa.scale = scale;
       sa.out = static_cast<__nv_bfloat16*>(dec->att);
+      sa.d_t = d_t;
       TCB_LAUNCH(TCB_K_ATTN, s, launch_dec_attn(sa, s));
       TCB_LAUNCH(TCB_K_GEMM_O, s, launch_linear_ln_bf16_tc(GemmMaps{dec->aAtt, m.o, dec->cX1, dec->cX},
                                                            A, d, d, dec->Lf(l, D_B_O), dec->Lf(l, D_LN1_G),
@@ -977,8 +992,87 @@ tcb_status tcb_decode_greedy(tcb_decoder* dec, const tcb_plan* plan, const void*
     TCB_LAUNCH(TCB_K_GEMM_QKV, s, launch_linear_bf16_tc(GemmMaps{dec->aX, dec->w_logits, dec->cLogits, dec->cLogits},
                                                         A, V, d, dec->zero_bias, TCB_EPI_BIAS, s));
     DecArgmaxArgs ga{static_cast<const __nv_bfloat16*>(dec->logits), V, A, t, 2, T, dec->act,
-                     dec->tmax, d_tokens, dec->out_len, dec->done, dec->flag};
+                     dec->tmax, d_tokens, dec->out_len, dec->done, dec->flag, d_t};
     TCB_LAUNCH(TCB_K_UNPACK, s, launch_dec_argmax(ga, s));
+    if (d_t) TCB_LAUNCH(TCB_K_UNPACK, s, launch_dec_step_advance(const_cast<int32_t*>(d_t), s));
+    return TCB_OK;
+  };
+  // CUDA graphs per bucket of rows: on a non-default stream the caller is not capturing,
+  // profiling off, TCB_NO_DEC_GRAPH unset
+  bool use_graphs = std::getenv("TCB_NO_DEC_GRAPH") == nullptr;
+  if (use_graphs) {
+    std::lock_guard<std::mutex> g(g_prof_mu);
+    use_graphs = !g_prof_on;
+  }
+  if (use_graphs && s != nullptr) {
+    cudaStreamCaptureStatus cs = cudaStreamCaptureStatusNone;
+    if (cudaStreamIsCapturing(s, &cs) != cudaSuccess || cs != cudaStreamCaptureStatusNone) {
+      cudaGetLastError();
+      use_graphs = false;
+    }
+  }
+  auto bucket_of = [&](int A) {
+    int b = 32;
+    while (b < A) b *= 2;
+    return std::min(b, dec->R);
+  };
+  int rows_up = -1;
+  if (use_graphs) {
+    e = cudaMemsetAsync(dec->tstep, 0, 4, s);
+    if (e != cudaSuccess) return cuda_fail(e, "tcb_decode_greedy: step index");
+  }
+  for (; t < max_steps && !act_h.empty(); ++t) {
+    const int A = static_cast<int>(act_h.size());
+    const int sl = t & 1;
+    if (use_graphs) {
+      // the step's kernels for a bucket of rows (the power of two >= A, at most R), captured
+      // once per bucket and output buffer, replayed with the step index in device memory
+      const int rows = bucket_of(A);
+      tcb_decoder::StepGraph* gph = nullptr;
+      for (auto& gg : dec->graphs)
+        if (gg.rows == rows && gg.tokens == d_tokens) gph = &gg;
+      if (!gph) {
+        if (dec->graphs.size() >= 16) {        // bounded cache: start over
+          for (auto& gg : dec->graphs) cudaGraphExecDestroy(gg.exec);
+          dec->graphs.clear();
+        }
+        cudaGraph_t graph = nullptr;
+        cudaStream_t cap = dec->cap_stream;
+        e = cudaStreamBeginCapture(cap, cudaStreamCaptureModeThreadLocal);
+        if (e != cudaSuccess) return cuda_fail(e, "tcb_decode_greedy: capture");
+        const uint64_t c0 = g_launches.load();
+        const tcb_status st = enqueue_step(rows, 0, dec->tstep, cap);
+        e = cudaStreamEndCapture(cap, &graph);
+        if (st != TCB_OK) { if (graph) cudaGraphDestroy(graph); return st; }
+        if (e != cudaSuccess) return cuda_fail(e, "tcb_decode_greedy: capture");
+        cudaGraphExec_t exec = nullptr;
+        e = cudaGraphInstantiate(&exec, graph, 0);
+        cudaGraphDestroy(graph);
+        if (e != cudaSuccess) return cuda_fail(e, "tcb_decode_greedy: graph instantiate");
+        dec->graphs.push_back({rows, d_tokens, exec, g_launches.load() - c0});
+        g_launches.fetch_sub(dec->graphs.back().launches);   // counted when replayed
+        gph = &dec->graphs.back();
+      }
+      if (act_dirty || rows != rows_up) {   // padded active list (rows >= A are -1)
+        std::memcpy(act_pin[sl], act_h.data(), 4 * static_cast<size_t>(A));
+        for (int i = A; i < rows; ++i) act_pin[sl][i] = -1;
+        e = cudaMemcpyAsync(dec->act, act_pin[sl], 4 * rows, cudaMemcpyHostToDevice, s);
+        if (e != cudaSuccess) return cuda_fail(e, "tcb_decode_greedy: active set upload");
+        act_dirty = false;
+        rows_up = rows;
+      }
+      e = cudaGraphLaunch(gph->exec, s);
+      if (e != cudaSuccess) return cuda_fail(e, "tcb_decode_greedy: graph launch");
+      g_launches.fetch_add(gph->launches, std::memory_order_relaxed);
+    } else {
+      if (act_dirty) {   // act_pin[sl]'s previous upload (step t-2) completed
+        std::memcpy(act_pin[sl], act_h.data(), 4 * static_cast<size_t>(A));
+        e = cudaMemcpyAsync(dec->act, act_pin[sl], 4 * A, cudaMemcpyHostToDevice, s);
+        if (e != cudaSuccess) return cuda_fail(e, "tcb_decode_greedy: active set upload");
+        act_dirty = false;
+      }
+      if (tcb_status st = enqueue_step(A, t, nullptr, s)) return st;
+    }
     e = cudaMemcpyAsync(done_pin[sl], dec->done, 4 * n, cudaMemcpyDeviceToHost, s);
     if (e == cudaSuccess) e = cudaEventRecord(dec->ev[sl], s);
     if (e != cudaSuccess) return cuda_fail(e, "tcb_decode_greedy: step");

@@ -38,13 +38,18 @@ dec_embed_kernel(DecEmbedArgs a) {
   pdl_trigger();
   if (warp >= a.rows) return;
   const int r = a.act[warp];
-  int tok = a.t == 0 ? a.bos : a.out_tok[static_cast<int64_t>(r) * a.ld_out + a.t - 1];
+  const int t = a.d_t ? *a.d_t : a.t;
+  __nv_bfloat16* x = a.x + static_cast<int64_t>(warp) * a.d;
+  if (r < 0) {                                   // padding row of a bucketed graph
+    for (int c = lane * 8; c < a.d; c += 256) *reinterpret_cast<uint4*>(x + c) = make_uint4(0, 0, 0, 0);
+    return;
+  }
+  int tok = t == 0 ? a.bos : a.out_tok[static_cast<int64_t>(r) * a.ld_out + t - 1];
   // a request that already finished (whole-batch mode keeps computing it; nothing of it is
   // recorded any more) has no next token: feed EOS
   if (tok < 0) tok = a.eos;
   const __nv_bfloat16* e = a.tok_emb + static_cast<int64_t>(tok) * a.d;
-  const float* pe = a.pe + static_cast<int64_t>(a.t) * a.d;
-  __nv_bfloat16* x = a.x + static_cast<int64_t>(warp) * a.d;
+  const float* pe = a.pe + static_cast<int64_t>(t) * a.d;
   for (int c = lane * 8; c < a.d; c += 256) {
     const uint4 v = *reinterpret_cast<const uint4*>(e + c);
     const __nv_bfloat162* h = reinterpret_cast<const __nv_bfloat162*>(&v);
@@ -74,14 +79,20 @@ dec_attn_kernel(DecAttnArgs a) {
   pdl_trigger();
   if (h >= a.heads) return;
   const int r = a.act[i];
+  if (r < 0) {                                   // padding row of a bucketed graph
+    reinterpret_cast<__nv_bfloat162*>(a.out + static_cast<int64_t>(i) * a.d + h * DH)[lane] =
+        __floats2bfloat162_rn(0.f, 0.f);
+    return;
+  }
+  const int t = a.d_t ? *a.d_t : a.t;
   int64_t kstart;
   int klen;
   if (a.self) {
     kstart = static_cast<int64_t>(r) * a.t_cap;
-    klen = a.t + 1;
+    klen = t + 1;
     // append this step's key and value (2 x 64 bf16) at cache position t
     const __nv_bfloat16* src = a.q + static_cast<int64_t>(i) * a.ldq;
-    __nv_bfloat16* dst = a.kv + (kstart + a.t) * a.ld_kv;
+    __nv_bfloat16* dst = a.kv + (kstart + t) * a.ld_kv;
     const uint32_t* sk = reinterpret_cast<const uint32_t*>(src + a.d + h * DH);
     const uint32_t* sv = reinterpret_cast<const uint32_t*>(src + 2 * a.d + h * DH);
     reinterpret_cast<uint32_t*>(dst + h * DH)[lane] = sk[lane];
@@ -182,19 +193,34 @@ dec_argmax_kernel(DecArgmaxArgs a) {
   }
   if (threadIdx.x == 0) {
     const int r = a.act[i];
+    if (r < 0) {                                 // padding row of a bucketed graph
+      a.flag[i] = 1;
+      return;
+    }
+    const int t = a.d_t ? *a.d_t : a.t;
     const int tok = si[0];
     if (!a.done[r]) {
-      a.out_tok[static_cast<int64_t>(r) * a.ld_out + a.t] = tok;
-      if (tok == a.eos || a.t + 1 >= a.t_max[r]) {
+      a.out_tok[static_cast<int64_t>(r) * a.ld_out + t] = tok;
+      if (tok == a.eos || t + 1 >= a.t_max[r]) {
         a.done[r] = 1;
-        a.out_len[r] = a.t + 1;
+        a.out_len[r] = t + 1;
       }
     }
     a.flag[i] = a.done[r];
   }
 }
 
+__global__ void dec_step_advance_kernel(int32_t* d_t) {
+  pdl_wait();
+  pdl_trigger();
+  *d_t += 1;
+}
+
 }  // namespace
+
+cudaError_t launch_dec_step_advance(int32_t* d_t, cudaStream_t s) {
+  return launch_ex(dec_step_advance_kernel, dim3(1), dim3(1), 0, s, 1, d_t);
+}
 
 cudaError_t launch_dec_embed(const DecEmbedArgs& a, cudaStream_t s) {
   if (a.rows == 0) return cudaSuccess;

@@ -136,6 +136,7 @@ struct DecEmbedArgs {
   const float* pe;             // [max_pos, d] fp32 sinusoidal table
   float emb_scale;
   __nv_bfloat16* x;            // out [rows, d]
+  const int32_t* d_t;          // if set: the step index is *d_t (CUDA-graph replay), not t
 };
 struct DecAttnArgs {
   const int32_t* act;
@@ -150,6 +151,7 @@ struct DecAttnArgs {
   int32_t d, heads, rows;
   float scale;
   __nv_bfloat16* out;          // [rows, d]
+  const int32_t* d_t;          // if set: the step index is *d_t, not t
 };
 struct DecArgmaxArgs {
   const __nv_bfloat16* logits; // [rows, vocab]
@@ -160,7 +162,11 @@ struct DecArgmaxArgs {
   int32_t* out_len;            // [R]
   int32_t* done;               // [R]
   int32_t* flag;               // [rows] finished after this step
+  const int32_t* d_t;          // if set: the step index is *d_t, not t
 };
+// Rows whose act[] entry is < 0 are padding (a graph captured for a bucket of rows): the
+// kernels write zeros for them and record nothing.
+cudaError_t launch_dec_step_advance(int32_t* d_t, cudaStream_t s);   // ++*d_t
 cudaError_t launch_dec_embed(const DecEmbedArgs& a, cudaStream_t s);
 cudaError_t launch_dec_attn(const DecAttnArgs& a, cudaStream_t s);
 cudaError_t launch_dec_argmax(const DecArgmaxArgs& a, cudaStream_t s);
