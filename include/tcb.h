@@ -206,11 +206,11 @@ tcb_status tcb_embed(const tcb_weights* w, const tcb_plan* plan, const int32_t* 
  * W_O GEMM + bias + residual -> LN1 -> FFN1 GEMM + bias + act -> FFN2 GEMM + bias +
  * residual -> LN2].  d_rows receives the last layer's hidden states [num_slots, d_model]
  * (pad slots 0).  The plan is read only for its shape (num_rows, row_len) and validation;
- * the device segment table is what the kernels use.  On a non-default stream that the caller
- * is not capturing, the call replays a CUDA graph of its own launch sequence (captured on the
- * first call with the same shape and the same d_segtab / d_token_ids / d_rows / d_workspace
- * pointers, at most 4 kept per weights handle; TCB_NO_FWD_GRAPH=1 launches directly); inside
- * a caller's capture the kernels are captured into that graph.  The workspace holds, for bf16
+ * the device segment table is what the kernels use.  Unless the caller is capturing
+ * `stream`, the call replays a CUDA graph of its own launch sequence (captured on a private
+ * stream on the first call with the same shape and the same d_segtab / d_token_ids / d_rows /
+ * d_workspace pointers, at most 4 kept per weights handle; TCB_NO_FWD_GRAPH=1 launches
+ * directly); inside a caller's capture the kernels are captured into that graph.  The workspace holds, for bf16
  * d in {512, 768, 1024}, the row-statistics scratch of the LayerNorm GEMMs; its counters are
  * zeroed by the call (one memset on the stream). */
 tcb_status tcb_encoder_forward(const tcb_weights* w, const tcb_plan* plan,

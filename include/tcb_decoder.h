@@ -56,7 +56,11 @@ void tcb_decoder_destroy(tcb_decoder* dec);
  * (the paper's baseline) -- the tokens are identical either way.
  * Outputs (caller-owned): d_tokens [num_requests, max_target] int32 device, -1 past the end
  * and for unplaced requests; h_lengths [num_requests] host, generated count (0 if unplaced).
- * Blocking: every step reads the finished flags back to build the next active set. */
+ * Blocking: while step t runs, the host reads the finished flags of step t-1 back to build
+ * the active set of step t+1 (so a finished request is computed once more, ignored).  Each
+ * step is replayed from a CUDA graph captured per bucket of rows (power of two >= the active
+ * count, at most max_requests) and per d_tokens buffer, unless the caller is capturing
+ * `stream` or TCB_NO_DEC_GRAPH=1. */
 tcb_status tcb_decode_greedy(tcb_decoder* dec, const tcb_plan* plan, const void* d_enc_rows,
                              int32_t early_clean, int32_t* d_tokens, int32_t* h_lengths,
                              tcb_stream_t stream);
