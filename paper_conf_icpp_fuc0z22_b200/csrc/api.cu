@@ -639,11 +639,12 @@ tcb_status tcb_op_linear_ln(int64_t M, int32_t N, int32_t K, const void* A, cons
   if (!tcb::k::make_gemm_a_map(&maps.a, A, M, K) || !tcb::k::make_gemm_w_map(&maps.w, W, N, K) ||
       !tcb::k::make_gemm_c_map(&maps.c, C, M, N) || !tcb::k::make_gemm_c_map(&maps.r, R, M, N))
     return fail(TCB_ERR_CUDA, "tcb_op_linear_ln: cuTensorMapEncodeTiled failed (alignment?)");
-  // d >= 768: the row-statistics scratch of the L2-exchange kernel, library-owned for this op
-  // (grown on demand; the encoder forward uses its workspace instead)
+  // the row-statistics scratch of the L2-exchange kernel (N = 512 / 1024 with K >= 2N, or
+  // every N under TCB_LN_KERNEL=global), library-owned for this op (grown on demand; the
+  // encoder forward uses its workspace instead)
   float2* st = nullptr;
   int* cnt = nullptr;
-  if (N >= 768) {
+  {
     static std::mutex mu;
     static void* buf = nullptr;
     static size_t cap = 0;

@@ -1408,8 +1408,16 @@ linear_lng_kernel(const __grid_constant__ CUtensorMap tmA, const __grid_constant
     const uint32_t tempty0 = mapa_rank(smem_u32(tempty), 0);
     int acc = 0;
     uint32_t acc_phase = 0, rphase = 0;
+#ifdef TCB_LN_PROBE
+    long long e0 = clock64(), e_tfull = 0, e_p1 = 0, e_x = 0, e_p2 = 0;
+    int nunits = 0;
+#endif
     for (int u = pair; u < num_units; u += num_pairs) {
       const int t = u / P, p = u % P;
+#ifdef TCB_LN_PROBE
+      long long ta = clock64();
+      ++nunits;
+#endif
       const int wid = p * kLncColGroups + cg;     // contribution slot of this warp
       const int row0 = t * 256 + static_cast<int>(r) * 128 + q * 32;
       const int col0 = p * 256 + cg * (32 * kLncChunks);
@@ -1426,6 +1434,10 @@ linear_lng_kernel(const __grid_constant__ CUtensorMap tmA, const __grid_constant
       }
       mbar_wait(&tfull[acc], acc_phase);
       tc_fence_after();
+#ifdef TCB_LN_PROBE
+      long long tb = clock64();
+      e_tfull += tb - ta;
+#endif
       const uint32_t tbase = tmem_base + (static_cast<uint32_t>(q * 32) << 16) +
                              static_cast<uint32_t>(acc * 256 + cg * (32 * kLncChunks));
       // pass 1: z = acc + bias + residual -> TMEM; row partial moments
@@ -1470,6 +1482,10 @@ linear_lng_kernel(const __grid_constant__ CUtensorMap tmA, const __grid_constant
       }
       rphase ^= 1;
       asm volatile("tcgen05.wait::st.sync.aligned;" ::: "memory");
+#ifdef TCB_LN_PROBE
+      long long tc2 = clock64();
+      e_p1 += tc2 - tb;
+#endif
       // publish this warp's partials of its 32 rows, then wait for all kContrib of them
       float2* tst = gstats + static_cast<size_t>(t) * kContrib * 256 + static_cast<int>(r) * 128 + srow;
       tst[wid * 256] = make_float2(sum, sumsq);
@@ -1498,6 +1514,10 @@ linear_lng_kernel(const __grid_constant__ CUtensorMap tmA, const __grid_constant
       const float mean = s1 * kInvN;
       const float rstd = rsqrtf(fmaxf(s2 * kInvN - mean * mean, 0.f) + eps);
       const float nmr = -mean * rstd;             // (z - mean) rstd = fma(z, rstd, nmr)
+#ifdef TCB_LN_PROBE
+      long long td = clock64();
+      e_x += td - tc2;
+#endif
       // pass 2: normalise -> bf16 -> staging -> TMA store
 #pragma unroll 1
       for (int j = 0; j < kLncChunks; ++j) {
@@ -1541,10 +1561,18 @@ linear_lng_kernel(const __grid_constant__ CUtensorMap tmA, const __grid_constant
           asm volatile("cp.async.bulk.commit_group;" ::: "memory");
         }
       }
+#ifdef TCB_LN_PROBE
+      e_p2 += clock64() - td;
+#endif
       acc ^= 1;
       if (acc == 0) acc_phase ^= 1;
     }
     if (lane == 0) bulk_wait_all();
+#ifdef TCB_LN_PROBE
+    if (lane == 0 && ew == 0 && blockIdx.x < 6)
+      printf("lngprobe epi cta %d total %lld wait_tfull %lld pass1 %lld exchange %lld pass2 %lld units %d\n",
+             blockIdx.x, clock64() - e0, e_tfull, e_p1, e_x, e_p2, nunits);
+#endif
   }
   __syncwarp();
   tc_fence_before();
