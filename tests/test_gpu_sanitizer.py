@@ -1,0 +1,29 @@
+"""compute-sanitizer over a small run of every kernel of the path:
+memcheck (out-of-bounds / misaligned accesses) and synccheck (barrier misuse) must report 0
+errors.  racecheck is not asserted: it reports the tcgen05.alloc write of the TMEM base
+address (ordered by tcgen05.fence + barrier, which it does not model) and the mbarrier
+hand-offs in which one lane arrives for its warp after __syncwarp."""
+import os
+import shutil
+import subprocess
+import sys
+
+import pytest
+
+pytestmark = pytest.mark.gpu
+ROOT = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+SAN = shutil.which("compute-sanitizer") or "/usr/local/cuda/bin/compute-sanitizer"
+
+
+@pytest.mark.parametrize("tool", ["memcheck", "synccheck"])
+def test_compute_sanitizer_clean(tool):
+    if not os.path.exists(SAN):
+        pytest.skip("compute-sanitizer not installed")
+    env = dict(os.environ, TCB_NO_FWD_GRAPH="1", TCB_NO_DEC_GRAPH="1")
+    r = subprocess.run([SAN, "--tool", tool, "--error-exitcode", "3", sys.executable,
+                        os.path.join(ROOT, "scripts", "sanitize_workload.py")],
+                       cwd=ROOT, env=env, capture_output=True, text=True, timeout=1500)
+    tail = (r.stdout + r.stderr)[-3000:]
+    assert r.returncode == 0, tail
+    assert "sanitize workload done" in r.stdout, tail
+    assert "ERROR SUMMARY: 0 errors" in r.stdout + r.stderr, tail
