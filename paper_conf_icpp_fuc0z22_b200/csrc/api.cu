@@ -16,6 +16,8 @@
 #include <string>
 #include <vector>
 
+#include <nvtx3/nvToolsExt.h>   // header-only NVTX3: host ranges for nsys / ncu timelines
+
 #include "kernels.h"
 #include "tcb_internal.h"
 
@@ -445,9 +447,15 @@ tcb_status tcb_encoder_forward(const tcb_weights* wc, const tcb_plan* plan,
 }
 
 namespace {
+struct NvtxRange {
+  explicit NvtxRange(const char* name) { nvtxRangePushA(name); }
+  ~NvtxRange() { nvtxRangePop(); }
+};
+
 tcb_status forward_impl(const tcb_weights* wc, const tcb_plan* plan, const int32_t* d_segtab,
                         const int32_t* d_token_ids, void* d_rows, void* d_ws, size_t ws_bytes,
                         tcb_stream_t stream) {
+  NvtxRange nvtx_fwd("tcb_encoder_forward");
   if (tcb_status st = validate_plan_for(wc, plan)) return st;
   tcb_weights* w = const_cast<tcb_weights*>(wc);
   const tcb_model_config& c = w->cfg;
@@ -507,6 +515,7 @@ tcb_status forward_impl(const tcb_weights* wc, const tcb_plan* plan, const int32
         cudaMemsetAsync(ws + L.lncnt, 0, L.lncnt_per_launch * 2 * c.num_layers, s) != cudaSuccess)
       return fail(TCB_ERR_CUDA, "tcb_encoder_forward: counter reset failed");
     for (int l = 0; l < c.num_layers; ++l) {
+      NvtxRange nvtx_layer("tcb encoder layer");
       const auto& mp = w->maps[l];
       const tcb::k::GemmMaps g_qkv{w->aX, mp.qkv, w->cQkv, w->cQkv};
       const tcb::k::GemmMaps g_o{w->aAtt, mp.o, w->cZ, w->cX};
@@ -580,6 +589,8 @@ tcb_status forward_impl(const tcb_weights* wc, const tcb_plan* plan, const int32
 tcb_status tcb_unpack(const tcb_weights* w, const tcb_plan* plan, const int32_t* d_segtab,
                       const void* d_rows, void* d_out, tcb_stream_t stream) {
   tcb::clear_error();
+  nvtxRangePushA("tcb_unpack");
+  struct Pop { ~Pop() { nvtxRangePop(); } } pop_;
   if (tcb_status st = validate_plan_for(w, plan)) return st;
   const int64_t M = plan->info.num_slots;
   if (M == 0) return TCB_OK;

@@ -7,6 +7,7 @@
 // put").  First-Fit here runs in O(n log B): a max-segment-tree over the
 // residual capacity of all candidate rows finds the leftmost row with room; rows not yet
 // opened have residual L, so "leftmost row with room" also opens new rows in order.
+#include <nvtx3/nvToolsExt.h>   // header-only NVTX3 host range
 #include <algorithm>
 #include <cstdint>
 #include <cstring>
@@ -187,6 +188,8 @@ const char* tcb_version(void) { return "tcb-b200 0.1 (sm_100a)"; }
 
 tcb_status tcb_pack(const int32_t* lengths, int32_t n, int32_t row_len, int32_t max_rows,
                     int32_t policy, tcb_plan** out) {
+  nvtxRangePushA("tcb_pack");
+  struct Pop { ~Pop() { nvtxRangePop(); } } pop_;
   tcb::clear_error();
   tcb_status st = tcb::validate_pack("tcb_pack", lengths, n, row_len, max_rows, out);
   if (st != TCB_OK) return st;
