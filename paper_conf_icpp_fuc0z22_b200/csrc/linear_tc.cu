@@ -221,6 +221,44 @@ __device__ __forceinline__ float gelu_erf(float x) {
   return x * (x >= 0.f ? 1.f - h : h);
 }
 
+// Packed fp32x2 arithmetic (sm_100: FFMA2 / FADD2 / FMUL2 -- two lanes of work per issue slot)
+__device__ __forceinline__ unsigned long long f2_u(float2 v) {
+  return *reinterpret_cast<unsigned long long*>(&v);
+}
+__device__ __forceinline__ float2 u_f2(unsigned long long v) { return *reinterpret_cast<float2*>(&v); }
+__device__ __forceinline__ float2 ffma2(float2 a, float2 b, float2 c) {
+  unsigned long long r;
+  asm("fma.rn.f32x2 %0, %1, %2, %3;" : "=l"(r) : "l"(f2_u(a)), "l"(f2_u(b)), "l"(f2_u(c)));
+  return u_f2(r);
+}
+__device__ __forceinline__ float2 fadd2(float2 a, float2 b) {
+  unsigned long long r;
+  asm("add.rn.f32x2 %0, %1, %2;" : "=l"(r) : "l"(f2_u(a)), "l"(f2_u(b)));
+  return u_f2(r);
+}
+__device__ __forceinline__ float2 fmul2(float2 a, float2 b) {
+  unsigned long long r;
+  asm("mul.rn.f32x2 %0, %1, %2;" : "=l"(r) : "l"(f2_u(a)), "l"(f2_u(b)));
+  return u_f2(r);
+}
+// gelu_erf on two elements: the polynomial and the final combination in packed fp32x2,
+// x Phi(x) = x/2 + |x| (1/2 - h) (either sign of x, no select)
+__device__ __forceinline__ float2 gelu_erf2(float2 x) {
+  const float2 ax = make_float2(fabsf(x.x), fabsf(x.y));
+  const float2 a = make_float2(fminf(ax.x, 5.0f), fminf(ax.y, 5.0f));
+  float2 p = make_float2(-4.724943100e-04f, -4.724943100e-04f);
+  p = ffma2(p, a, make_float2(7.075486431e-03f, 7.075486431e-03f));
+  p = ffma2(p, a, make_float2(-5.179505318e-02f, -5.179505318e-02f));
+  p = ffma2(p, a, make_float2(-4.600401928e-01f, -4.600401928e-01f));
+  p = ffma2(p, a, make_float2(-1.150758799e+00f, -1.150758799e+00f));
+  p = ffma2(p, a, make_float2(-1.000043237e+00f, -1.000043237e+00f));
+  float2 h;
+  asm("ex2.approx.ftz.f32 %0, %1;" : "=f"(h.x) : "f"(p.x));
+  asm("ex2.approx.ftz.f32 %0, %1;" : "=f"(h.y) : "f"(p.y));
+  const float2 t = fadd2(make_float2(0.5f, 0.5f), make_float2(-h.x, -h.y));
+  return ffma2(ax, t, fmul2(make_float2(0.5f, 0.5f), x));
+}
+
 __device__ __forceinline__ void st_shared_v4(uint32_t addr, uint4 v) {
   asm volatile("st.shared.v4.b32 [%0], {%1, %2, %3, %4};" ::"r"(addr), "r"(v.x), "r"(v.y),
                "r"(v.z), "r"(v.w)
@@ -482,7 +520,11 @@ linear_tc_kernel(const __grid_constant__ CUtensorMap tmA, const __grid_constant_
         }
         if constexpr (EPI == TCB_EPI_BIAS_GELU) {
 #pragma unroll
-          for (int t = 0; t < 32; ++t) v[t] = gelu_erf(v[t]);
+          for (int t = 0; t < 32; t += 2) {
+            const float2 g = gelu_erf2(make_float2(v[t], v[t + 1]));
+            v[t] = g.x;
+            v[t + 1] = g.y;
+          }
         } else if constexpr (EPI == TCB_EPI_BIAS_RELU) {
 #pragma unroll
           for (int t = 0; t < 32; ++t) v[t] = fmaxf(v[t], 0.f);
