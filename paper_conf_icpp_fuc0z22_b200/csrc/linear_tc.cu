@@ -849,10 +849,12 @@ linear_ln_kernel(const __grid_constant__ CUtensorMap tmA, const __grid_constant_
 #pragma unroll
         for (int t = 0; t < 8; ++t) {
           const float4 bb = b4[t];
-          v[4 * t + 0] += bb.x;
-          v[4 * t + 1] += bb.y;
-          v[4 * t + 2] += bb.z;
-          v[4 * t + 3] += bb.w;
+          const float2 s0 = fadd2(make_float2(v[4 * t + 0], v[4 * t + 1]), make_float2(bb.x, bb.y));
+          const float2 s1 = fadd2(make_float2(v[4 * t + 2], v[4 * t + 3]), make_float2(bb.z, bb.w));
+          v[4 * t + 0] = s0.x;
+          v[4 * t + 1] = s0.y;
+          v[4 * t + 2] = s1.x;
+          v[4 * t + 3] = s1.y;
         }
 #ifdef TCB_LN_PROBE
         long long tr = clock64();
@@ -869,18 +871,21 @@ linear_ln_kernel(const __grid_constant__ CUtensorMap tmA, const __grid_constant_
 #pragma unroll
           for (int e = 0; e < 4; ++e) {
             const float2 f = __bfloat1622float2(hh[e]);
-            v[8 * t + 2 * e] += f.x;
-            v[8 * t + 2 * e + 1] += f.y;
+            const float2 s = fadd2(make_float2(v[8 * t + 2 * e], v[8 * t + 2 * e + 1]), f);
+            v[8 * t + 2 * e] = s.x;
+            v[8 * t + 2 * e + 1] = s.y;
           }
         }
-        float ps[4] = {0.f, 0.f, 0.f, 0.f}, pq[4] = {0.f, 0.f, 0.f, 0.f};   // short chains
+        float2 ps[2] = {make_float2(0.f, 0.f), make_float2(0.f, 0.f)};   // packed, short chains
+        float2 pq[2] = {make_float2(0.f, 0.f), make_float2(0.f, 0.f)};
 #pragma unroll
-        for (int t = 0; t < 32; ++t) {
-          ps[t & 3] += v[t];
-          pq[t & 3] = fmaf(v[t], v[t], pq[t & 3]);
+        for (int t = 0; t < 32; t += 2) {
+          const float2 vv = make_float2(v[t], v[t + 1]);
+          ps[(t >> 1) & 1] = fadd2(ps[(t >> 1) & 1], vv);
+          pq[(t >> 1) & 1] = ffma2(vv, vv, pq[(t >> 1) & 1]);
         }
-        sum += (ps[0] + ps[1]) + (ps[2] + ps[3]);
-        sumsq += (pq[0] + pq[1]) + (pq[2] + pq[3]);
+        sum += (ps[0].x + ps[0].y) + (ps[1].x + ps[1].y);
+        sumsq += (pq[0].x + pq[0].y) + (pq[1].x + pq[1].y);
         tmem_st32(taddr, *reinterpret_cast<float(*)[32]>(v));
         __syncwarp();                             // every lane has read buffer b
         if (j + 2 < 4 && lane == 0) {
@@ -908,6 +913,7 @@ linear_ln_kernel(const __grid_constant__ CUtensorMap tmA, const __grid_constant_
                          (1.f / kLnN);
       const float rstd = rsqrtf(fmaxf(ex2m - mean * mean, 0.f) + eps);
       const float nmr = -mean * rstd;             // (z - mean) rstd = fma(z, rstd, nmr)
+      const float2 rs2 = make_float2(rstd, rstd), nm2 = make_float2(nmr, nmr);
       // pass 2: normalise, bf16, TMA store; each half is released to the MMA as soon as its
       // last read is done
 #pragma unroll 1
@@ -929,10 +935,14 @@ linear_ln_kernel(const __grid_constant__ CUtensorMap tmA, const __grid_constant_
 #pragma unroll
         for (int t = 0; t < 8; ++t) {
           const float4 gg = g4[t], ee = e4[t];
-          y[4 * t + 0] = pad ? 0.f : fmaf(fmaf(y[4 * t + 0], rstd, nmr), gg.x, ee.x);
-          y[4 * t + 1] = pad ? 0.f : fmaf(fmaf(y[4 * t + 1], rstd, nmr), gg.y, ee.y);
-          y[4 * t + 2] = pad ? 0.f : fmaf(fmaf(y[4 * t + 2], rstd, nmr), gg.z, ee.z);
-          y[4 * t + 3] = pad ? 0.f : fmaf(fmaf(y[4 * t + 3], rstd, nmr), gg.w, ee.w);
+          const float2 y0 = ffma2(ffma2(make_float2(y[4 * t + 0], y[4 * t + 1]), rs2, nm2),
+                                  make_float2(gg.x, gg.y), make_float2(ee.x, ee.y));
+          const float2 y1 = ffma2(ffma2(make_float2(y[4 * t + 2], y[4 * t + 3]), rs2, nm2),
+                                  make_float2(gg.z, gg.w), make_float2(ee.z, ee.w));
+          y[4 * t + 0] = pad ? 0.f : y0.x;
+          y[4 * t + 1] = pad ? 0.f : y0.y;
+          y[4 * t + 2] = pad ? 0.f : y1.x;
+          y[4 * t + 3] = pad ? 0.f : y1.y;
         }
         if (lane == 0) bulk_wait_read<1>();       // the store that last used `buf` has read it
         __syncwarp();
@@ -1210,10 +1220,12 @@ linear_lnc_kernel(const __grid_constant__ CUtensorMap tmA, const __grid_constant
 #pragma unroll
         for (int t = 0; t < 8; ++t) {
           const float4 bb = __ldg(b4 + t);
-          v[4 * t + 0] += bb.x;
-          v[4 * t + 1] += bb.y;
-          v[4 * t + 2] += bb.z;
-          v[4 * t + 3] += bb.w;
+          const float2 s0 = fadd2(make_float2(v[4 * t + 0], v[4 * t + 1]), make_float2(bb.x, bb.y));
+          const float2 s1 = fadd2(make_float2(v[4 * t + 2], v[4 * t + 3]), make_float2(bb.z, bb.w));
+          v[4 * t + 0] = s0.x;
+          v[4 * t + 1] = s0.y;
+          v[4 * t + 2] = s1.x;
+          v[4 * t + 3] = s1.y;
         }
         mbar_wait(&my_rbar[j], rphase);
         const uint32_t buf = bufs + j * kStageBufBytes;
@@ -1224,18 +1236,21 @@ linear_lnc_kernel(const __grid_constant__ CUtensorMap tmA, const __grid_constant
 #pragma unroll
           for (int e = 0; e < 4; ++e) {
             const float2 f = __bfloat1622float2(hh[e]);
-            v[8 * t + 2 * e] += f.x;
-            v[8 * t + 2 * e + 1] += f.y;
+            const float2 s = fadd2(make_float2(v[8 * t + 2 * e], v[8 * t + 2 * e + 1]), f);
+            v[8 * t + 2 * e] = s.x;
+            v[8 * t + 2 * e + 1] = s.y;
           }
         }
-        float ps[4] = {0.f, 0.f, 0.f, 0.f}, pq[4] = {0.f, 0.f, 0.f, 0.f};   // short chains
+        float2 ps[2] = {make_float2(0.f, 0.f), make_float2(0.f, 0.f)};   // packed, short chains
+        float2 pq[2] = {make_float2(0.f, 0.f), make_float2(0.f, 0.f)};
 #pragma unroll
-        for (int t = 0; t < 32; ++t) {
-          ps[t & 3] += v[t];
-          pq[t & 3] = fmaf(v[t], v[t], pq[t & 3]);
+        for (int t = 0; t < 32; t += 2) {
+          const float2 vv = make_float2(v[t], v[t + 1]);
+          ps[(t >> 1) & 1] = fadd2(ps[(t >> 1) & 1], vv);
+          pq[(t >> 1) & 1] = ffma2(vv, vv, pq[(t >> 1) & 1]);
         }
-        sum += (ps[0] + ps[1]) + (ps[2] + ps[3]);
-        sumsq += (pq[0] + pq[1]) + (pq[2] + pq[3]);
+        sum += (ps[0].x + ps[0].y) + (ps[1].x + ps[1].y);
+        sumsq += (pq[0].x + pq[0].y) + (pq[1].x + pq[1].y);
         tmem_st32(tbase + 32 * j, *reinterpret_cast<float(*)[32]>(v));
       }
       rphase ^= 1;
@@ -1268,6 +1283,7 @@ linear_lnc_kernel(const __grid_constant__ CUtensorMap tmA, const __grid_constant
       const float mean = s1 * kInvN;
       const float rstd = rsqrtf(fmaxf(s2 * kInvN - mean * mean, 0.f) + eps);
       const float nmr = -mean * rstd;             // (z - mean) rstd = fma(z, rstd, nmr)
+      const float2 rs2 = make_float2(rstd, rstd), nm2 = make_float2(nmr, nmr);
       // pass 2: normalise -> bf16 -> staging (the residual chunks are consumed) -> TMA store
 #pragma unroll 1
       for (int j = 0; j < kLncChunks; ++j) {
@@ -1286,10 +1302,14 @@ linear_lnc_kernel(const __grid_constant__ CUtensorMap tmA, const __grid_constant
 #pragma unroll
         for (int t = 0; t < 8; ++t) {
           const float4 gg = __ldg(g4 + t), ee = __ldg(e4 + t);
-          y[4 * t + 0] = pad ? 0.f : fmaf(fmaf(y[4 * t + 0], rstd, nmr), gg.x, ee.x);
-          y[4 * t + 1] = pad ? 0.f : fmaf(fmaf(y[4 * t + 1], rstd, nmr), gg.y, ee.y);
-          y[4 * t + 2] = pad ? 0.f : fmaf(fmaf(y[4 * t + 2], rstd, nmr), gg.z, ee.z);
-          y[4 * t + 3] = pad ? 0.f : fmaf(fmaf(y[4 * t + 3], rstd, nmr), gg.w, ee.w);
+          const float2 y0 = ffma2(ffma2(make_float2(y[4 * t + 0], y[4 * t + 1]), rs2, nm2),
+                                  make_float2(gg.x, gg.y), make_float2(ee.x, ee.y));
+          const float2 y1 = ffma2(ffma2(make_float2(y[4 * t + 2], y[4 * t + 3]), rs2, nm2),
+                                  make_float2(gg.z, gg.w), make_float2(ee.z, ee.w));
+          y[4 * t + 0] = pad ? 0.f : y0.x;
+          y[4 * t + 1] = pad ? 0.f : y0.y;
+          y[4 * t + 2] = pad ? 0.f : y1.x;
+          y[4 * t + 3] = pad ? 0.f : y1.y;
         }
         const uint32_t buf = bufs + j * kStageBufBytes;
 #pragma unroll
@@ -1494,10 +1514,12 @@ linear_lng_kernel(const __grid_constant__ CUtensorMap tmA, const __grid_constant
 #pragma unroll
         for (int tt = 0; tt < 8; ++tt) {
           const float4 bb = __ldg(b4 + tt);
-          v[4 * tt + 0] += bb.x;
-          v[4 * tt + 1] += bb.y;
-          v[4 * tt + 2] += bb.z;
-          v[4 * tt + 3] += bb.w;
+          const float2 s0 = fadd2(make_float2(v[4 * tt + 0], v[4 * tt + 1]), make_float2(bb.x, bb.y));
+          const float2 s1 = fadd2(make_float2(v[4 * tt + 2], v[4 * tt + 3]), make_float2(bb.z, bb.w));
+          v[4 * tt + 0] = s0.x;
+          v[4 * tt + 1] = s0.y;
+          v[4 * tt + 2] = s1.x;
+          v[4 * tt + 3] = s1.y;
         }
         mbar_wait(&my_rbar[j], rphase);
         const uint32_t buf = bufs + j * kStageBufBytes;
@@ -1508,18 +1530,21 @@ linear_lng_kernel(const __grid_constant__ CUtensorMap tmA, const __grid_constant
 #pragma unroll
           for (int e = 0; e < 4; ++e) {
             const float2 f = __bfloat1622float2(hh[e]);
-            v[8 * tt + 2 * e] += f.x;
-            v[8 * tt + 2 * e + 1] += f.y;
+            const float2 s = fadd2(make_float2(v[8 * tt + 2 * e], v[8 * tt + 2 * e + 1]), f);
+            v[8 * tt + 2 * e] = s.x;
+            v[8 * tt + 2 * e + 1] = s.y;
           }
         }
-        float ps[4] = {0.f, 0.f, 0.f, 0.f}, pq[4] = {0.f, 0.f, 0.f, 0.f};   // short chains
+        float2 ps[2] = {make_float2(0.f, 0.f), make_float2(0.f, 0.f)};   // packed, short chains
+        float2 pq[2] = {make_float2(0.f, 0.f), make_float2(0.f, 0.f)};
 #pragma unroll
-        for (int tt = 0; tt < 32; ++tt) {
-          ps[tt & 3] += v[tt];
-          pq[tt & 3] = fmaf(v[tt], v[tt], pq[tt & 3]);
+        for (int tt = 0; tt < 32; tt += 2) {
+          const float2 vv = make_float2(v[tt], v[tt + 1]);
+          ps[(tt >> 1) & 1] = fadd2(ps[(tt >> 1) & 1], vv);
+          pq[(tt >> 1) & 1] = ffma2(vv, vv, pq[(tt >> 1) & 1]);
         }
-        sum += (ps[0] + ps[1]) + (ps[2] + ps[3]);
-        sumsq += (pq[0] + pq[1]) + (pq[2] + pq[3]);
+        sum += (ps[0].x + ps[0].y) + (ps[1].x + ps[1].y);
+        sumsq += (pq[0].x + pq[0].y) + (pq[1].x + pq[1].y);
         tmem_st32(tbase + 32 * j, *reinterpret_cast<float(*)[32]>(v));
       }
       rphase ^= 1;
@@ -1556,6 +1581,7 @@ linear_lng_kernel(const __grid_constant__ CUtensorMap tmA, const __grid_constant
       const float mean = s1 * kInvN;
       const float rstd = rsqrtf(fmaxf(s2 * kInvN - mean * mean, 0.f) + eps);
       const float nmr = -mean * rstd;             // (z - mean) rstd = fma(z, rstd, nmr)
+      const float2 rs2 = make_float2(rstd, rstd), nm2 = make_float2(nmr, nmr);
 #ifdef TCB_LN_PROBE
       long long td = clock64();
       e_x += td - tc2;
@@ -1578,10 +1604,14 @@ linear_lng_kernel(const __grid_constant__ CUtensorMap tmA, const __grid_constant
 #pragma unroll
         for (int tt = 0; tt < 8; ++tt) {
           const float4 gg = __ldg(g4 + tt), ee = __ldg(e4 + tt);
-          y[4 * tt + 0] = pad ? 0.f : fmaf(fmaf(y[4 * tt + 0], rstd, nmr), gg.x, ee.x);
-          y[4 * tt + 1] = pad ? 0.f : fmaf(fmaf(y[4 * tt + 1], rstd, nmr), gg.y, ee.y);
-          y[4 * tt + 2] = pad ? 0.f : fmaf(fmaf(y[4 * tt + 2], rstd, nmr), gg.z, ee.z);
-          y[4 * tt + 3] = pad ? 0.f : fmaf(fmaf(y[4 * tt + 3], rstd, nmr), gg.w, ee.w);
+          const float2 y0 = ffma2(ffma2(make_float2(y[4 * tt + 0], y[4 * tt + 1]), rs2, nm2),
+                                  make_float2(gg.x, gg.y), make_float2(ee.x, ee.y));
+          const float2 y1 = ffma2(ffma2(make_float2(y[4 * tt + 2], y[4 * tt + 3]), rs2, nm2),
+                                  make_float2(gg.z, gg.w), make_float2(ee.z, ee.w));
+          y[4 * tt + 0] = pad ? 0.f : y0.x;
+          y[4 * tt + 1] = pad ? 0.f : y0.y;
+          y[4 * tt + 2] = pad ? 0.f : y1.x;
+          y[4 * tt + 3] = pad ? 0.f : y1.y;
         }
         const uint32_t buf = bufs + j * kStageBufBytes;
 #pragma unroll
