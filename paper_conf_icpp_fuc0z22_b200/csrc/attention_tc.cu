@@ -179,6 +179,22 @@ __device__ __forceinline__ float ex2(float x) {
   asm("ex2.approx.ftz.f32 %0, %1;" : "=f"(y) : "f"(x));
   return y;
 }
+// packed fp32x2 arithmetic (sm_100 FFMA2 / FADD2: two lanes of work per issue slot)
+__device__ __forceinline__ float2 ffma2(float2 a, float2 b, float2 c) {
+  unsigned long long r;
+  asm("fma.rn.f32x2 %0, %1, %2, %3;"
+      : "=l"(r)
+      : "l"(*reinterpret_cast<unsigned long long*>(&a)), "l"(*reinterpret_cast<unsigned long long*>(&b)),
+        "l"(*reinterpret_cast<unsigned long long*>(&c)));
+  return *reinterpret_cast<float2*>(&r);
+}
+__device__ __forceinline__ float2 fadd2(float2 a, float2 b) {
+  unsigned long long r;
+  asm("add.rn.f32x2 %0, %1, %2;"
+      : "=l"(r)
+      : "l"(*reinterpret_cast<unsigned long long*>(&a)), "l"(*reinterpret_cast<unsigned long long*>(&b)));
+  return *reinterpret_cast<float2*>(&r);
+}
 // K-major operand, rows of 128 B, 128B swizzle, 8-row groups 1024 B apart (SBO).
 __device__ __forceinline__ uint64_t desc_kmajor(uint32_t saddr) {
   return static_cast<uint64_t>((saddr & 0x3FFFFu) >> 4) | (static_cast<uint64_t>(1) << 16) |
@@ -634,7 +650,9 @@ attn_tc_kernel(const __grid_constant__ CUtensorMap tmQKV, const int32_t* __restr
         p_pempty += t5 - t4;
 #endif
         const uint32_t prow = sP + b * kPBytes + half * kTileBytes + row * 128;
-        float lp[4] = {0.f, 0.f, 0.f, 0.f};    // independent partial row sums
+        // independent partial row sums, packed pairs (FFMA2 / FADD2 on sm_100)
+        float2 lp[2] = {make_float2(0.f, 0.f), make_float2(0.f, 0.f)};
+        const float2 sc2 = make_float2(scale_log2, scale_log2), off2 = make_float2(off, off);
 #pragma unroll
         for (int cch = 0; cch < 8; ++cch) {
           uint32_t w4[4] = {0u, 0u, 0u, 0u};
@@ -643,10 +661,11 @@ attn_tc_kernel(const __grid_constant__ CUtensorMap tmQKV, const int32_t* __restr
             for (int e = 0; e < 4; ++e) {
               const int j = cch * 8 + 2 * e;
               // masked scores are -inf: 2^-inf = 0 exactly
-              const float p0 = ex2(fmaf(__uint_as_float(sr[j]), scale_log2, off));
-              const float p1 = ex2(fmaf(__uint_as_float(sr[j + 1]), scale_log2, off));
-              lp[e] += p0 + p1;
-              __nv_bfloat162 hv = __floats2bfloat162_rn(p0, p1);
+              const float2 x = ffma2(make_float2(__uint_as_float(sr[j]), __uint_as_float(sr[j + 1])),
+                                     sc2, off2);
+              const float2 pp = make_float2(ex2(x.x), ex2(x.y));
+              lp[e & 1] = fadd2(lp[e & 1], pp);
+              __nv_bfloat162 hv = __floats2bfloat162_rn(pp.x, pp.y);
               w4[e] = *reinterpret_cast<uint32_t*>(&hv);
             }
           }
@@ -655,7 +674,7 @@ attn_tc_kernel(const __grid_constant__ CUtensorMap tmQKV, const int32_t* __restr
                        "r"(w4[1]), "r"(w4[2]), "r"(w4[3])
                        : "memory");
         }
-        l += (lp[0] + lp[1]) + (lp[2] + lp[3]);
+        l += (lp[0].x + lp[0].y) + (lp[1].x + lp[1].y);
 #ifdef TCB_ATTN_PROBE
         p_exp += clock64() - t5;
 #endif
