@@ -513,10 +513,14 @@ linear_tc_kernel(const __grid_constant__ CUtensorMap tmA, const __grid_constant_
 #pragma unroll
         for (int t = 0; t < 8; ++t) {
           const float4 bb = __ldg(b4 + t);
-          v[4 * t + 0] = __uint_as_float(r[4 * t + 0]) + bb.x;
-          v[4 * t + 1] = __uint_as_float(r[4 * t + 1]) + bb.y;
-          v[4 * t + 2] = __uint_as_float(r[4 * t + 2]) + bb.z;
-          v[4 * t + 3] = __uint_as_float(r[4 * t + 3]) + bb.w;
+          const float2 s0 = fadd2(make_float2(__uint_as_float(r[4 * t + 0]), __uint_as_float(r[4 * t + 1])),
+                                  make_float2(bb.x, bb.y));
+          const float2 s1 = fadd2(make_float2(__uint_as_float(r[4 * t + 2]), __uint_as_float(r[4 * t + 3])),
+                                  make_float2(bb.z, bb.w));
+          v[4 * t + 0] = s0.x;
+          v[4 * t + 1] = s0.y;
+          v[4 * t + 2] = s1.x;
+          v[4 * t + 3] = s1.y;
         }
         if constexpr (EPI == TCB_EPI_BIAS_GELU) {
 #pragma unroll
@@ -536,9 +540,10 @@ linear_tc_kernel(const __grid_constant__ CUtensorMap tmA, const __grid_constant_
             const __nv_bfloat162* h = reinterpret_cast<const __nv_bfloat162*>(&x);
 #pragma unroll
             for (int e = 0; e < 4; ++e) {
-              const float2 f = __bfloat1622float2(h[e]);
-              v[8 * t + 2 * e] += f.x;
-              v[8 * t + 2 * e + 1] += f.y;
+              const float2 f = fadd2(make_float2(v[8 * t + 2 * e], v[8 * t + 2 * e + 1]),
+                                     __bfloat1622float2(h[e]));
+              v[8 * t + 2 * e] = f.x;
+              v[8 * t + 2 * e + 1] = f.y;
             }
           }
         }
