@@ -191,3 +191,49 @@ def test_empty_and_tiny_batches():
     ref = oracle.run(model, w, wl.weight_names(model), lengths, ids, 8)
     e = np.max(np.abs(out - ref["out"])) / np.max(np.abs(ref["out"]))
     assert e <= TOL["bf16"]
+
+
+def test_internal_graph_replay_with_new_plan_contents():
+    """tcb_encoder_forward's own graph cache (include/tcb.h): captured with plan A, replayed
+    for plan B written into the same device buffers (same B x L) -- the kernels read every
+    plan-specific value from the device segment table -- equals a fresh capture for B and the
+    directly launched forward (TCB_NO_FWD_GRAPH semantics via a caller capture)."""
+    wlc = wl.WORKLOADS["c2"]
+    model = wlc.model
+    lengths_a, ids_a, w = wl.workload_inputs("c2", rows=8)
+    lengths_b = wl.lengths_filling(wlc.lengths, 8, wlc.row_len, 123)
+    ids_b = wl.draw_token_ids(int(lengths_b.sum()), model.vocab, 124)
+    enc = tcb.Encoder(model, w, wl.weight_names(model))
+    pa = tcb.tcb_pack(lengths_a, wlc.row_len, 8)
+    pb = tcb.tcb_pack(lengths_b, wlc.row_len, 8)
+    assert pa.num_slots == pb.num_slots
+    words = max(pa.segtab().size, pb.segtab().size)
+    seg = torch.zeros(words, dtype=torch.int32, device="cuda")
+    ids = torch.zeros(max(len(ids_a), len(ids_b)), dtype=torch.int32, device="cuda")
+    rows = enc.alloc_rows(pa.num_slots)
+    s = torch.cuda.Stream()
+
+    def load(plan, tok):
+        st = torch.from_numpy(plan.segtab())
+        seg[:st.numel()].copy_(st.cuda())
+        ids[:len(tok)].copy_(torch.from_numpy(tok).cuda())
+
+    load(pa, ids_a)
+    enc.encoder_forward(pa, seg, ids, rows, stream=s)          # captures the graph (plan A)
+    s.synchronize()
+    load(pb, ids_b)
+    enc.encoder_forward(pb, seg, ids, rows, stream=s)          # replays it for plan B
+    s.synchronize()
+    got = rows.clone()
+    rows2 = enc.alloc_rows(pb.num_slots)                        # new buffers: new capture
+    enc.encoder_forward(pb, seg, ids, rows2, stream=s)
+    s.synchronize()
+    assert torch.equal(got, rows2)
+    # directly launched kernels (inside a caller's capture the library does not use its cache)
+    rows3 = enc.alloc_rows(pb.num_slots)
+    g = torch.cuda.CUDAGraph()
+    with torch.cuda.graph(g, stream=s):
+        enc.encoder_forward(pb, seg, ids, rows3, stream=s)
+    g.replay()
+    torch.cuda.synchronize()
+    assert torch.equal(got, rows3)
