@@ -594,9 +594,14 @@ attn_tc_kernel(const __grid_constant__ CUtensorMap tmQKV, const int32_t* __restr
             for (int j = 32 * gi; j < 32 * gi + 32; j += 2)
               mxp[(j >> 1) & 7] = fmax3(mxp[(j >> 1) & 7], __uint_as_float(sr[j]), __uint_as_float(sr[j + 1]));
           } else {
+            // valid keys of this row in the group as a bit mask: one bit test per score
+            const int lo = min(max(jlo - 32 * gi, 0), 32), hi = min(max(jhi - 32 * gi, 0), 32);
+            const uint32_t below_hi = hi >= 32 ? 0xffffffffu : (1u << hi) - 1u;
+            const uint32_t from_lo = lo >= 32 ? 0u : ~((1u << lo) - 1u);   // no shift by 32
+            const uint32_t vm = below_hi & from_lo;
 #pragma unroll
             for (int j = 32 * gi; j < 32 * gi + 32; ++j) {
-              const float v = (j >= jlo && j < jhi) ? __uint_as_float(sr[j]) : -INFINITY;
+              const float v = (vm & (1u << (j - 32 * gi))) ? __uint_as_float(sr[j]) : -INFINITY;
               sr[j] = __float_as_uint(v);
               mxp[j & 7] = fmaxf(mxp[j & 7], v);
             }
