@@ -600,10 +600,12 @@ attn_tc_kernel(const __grid_constant__ CUtensorMap tmQKV, const int32_t* __restr
             const uint32_t from_lo = lo >= 32 ? 0u : ~((1u << lo) - 1u);   // no shift by 32
             const uint32_t vm = below_hi & from_lo;
 #pragma unroll
-            for (int j = 32 * gi; j < 32 * gi + 32; ++j) {
-              const float v = (vm & (1u << (j - 32 * gi))) ? __uint_as_float(sr[j]) : -INFINITY;
-              sr[j] = __float_as_uint(v);
-              mxp[j & 7] = fmaxf(mxp[j & 7], v);
+            for (int j = 32 * gi; j < 32 * gi + 32; j += 2) {
+              const float v0 = (vm & (1u << (j - 32 * gi))) ? __uint_as_float(sr[j]) : -INFINITY;
+              const float v1 = (vm & (2u << (j - 32 * gi))) ? __uint_as_float(sr[j + 1]) : -INFINITY;
+              sr[j] = __float_as_uint(v0);
+              sr[j + 1] = __float_as_uint(v1);
+              mxp[(j >> 1) & 7] = fmax3(mxp[(j >> 1) & 7], v0, v1);
             }
           }
         }
