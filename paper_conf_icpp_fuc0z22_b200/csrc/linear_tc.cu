@@ -919,6 +919,7 @@ linear_ln_kernel(const __grid_constant__ CUtensorMap tmA, const __grid_constant_
       const float rstd = rsqrtf(fmaxf(ex2m - mean * mean, 0.f) + eps);
       const float nmr = -mean * rstd;             // (z - mean) rstd = fma(z, rstd, nmr)
       const float2 rs2 = make_float2(rstd, rstd), nm2 = make_float2(nmr, nmr);
+      const float2 keep2 = pad ? make_float2(0.f, 0.f) : make_float2(1.f, 1.f);
       // pass 2: normalise, bf16, TMA store; each half is released to the MMA as soon as its
       // last read is done
 #pragma unroll 1
@@ -944,10 +945,11 @@ linear_ln_kernel(const __grid_constant__ CUtensorMap tmA, const __grid_constant_
                                   make_float2(gg.x, gg.y), make_float2(ee.x, ee.y));
           const float2 y1 = ffma2(ffma2(make_float2(y[4 * t + 2], y[4 * t + 3]), rs2, nm2),
                                   make_float2(gg.z, gg.w), make_float2(ee.z, ee.w));
-          y[4 * t + 0] = pad ? 0.f : y0.x;
-          y[4 * t + 1] = pad ? 0.f : y0.y;
-          y[4 * t + 2] = pad ? 0.f : y1.x;
-          y[4 * t + 3] = pad ? 0.f : y1.y;
+          const float2 z0 = fmul2(y0, keep2), z1 = fmul2(y1, keep2);   // pad rows -> 0
+          y[4 * t + 0] = z0.x;
+          y[4 * t + 1] = z0.y;
+          y[4 * t + 2] = z1.x;
+          y[4 * t + 3] = z1.y;
         }
         if (lane == 0) bulk_wait_read<1>();       // the store that last used `buf` has read it
         __syncwarp();
@@ -1289,6 +1291,7 @@ linear_lnc_kernel(const __grid_constant__ CUtensorMap tmA, const __grid_constant
       const float rstd = rsqrtf(fmaxf(s2 * kInvN - mean * mean, 0.f) + eps);
       const float nmr = -mean * rstd;             // (z - mean) rstd = fma(z, rstd, nmr)
       const float2 rs2 = make_float2(rstd, rstd), nm2 = make_float2(nmr, nmr);
+      const float2 keep2 = pad ? make_float2(0.f, 0.f) : make_float2(1.f, 1.f);
       // pass 2: normalise -> bf16 -> staging (the residual chunks are consumed) -> TMA store
 #pragma unroll 1
       for (int j = 0; j < kLncChunks; ++j) {
@@ -1311,10 +1314,11 @@ linear_lnc_kernel(const __grid_constant__ CUtensorMap tmA, const __grid_constant
                                   make_float2(gg.x, gg.y), make_float2(ee.x, ee.y));
           const float2 y1 = ffma2(ffma2(make_float2(y[4 * t + 2], y[4 * t + 3]), rs2, nm2),
                                   make_float2(gg.z, gg.w), make_float2(ee.z, ee.w));
-          y[4 * t + 0] = pad ? 0.f : y0.x;
-          y[4 * t + 1] = pad ? 0.f : y0.y;
-          y[4 * t + 2] = pad ? 0.f : y1.x;
-          y[4 * t + 3] = pad ? 0.f : y1.y;
+          const float2 z0 = fmul2(y0, keep2), z1 = fmul2(y1, keep2);   // pad rows -> 0
+          y[4 * t + 0] = z0.x;
+          y[4 * t + 1] = z0.y;
+          y[4 * t + 2] = z1.x;
+          y[4 * t + 3] = z1.y;
         }
         const uint32_t buf = bufs + j * kStageBufBytes;
 #pragma unroll
@@ -1587,6 +1591,7 @@ linear_lng_kernel(const __grid_constant__ CUtensorMap tmA, const __grid_constant
       const float rstd = rsqrtf(fmaxf(s2 * kInvN - mean * mean, 0.f) + eps);
       const float nmr = -mean * rstd;             // (z - mean) rstd = fma(z, rstd, nmr)
       const float2 rs2 = make_float2(rstd, rstd), nm2 = make_float2(nmr, nmr);
+      const float2 keep2 = pad ? make_float2(0.f, 0.f) : make_float2(1.f, 1.f);
 #ifdef TCB_LN_PROBE
       long long td = clock64();
       e_x += td - tc2;
@@ -1613,10 +1618,11 @@ linear_lng_kernel(const __grid_constant__ CUtensorMap tmA, const __grid_constant
                                   make_float2(gg.x, gg.y), make_float2(ee.x, ee.y));
           const float2 y1 = ffma2(ffma2(make_float2(y[4 * tt + 2], y[4 * tt + 3]), rs2, nm2),
                                   make_float2(gg.z, gg.w), make_float2(ee.z, ee.w));
-          y[4 * tt + 0] = pad ? 0.f : y0.x;
-          y[4 * tt + 1] = pad ? 0.f : y0.y;
-          y[4 * tt + 2] = pad ? 0.f : y1.x;
-          y[4 * tt + 3] = pad ? 0.f : y1.y;
+          const float2 z0 = fmul2(y0, keep2), z1 = fmul2(y1, keep2);   // pad rows -> 0
+          y[4 * tt + 0] = z0.x;
+          y[4 * tt + 1] = z0.y;
+          y[4 * tt + 2] = z1.x;
+          y[4 * tt + 3] = z1.y;
         }
         const uint32_t buf = bufs + j * kStageBufBytes;
 #pragma unroll
