@@ -260,44 +260,70 @@ layernorm_kernel(int64_t rows, int d, const T* __restrict__ Z, const float* __re
   }
 }
 
-// unpack: one CTA per (batch row, 64-slot chunk); the part of each segment inside the
-// chunk is a contiguous block in both the rows buffer and the request-order output, so the
-// CTA copies it with 16-byte vectors (4 independent loads in flight per thread).
+// unpack: one CTA per (batch row, kRowChunk-slot chunk).  The chunk's slots are contiguous in
+// the rows buffer, so every thread first issues its 16-byte loads of them (independent of the
+// segment layout), and only then resolves, one thread per slot, where each slot goes in the
+// request-order output (binary search over the row's segment records staged in smem): the
+// metadata's dependent loads overlap the data loads instead of preceding them.  Pad slots are
+// loaded but not stored.
 __global__ void __launch_bounds__(kWarpsPerBlock * 32)
 unpack_kernel(const int4* __restrict__ segtab, int row_len, int row_bytes_per_slot,
               const uint8_t* __restrict__ rows, uint8_t* __restrict__ out) {
+  constexpr int U = 4;
+  extern __shared__ int4 recs[];
+  __shared__ int64_t s_dst[kRowChunk];   // output token index of each slot of the chunk, -1 at pad
   const int row = blockIdx.x;
+  const int jc0 = static_cast<int>(blockIdx.y) * kRowChunk;
+  const int nslots = min(kRowChunk, row_len - jc0);
+  const int64_t c0 = static_cast<int64_t>(row) * row_len + jc0;
+  const int vps = row_bytes_per_slot / 16;             // 16-byte vectors per slot
+  const int nvec = nslots * vps;
+  const uint4* src = reinterpret_cast<const uint4*>(rows + c0 * row_bytes_per_slot);
+  uint4* dst = reinterpret_cast<uint4*>(out);
   pdl_wait();
   pdl_trigger();
+  uint4 t[U];
+#pragma unroll
+  for (int u = 0; u < U; ++u) {
+    const int i = threadIdx.x + u * blockDim.x;
+    if (i < nvec) t[u] = __ldg(src + i);
+  }
   const int S = segtab[0].x;
   const int* row_first = reinterpret_cast<const int*>(segtab + 1 + S);
-  const int f = __ldg(&row_first[row]), e = __ldg(&row_first[row + 1]);
-  const int64_t c0 = static_cast<int64_t>(row) * row_len + blockIdx.y * kRowChunk;
-  const int64_t c1 = min(c0 + kRowChunk, static_cast<int64_t>(row + 1) * row_len);
-  constexpr int U = 4;
-  for (int sg = f; sg < e; ++sg) {
-    const int4 rec = __ldg(&segtab[1 + sg]);
-    const int64_t a0 = rec.x > c0 ? static_cast<int64_t>(rec.x) : c0;
-    const int64_t a1 = rec.x + rec.y < c1 ? static_cast<int64_t>(rec.x + rec.y) : c1;
-    if (a0 >= a1) continue;
-    const int64_t nvec = (a1 - a0) * row_bytes_per_slot / 16;
-    const uint4* src = reinterpret_cast<const uint4*>(rows + a0 * row_bytes_per_slot);
-    uint4* dst = reinterpret_cast<uint4*>(out + (rec.z + (a0 - rec.x)) * row_bytes_per_slot);
-    for (int64_t i0 = threadIdx.x; i0 < nvec; i0 += static_cast<int64_t>(blockDim.x) * U) {
-      uint4 t[U];
+  const int f = __ldg(&row_first[row]);
+  const int nseg = __ldg(&row_first[row + 1]) - f;
+  for (int i = threadIdx.x; i < nseg; i += blockDim.x) recs[i] = __ldg(&segtab[1 + f + i]);
+  __syncthreads();
+  if (threadIdx.x < nslots) {
+    const int64_t slot = c0 + threadIdx.x;
+    int lo = 0, hi = nseg - 1, k = -1;                 // last record with start <= slot
+    while (lo <= hi) {
+      const int mid = (lo + hi) >> 1;
+      if (recs[mid].x <= slot) { k = mid; lo = mid + 1; } else { hi = mid - 1; }
+    }
+    int64_t o = -1;
+    if (k >= 0 && slot < recs[k].x + recs[k].y) o = recs[k].z + (slot - recs[k].x);
+    s_dst[threadIdx.x] = o;
+  }
+  __syncthreads();
+  for (int i0 = threadIdx.x;;) {
 #pragma unroll
-      for (int u = 0; u < U; ++u) {
-        const int64_t i = i0 + static_cast<int64_t>(u) * blockDim.x;
-        if (i < nvec) t[u] = __ldg(src + i);
-      }
-#pragma unroll
-      for (int u = 0; u < U; ++u) {
-        const int64_t i = i0 + static_cast<int64_t>(u) * blockDim.x;
-        if (i < nvec) dst[i] = t[u];
+    for (int u = 0; u < U; ++u) {
+      const int i = i0 + u * blockDim.x;
+      if (i < nvec) {
+        const int j = i / vps;
+        const int64_t o = s_dst[j];
+        if (o >= 0) dst[o * vps + (i - j * vps)] = t[u];
       }
     }
+    i0 += U * blockDim.x;
+    if (i0 >= nvec) break;
+#pragma unroll
+    for (int u = 0; u < U; ++u) {
+      const int i = i0 + u * blockDim.x;
+      if (i < nvec) t[u] = __ldg(src + i);
+    }
   }
-  (void)row_len;
 }
 
 __global__ void pe_table_kernel(float* table, int max_pos, int d, int variant) {
@@ -385,7 +411,14 @@ cudaError_t launch_unpack(int dtype, const int4* segtab, int num_rows, int row_l
   if (num_rows == 0) return cudaSuccess;
   const int bytes_per_slot = d * (dtype == 0 ? 4 : 2);
   const dim3 grid(static_cast<unsigned>(num_rows), static_cast<unsigned>((row_len + kRowChunk - 1) / kRowChunk));
-  return launch_ex(unpack_kernel, grid, dim3(kWarpsPerBlock * 32), 0, s, 1, segtab, row_len,
+  // <= row_len segment records per row
+  const size_t smem = static_cast<size_t>(row_len) * sizeof(int4);
+  if (smem > 48 * 1024) {
+    const cudaError_t e = cudaFuncSetAttribute(unpack_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize,
+                                               static_cast<int>(smem));
+    if (e != cudaSuccess) return e;
+  }
+  return launch_ex(unpack_kernel, grid, dim3(kWarpsPerBlock * 32), smem, s, 1, segtab, row_len,
                    bytes_per_slot, static_cast<const uint8_t*>(rows), static_cast<uint8_t*>(out));
 }
 
