@@ -64,6 +64,7 @@ __device__ __forceinline__ float warp_sum(float v) {
 #define TCB_ROW_CHUNK 16
 #endif
 constexpr int kRowChunk = TCB_ROW_CHUNK;   // slots per CTA (64 measured slower: fewer CTAs in flight)
+static_assert(kRowChunk <= kWarpsPerBlock * 32, "one metadata thread per slot of a chunk");
 template <typename T, int NV>
 __global__ void __launch_bounds__(kWarpsPerBlock * 32) pack_embed_kernel(EmbedArgs a) {
   constexpr int V = Vec<T>::N;
@@ -91,32 +92,39 @@ __global__ void __launch_bounds__(kWarpsPerBlock * 32) pack_embed_kernel(EmbedAr
   const int d = a.d;
   const int nvec = d / V;
   const int64_t row0 = static_cast<int64_t>(row) * a.row_len;
-  const int j_end = min(a.row_len, static_cast<int>(blockIdx.y + 1) * kRowChunk);
-  for (int j = static_cast<int>(blockIdx.y) * kRowChunk + warp; j < j_end; j += kWarpsPerBlock) {
-    const int64_t slot = row0 + j;
-    T* x = reinterpret_cast<T*>(a.X) + slot * d;
-    // last record with start <= slot
-    int lo = 0, hi = nseg - 1, k = -1;
+  const int jc0 = static_cast<int>(blockIdx.y) * kRowChunk;
+  const int j_end = min(a.row_len, jc0 + kRowChunk);
+  // one thread per slot of the chunk resolves (segment, position, token id) -- every id load
+  // of the chunk in flight together -- and writes the slot metadata coalesced; the warps then
+  // wait on only the embedding-row load per slot
+  __shared__ int2 s_meta[kRowChunk];   // (position, token id); position -1 at pad
+  if (jc0 + static_cast<int>(threadIdx.x) < j_end) {
+    const int64_t slot = row0 + jc0 + threadIdx.x;
+    int lo = 0, hi = nseg - 1, k = -1;   // last record with start <= slot
     while (lo <= hi) {
       const int mid = (lo + hi) >> 1;
       if (row_recs[mid].x <= slot) { k = mid; lo = mid + 1; } else { hi = mid - 1; }
     }
-    const int4 rec = k >= 0 ? row_recs[k] : make_int4(0, 0, 0, 0);
-    if (k < 0 || slot >= rec.x + rec.y) {  // pad slot: zeros, segment -1, position -1 (R12)
+    int seg = -1, pos = -1, id = 0;      // pad slot: segment -1, position -1 (R12)
+    if (k >= 0 && slot < row_recs[k].x + row_recs[k].y) {
+      seg = f + k;
+      pos = static_cast<int>(slot - row_recs[k].x);      // restarts at 0 per request
+      id = __ldg(&a.ids[row_recs[k].z + pos]);
+    }
+    if (a.seg_ids) a.seg_ids[slot] = seg;
+    if (a.positions) a.positions[slot] = pos;
+    s_meta[threadIdx.x] = make_int2(pos, id);
+  }
+  __syncthreads();
+  for (int j = jc0 + warp; j < j_end; j += kWarpsPerBlock) {
+    const int64_t slot = row0 + j;
+    T* x = reinterpret_cast<T*>(a.X) + slot * d;
+    const int2 m = s_meta[j - jc0];
+    const int pos = m.x, id = m.y;
+    if (pos < 0) {                        // pad slot: zeros
       float z[V] = {};
       for (int i = lane; i < nvec; i += 32) Vec<T>::store(x + i * V, z);
-      if (lane == 0) {
-        if (a.seg_ids) a.seg_ids[slot] = -1;
-        if (a.positions) a.positions[slot] = -1;
-      }
       continue;
-    }
-    const int seg = f + k;
-    const int pos = static_cast<int>(slot - rec.x);           // restarts at 0 per request
-    const int id = __ldg(&a.ids[rec.z + pos]);
-    if (lane == 0) {
-      if (a.seg_ids) a.seg_ids[slot] = seg;
-      if (a.positions) a.positions[slot] = pos;
     }
     const T* e = reinterpret_cast<const T*>(a.tok_emb) + static_cast<int64_t>(id) * d;
     float v[NV][V];
