@@ -274,15 +274,23 @@ layernorm_kernel(int64_t rows, int d, const T* __restrict__ Z, const float* __re
 // request-order output (binary search over the row's segment records staged in smem): the
 // metadata's dependent loads overlap the data loads instead of preceding them.  Pad slots are
 // loaded but not stored.
+#ifndef TCB_UNPACK_CHUNK
+#define TCB_UNPACK_CHUNK 16
+#endif
+#ifndef TCB_UNPACK_U
+#define TCB_UNPACK_U 4
+#endif
+constexpr int kUnpackChunk = TCB_UNPACK_CHUNK;   // slots per CTA
+static_assert(kUnpackChunk <= kWarpsPerBlock * 32, "one lookup thread per slot of a chunk");
 __global__ void __launch_bounds__(kWarpsPerBlock * 32)
 unpack_kernel(const int4* __restrict__ segtab, int row_len, int row_bytes_per_slot,
               const uint8_t* __restrict__ rows, uint8_t* __restrict__ out) {
-  constexpr int U = 4;
+  constexpr int U = TCB_UNPACK_U;
   extern __shared__ int4 recs[];
-  __shared__ int64_t s_dst[kRowChunk];   // output token index of each slot of the chunk, -1 at pad
+  __shared__ int64_t s_dst[kUnpackChunk];   // output token index of each slot of the chunk, -1 at pad
   const int row = blockIdx.x;
-  const int jc0 = static_cast<int>(blockIdx.y) * kRowChunk;
-  const int nslots = min(kRowChunk, row_len - jc0);
+  const int jc0 = static_cast<int>(blockIdx.y) * kUnpackChunk;
+  const int nslots = min(kUnpackChunk, row_len - jc0);
   const int64_t c0 = static_cast<int64_t>(row) * row_len + jc0;
   const int vps = row_bytes_per_slot / 16;             // 16-byte vectors per slot
   const int nvec = nslots * vps;
@@ -418,7 +426,7 @@ cudaError_t launch_unpack(int dtype, const int4* segtab, int num_rows, int row_l
                           const void* rows, void* out, cudaStream_t s) {
   if (num_rows == 0) return cudaSuccess;
   const int bytes_per_slot = d * (dtype == 0 ? 4 : 2);
-  const dim3 grid(static_cast<unsigned>(num_rows), static_cast<unsigned>((row_len + kRowChunk - 1) / kRowChunk));
+  const dim3 grid(static_cast<unsigned>(num_rows), static_cast<unsigned>((row_len + kUnpackChunk - 1) / kUnpackChunk));
   // <= row_len segment records per row
   const size_t smem = static_cast<size_t>(row_len) * sizeof(int4);
   if (smem > 48 * 1024) {
