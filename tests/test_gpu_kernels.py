@@ -296,6 +296,39 @@ def test_pack_embed_metadata_bit_exact_and_values(mkey):
     assert np.all(np.abs(got - ref) <= tol * np.abs(ref) + (1e-6 if model.dtype == "fp32" else 1e-3))
 
 
+@pytest.mark.gpu
+@pytest.mark.parametrize("dtype,d,L,lengths", [
+    # fp32 d = 1024: 256 vectors per slot, a 16-slot chunk takes four load batches
+    ("fp32", 1024, 40, [5, 17, 3, 30, 1, 8, 37, 2]),
+    # bf16 d = 768, ragged last chunk of each row (40 = 2 x 16 + 8), pad slots
+    ("bf16", 768, 40, [36, 1, 20, 20, 9, 4]),
+    # row_len 4104: the row's segment records need > 48 KB of smem
+    ("bf16", 64, 4104, [4104, 1, 4099, 7, 2000, 2000, 64] + [1] * 3100),
+])
+def test_unpack_exact_shapes(dtype, d, L, lengths):
+    """a10: every request's tokens come back bit-exact and nothing else is written
+    (sentinel-filled output), across load batches, ragged chunks and large row records."""
+    model = small_model(dtype=dtype, d=d, h=d // 64, f=4 * d, max_pos=max(512, L))
+    w = wl.draw_weights(model, 1)
+    enc = tcb.Encoder(model, w, wl.weight_names(model))
+    lengths = np.array(lengths, np.int32)
+    plan = tcb.tcb_pack(lengths, L, 0)
+    segtab = _dev(plan.segtab())
+    tdt = torch.float32 if dtype == "fp32" else torch.bfloat16
+    rows = torch.randn(plan.num_slots, d, device="cuda").to(tdt)
+    T = int(lengths.sum())
+    out = torch.full((T + 3, d), 12345.0, device="cuda").to(tdt)
+    enc.unpack(plan, segtab, rows, out)
+    torch.cuda.synchronize()
+    a = plan.arrays()
+    cu = np.concatenate([[0], np.cumsum(lengths)])
+    r, o = rows.cpu(), out.cpu()
+    for s, req in enumerate(a["seg_req"]):
+        st = a["seg_start"][s]
+        assert torch.equal(o[cu[req]:cu[req + 1]], r[st:st + lengths[req]])
+    assert torch.all(o[T:] == 12345.0)
+
+
 def test_unpack_roundtrip_exact():
     model = small_model(dtype="bf16", d=128, h=2, f=256)
     w = wl.draw_weights(model, 1)
