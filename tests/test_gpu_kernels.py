@@ -268,12 +268,13 @@ def test_layernorm_bf16_vs_oracle(d):
     assert np.all(got[-5:] == 0)
 
 
-@pytest.mark.parametrize("mkey", ["toy", "transformer-base", "bert-base"])
-def test_pack_embed_metadata_bit_exact_and_values(mkey):
+@pytest.mark.parametrize("mkey,L", [("toy", 32), ("transformer-base", 128), ("bert-base", 128),
+                                    # ragged last 16-slot chunk of every row (40 = 2 x 16 + 8)
+                                    ("toy", 40), ("bert-base", 40)])
+def test_pack_embed_metadata_bit_exact_and_values(mkey, L):
     model = wl.MODELS[mkey]
     w = wl.draw_weights(model, 2)
     names = wl.weight_names(model)
-    L = 32 if mkey == "toy" else 128
     lengths = np.minimum(wl.draw_lengths("paracrawl", 90, 4), L).astype(np.int32)
     ids = wl.draw_token_ids(int(lengths.sum()), model.vocab, 5)
     enc = tcb.Encoder(model, w, names)
