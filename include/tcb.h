@@ -112,8 +112,12 @@ typedef struct {
   int64_t kv_tiles_dense;      /* num_rows * (row_len/128)^2: pure ConcatBatching's dense
                                   work; -1 when row_len % 128 != 0             */
   int64_t useful_score_elems;  /* sum_i l_i^2 over placed requests                          */
-  int64_t executed_score_elems;/* score elements the attention kernel evaluates (16x16
-                                  sub-blocks visited per 16-query warp group)              */
+  int64_t executed_score_elems;/* per head: S = QK^T elements the attention kernel computes
+                                  on the tensor cores (128-query x 128-key chunks over each
+                                  query block's key interval)                             */
+  int64_t softmax_score_elems; /* per head: of those, the elements that go through the
+                                  softmax exponentials (32-row x 32-key groups intersecting
+                                  the rows' own requests; dead groups are skipped)         */
 } tcb_plan_info;
 
 tcb_status tcb_plan_info_get(const tcb_plan* plan, tcb_plan_info* info);

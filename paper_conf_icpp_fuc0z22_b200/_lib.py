@@ -50,7 +50,8 @@ class PlanInfo(ctypes.Structure):
                 ("num_slots", ctypes.c_int64), ("qtiles", ctypes.c_int64),
                 ("kv_tiles_visited", ctypes.c_int64), ("kv_tiles_dense", ctypes.c_int64),
                 ("useful_score_elems", ctypes.c_int64),
-                ("executed_score_elems", ctypes.c_int64)]
+                ("executed_score_elems", ctypes.c_int64),
+                ("softmax_score_elems", ctypes.c_int64)]
 
     def as_dict(self):
         return {f: getattr(self, f) for f, _ in self._fields_}

@@ -99,7 +99,7 @@ tcb_status check_device() {
 constexpr size_t align256(size_t x) { return (x + 255) & ~static_cast<size_t>(255); }
 
 struct WsLayout {
-  size_t seg, qkv, att, z, x1, h, lnst, lncnt, lncnt_per_launch, total;
+  size_t seg, qkv, att, z, x1, h, lnst, lncnt, lncnt_per_launch, attn_cnt, total;
 };
 WsLayout ws_layout(const tcb_model_config& c, int64_t M) {
   const size_t es = c.dtype == 0 ? 4 : 2;
@@ -122,6 +122,10 @@ WsLayout ws_layout(const tcb_model_config& c, int64_t M) {
     L.lncnt_per_launch = align256(tcb::k::linear_ln_scratch_cnt_bytes(M));
     off += L.lncnt_per_launch * 2 * static_cast<size_t>(c.num_layers);
   }
+  // bf16 attention: one dynamic item counter per layer.  [lncnt, total) is the zeroed region
+  // (one memset per forward).
+  L.attn_cnt = off;
+  if (c.dtype == 1) off += align256(sizeof(int32_t) * static_cast<size_t>(c.num_layers));
   L.total = off;
   return L;
 }
@@ -192,16 +196,10 @@ namespace {
 
 enum { W_QKV = 0, B_QKV, W_O, B_O, LN1_G, LN1_B, W_1, B_1, W_2, B_2, LN2_G, LN2_B };
 
-// bf16 attention: tcgen05 kernel (attention_tc.cu); TCB_ATTN=mma selects the warp-level
-// mma.sync kernel (attention.cu) for A/B measurements.
+// bf16 attention: the tcgen05 kernel (attention_tc.cu).
 cudaError_t attention_bf16(int64_t M, int d, int heads, const void* qkv, const int32_t* seg,
-                           const int4* segtab, void* out, cudaStream_t s) {
-  static const bool use_mma = [] {
-    const char* v = std::getenv("TCB_ATTN");
-    return v && std::string(v) == "mma";
-  }();
-  return use_mma ? tcb::k::launch_attention_bf16(M, d, heads, qkv, seg, segtab, out, s)
-                 : tcb::k::launch_attention_bf16_tc(M, d, heads, qkv, seg, segtab, out, s);
+                           const int4* segtab, void* out, int* item_counter, cudaStream_t s) {
+  return tcb::k::launch_attention_bf16_tc(M, d, heads, qkv, seg, segtab, out, item_counter, s);
 }
 
 tcb_status embed_impl(const tcb_weights* w, const tcb_plan* plan, const int32_t* d_segtab,
@@ -389,6 +387,10 @@ tcb_status tcb_encoder_forward(const tcb_weights* wc, const tcb_plan* plan,
   if (!use_graph)
     return forward_impl(wc, plan, d_segtab, d_token_ids, d_rows, d_ws, ws_bytes, stream);
   if (tcb_status st = validate_plan_for(wc, plan)) return st;
+  // the same argument checks as forward_impl BEFORE a cache hit can replay (a graph captured
+  // for an all-pad plan with NULL ids must not serve a plan that has tokens)
+  if (plan->info.total_tokens > 0 && !d_token_ids)
+    return fail(TCB_ERR_INVALID_ARGUMENT, "tcb_encoder_forward: NULL device pointer");
   tcb_weights* w = const_cast<tcb_weights*>(wc);
   const int64_t M = plan->info.num_slots;
   std::lock_guard<std::mutex> gl(w->graph_mu);
@@ -483,6 +485,10 @@ tcb_status forward_impl(const tcb_weights* wc, const tcb_plan* plan, const int32
   if (tcb_status st = embed_impl(w, plan, d_segtab, d_token_ids, d_rows, seg, nullptr, s)) return st;
 
   if (c.dtype == 1) {
+    // Activation TMA descriptors: cached per weights handle for the last (rows, workspace, M)
+    // and COPIED into this call's locals under the lock, so concurrent forwards with other
+    // buffers (direct launches on other streams) never read a descriptor being rewritten.
+    CUtensorMap aX, aAtt, aX1, aH, cQkv, cZ, cH, cX, cX1;
     {
       std::lock_guard<std::mutex> g(w->mu);
       if (w->c_rows != d_rows || w->c_ws != d_ws || w->c_M != M) {
@@ -495,11 +501,17 @@ tcb_status forward_impl(const tcb_weights* wc, const tcb_plan* plan, const int32
                         make_gemm_c_map(&w->cZ, z, M, d) && make_gemm_c_map(&w->cH, hbuf, M, f) &&
                         make_gemm_c_map(&w->cX, d_rows, M, d) &&
                         make_gemm_c_map(&w->cX1, x1, M, d);
-        if (!ok) return fail(TCB_ERR_CUDA, "cuTensorMapEncodeTiled failed for an activation");
+        if (!ok) {
+          w->c_rows = w->c_ws = nullptr;         // a half-written set is never reused
+          w->c_M = -1;
+          return fail(TCB_ERR_CUDA, "cuTensorMapEncodeTiled failed for an activation");
+        }
         w->c_rows = d_rows;
         w->c_ws = d_ws;
         w->c_M = M;
       }
+      aX = w->aX; aAtt = w->aAtt; aX1 = w->aX1; aH = w->aH;
+      cQkv = w->cQkv; cZ = w->cZ; cH = w->cH; cX = w->cX; cX1 = w->cX1;
     }
     // bias + residual + LayerNorm fused into the W_O / FFN2 GEMMs (d = 512, 768, 1024: a
     // cluster of d / 256 CTA pairs owns complete rows); TCB_NO_LN_FUSION=1 forces the unfused
@@ -511,21 +523,22 @@ tcb_status forward_impl(const tcb_weights* wc, const tcb_plan* plan, const int32
       return L.lncnt_per_launch ? reinterpret_cast<int*>(ws + L.lncnt + L.lncnt_per_launch * launch)
                                 : nullptr;
     };
-    if (fuse_ln && L.lncnt_per_launch &&
-        cudaMemsetAsync(ws + L.lncnt, 0, L.lncnt_per_launch * 2 * c.num_layers, s) != cudaSuccess)
+    // LayerNorm-exchange counters and attention item counters: one reset per forward
+    if (cudaMemsetAsync(ws + L.lncnt, 0, L.total - L.lncnt, s) != cudaSuccess)
       return fail(TCB_ERR_CUDA, "tcb_encoder_forward: counter reset failed");
+    int* attn_cnt = reinterpret_cast<int*>(ws + L.attn_cnt);
     for (int l = 0; l < c.num_layers; ++l) {
       NvtxRange nvtx_layer("tcb encoder layer");
       const auto& mp = w->maps[l];
-      const tcb::k::GemmMaps g_qkv{w->aX, mp.qkv, w->cQkv, w->cQkv};
-      const tcb::k::GemmMaps g_o{w->aAtt, mp.o, w->cZ, w->cX};
-      const tcb::k::GemmMaps g_1{w->aX1, mp.w1, w->cH, w->cH};
-      const tcb::k::GemmMaps g_2{w->aH, mp.w2, w->cZ, w->cX1};
+      const tcb::k::GemmMaps g_qkv{aX, mp.qkv, cQkv, cQkv};
+      const tcb::k::GemmMaps g_o{aAtt, mp.o, cZ, cX};
+      const tcb::k::GemmMaps g_1{aX1, mp.w1, cH, cH};
+      const tcb::k::GemmMaps g_2{aH, mp.w2, cZ, cX1};
       TCB_LAUNCH(TCB_K_GEMM_QKV, s, tcb::k::launch_linear_bf16_tc(g_qkv, M, 3 * d, d,
                                                                   w->Lf(l, B_QKV), TCB_EPI_BIAS, s));
-      TCB_LAUNCH(TCB_K_ATTN, s, attention_bf16(M, d, c.num_heads, qkv, seg, segtab, att, s));
+      TCB_LAUNCH(TCB_K_ATTN, s, attention_bf16(M, d, c.num_heads, qkv, seg, segtab, att, attn_cnt + l, s));
       if (fuse_ln) {   // W_O + bias + residual + LN1 in one kernel -> x1
-        const tcb::k::GemmMaps g_o_ln{w->aAtt, mp.o, w->cX1, w->cX};
+        const tcb::k::GemmMaps g_o_ln{aAtt, mp.o, cX1, cX};
         TCB_LAUNCH(TCB_K_GEMM_O, s, tcb::k::launch_linear_ln_bf16_tc(
                                         g_o_ln, M, d, d, w->Lf(l, B_O), w->Lf(l, LN1_G),
                                         w->Lf(l, LN1_B), c.ln_eps, seg, s, lnst, lncnt(2 * l)));
@@ -538,7 +551,7 @@ tcb_status forward_impl(const tcb_weights* wc, const tcb_plan* plan, const int32
       TCB_LAUNCH(TCB_K_GEMM_FFN1, s, tcb::k::launch_linear_bf16_tc(g_1, M, f, d, w->Lf(l, B_1),
                                                                    act_epi, s));
       if (fuse_ln) {   // FFN2 + bias + residual + LN2 in one kernel -> X
-        const tcb::k::GemmMaps g_2_ln{w->aH, mp.w2, w->cX, w->cX1};
+        const tcb::k::GemmMaps g_2_ln{aH, mp.w2, cX, cX1};
         TCB_LAUNCH(TCB_K_GEMM_FFN2, s, tcb::k::launch_linear_ln_bf16_tc(
                                            g_2_ln, M, d, f, w->Lf(l, B_2), w->Lf(l, LN2_G),
                                            w->Lf(l, LN2_B), c.ln_eps, seg, s, lnst, lncnt(2 * l + 1)));
@@ -651,30 +664,26 @@ tcb_status tcb_op_linear_ln(int64_t M, int32_t N, int32_t K, const void* A, cons
       !tcb::k::make_gemm_c_map(&maps.c, C, M, N) || !tcb::k::make_gemm_c_map(&maps.r, R, M, N))
     return fail(TCB_ERR_CUDA, "tcb_op_linear_ln: cuTensorMapEncodeTiled failed (alignment?)");
   // the row-statistics scratch of the L2-exchange kernel (N = 512 / 1024 with K >= 2N, or
-  // every N under TCB_LN_KERNEL=global), library-owned for this op (grown on demand; the
-  // encoder forward uses its workspace instead)
-  float2* st = nullptr;
-  int* cnt = nullptr;
-  {
-    static std::mutex mu;
-    static void* buf = nullptr;
-    static size_t cap = 0;
-    const size_t sb = (tcb::k::linear_ln_scratch_stats_bytes(M, N) + 255) & ~size_t(255);
-    const size_t need = sb + tcb::k::linear_ln_scratch_cnt_bytes(M);
-    std::lock_guard<std::mutex> g(mu);
-    if (need > cap) {
-      if (buf) cudaFree(buf);
-      buf = nullptr;
-      cap = 0;
-      if (cudaMalloc(&buf, need) != cudaSuccess)
-        return fail(TCB_ERR_OUT_OF_MEMORY, "tcb_op_linear_ln: scratch allocation failed");
-      cap = need;
-    }
-    st = static_cast<float2*>(buf);
-    cnt = reinterpret_cast<int*>(static_cast<uint8_t*>(buf) + sb);
-    if (cudaMemsetAsync(cnt, 0, tcb::k::linear_ln_scratch_cnt_bytes(M), s) != cudaSuccess)
-      return fail(TCB_ERR_CUDA, "tcb_op_linear_ln: counter reset failed");
+  // every N under TCB_LN_KERNEL=global): stream-ordered allocation per call, so calls on
+  // different streams never share counters (the encoder forward uses its workspace instead)
+  const size_t sb = (tcb::k::linear_ln_scratch_stats_bytes(M, N) + 255) & ~size_t(255);
+  const size_t cb = tcb::k::linear_ln_scratch_cnt_bytes(M);
+  void* buf = nullptr;
+  if (cudaMallocAsync(&buf, sb + cb, s) != cudaSuccess) {
+    cudaGetLastError();
+    return fail(TCB_ERR_OUT_OF_MEMORY, "tcb_op_linear_ln: scratch allocation failed");
   }
+  float2* st = static_cast<float2*>(buf);
+  int* cnt = reinterpret_cast<int*>(static_cast<uint8_t*>(buf) + sb);
+  if (cudaMemsetAsync(cnt, 0, cb, s) != cudaSuccess) {
+    cudaFreeAsync(buf, s);
+    return fail(TCB_ERR_CUDA, "tcb_op_linear_ln: counter reset failed");
+  }
+  struct FreeAfter {                              // after the launch, in stream order
+    void* p;
+    cudaStream_t s;
+    ~FreeAfter() { cudaFreeAsync(p, s); }
+  } free_after{buf, s};
   TCB_LAUNCH(TCB_K_GEMM_O, s, tcb::k::launch_linear_ln_bf16_tc(maps, M, N, K, bias, gamma, beta,
                                                                eps, d_seg, s, st, cnt));
   return TCB_OK;
@@ -695,8 +704,23 @@ tcb_status tcb_op_attention(int32_t dtype, int64_t num_slots, int32_t d_model,
   if (tcb_status st = check_device()) return st;
   cudaStream_t s = reinterpret_cast<cudaStream_t>(stream);
   const int4* segtab = reinterpret_cast<const int4*>(d_segtab);
-  if (dtype == 1)
-    TCB_LAUNCH(TCB_K_ATTN, s, attention_bf16(num_slots, d_model, num_heads, qkv, d_seg, segtab, O, s));
+  if (dtype == 1) {
+    // the kernel's dynamic item counter: stream-ordered scratch, zeroed per call
+    void* cnt = nullptr;
+    if (cudaMallocAsync(&cnt, sizeof(int), s) != cudaSuccess) {
+      cudaGetLastError();
+      return fail(TCB_ERR_OUT_OF_MEMORY, "tcb_op_attention: counter allocation failed");
+    }
+    struct FreeAfter {
+      void* p;
+      cudaStream_t s;
+      ~FreeAfter() { cudaFreeAsync(p, s); }
+    } free_after{cnt, s};
+    if (cudaMemsetAsync(cnt, 0, sizeof(int), s) != cudaSuccess)
+      return fail(TCB_ERR_CUDA, "tcb_op_attention: counter reset failed");
+    TCB_LAUNCH(TCB_K_ATTN, s, attention_bf16(num_slots, d_model, num_heads, qkv, d_seg, segtab, O,
+                                             static_cast<int*>(cnt), s));
+  }
   else
     TCB_LAUNCH(TCB_K_ATTN, s, tcb::k::launch_attention_f32(num_slots, d_model, num_heads,
                                                            static_cast<const float*>(qkv), d_seg,
@@ -818,8 +842,10 @@ tcb_status tcb_decoder_create(const tcb_weights* enc, const void* const* tensors
     if (!tensors[i] || (reinterpret_cast<uintptr_t>(tensors[i]) & 15))
       return fail(TCB_ERR_INVALID_ARGUMENT, "tcb_decoder_create: tensor " + std::to_string(i) +
                                                 " is NULL or not 16-byte aligned");
+  // (dec_attn walks any number of keys in chunks of its smem score buffer, so neither the
+  // self-attention length max_target nor a request's source length is bounded by it)
   if (max_requests <= 0 || max_slots <= 0 || max_target <= 0 || max_target >= c.max_pos ||
-      max_target > tcb::k::dec_max_keys() || max_slots > INT32_MAX)
+      max_slots > INT32_MAX)
     return fail(TCB_ERR_INVALID_ARGUMENT, "tcb_decoder_create: bad capacities");
   if (tcb_status st = check_device()) return st;
   tcb_decoder* dec = new (std::nothrow) tcb_decoder();

@@ -28,7 +28,7 @@ namespace {
 
 constexpr int DH = 64;
 constexpr int kAttnWarps = 4;            // heads per CTA
-constexpr int kMaxKeys = 1024;           // smem score buffer per warp
+constexpr int kMaxKeys = 1024;           // smem score buffer per warp (keys are processed in chunks of it)
 
 __global__ void __launch_bounds__(256)
 dec_embed_kernel(DecEmbedArgs a) {
@@ -116,44 +116,57 @@ dec_attn_kernel(DecAttnArgs a) {
       q[8 * v + 2 * e + 1] = f.y * a.scale;
     }
   }
-  // scores: lane j takes keys j, j + 32, ...
-  float m = -INFINITY;
-  for (int j = lane; j < klen; j += 32) {
-    const uint4* k4 = reinterpret_cast<const uint4*>(a.kv + (kstart + j) * a.ld_kv + h * DH);
-    float s = 0.f;
+  // Keys in chunks of kMaxKeys (the smem score buffer) with an online max / sum across
+  // chunks, so any klen is safe (cross-attention keys = the request's source length, which can
+  // exceed the self-attention bound).  For klen <= kMaxKeys this is exactly one pass.
+  float m_run = -INFINITY, l = 0.f, o0 = 0.f, o1 = 0.f;
+  for (int base = 0; base < klen; base += kMaxKeys) {
+    const int n = min(kMaxKeys, klen - base);
+    // scores: lane j takes keys j, j + 32, ...
+    float m = -INFINITY;
+    for (int j = lane; j < n; j += 32) {
+      const uint4* k4 = reinterpret_cast<const uint4*>(a.kv + (kstart + base + j) * a.ld_kv + h * DH);
+      float s = 0.f;
 #pragma unroll
-    for (int v = 0; v < DH / 8; ++v) {
-      const uint4 x = k4[v];
-      const __nv_bfloat162* hh = reinterpret_cast<const __nv_bfloat162*>(&x);
+      for (int v = 0; v < DH / 8; ++v) {
+        const uint4 x = k4[v];
+        const __nv_bfloat162* hh = reinterpret_cast<const __nv_bfloat162*>(&x);
 #pragma unroll
-      for (int e = 0; e < 4; ++e) {
-        const float2 f = __bfloat1622float2(hh[e]);
-        s = fmaf(q[8 * v + 2 * e], f.x, s);
-        s = fmaf(q[8 * v + 2 * e + 1], f.y, s);
+        for (int e = 0; e < 4; ++e) {
+          const float2 f = __bfloat1622float2(hh[e]);
+          s = fmaf(q[8 * v + 2 * e], f.x, s);
+          s = fmaf(q[8 * v + 2 * e + 1], f.y, s);
+        }
       }
+      sp[w][j] = s;
+      m = fmaxf(m, s);
     }
-    sp[w][j] = s;
-    m = fmaxf(m, s);
-  }
 #pragma unroll
-  for (int o = 16; o > 0; o >>= 1) m = fmaxf(m, __shfl_xor_sync(0xffffffffu, m, o));
-  float l = 0.f;
-  for (int j = lane; j < klen; j += 32) {
-    const float p = __expf(sp[w][j] - m);
-    sp[w][j] = p;
-    l += p;
-  }
+    for (int o = 16; o > 0; o >>= 1) m = fmaxf(m, __shfl_xor_sync(0xffffffffu, m, o));
+    const float mn = fmaxf(m_run, m);
+    const float f = m_run == -INFINITY ? 0.f : __expf(m_run - mn);   // rescale earlier chunks
+    float lc = 0.f;
+    for (int j = lane; j < n; j += 32) {
+      const float p = __expf(sp[w][j] - mn);
+      sp[w][j] = p;
+      lc += p;
+    }
 #pragma unroll
-  for (int o = 16; o > 0; o >>= 1) l += __shfl_xor_sync(0xffffffffu, l, o);
-  __syncwarp();
-  // o = sum_j p_j v_j: lane owns dims 2*lane, 2*lane + 1 (coalesced 128-byte V rows)
-  float o0 = 0.f, o1 = 0.f;
-  const __nv_bfloat16* vb = a.kv + kstart * a.ld_kv + a.voff + h * DH + 2 * lane;
-  for (int j = 0; j < klen; ++j) {
-    const float2 f = __bfloat1622float2(*reinterpret_cast<const __nv_bfloat162*>(vb + j * a.ld_kv));
-    const float p = sp[w][j];
-    o0 = fmaf(p, f.x, o0);
-    o1 = fmaf(p, f.y, o1);
+    for (int o = 16; o > 0; o >>= 1) lc += __shfl_xor_sync(0xffffffffu, lc, o);
+    __syncwarp();
+    l = l * f + lc;
+    o0 *= f;
+    o1 *= f;
+    // o = sum_j p_j v_j: lane owns dims 2*lane, 2*lane + 1 (coalesced 128-byte V rows)
+    const __nv_bfloat16* vb = a.kv + (kstart + base) * a.ld_kv + a.voff + h * DH + 2 * lane;
+    for (int j = 0; j < n; ++j) {
+      const float2 fv = __bfloat1622float2(*reinterpret_cast<const __nv_bfloat162*>(vb + j * a.ld_kv));
+      const float p = sp[w][j];
+      o0 = fmaf(p, fv.x, o0);
+      o1 = fmaf(p, fv.y, o1);
+    }
+    m_run = mn;
+    __syncwarp();                                // sp is rewritten by the next chunk
   }
   const float inv = klen > 0 ? 1.f / l : 0.f;
   reinterpret_cast<__nv_bfloat162*>(a.out + static_cast<int64_t>(i) * a.d + h * DH)[lane] =
@@ -239,7 +252,6 @@ cudaError_t launch_dec_argmax(const DecArgmaxArgs& a, cudaStream_t s) {
   return launch_ex(dec_argmax_kernel, dim3(a.rows), dim3(256), 0, s, 1, a);
 }
 
-int dec_max_keys() { return kMaxKeys; }
 
 }  // namespace k
 }  // namespace tcb

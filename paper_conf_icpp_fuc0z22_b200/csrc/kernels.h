@@ -116,13 +116,11 @@ size_t linear_ln_scratch_stats_bytes(int64_t M, int N);
 size_t linear_ln_scratch_cnt_bytes(int64_t M);
 
 // Attention ------------------------------------------------------------------------------
-cudaError_t launch_attention_bf16(int64_t num_slots, int d_model, int num_heads,
-                                  const void* qkv, const int32_t* seg_ids, const int4* segtab,
-                                  void* O, cudaStream_t s);
-// tcgen05 variant (attention_tc.cu): S and O in TMEM, 128-query x 128-key chunks.
+// tcgen05 kernel (attention_tc.cu): S and O in TMEM, 128-query x 128-key chunks.  item_counter:
+// one int32 in device memory, zero at launch (dynamic item scheduling); NULL = static order.
 cudaError_t launch_attention_bf16_tc(int64_t num_slots, int d_model, int num_heads,
                                      const void* qkv, const int32_t* seg_ids, const int4* segtab,
-                                     void* O, cudaStream_t s);
+                                     void* O, int* item_counter, cudaStream_t s);
 cudaError_t launch_attention_f32(int64_t num_slots, int d_model, int num_heads,
                                  const float* qkv, const int32_t* seg_ids, const int4* segtab,
                                  float* O, cudaStream_t s);
@@ -170,7 +168,6 @@ cudaError_t launch_dec_step_advance(int32_t* d_t, cudaStream_t s);   // ++*d_t
 cudaError_t launch_dec_embed(const DecEmbedArgs& a, cudaStream_t s);
 cudaError_t launch_dec_attn(const DecAttnArgs& a, cudaStream_t s);
 cudaError_t launch_dec_argmax(const DecArgmaxArgs& a, cudaStream_t s);
-int dec_max_keys();
 
 }  // namespace k
 }  // namespace tcb

@@ -1815,6 +1815,10 @@ cudaError_t launch_lng(const GemmMaps& m, int M, int K, const float* bias, const
     }
     max_pairs = n;               // every CTA of the grid must be co-resident (see the kernel)
   }
+  // The P units of a tile must sit on P distinct pairs (a unit waits for its tile's other
+  // units; two on one pair would wait for themselves): with fewer co-resident pairs than P
+  // (an SM-limited context) use the cluster kernel instead.
+  if (max_pairs < P) return launch_lnc<P>(m, M, K, bias, gamma, beta, eps, seg_ids, s);
   const int units = ((M + 255) / 256) * P;
   const int pairs = units < max_pairs ? units : max_pairs;
   cfg.gridDim = dim3(2 * pairs);

@@ -93,32 +93,38 @@ void compute_info(tcb_plan* p) {
     I.kv_tiles_dense = -1;
     I.kv_tiles_visited = -1;
   }
-  // Score elements the attention kernel evaluates: per 64-slot CTA, 16-key sub-blocks
-  // starting at the CTA's interval start; a warp (16 query rows) evaluates a sub-block iff
-  // it intersects the warp's own interval.
+  // Score elements the tcgen05 attention kernel (attention_tc.cu) evaluates, per head.  An
+  // item is a block of kAttnQBlock query slots; its key interval [lo, hi) spans its first to
+  // its last request, walked in kAttnKChunk-key chunks from kbase = lo rounded down to 8:
+  //   executed: every chunk is a full kAttnQBlock x kAttnKChunk S = QK^T tile on the tensor core;
+  //   softmax : inside a chunk, a group of kAttnSmRows query rows x kAttnSmKeys keys goes
+  //             through the exponentials iff it intersects the union of those rows' intervals
+  //             (dead groups are skipped, P = 0).
   for (int64_t q0 = 0; q0 < I.num_slots; q0 += kAttnQBlock) {
-    int64_t clo = -1, chi = -1;
-    int64_t wlo[kAttnQBlock / kAttnWarpRows], whi[kAttnQBlock / kAttnWarpRows];
-    for (int w = 0; w < kAttnQBlock / kAttnWarpRows; ++w) {
-      wlo[w] = -1; whi[w] = -1;
-      for (int64_t k = q0 + w * kAttnWarpRows;
-           k < std::min<int64_t>(I.num_slots, q0 + (w + 1) * kAttnWarpRows); ++k) {
+    constexpr int kG = kAttnQBlock / kAttnSmRows;
+    int64_t glo[kG], ghi[kG];
+    int64_t lo = -1, hi = -1;
+    for (int g = 0; g < kG; ++g) {
+      glo[g] = -1; ghi[g] = -1;
+      for (int64_t k = q0 + g * kAttnSmRows; k < std::min<int64_t>(I.num_slots, q0 + (g + 1) * kAttnSmRows); ++k) {
         if (seg_of[k] < 0) continue;
         const int64_t a = p->seg_start[seg_of[k]], b = seg_end[seg_of[k]];
-        if (wlo[w] < 0 || a < wlo[w]) wlo[w] = a;
-        if (b > whi[w]) whi[w] = b;
+        if (glo[g] < 0 || a < glo[g]) glo[g] = a;
+        if (b > ghi[g]) ghi[g] = b;
       }
-      if (wlo[w] >= 0) {
-        if (clo < 0 || wlo[w] < clo) clo = wlo[w];
-        if (whi[w] > chi) chi = whi[w];
+      if (glo[g] >= 0) {
+        if (lo < 0 || glo[g] < lo) lo = glo[g];
+        if (ghi[g] > hi) hi = ghi[g];
       }
     }
-    if (clo < 0) continue;
-    for (int w = 0; w < kAttnQBlock / kAttnWarpRows; ++w) {
-      if (wlo[w] < 0) continue;
-      for (int64_t kb = clo; kb < chi; kb += kAttnKSub)
-        if (kb < whi[w] && kb + kAttnKSub > wlo[w])
-          I.executed_score_elems += kAttnWarpRows * kAttnKSub;
+    if (lo < 0) continue;
+    const int64_t kbase = lo & ~static_cast<int64_t>(7);
+    const int64_t nch = (hi - kbase + kAttnKChunk - 1) / kAttnKChunk;
+    I.executed_score_elems += nch * kAttnQBlock * kAttnKChunk;
+    for (int g = 0; g < kG; ++g) {
+      if (glo[g] < 0) continue;
+      for (int64_t gk = kbase; gk < kbase + nch * kAttnKChunk; gk += kAttnSmKeys)
+        if (gk < ghi[g] && gk + kAttnSmKeys > glo[g]) I.softmax_score_elems += kAttnSmRows * kAttnSmKeys;
     }
   }
 }

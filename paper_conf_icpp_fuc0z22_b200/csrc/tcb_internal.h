@@ -9,11 +9,12 @@
 #include "../../include/tcb.h"
 #include "../../include/tcb_ops.h"
 
-// Geometry of the segment-masked attention kernel (attn.cu); the host plan uses it to
-// report how many score elements the kernel evaluates (tcb_plan_info).
-constexpr int kAttnQBlock = 128;   // query slots per CTA (8 warps x 16 rows)
-constexpr int kAttnWarpRows = 16;  // query rows per warp (one m16 MMA tile)
-constexpr int kAttnKSub = 16;      // keys per skip decision (one k16 MMA step of P.V)
+// Geometry of the tcgen05 segment-masked attention kernel (attention_tc.cu); the host plan
+// uses it to report the score elements the kernel evaluates (tcb_plan_info).
+constexpr int kAttnQBlock = 128;   // query slots per item (TMEM lanes of S)
+constexpr int kAttnKChunk = 128;   // keys per S = QK^T tile
+constexpr int kAttnSmRows = 32;    // query rows of one softmax warp
+constexpr int kAttnSmKeys = 32;    // keys per liveness decision of the softmax
 
 struct tcb_plan;
 

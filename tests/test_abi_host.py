@@ -177,8 +177,9 @@ def test_pack_errors():
 
 def test_plan_counters_vs_brute_force():
     """P9 on the product's plan counters: 128x128 tiles touching a diagonal block, the
-    dense count, sum l^2, and the kernel's executed 16x16 sub-blocks (re-derived here from
-    its stated geometry: 128-slot CTAs, 16-row warps, 16-key sub-blocks from the CTA start)."""
+    dense count, sum l^2, and the tcgen05 attention kernel's executed S elements and softmax
+    elements (re-derived here from its stated geometry: 128-query items, 128-key chunks from
+    the item's interval start rounded down to 8, 32-row x 32-key softmax liveness groups)."""
     lengths = np.minimum(wl.draw_lengths("dia", 300, 5), 512).astype(np.int32)
     plan = tcb.tcb_pack(lengths, 512, 16)
     a = plan.arrays()
@@ -198,21 +199,26 @@ def test_plan_counters_vs_brute_force():
     placed = a["req_row"] >= 0
     assert info["useful_score_elems"] == int(np.sum(lengths[placed].astype(np.int64) ** 2))
     starts, lens = a["seg_start"], lengths[a["seg_req"]]
-    ex = 0
+    ex = sm = 0
     for q0 in range(0, M, 128):
         iv = []
-        for w in range(8):
-            ss = [s for s in seg[q0 + 16 * w:q0 + 16 * w + 16] if s >= 0]
+        for g in range(4):
+            ss = [s for s in seg[q0 + 32 * g:q0 + 32 * g + 32] if s >= 0]
             iv.append((min(starts[s] for s in ss), max(starts[s] + lens[s] for s in ss))
                       if ss else None)
         real = [x for x in iv if x]
         if not real:
             continue
-        clo, chi = min(x[0] for x in real), max(x[1] for x in real)
+        lo, hi = min(x[0] for x in real), max(x[1] for x in real)
+        kb = lo - lo % 8
+        nch = -(-(hi - kb) // 128)
+        ex += nch * 128 * 128
         for x in real:
-            ex += 256 * sum(1 for kb in range(clo, chi, 16) if kb < x[1] and kb + 16 > x[0])
+            sm += 32 * 32 * sum(1 for gk in range(kb, kb + 128 * nch, 32)
+                                if gk < x[1] and gk + 32 > x[0])
     assert info["executed_score_elems"] == ex
-    assert info["useful_score_elems"] <= ex
+    assert info["softmax_score_elems"] == sm
+    assert info["useful_score_elems"] <= sm <= ex
 
 
 def test_device_calls_fail_loudly_without_gpu():

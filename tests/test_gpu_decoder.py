@@ -101,3 +101,30 @@ def test_decoder_tokens_valid_under_oracle_and_early_clean_bitwise():
             lg = out[k] @ E.T
             tol = 2 * 2e-2 * np.max(np.abs(lg))
             assert lg[seq[k]] >= lg.max() - tol, (r, k, lg[seq[k]], lg.max())
+
+
+def test_decoder_cross_attention_longer_than_score_buffer():
+    """A request whose source (the cross-attention keys) is longer than dec_attn's 1024-key
+    smem score buffer: the keys are walked in chunks with an online max / sum,
+    step-1 logits vs the oracle <= 2e-2 normwise."""
+    model = wl.ModelConfig("dec-long", 1, 512, 8, 2048, 512, 2048, "bf16", "relu", "sin_paper",
+                           False, False, 1e-5, 1e-5, 1.0)
+    lengths = np.array([1300, 40], np.int32)
+    w = wl.draw_weights(model, 13)
+    names = wl.weight_names(model)
+    dw = wl.draw_dec_weights(model, 113)
+    dn = wl.dec_weight_names(model)
+    ids = wl.draw_token_ids(int(lengths.sum()), model.vocab, 14)
+    enc = tcb.Encoder(model, w, names)
+    plan, rows, _ = enc.run(lengths, ids, 1536)
+    dec = tcb.Decoder(enc, dw, dn, max_requests=len(lengths), max_slots=plan.num_slots,
+                      max_target=1)
+    tokens, lens = dec.decode(plan, rows, early_clean=True)
+    torch.cuda.synchronize()
+    got = dec.last_logits()
+    cu = np.concatenate([[0], np.cumsum(lengths)])
+    for r in range(len(lengths)):
+        _, lg = oracle.decode_greedy(model, w, names, dw, dn, ids[cu[r]:cu[r + 1]], 1,
+                                     with_logits=True)
+        e = np.max(np.abs(got[r] - lg[0])) / np.max(np.abs(lg[0]))
+        assert e <= 2e-2, (r, e)
