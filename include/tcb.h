@@ -141,8 +141,12 @@ tcb_status tcb_plan_copy(const tcb_plan* plan, int32_t* req_row, int32_t* req_co
  *                     {slot_start, length, token_offset (request-order index of its first
  *                      token), request};
  *   row index (num_rows + 1 words, padded to a multiple of 4): row_first[r] = index of the
- *                     first segment of row r, row_first[num_rows] = S.
- * tcb_plan_segtab_words gives the word count (4 * (1 + S) + round_up(num_rows + 1, 4));
+ *                     first segment of row r, row_first[num_rows] = S;
+ *   query-block order (qtiles words, padded to a multiple of 4): the 128-slot query blocks
+ *                     by decreasing number of 128-key chunks of their key interval (ties by
+ *                     index) -- the attention kernel hands out its items in this order.
+ * tcb_plan_segtab_words gives the word count
+ * (4 * (1 + S) + round_up(num_rows + 1, 4) + round_up(qtiles, 4));
  * tcb_plan_write_segtab writes it into a HOST buffer of at least that many words; the caller
  * copies it to the device (16-byte aligned) and passes that pointer as d_segtab below.  A
  * plan of the same (num_rows, row_len) may later be written into the same device buffer (if

@@ -358,7 +358,8 @@ tcb_status tcb_plan_copy(const tcb_plan* p, int32_t* req_row, int32_t* req_col,
 
 int64_t tcb_plan_segtab_words(const tcb_plan* p) {
   if (!p) return -1;
-  return 4 * (1 + static_cast<int64_t>(p->seg_req.size())) + (p->num_rows + 1 + 3) / 4 * 4;
+  return 4 * (1 + static_cast<int64_t>(p->seg_req.size())) + (p->num_rows + 1 + 3) / 4 * 4 +
+         (p->info.qtiles + 3) / 4 * 4;
 }
 
 tcb_status tcb_plan_write_segtab(const tcb_plan* p, int32_t* dst, int64_t capacity_words) {
@@ -391,6 +392,34 @@ tcb_status tcb_plan_write_segtab(const tcb_plan* p, int32_t* dst, int64_t capaci
     while (s < S && p->seg_start[s] < static_cast<int64_t>(k) * p->row_len) ++s;
     row_first[k] = s;
   }
+  // attention work order: the 128-slot query blocks by decreasing number of 128-key chunks
+  // of their key interval (the attention kernel's item cost; longest first, ties by index),
+  // so a dynamically scheduled grid ends on short items
+  int32_t* qorder = row_first + (p->num_rows + 1 + 3) / 4 * 4;
+  const int64_t QT = p->info.qtiles, M = p->info.num_slots;
+  std::vector<int32_t> nch(static_cast<size_t>(QT), 0);
+  {
+    int64_t s0 = 0;
+    for (int64_t t = 0; t < QT; ++t) {
+      const int64_t q0 = t * 128, q1 = std::min<int64_t>(M, q0 + 128);
+      while (s0 < S && static_cast<int64_t>(p->seg_start[s0]) + p->lengths[p->seg_req[s0]] <= q0) ++s0;
+      int64_t lo = -1, hi = -1;
+      for (int64_t k = s0; k < S && p->seg_start[k] < q1; ++k) {
+        const int64_t a = p->seg_start[k], b = a + p->lengths[p->seg_req[k]];
+        if (b <= q0) continue;
+        if (lo < 0) lo = a;
+        hi = b;
+      }
+      if (lo >= 0) {
+        const int64_t kb = lo & ~static_cast<int64_t>(7);
+        nch[t] = static_cast<int32_t>((hi - kb + 127) / 128);
+      }
+    }
+  }
+  std::vector<int32_t> ord(static_cast<size_t>(QT));
+  for (int64_t t = 0; t < QT; ++t) ord[t] = static_cast<int32_t>(t);
+  std::stable_sort(ord.begin(), ord.end(), [&](int32_t a, int32_t b) { return nch[a] > nch[b]; });
+  for (int64_t t = 0; t < (QT + 3) / 4 * 4; ++t) qorder[t] = t < QT ? ord[t] : 0;
   const int64_t padded = (p->num_rows + 1 + 3) / 4 * 4;
   for (int64_t k = p->num_rows + 1; k < padded; ++k) row_first[k] = S;
   return TCB_OK;

@@ -45,8 +45,8 @@ class Server:
         M = self.B * self.L
         d = encoder.model.d_model
         dev = encoder.device
-        # segment table of at most M segments (one per slot) + row index
-        self.seg_words = 4 * (1 + M) + ((self.B + 1 + 3) // 4) * 4
+        # segment table of at most M segments (one per slot) + row index + query-block order
+        self.seg_words = 4 * (1 + M) + ((self.B + 1 + 3) // 4) * 4 + ((M + 127) // 128 + 3) // 4 * 4
         self.d_segtab = torch.zeros(self.seg_words, dtype=torch.int32, device=dev)
         self.h_segtab = torch.zeros(self.seg_words, dtype=torch.int32).pin_memory()
         self.d_ids = torch.zeros(M, dtype=torch.int32, device=dev)

@@ -757,9 +757,12 @@ attn_tc_kernel(const __grid_constant__ CUtensorMap tmQKV, const int32_t* __restr
 // warp.  Items are handed out dynamically (an atomic counter in global memory, zeroed before
 // the launch), so the 1- to 5-chunk items of a mixed-length batch balance across the 296 CTAs.
 namespace v3 {
-constexpr int kWarps = 6;                    // 0 producer, 1 MMA + TMEM, 2..5 softmax / epilogue
+constexpr int kWarps = 8;                    // warpgroup 0: 0 TMA producer, 1 MMA + TMEM,
+                                             // 2 item scheduler (metadata), 3 idle;
+                                             // warpgroup 1: 4..7 softmax / epilogue
+constexpr int kCtrlRegs = 56, kSoftmaxRegs = 168;   // setmaxnreg split (2 CTAs x 256 threads)
 constexpr int kThreads = kWarps * 32;
-constexpr int kQStages = 2, kKStages = 2, kVStages = 2;
+constexpr int kQStages = 2, kKStages = 2, kVStages = 2, kInfoStages = 2;
 constexpr uint32_t kTmemCols = 256;          // S [0,128), O [128,192), P [192,256)
 constexpr uint32_t kOCol = 128, kPCol = 192;
 
@@ -777,7 +780,7 @@ struct Info {
   int qb, h;       // query block, head
 };
 constexpr int kSmemBytes = 1024 + (kQStages + kKStages + kVStages) * kTileBytes +
-                           kQStages * static_cast<int>(sizeof(Info)) + 256;
+                           kInfoStages * static_cast<int>(sizeof(Info)) + 256;
 
 // the segment table's query-block order (tcb.h: after the records and the row index), longest
 // key interval first
@@ -889,14 +892,15 @@ attn_tc3_kernel(const __grid_constant__ CUtensorMap tmQKV, const __grid_constant
   const uint32_t sK = sQ + kQStages * kTileBytes;              // [2][128 x 64]
   const uint32_t sV = sK + kKStages * kTileBytes;              // [2][128 x 64]
   uint8_t* gen = smem_raw + (sV + kVStages * kTileBytes - raw);
-  Info* infos = reinterpret_cast<Info*>(gen);                  // [2]
-  uint32_t* tmem_slot = reinterpret_cast<uint32_t*>(gen + kQStages * sizeof(Info));
+  Info* infos = reinterpret_cast<Info*>(gen);                  // [kInfoStages]
+  uint32_t* tmem_slot = reinterpret_cast<uint32_t*>(gen + kInfoStages * sizeof(Info));
   const uint32_t bars = (smem_u32(tmem_slot + 2) + 7) & ~7u;
   const uint32_t q_full = bars, q_empty = q_full + 8 * kQStages;
   const uint32_t k_full = q_empty + 8 * kQStages, k_empty = k_full + 8 * kKStages;
   const uint32_t v_full = k_empty + 8 * kKStages, v_empty = v_full + 8 * kVStages;
   const uint32_t s_full = v_empty + 8 * kVStages, s_free = s_full + 8;
   const uint32_t p_full = s_free + 8, pv_done = p_full + 8;
+  const uint32_t i_full = pv_done + 8, i_empty = i_full + 8 * kInfoStages;
 
   const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
   if (threadIdx.x == 0) {
@@ -911,6 +915,10 @@ attn_tc3_kernel(const __grid_constant__ CUtensorMap tmQKV, const __grid_constant
     mbar_init(s_free, 4);
     mbar_init(p_full, 4);
     mbar_init(pv_done, 1);
+    for (int i = 0; i < kInfoStages; ++i) {
+      mbar_init(i_full + 8 * i, 1);
+      mbar_init(i_empty + 8 * i, 1 + 1 + 4);  // TMA producer + MMA + 4 softmax warps
+    }
     asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
   }
   if (warp == 1) {
@@ -924,13 +932,14 @@ attn_tc3_kernel(const __grid_constant__ CUtensorMap tmQKV, const __grid_constant
   const uint32_t tmem = *tmem_slot;
   pdl_wait();                                 // QKV / segment ids come from earlier kernels
   pdl_trigger();
-
-  if (warp == 0) {
-    // ================= producer: next item, its metadata, Q, then its K/V chunks ==========
-    if (lane == 0) asm volatile("prefetch.tensormap [%0];" ::"l"(reinterpret_cast<uint64_t>(&tmQKV)) : "memory");
+  // registers: the control warpgroup hands most of its share to the softmax warpgroup
+  if (warp < 4) {
+  asm volatile("setmaxnreg.dec.sync.aligned.u32 %0;" ::"n"(kCtrlRegs));
+  if (warp == 2) {
+    // ================= item scheduler: next item -> metadata ring ==========================
     const int32_t* qorder = qblock_order(segtab);
-    int qs = 0, ks = 0, vs = 0;
-    uint32_t qph = 0, kph = 0, vph = 0;
+    int is = 0;
+    uint32_t iph = 0;
     for (int k = 0;; ++k) {
       int item = 0;
       if (item_counter) {
@@ -939,31 +948,49 @@ attn_tc3_kernel(const __grid_constant__ CUtensorMap tmQKV, const __grid_constant
       } else {
         item = blockIdx.x + k * gridDim.x;
       }
-      if (lane == 0) mbar_wait(q_empty + 8 * qs, qph ^ 1);
+      if (lane == 0) mbar_wait(i_empty + 8 * is, iph ^ 1);
       __syncwarp();
-      Info* inf = infos + qs;
+      Info* inf = infos + is;
       if (item >= num_items) {
         if (lane == 0) {
           inf->nch = -1;
-          mbar_arrive(q_full + 8 * qs);
+          mbar_arrive(i_full + 8 * is);
         }
         break;
       }
-      const int qb = __ldg(&qorder[item / num_heads]), h = item % num_heads;
-      const int64_t q0 = static_cast<int64_t>(qb) * TQ;
-      compute_info(reinterpret_cast<ItemInfo*>(inf), seg_ids, segtab, q0, num_slots, lane);
-      const int nch = inf->nch;
+      const int qb = __ldg(&qorder[item / num_heads]);
+      compute_info(reinterpret_cast<ItemInfo*>(inf), seg_ids, segtab, static_cast<int64_t>(qb) * TQ,
+                   num_slots, lane);
       if (lane == 0) {
         inf->qb = qb;
-        inf->h = h;
+        inf->h = item % num_heads;
+        mbar_arrive(i_full + 8 * is);
+      }
+      __syncwarp();
+      if (++is == kInfoStages) { is = 0; iph ^= 1; }
+    }
+  } else if (warp == 0) {
+    // ================= TMA producer: per item its Q tile, then K one chunk ahead of V =========
+    if (lane == 0) {
+      asm volatile("prefetch.tensormap [%0];" ::"l"(reinterpret_cast<uint64_t>(&tmQKV)) : "memory");
+      int qs = 0, ks = 0, vs = 0, is = 0;
+      uint32_t qph = 0, kph = 0, vph = 0, iph = 0;
+      for (;;) {
+        mbar_wait(i_full + 8 * is, iph);
+        const Info* inf = infos + is;
+        const int nch = inf->nch, kbase = inf->kbase, qb = inf->qb, h = inf->h;
+        mbar_arrive(i_empty + 8 * is);
+        if (++is == kInfoStages) { is = 0; iph ^= 1; }
+        if (nch < 0) break;
+        mbar_wait(q_empty + 8 * qs, qph ^ 1);  // the slot is ours (also for an empty item:
+                                               // the softmax warps stage its output there)
         if (nch == 0) {
           mbar_arrive(q_full + 8 * qs);
         } else {
           mbar_expect_tx(q_full + 8 * qs, kTileBytes);
-          tma_load(sQ + qs * kTileBytes, &tmQKV, q_full + 8 * qs, h * DH, static_cast<int>(q0));
+          tma_load(sQ + qs * kTileBytes, &tmQKV, q_full + 8 * qs, h * DH, qb * TQ);
         }
         // K one chunk ahead of V (K is released by S, V only by P V)
-        const int kbase = inf->kbase;
         for (int c = 0; c <= nch; ++c) {
           if (c < nch) {
             mbar_wait(k_empty + 8 * ks, kph ^ 1);
@@ -978,9 +1005,8 @@ attn_tc3_kernel(const __grid_constant__ CUtensorMap tmQKV, const __grid_constant
             if (++vs == kVStages) { vs = 0; vph ^= 1; }
           }
         }
+        if (++qs == kQStages) { qs = 0; qph ^= 1; }
       }
-      __syncwarp();
-      if (++qs == kQStages) { qs = 0; qph ^= 1; }
     }
   } else if (warp == 1) {
     // ================= MMA issuer ===========================================================
@@ -1013,12 +1039,18 @@ attn_tc3_kernel(const __grid_constant__ CUtensorMap tmQKV, const __grid_constant
       __syncwarp();
       if (++vs == kVStages) { vs = 0; vph ^= 1; }
     };
+    int is = 0;
+    uint32_t iph = 0;
     for (;;) {
       PRB(t0);
+      mbar_wait(i_full + 8 * is, iph);
+      const int nch = infos[is].nch;
+      __syncwarp();
+      if (lane == 0) mbar_arrive(i_empty + 8 * is);
+      if (++is == kInfoStages) { is = 0; iph ^= 1; }
+      if (nch < 0) break;
       mbar_wait(q_full + 8 * qs, qph);
       PRB_ADD(a_q, t0);
-      const int nch = infos[qs].nch;
-      if (nch < 0) break;
       tc_fence_after();
       const uint32_t qaddr = sQ + qs * kTileBytes;
       if (nch == 0) {
@@ -1065,28 +1097,35 @@ attn_tc3_kernel(const __grid_constant__ CUtensorMap tmQKV, const __grid_constant
       printf("a3probe mma cta %d total %lld wait_q %lld wait_kv %lld wait_sfree %lld wait_p %lld chunks %u\n",
              blockIdx.x, clock64() - a_start, a_q, a_kv, a_sf, a_p, g);
 #endif
+  }
   } else {
-    // ================= softmax + output (warps 2..5, thread = query row) ===================
+    asm volatile("setmaxnreg.inc.sync.aligned.u32 %0;" ::"n"(kSoftmaxRegs));
+    // ================= softmax + output (warps 4..7, thread = query row) ===================
     const int q = warp & 3;                 // TMEM lane quarter
     const int row = q * 32 + lane;
     const uint32_t lane_off = static_cast<uint32_t>(q * 32) << 16;
     const uint32_t s_addr = tmem + lane_off, o_addr = tmem + lane_off + kOCol, p_addr = tmem + lane_off + kPCol;
-    int qs = 0;
-    uint32_t qph = 0, g = 0;
+    int qs = 0, is = 0;
+    uint32_t iph = 0, g = 0;
 #ifdef TCB_ATTN_PROBE
     long long b_q = 0, b_s = 0, b_p1 = 0, b_pv = 0, b_e1 = 0, b_e0 = 0, b_epi = 0, b_start = clock64();
 #endif
     for (;;) {
       PRB(t0);
-      mbar_wait(q_full + 8 * qs, qph);
+      mbar_wait(i_full + 8 * is, iph);
       PRB_ADD(b_q, t0);
-      const Info* inf = infos + qs;
+      const Info* inf = infos + is;
       const int nch = inf->nch;
-      if (nch < 0) break;
       const int2 rr = inf->rows[row];
       const int kbase = inf->kbase, qb = inf->qb, h = inf->h;
-      const int my_qs = qs;                 // the item's Q slot stages its output tile
-      if (++qs == kQStages) { qs = 0; qph ^= 1; }
+      __syncwarp();
+      if (lane == 0) mbar_arrive(i_empty + 8 * is);   // metadata copied to registers
+      if (++is == kInfoStages) { is = 0; iph ^= 1; }
+      if (nch < 0) break;
+      // the item's Q slot (acquired by the producer, read by the item's S MMAs) stages the
+      // output tile; no wait needed: the epilogue runs after the item's last P V
+      const int my_qs = qs;
+      if (++qs == kQStages) { qs = 0; }
       // key interval of this warp's 32 rows: union [ulo, uhi) and intersection [ilo, ihi)
       const bool real = rr.y > rr.x;
       int ulo = real ? rr.x : INT_MAX, uhi = real ? rr.y : -1;
@@ -1224,7 +1263,7 @@ attn_tc3_kernel(const __grid_constant__ CUtensorMap tmQKV, const __grid_constant
       PRB_ADD(b_epi, t6);
     }
 #ifdef TCB_ATTN_PROBE
-    if (lane == 0 && blockIdx.x < 3 && warp == 2)
+    if (lane == 0 && blockIdx.x < 3 && warp == 4)
       printf("a3probe sm cta %d total %lld wait_q %lld wait_s %lld pass1 %lld wait_pv %lld exp1 %lld exp0 %lld epi %lld chunks %u\n",
              blockIdx.x, clock64() - b_start, b_q, b_s, b_p1, b_pv, b_e1, b_e0, b_epi, g);
 #endif

@@ -1,7 +1,8 @@
-cd $GRAFT_REPO_ROOT; mkdir -p gpurun_out/r02j
-python -c "import __graft_entry__ as g; g.build()" > gpurun_out/r02j/build.log 2>&1; echo build rc $?
-timeout 600 python -m pytest tests/test_gpu_kernels.py -q -x -k "attention or attn" -p no:cacheprovider > gpurun_out/r02j/pytest_attn.log 2>&1; echo pytest attn rc $?; tail -3 gpurun_out/r02j/pytest_attn.log
-timeout 300 python scripts/attn_bench.py c2 c3 c4 c5 2>&1 | tee gpurun_out/r02j/attn_v3.txt
+cd $GRAFT_REPO_ROOT; mkdir -p gpurun_out/r02l
+python -c "import __graft_entry__ as g; g.build()" > gpurun_out/r02l/build.log 2>&1; echo build rc $?
+timeout 600 python -m pytest tests/test_gpu_kernels.py -q -x -k "attention or attn" -p no:cacheprovider > gpurun_out/r02l/pytest_attn.log 2>&1; echo pytest attn rc $?; tail -3 gpurun_out/r02l/pytest_attn.log
+timeout 300 python scripts/attn_bench.py c2 c3 c4 c5 2>&1 | tee gpurun_out/r02l/attn_v3.txt
 sed -i 's/FLAGS = \["-O3"/FLAGS = ["-DTCB_ATTN_PROBE", "-O3"/' paper_conf_icpp_fuc0z22_b200/_build.py
-python -c "import sys; sys.path.insert(0,'paper_conf_icpp_fuc0z22_b200'); import _build; _build.build(force=True)" > gpurun_out/r02j/build_probe.log 2>&1
-for w in c2 c3; do timeout 120 python scripts/attn_bench.py $w 2>&1 | grep -E "a3probe|workload" | tail -7; done | tee gpurun_out/r02j/probe.txt
+python -c "import sys; sys.path.insert(0,'paper_conf_icpp_fuc0z22_b200'); import _build; _build.build(force=True)" > gpurun_out/r02l/build_probe.log 2>&1
+for w in c2 c3; do timeout 120 python scripts/attn_bench.py $w 2>&1 | grep -E "a3probe|workload" | tail -7; done | tee gpurun_out/r02l/probe.txt
+cp /tmp/_b.py paper_conf_icpp_fuc0z22_b200/_build.py 2>/dev/null

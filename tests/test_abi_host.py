@@ -79,8 +79,9 @@ def test_pack_golden_f1(golden_dir):
     assert a["qtile_kv"].tolist() == f1["qtile_kv_128"]
     st = plan.segtab()
     assert st[:4].tolist() == [8, 64, 32, 58]
-    assert len(st) == 4 * 9 + 4
+    assert len(st) == 4 * 9 + 4 + 4
     assert st[36:39].tolist() == [0, 3, 8]          # row_first: row 0 -> seg 0, row 1 -> 3, end
+    assert st[40] == 0                              # query-block order: the single q-block
     recs = st[4:36].reshape(-1, 4)
     assert recs[:, 0].tolist() == f1["seg_start"]
     assert recs[:, 1].tolist() == [f1["lengths"][r] for r in f1["seg_req"]]
@@ -255,3 +256,34 @@ def test_decoder_abi_validates_without_a_gpu():
     st = _lib.DecodeStats()
     assert L.tcb_decoder_stats(None, ctypes.byref(st)) == -1
     assert len(wl.dec_weight_names(m)) == 20 * m.num_layers
+
+
+@pytest.mark.parametrize("dist,L,B,seed", [("dia", 512, 16, 3), ("paracrawl", 128, 64, 4),
+                                           ("mixed_8_512", 512, 16, 5), ("wmt", 256, 32, 6)])
+def test_segtab_query_block_order(dist, L, B, seed):
+    """The segment table's query-block order (attention work order): a permutation of the
+    q-blocks, chunk counts non-increasing, ties by index -- chunk counts re-derived here from
+    the layout (128-key chunks from the block's interval start rounded down to 8)."""
+    lengths = np.minimum(wl.draw_lengths(dist, 4 * B, seed), L).astype(np.int32)
+    plan = tcb.tcb_pack(lengths, L, B)
+    a = plan.arrays()
+    seg, starts, lens = a["segment_ids"], a["seg_start"], lengths[a["seg_req"]]
+    M = len(seg)
+    QT = -(-M // 128)
+    S = len(a["seg_req"])
+    st = plan.segtab()
+    off = 4 * (1 + S) + (plan.info["num_rows"] + 1 + 3) // 4 * 4
+    order = st[off:off + QT].tolist()
+    assert len(st) == off + (QT + 3) // 4 * 4
+    nch = []
+    for t in range(QT):
+        ss = [s for s in seg[t * 128:(t + 1) * 128] if s >= 0]
+        if not ss:
+            nch.append(0)
+            continue
+        lo, hi = min(starts[s] for s in ss), max(starts[s] + lens[s] for s in ss)
+        kb = lo - lo % 8
+        nch.append(-(-(hi - kb) // 128))
+    assert sorted(order) == list(range(QT))
+    keys = [(-nch[q], q) for q in order]
+    assert keys == sorted(keys)
