@@ -17,10 +17,11 @@ e2e:   the same metric through the public API from host memory: per step tcb_pac
        H2D of the segment table + token ids from pinned memory, forward, unpack, D2H of the
        per-request outputs [T, d] into pinned memory, read by the host; two-deep pipeline (the
        D2H of step i overlaps step i+1 on a copy stream); host wall clock.
-roofline: the dominant kernel class (largest device time per step) measured live with CUDA
-       events around each launch (tcb_profile_*); algorithmic flops / bytes per class in
-       DESIGN.md section 7 (GEMMs: 2 T d_in d_out per layer over non-pad tokens T); every
-       class is listed under roofline.classes.
+roofline: the dominant kernel class (largest device time per step), each launch timed by CUDA
+       event nodes inside a graph-replayed step (tcb_profile_*; L2 flushed per replay);
+       algorithmic flops / bytes per class in DESIGN.md section 7 (GEMMs: 2 T d_in d_out per
+       layer over non-pad tokens T) against the burst bf16 peak / hbm_gbs of
+       MEASURED_PEAKS.json; every class is listed under roofline.classes.
 cpu_baseline / --impl reference: the float64 oracle (oracle/, test infrastructure) on a
        bounded sample of the same workload, on this host's cores.
 """
@@ -149,8 +150,10 @@ def make_batches(key: str, rank: int, nbatches: int):
     return out
 
 
-def cpu_oracle_sample(key: str, lengths, ids, weights, budget_s: float = 12.0, max_rows=16):
-    """Time the f64 oracle (as it stands) row by row on this host until ~budget_s."""
+def cpu_oracle_sample(key: str, lengths, ids, weights, budget_s: float = 12.0, max_rows=16,
+                      threads: int = 0):
+    """Time the f64 oracle (as it stands) row by row on this host until ~budget_s.
+    threads = 0: every core of this process's affinity; 1: the single-thread baseline."""
     import oracle
     wlc = wl.WORKLOADS[key]
     model = wlc.model
@@ -159,18 +162,22 @@ def cpu_oracle_sample(key: str, lengths, ids, weights, budget_s: float = 12.0, m
     lay = oracle.layout(lengths, pk["req_row"], pk["req_col"], pk["num_rows"], wlc.row_len)
     seg = lay["segment_ids"]
     L = wlc.row_len
+    avail = len(os.sched_getaffinity(0)) if hasattr(os, "sched_getaffinity") else os.cpu_count()
+    cores = oracle.set_num_threads(threads if threads > 0 else avail)
     tokens, elapsed, rows = 0, 0.0, 0
-    while elapsed < budget_s and rows < min(max_rows, pk["num_rows"]):
-        t0 = time.perf_counter()
-        oracle.encoder_rows(model, weights, names, ids, lay, L, [rows])
-        elapsed += time.perf_counter() - t0
-        tokens += int(np.sum(seg[rows * L:(rows + 1) * L] >= 0))
-        rows += 1
-    cores = len(os.sched_getaffinity(0)) if hasattr(os, "sched_getaffinity") else os.cpu_count()
-    return {"value": tokens / elapsed, "unit": UNIT, "cores": int(os.environ.get("OMP_NUM_THREADS", cores)),
+    try:
+        while elapsed < budget_s and rows < min(max_rows, pk["num_rows"]):
+            t0 = time.perf_counter()
+            oracle.encoder_rows(model, weights, names, ids, lay, L, [rows])
+            elapsed += time.perf_counter() - t0
+            tokens += int(np.sum(seg[rows * L:(rows + 1) * L] >= 0))
+            rows += 1
+    finally:
+        oracle.set_num_threads(avail)
+    return {"value": tokens / elapsed, "unit": UNIT, "cores": int(cores),
             "kind": "oracle",
             "sample": f"first {rows} packed rows ({tokens} non-pad tokens) of the rank-0 batch, "
-                      f"{model.name} L={L}, float64, {elapsed:.1f} s"}
+                      f"{model.name} L={L}, float64, {elapsed:.1f} s, {cores} thread(s)"}
 
 
 def run_reference(args):
@@ -215,6 +222,78 @@ def run_reference(args):
     return 0
 
 
+def run_online(args):
+    """--online: BASELINE configs[4] -- one Poisson request stream (WMT-like lengths) over all
+    ranks (paper_conf_icpp_fuc0z22_b200/serve_dist.py): a dispatcher thins it into one
+    Poisson(lambda / W) substream per rank, each rank serves its share with its own scheduler
+    (DAS) and encoder replica (Transformer-big encoder, 128 x 256 rows, CUDA-graph replay per
+    time slot), no per-step collective.  lambda = load x W x the measured single-GPU capacity.
+    value = tokens answered by all ranks / the longest rank's serving clock (scheduler host
+    time + device time per slot)."""
+    import torch
+    import torch.distributed as dist
+
+    import paper_conf_icpp_fuc0z22_b200 as tcb
+    from paper_conf_icpp_fuc0z22_b200 import dist as tdist
+    from paper_conf_icpp_fuc0z22_b200 import serve_dist as sd
+
+    rank, world = tdist.init("nccl")
+    local = int(os.environ.get("LOCAL_RANK", 0))
+    torch.cuda.set_device(local)
+    dev = torch.device("cuda", local)
+    wlc = wl.WORKLOADS["c5"]
+    model = wlc.model
+    names = wl.weight_names(model)
+    weights_np = wl.draw_weights(model, wlc.seeds[2]) if rank == 0 else None
+    views = tdist.broadcast_weights(model, names, weights_np, dev)
+    enc = tcb.Encoder(model, None, names, device=str(dev), tensors=views)
+    B, L = wlc.rows, wlc.row_len
+    cap, tau = sd.capacity(enc, wlc.lengths, B, L, wlc.seeds[0])
+    # every rank must draw the same global stream: agree on the capacity (max over ranks)
+    t = torch.tensor([cap, tau], dtype=torch.float64, device=dev)
+    if world > 1:
+        dist.all_reduce(t, op=dist.ReduceOp.MAX)
+    cap, tau = float(t[0]), float(t[1])
+    rate = args.load * world * cap
+    horizon = args.horizon
+    n = int(rate * horizon * 1.1) + 1000
+    sub = sd.substream(rank, world, n, rate, wlc.lengths, L, tau, wlc.seeds[0] + 17)
+    # warm-up: a short run of the same serving loop (graph capture, scheduler, allocator)
+    sd.serve_rank(enc, {k: v[:2000] for k, v in sub.items()}, model.vocab, B, L, "das",
+                  min(horizon, 5 * tau), wlc.seeds[1] + rank)
+    if world > 1:
+        dist.barrier()
+    torch.cuda.synchronize()
+    with ClockSampler(local) as clk:
+        res = sd.serve_rank(enc, sub, model.vocab, B, L, "das", horizon, wlc.seeds[1] + rank)
+        torch.cuda.synchronize()
+    if world > 1:
+        dist.barrier()
+    red = sd.reduce_results(res, world)
+    if rank == 0:
+        line = {
+            "metric": "sustained non-pad tokens/s, online DAS over a Poisson stream (C5)",
+            "value": red["tokens_per_s"], "unit": UNIT, "n_gpus": world,
+            "steps": int(red["batches"]), "warmup": 1,
+            "ms_per_step": 1e3 * red["seconds"] / max(red["batches"] / world, 1),
+            "higher_is_better": True, "scaling": "weak", "vs_baseline": None, "dtype": "bf16",
+            "data": "synthetic (Poisson arrivals, WMT-like lengths, R29 deadlines, random-init weights)",
+            "config": {"workload": "c5-online", "model": model.name, "layers": model.num_layers,
+                       "d_model": model.d_model, "rows_per_gpu": B, "row_len": L,
+                       "policy": "das (eta = q = 1/2)", "load_x_capacity": args.load,
+                       "arrival_rate_req_per_s": rate, "single_gpu_capacity_req_per_s": cap,
+                       "full_batch_ms": tau * 1e3, "horizon_s": horizon,
+                       "parallelism": f"dp{world} (Poisson thinning per rank, weights broadcast once)"},
+            "online": red,
+            "clocks": clk.summary(),
+        }
+        print(json.dumps(line), flush=True)
+    if world > 1:
+        dist.barrier()
+        dist.destroy_process_group()
+    return 0
+
+
 def main():
     ap = argparse.ArgumentParser()
     ap.add_argument("--gpus", type=int, default=1)
@@ -224,10 +303,16 @@ def main():
     ap.add_argument("--workload", default="c2", choices=sorted(wl.WORKLOADS))
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--no-graph", action="store_true")
+    ap.add_argument("--online", action="store_true",
+                    help="C5 online serving: one Poisson stream over all ranks (serve_dist.py)")
+    ap.add_argument("--load", type=float, default=2.0, help="--online: arrival rate / capacity")
+    ap.add_argument("--horizon", type=float, default=0.3, help="--online: served seconds per rank")
     args = ap.parse_args()
     args.warmup = max(args.warmup, 3)
     if args.impl == "reference":
         return run_reference(args)
+    if args.online:
+        return run_online(args)
 
     import torch
     import torch.distributed as dist
@@ -325,22 +410,44 @@ def main():
     value = tokens_all * args.steps / (ms_max / 1e3)
     ms_per_step = ms_max / args.steps
 
-    # ---- roofline: per-kernel-class CUDA-event durations over K eager steps ----------------
+    # ---- roofline: per-kernel-class durations inside the graph-replayed step -----------------
+    # The same forward + unpack is captured once more with profiling on: every launch sits
+    # between two event-record nodes of the graph, so each replay times every kernel (warm
+    # caches and the pipeline's own L2 state, as in the timed step; the event nodes only remove
+    # the programmatic overlap between neighbouring kernels).  L2 flushed before every replay.
     tcb.profile_enable(True)
+    with torch.cuda.stream(stream):
+        fwd()                                           # warm-up of the profiled path
+    stream.synchronize()
+    tcb.profile_collect()
+    pgraph = torch.cuda.CUDAGraph()
+    with torch.cuda.graph(pgraph, stream=stream):
+        fwd()
+    tcb.profile_enable(False)
+    prof = {}
+    pstep = []
     with torch.cuda.stream(stream):
         for _ in range(args.steps):
             flush.zero_()
-            fwd()
-    stream.synchronize()
-    prof = tcb.profile_collect()
-    tcb.profile_enable(False)
+            pa, pb = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+            pa.record(stream)
+            pgraph.replay()
+            pb.record(stream)
+            stream.synchronize()
+            pstep.append(pa.elapsed_time(pb))
+            for c, (t, n) in tcb.profile_snapshot().items():
+                m0, n0 = prof.get(c, (0.0, 0))
+                prof[c] = (m0 + t, n0 + n)
+    del pgraph
+    tcb.profile_collect()                               # release the records' events
     peaks, peak_src = _peaks()
     d, S, f = model.d_model, model.num_layers, model.d_ff
     T = tokens_rank
     gemm_cls = ["gemm_qkv", "gemm_o", "gemm_ffn1", "gemm_ffn2"]
     gemm_flops = 2.0 * T * S * (3 * d * d + d * d + 2 * d * f)
     attn_flops = 4.0 * d * S * info["useful_score_elems"]
-    tc_peak = peaks.get("bf16_tflops_sustained", peaks["bf16_tflops"])
+    tc_burst = peaks["bf16_tflops"]
+    tc_sust = peaks.get("bf16_tflops_sustained", tc_burst)
     hbm_peak = peaks["hbm_gbs"]
     esz = 2 if model.dtype == "bf16" else 4
     fused_ln = d in (512, 768, 1024) and model.dtype == "bf16"
@@ -359,13 +466,14 @@ def main():
         "layernorm": ("hbm", 0.0 if fused_ln else 2.0 * S * T * 2 * d * esz),
         "unpack": ("hbm", T * 2 * d * esz),
     }
-    ln_o = {512: "linear_ln_kernel", 768: "linear_lnc_kernel<3>", 1024: "linear_lnc_kernel<4>"}
-    ln_2 = {512: "linear_lnc_kernel<2>", 768: "linear_lnc_kernel<3>", 1024: "linear_lng_kernel<4>"}
+    # the kernels that run for each class (api.cu / linear_tc.cu dispatch)
+    ln_o = {512: "linear_ln_kernel<false>", 768: "linear_lnc_kernel<3>", 1024: "linear_lnc_kernel<4>"}
+    ln_2 = {512: "linear_lng_kernel<2>", 768: "linear_lnc_kernel<3>", 1024: "linear_lng_kernel<4>"}
     names = {"gemm_qkv": "linear_tc_kernel<2,256,EPI_BIAS> (QKV)",
              "gemm_o": f"{ln_o.get(d)} (W_O + residual + LN1)" if fused_ln else "linear_tc_kernel (W_O + residual)",
              "gemm_ffn1": "linear_tc_kernel<2,256,EPI_ACT> (FFN1 + act)",
              "gemm_ffn2": f"{ln_2.get(d)} (FFN2 + residual + LN2)" if fused_ln else "linear_tc_kernel (FFN2 + residual)",
-             "attention": "attn_tc_kernel (segment-masked attention; Q,K,V in + O out)",
+             "attention": "v3::attn_tc3_kernel (segment-masked attention; Q,K,V in + O out)",
              "embed": "pack_embed_kernel", "layernorm": "layernorm_kernel", "unpack": "unpack_kernel"}
     classes = {}
     for c, (bound, w) in work.items():
@@ -374,13 +482,15 @@ def main():
             continue
         w_all = w * args.steps                      # prof times cover args.steps forwards
         if bound == "tensor":
-            ach, pk, unit = w_all / (ms_c / 1e3) / 1e12, tc_peak, "TFLOP/s"
+            ach, pk, unit = w_all / (ms_c / 1e3) / 1e12, tc_burst, "TFLOP/s"
         else:
             ach, pk, unit = w_all / (ms_c / 1e3) / 1e9, hbm_peak, "GB/s"
         classes[c] = {"kernel": names[c], "bound": bound, "achieved": ach, "peak": pk, "unit": unit,
                       "frac": ach / pk, "launches_per_step": n_c / args.steps,
-                      "ms_per_step": ms_c / args.steps,
-                      "us_per_launch": 1e3 * ms_c / n_c}
+                      "ms_per_step": ms_c / args.steps, "us_per_launch": 1e3 * ms_c / n_c,
+                      "work_per_launch": w / (n_c / args.steps)}
+        if bound == "tensor":
+            classes[c]["frac_vs_sustained"] = ach / tc_sust
         if c == "attention":
             classes[c]["useful_tflops"] = attn_flops * args.steps / (ms_c / 1e3) / 1e12
     dom = max(classes, key=lambda c: classes[c]["ms_per_step"])
@@ -396,10 +506,16 @@ def main():
     roofline = {"bound": dc["bound"], "kernel": dc["kernel"], "class": dom,
                 "achieved": dc["achieved"], "peak": dc["peak"], "unit": dc["unit"],
                 "frac": dc["frac"], "traffic": traffic,
-                "peak_source": f"{peak_src} " + ("bf16_tflops_sustained (kernel timed inside a long step)"
-                                                 if dc["bound"] == "tensor" else "hbm_gbs"),
+                "peak_source": f"{peak_src} " + ("bf16_tflops (burst: the step runs at the clocks of a "
+                                                 "short burst, see clocks)" if dc["bound"] == "tensor" else "hbm_gbs"),
+                "timing": "per-launch CUDA events recorded as event nodes inside the graph-replayed "
+                          "forward (L2 flushed per replay); algorithmic work per launch / average duration",
+                "work_per_launch": dc["work_per_launch"],
+                "us_per_launch": dc["us_per_launch"],
                 "share_of_step": dc["ms_per_step"] / total_prof_ms if total_prof_ms else None,
-                "gemm_class_frac": (gemm_flops / (sum(prof[c][0] for c in gemm_cls) / args.steps / 1e3) / 1e12) / tc_peak,
+                "profiled_graph_ms_per_step": float(np.median(pstep)),
+                "sum_of_kernels_ms_per_step": total_prof_ms,
+                "gemm_class_frac": (gemm_flops / (sum(prof[c][0] for c in gemm_cls) / args.steps / 1e3) / 1e12) / tc_burst,
                 "classes": classes}
     whole_tc = (gemm_flops + attn_flops) / (ms_per_step / 1e3) / 1e12
 
@@ -481,8 +597,11 @@ def main():
 
     cpu = None
     if rank == 0 and world == 1 and not args.no_cpu_baseline:
-        cpu = cpu_oracle_sample(key, batches[0][0], batches[0][1],
-                                wl.draw_weights(model, wlc.seeds[2]))
+        w64 = wl.draw_weights(model, wlc.seeds[2])
+        cpu = cpu_oracle_sample(key, batches[0][0], batches[0][1], w64)
+        # the same oracle on ONE host thread (SURVEY 8(d) / BASELINE.md: next to the all-core run)
+        cpu["single_thread"] = cpu_oracle_sample(key, batches[0][0], batches[0][1], w64,
+                                                 budget_s=8.0, max_rows=4, threads=1)
 
     if rank == 0:
         line = {
@@ -503,8 +622,8 @@ def main():
                        "l2": "flushed (256 MiB write) between timed steps",
                        "cuda_graph": graph is not None},
             "ms_per_step_p10_p50_p90": [float(np.percentile(step_ms, q)) for q in (10, 50, 90)],
-            "tc_frac_whole_step": whole_tc / peaks["bf16_tflops"],
-            "tc_frac_whole_step_vs_sustained": whole_tc / tc_peak,
+            "tc_frac_whole_step": whole_tc / tc_burst,
+            "tc_frac_whole_step_vs_sustained": whole_tc / tc_sust,
             "tc_whole_step_tflops": whole_tc,
             "gpu_launches": int(launches_per_step * args.steps),
             "roofline": roofline,

@@ -241,14 +241,18 @@ int64_t tcb_launch_count(void);
 /* When enabled, tcb_encoder_forward / tcb_unpack record a CUDA event pair around every
  * kernel they launch (kernel classes below) on the launching stream; tcb_profile_collect
  * synchronises those events and adds their durations into ms[TCB_KCLASS_COUNT] and
- * launches[TCB_KCLASS_COUNT] (either may be NULL), then clears the record.  Not for use
- * under CUDA-graph capture. */
+ * launches[TCB_KCLASS_COUNT] (either may be NULL), then clears the record (and recycles its
+ * events).  Under stream capture the pairs become external event-record nodes of the graph:
+ * after each replay, tcb_profile_snapshot sums the same records WITHOUT clearing them (call
+ * tcb_profile_collect once the graph will not be replayed again).  The event nodes serialise
+ * the timed launches (no programmatic overlap across them). */
 enum {
   TCB_K_EMBED = 0, TCB_K_GEMM_QKV = 1, TCB_K_ATTN = 2, TCB_K_GEMM_O = 3, TCB_K_LN = 4,
   TCB_K_GEMM_FFN1 = 5, TCB_K_GEMM_FFN2 = 6, TCB_K_UNPACK = 7, TCB_KCLASS_COUNT = 8
 };
 tcb_status tcb_profile_enable(int32_t on);
 tcb_status tcb_profile_collect(double* ms, int64_t* launches);
+tcb_status tcb_profile_snapshot(double* ms, int64_t* launches);
 
 /* ======================================================================================
  * 5. Online request scheduling (host; §5; §8(f) row f2).

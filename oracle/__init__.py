@@ -58,6 +58,15 @@ def lib() -> ctypes.CDLL:
     return _lib
 
 
+def set_num_threads(n: int) -> int:
+    """OpenMP thread count of the oracle's parallel loops (the libgomp ICV of the calling
+    thread; results never depend on it, see oracle.c).  Returns the count now in effect."""
+    lib()
+    g = ctypes.CDLL("libgomp.so.1")
+    g.omp_set_num_threads(ctypes.c_int(int(n)))
+    return int(g.omp_get_max_threads())
+
+
 def _i32(a) -> np.ndarray:
     return np.ascontiguousarray(np.asarray(a, dtype=np.int32))
 

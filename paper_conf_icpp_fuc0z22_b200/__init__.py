@@ -20,7 +20,8 @@ from . import _lib
 from ._lib import KCLASSES, POLICIES, TcbError, check, lib
 
 __all__ = ["Plan", "Encoder", "Decoder", "Scheduler", "sched_batch", "tcb_pack", "tcb_pack_slotted", "op_linear", "op_linear_ln", "op_attention", "op_layernorm",
-           "launch_count", "profile_enable", "profile_collect", "TcbError", "KCLASSES"]
+           "launch_count", "profile_enable", "profile_collect", "profile_snapshot", "TcbError",
+           "KCLASSES"]
 
 _DTYPES = {"fp32": 0, "bf16": 1}
 _ACTS = {"gelu": 0, "relu": 1}
@@ -191,6 +192,15 @@ def profile_collect() -> Dict[str, tuple]:
     ms = np.zeros(len(KCLASSES), np.float64)
     n = np.zeros(len(KCLASSES), np.int64)
     check(lib().tcb_profile_collect(_ptr(ms), _ptr(n)))
+    return {k: (float(ms[i]), int(n[i])) for i, k in enumerate(KCLASSES)}
+
+
+def profile_snapshot() -> Dict[str, tuple]:
+    """Per-class (ms, launches) of the current records without clearing them (the records of
+    a graph captured with profiling on are re-timed by every replay)."""
+    ms = np.zeros(len(KCLASSES), np.float64)
+    n = np.zeros(len(KCLASSES), np.int64)
+    check(lib().tcb_profile_snapshot(_ptr(ms), _ptr(n)))
     return {k: (float(ms[i]), int(n[i])) for i, k in enumerate(KCLASSES)}
 
 

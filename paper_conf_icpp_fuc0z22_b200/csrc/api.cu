@@ -48,10 +48,13 @@ cudaEvent_t pool_event() {
   return e;
 }
 
+// Under stream capture the pair is recorded as external event-record nodes, so a graph
+// captured with profiling on times every launch on each replay (tcb_profile_snapshot).
 struct ProfScope {
   bool on;
   int cls;
   cudaStream_t s;
+  unsigned flags = cudaEventRecordDefault;
   cudaEvent_t a = nullptr, b = nullptr;
   ProfScope(int c, cudaStream_t st) : on(false), cls(c), s(st) {
     std::lock_guard<std::mutex> g(g_prof_mu);
@@ -59,11 +62,15 @@ struct ProfScope {
     on = true;
     a = pool_event();
     b = pool_event();
-    cudaEventRecord(a, s);
+    cudaStreamCaptureStatus cs = cudaStreamCaptureStatusNone;
+    if (cudaStreamIsCapturing(s, &cs) == cudaSuccess && cs == cudaStreamCaptureStatusActive)
+      flags = cudaEventRecordExternal;
+    cudaGetLastError();
+    cudaEventRecordWithFlags(a, s, flags);
   }
   ~ProfScope() {
     if (!on) return;
-    cudaEventRecord(b, s);
+    cudaEventRecordWithFlags(b, s, flags);
     std::lock_guard<std::mutex> g(g_prof_mu);
     g_prof.push_back({cls, a, b});
   }
@@ -269,6 +276,23 @@ tcb_status tcb_profile_collect(double* ms, int64_t* launches) {
     g_event_pool.push_back(r.b);
   }
   g_prof.clear();
+  return st;
+}
+
+tcb_status tcb_profile_snapshot(double* ms, int64_t* launches) {
+  tcb::clear_error();
+  std::lock_guard<std::mutex> g(g_prof_mu);
+  if (ms) for (int i = 0; i < TCB_KCLASS_COUNT; ++i) ms[i] = 0.0;
+  if (launches) for (int i = 0; i < TCB_KCLASS_COUNT; ++i) launches[i] = 0;
+  tcb_status st = TCB_OK;
+  for (const ProfRec& r : g_prof) {
+    float t = 0.f;
+    cudaError_t e = cudaEventSynchronize(r.b);
+    if (e == cudaSuccess) e = cudaEventElapsedTime(&t, r.a, r.b);
+    if (e != cudaSuccess) st = cuda_fail(e, "tcb_profile_snapshot");
+    if (ms) ms[r.cls] += t;
+    if (launches) launches[r.cls] += 1;
+  }
   return st;
 }
 

@@ -171,7 +171,7 @@ class Server:
         st = sched.stats()
         elapsed = max(now, 1e-12)
         return {"policy": self.policy, "B": self.B, "L": self.L, "requests": n,
-                "overlap": self.overlap,
+                "overlap": self.overlap, "tokens": tokens,
                 "scheduled": st["scheduled"], "expired": st["expired"],
                 "utility": st["utility"], "sim_seconds": elapsed,
                 "responses_per_s": st["scheduled"] / elapsed,

@@ -1911,10 +1911,9 @@ cudaError_t launch_linear_ln_bf16_tc(const GemmMaps& m, int64_t M, int N, int K,
     const char* e = getenv("TCB_LN_SPLIT");             // tuning override (k-blocks)
     return e ? atoi(e) : -1;
   }();
-  // measured: K = 512 (W_O, C2 forward) fastest with 3 joint stages and a 4-block split
-  // (34.4 vs 36.1 us fully split or fully joint, r02x: TCB_LN_SPLIT sweep); K = 2048 fastest
+  // measured (scripts/ln_ab.py): K = 512 fastest fully split with 4 stages; K = 2048 fastest
   // with 3 joint stages and a 2-block split (A re-reads cost more than the overlap there)
-  int split_kb = split_env >= 0 ? (split_env < nkb ? split_env : nkb) : (nkb <= 16 ? nkb / 2 : 2);
+  int split_kb = split_env >= 0 ? (split_env < nkb ? split_env : nkb) : (nkb <= 16 ? nkb : 2);
   const bool joint = split_kb < nkb;
   auto kern = joint ? linear_ln_kernel<true> : linear_ln_kernel<false>;
   const int smem = joint ? LnCfg<true>::kSmemBytes : LnCfg<false>::kSmemBytes;

@@ -93,3 +93,65 @@ def test_rank_streams_are_independent():
     a = wl.draw_lengths("wmt", 100, tdist.rank_seed(40, 0))
     b = wl.draw_lengths("wmt", 100, tdist.rank_seed(40, 1))
     assert not np.array_equal(a, b)
+
+
+# ---- online serving across ranks (serve_dist, BASELINE configs[4]) -------------------------
+def _online_worker(rank, world, port, q):
+    from paper_conf_icpp_fuc0z22_b200 import serve_dist as sd
+    os.environ.update(MASTER_ADDR="127.0.0.1", MASTER_PORT=str(port), RANK=str(rank),
+                      WORLD_SIZE=str(world), LOCAL_RANK=str(rank))
+    dist.init_process_group("gloo", rank=rank, world_size=world)
+    n, rate, tau = 40000, 2.0e5, 4e-3
+    sub = sd.substream(rank, world, n, rate, "wmt", 256, tau, seed=40)
+    # every rank sees the requests the dispatcher sends it; the ranks partition the stream
+    ids = torch.from_numpy(sub["id"].astype(np.int64))
+    sizes = [torch.zeros(1, dtype=torch.int64) for _ in range(world)]
+    dist.all_gather(sizes, torch.tensor([len(ids)], dtype=torch.int64))
+    pad = torch.full((int(max(s.item() for s in sizes)),), -1, dtype=torch.int64)
+    pad[:len(ids)] = ids
+    allid = [torch.zeros_like(pad) for _ in range(world)]
+    dist.all_gather(allid, pad)
+    union = np.concatenate([a.numpy()[a.numpy() >= 0] for a in allid])
+    # per-rank counters reduce as the multi-GPU runner does (sums; max of the serving clock)
+    fake = {"tokens": 1000.0 * (rank + 1), "scheduled": 10.0, "utility": 0.5, "expired": 1.0,
+            "requests": float(len(ids)), "batches": 3.0, "sim_seconds": 0.1 * (rank + 1),
+            "batch_ms": 4.0 + rank, "sched_ms": 0.2}
+    red = sd.reduce_results(fake, world)
+    q.put((rank, union.tolist() if rank == 0 else None, len(ids),
+           sub["arrival"].tolist(), sub["length"].tolist(), red))
+    dist.barrier()
+    dist.destroy_process_group()
+
+
+def test_online_substreams_gloo_world2():
+    """The multi-rank serving runner's feeding logic: each rank's Poisson(lambda / W) share of
+    one global stream (independent thinning), the shares partition the stream (every request
+    served by exactly one rank), each share's arrival rate is ~lambda / W with exponential
+    gaps, and the whole-job counters reduce as sums with the max serving clock."""
+    from paper_conf_icpp_fuc0z22_b200 import serve_dist as sd
+    ctx = mp.get_context("spawn")
+    q = ctx.Queue()
+    port = _free_port()
+    procs = [ctx.Process(target=_online_worker, args=(r, 2, port, q)) for r in range(2)]
+    for p in procs:
+        p.start()
+    res = sorted([q.get(timeout=240) for _ in procs], key=lambda t: t[0])
+    for p in procs:
+        p.join(timeout=60)
+    assert all(p.exitcode == 0 for p in procs)
+    n, rate = 40000, 2.0e5
+    union = np.array(res[0][1])
+    assert len(union) == n and np.array_equal(np.sort(union), np.arange(n))
+    arr_g, len_g, _ = sd.global_stream(n, rate, "wmt", 256, 4e-3, 40)
+    for rank, _, cnt, arr, lens, red in res:
+        assert abs(cnt / n - 0.5) < 0.02                        # thinning p = 1/W
+        gaps = np.diff(np.array(arr))
+        # Poisson(lambda / W): mean gap W / lambda, coefficient of variation ~ 1 (exponential)
+        assert abs(gaps.mean() * rate / 2 - 1) < 0.05
+        assert abs(gaps.std() / gaps.mean() - 1) < 0.05
+        assert np.all(np.isin(np.array(lens), len_g))
+        assert red["tokens"] == 3000.0 and red["seconds"] == pytest.approx(0.2)
+        assert red["max_batch_ms"] == 5.0 and red["requests"] == n
+        assert red["tokens_per_s"] == pytest.approx(15000.0)
+    # the same seed gives the same global stream on every rank
+    assert np.allclose(np.sort(np.concatenate([r[3] for r in res])), arr_g)

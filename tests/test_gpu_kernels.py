@@ -54,7 +54,8 @@ def test_linear_bf16_tcgen05_vs_oracle(M, N, K, epi):
 @pytest.mark.parametrize("M,K,N", [(1, 512, 512), (300, 512, 512), (4133, 512, 512),
                                    (1000, 1024, 512), (1000, 2048, 512), (513, 4096, 512),
                                    (32768, 512, 512), (1, 768, 768), (777, 768, 768),
-                                   (3001, 3072, 768), (300, 1024, 1024), (2049, 4096, 1024),
+                                   (3001, 3072, 768), (32768, 768, 768), (32768, 3072, 768),
+                                   (300, 1024, 1024), (2049, 4096, 1024),
                                    (1, 4096, 1024), (300, 2048, 1024), (32768, 1024, 1024),
                                    (32768, 4096, 1024)])
 def test_linear_ln_fused_vs_oracle(M, K, N):
@@ -79,7 +80,9 @@ def test_linear_ln_fused_vs_oracle(M, K, N):
     ref = oracle.layernorm(z, g, be, 1e-5)
     real = seg >= 0
     err = np.abs(got[real] - ref[real])
-    assert np.all(err <= 2.0 ** -8 * np.abs(ref[real]) + 2e-2), float(err.max())
+    # one bf16 rounding of the output (2^-8 relative) + fp32 statistics / accumulation noise
+    bound = 2.0 ** -8 * np.abs(ref[real]) + 1e-3
+    assert np.all(err <= bound), float(np.max(err / bound))
     assert np.all(got[~real] == 0)
 
 
@@ -268,11 +271,22 @@ def test_layernorm_bf16_vs_oracle(d):
     assert np.all(got[-5:] == 0)
 
 
-@pytest.mark.parametrize("mkey,L", [("toy", 32), ("transformer-base", 128), ("bert-base", 128),
-                                    # ragged last 16-slot chunk of every row (40 = 2 x 16 + 8)
-                                    ("toy", 40), ("bert-base", 40)])
-def test_pack_embed_metadata_bit_exact_and_values(mkey, L):
-    model = wl.MODELS[mkey]
+def _scaled(mkey, pe, scale):
+    import dataclasses
+    m = wl.MODELS[mkey]
+    return dataclasses.replace(m, name=f"{m.name}-{pe}-x{scale:g}", pe=pe, emb_scale=scale)
+
+
+@pytest.mark.parametrize("mkey,L,pe,scale", [("toy", 32, None, None), ("transformer-base", 128, None, None),
+                                             ("bert-base", 128, None, None),
+                                             # ragged last 16-slot chunk of every row (40 = 2 x 16 + 8)
+                                             ("toy", 40, None, None), ("bert-base", 40, None, None),
+                                             # both sinusoidal readings (R1) with emb_scale != 1 (R3)
+                                             ("transformer-base", 128, "sin_paper", 22.627416997969522),
+                                             ("transformer-base", 128, "sin_vaswani", 2.5),
+                                             ("toy", 32, "sin_vaswani", 8.0)])
+def test_pack_embed_metadata_bit_exact_and_values(mkey, L, pe, scale):
+    model = wl.MODELS[mkey] if pe is None else _scaled(mkey, pe, scale)
     w = wl.draw_weights(model, 2)
     names = wl.weight_names(model)
     lengths = np.minimum(wl.draw_lengths("paracrawl", 90, 4), L).astype(np.int32)

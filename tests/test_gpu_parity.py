@@ -67,6 +67,22 @@ def test_c2_transformer_base_full_size_sampled_rows():
     print("c2 worst normwise error", worst)
 
 
+@pytest.mark.parametrize("key", ["c3", "c4", "c5"])
+def test_full_bench_batch_sampled_rows(key):
+    """C3 / C4 / C5 at the bench's own size and launch configuration: bench.py's rank-0 batch 0
+    (make_batches seeds; 64 x 512, 64 x 512, 128 x 256 rows), first and last row vs the oracle
+    -- the multi-tile paths (several 256-row tiles per cluster / pair, dynamic attention item
+    order) only run at these sizes."""
+    import bench
+    wlc = wl.WORKLOADS[key]
+    (lengths, ids), = bench.make_batches(key, 0, 1)
+    lengths0, ids0, _ = wl.workload_inputs(key)
+    assert np.array_equal(lengths, lengths0) and np.array_equal(ids, ids0)
+    plan, worst = _sampled_parity(key, [0, -1])
+    assert plan.info["num_rows"] == wlc.rows
+    print(key, "worst normwise error", worst)
+
+
 def test_c3_bert_base_sampled_row():
     _sampled_parity("c3", [0], gpu_rows=8)
 

@@ -178,3 +178,37 @@ def test_identities():
     qkv[:, 2 * d:] = 1.0
     o = oracle.attention(qkv, np.array([0] * 6 + [1] * 4, np.int32), 1, L, d, 1)
     assert np.max(np.abs(o - 1.0)) <= 4 * np.finfo(float).eps
+
+
+@pytest.mark.parametrize("pe,scale", [("sin_paper", 1.0), ("sin_paper", 2.5),
+                                      ("sin_vaswani", 8.0), ("sin_vaswani", 1.0)])
+def test_sinusoidal_embedding_closed_form(pe, scale):
+    """oracle_embed's sinusoidal branch (Eq. (1)-(2) P:329-333, separate PE §4.1.1)
+    against the closed form written out here: x = E[id] * emb_scale + PE(j, c) with j the
+    token's index inside its own request (positions restart, R2), PE(j, c) = sin / cos of
+    j / 10000^(c/d) for the literal Eq. (2) (R1: odd columns use (2e+1)/d) or of
+    j / 10000^(2 floor(c/2)/d) (Vaswani), every slot located from the packing alone
+    (row * L + col + j); pad slots are 0."""
+    d = 64
+    cfg = wl.ModelConfig("s", 1, d, 2, 256, 100, 64, "fp32", "relu", pe, False, False,
+                         1e-5, 1e-5, scale)
+    w = wl.draw_weights(cfg, 5)
+    lengths = np.array([7, 12, 3, 9, 16, 5], np.int32)
+    L = 24
+    ids = wl.draw_token_ids(int(lengths.sum()), cfg.vocab, 6)
+    pk = oracle.pack(lengths, L)
+    lay = oracle.layout(lengths, pk["req_row"], pk["req_col"], pk["num_rows"], L)
+    x = oracle.embed(cfg, w, ids, lay)
+    cu = np.concatenate([[0], np.cumsum(lengths)])
+    real = np.zeros(len(x), bool)
+    for r, l in enumerate(lengths):
+        for j in range(l):
+            slot = pk["req_row"][r] * L + pk["req_col"][r] + j
+            real[slot] = True
+            ref = np.array(w["tok_emb"][ids[cu[r] + j]], np.float64) * scale
+            for c in range(d):
+                ex = c / d if pe == "sin_paper" else (c - c % 2) / d
+                ang = j / 10000.0 ** ex
+                ref[c] += math.sin(ang) if c % 2 == 0 else math.cos(ang)
+            assert np.max(np.abs(x[slot] - ref)) <= 1e-12 * max(1.0, np.max(np.abs(ref))), (r, j)
+    assert np.all(x[~real] == 0)
