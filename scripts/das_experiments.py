@@ -11,7 +11,7 @@ paper (reading R29): d_n = a_n + U(1, 10) * tau, tau = the full-batch device tim
 
 Every run goes through paper_conf_icpp_fuc0z22_b200.serve.Server (C++ scheduler + CUDA-
 graph replay of the encoder per time slot).  One JSON line per run.
-Usage: python scripts/das_experiments.py [e1|e7|c5|all] [slots]
+Usage: python scripts/das_experiments.py [e1|e7|c5|deadlines|overlap|all] [slots]
 """
 import json
 import os
@@ -59,7 +59,18 @@ def full_batch_ms(enc, lengths, B, L):
     return a.elapsed_time(b) / 10, per_batch
 
 
-def run(enc, model, policy, B, L, rate_mult, var, slots, seed, dist=None, overlap=False):
+# deadline models (the paper gives none, reading R29): budget in units of tau = full-batch time
+DEADLINES = {
+    "u1_10": lambda rng, l, n: rng.uniform(1.0, 10.0, size=n),          # R29 (default)
+    "u1_3": lambda rng, l, n: rng.uniform(1.0, 3.0, size=n),            # tight
+    "const3": lambda rng, l, n: np.full(n, 3.0),                        # one SLA for all
+    "len": lambda rng, l, n: 1.0 + 9.0 * l / 100.0,                     # budget grows with length
+    "inv_len": lambda rng, l, n: 1.0 + 9.0 * (1.0 - l / 100.0),         # short = interactive
+}
+
+
+def run(enc, model, policy, B, L, rate_mult, var, slots, seed, dist=None, overlap=False,
+        deadlines="u1_10"):
     probe = lengths_normal(20000, var, seed + 7) if dist is None else \
         np.minimum(wl.draw_lengths(dist, 20000, seed + 7), L).astype(np.int32)
     tau_ms, per_batch = full_batch_ms(enc, probe, B, L)
@@ -71,14 +82,14 @@ def run(enc, model, policy, B, L, rate_mult, var, slots, seed, dist=None, overla
     arrival = np.cumsum(rng.exponential(1.0 / rate, size=n))
     lengths = lengths_normal(n, var, seed + 1) if dist is None else \
         np.minimum(wl.draw_lengths(dist, n, seed + 1), L).astype(np.int32)
-    deadline = arrival + rng.uniform(1.0, 10.0, size=n) * (tau_ms / 1e3)
+    deadline = arrival + DEADLINES[deadlines](rng, lengths, n) * (tau_ms / 1e3)
     offs = np.concatenate([[0], np.cumsum(lengths)])[:-1].astype(np.int64)
     ids = wl.draw_token_ids(int(lengths.sum()), model.vocab, seed + 2)
     srv = Server(enc, policy, B, L, overlap=overlap)
     res = srv.run(lengths, arrival, deadline, ids, offs, horizon)
     res.update({"model": model.name, "rate_x_capacity": rate_mult, "rate_req_s": rate,
                 "capacity_req_s": cap, "full_batch_ms": tau_ms, "length_var": var,
-                "dist": dist or f"normal(20,{var})", "slots_target": slots})
+                "dist": dist or f"normal(20,{var})", "slots_target": slots, "deadlines": deadlines})
     print(json.dumps(res), flush=True)
     return res
 
@@ -102,6 +113,11 @@ def main():
         for L in (104, 200, 304):
             for pol in POLICIES:
                 run(enc, base, pol, 16, L, 2.0, 20, slots, 400)
+    if what == "deadlines":            # DAS vs SJF under other deadline models (R29 is a guess)
+        for dl in DEADLINES:
+            for B, rm in ((16, 2.0), (64, 1.0), (64, 2.0)):
+                for pol in ("das", "sjf", "fcfs"):
+                    run(enc, base, pol, B, 128, rm, 50, slots, 600, deadlines=dl)
     if what == "overlap":              # serial vs pipelined scheduler + GPU (Server overlap)
         for rm in (0.5, 1.0, 2.0, 3.0):
             for pol in ("das", "fcfs"):
