@@ -106,7 +106,8 @@ tcb_status check_device() {
 constexpr size_t align256(size_t x) { return (x + 255) & ~static_cast<size_t>(255); }
 
 struct WsLayout {
-  size_t seg, qkv, att, z, x1, h, lnst, lncnt, lncnt_per_launch, attn_cnt, total;
+  size_t seg, qkv, att, z, x1, h, lnst, lncnt, lncnt_per_launch, attn_cnt, gemm_cnt, ready,
+      ready_per_launch, total;
 };
 WsLayout ws_layout(const tcb_model_config& c, int64_t M) {
   const size_t es = c.dtype == 0 ? 4 : 2;
@@ -133,6 +134,18 @@ WsLayout ws_layout(const tcb_model_config& c, int64_t M) {
   // (one memset per forward).
   L.attn_cnt = off;
   if (c.dtype == 1) off += align256(sizeof(int32_t) * static_cast<size_t>(c.num_layers));
+  // bf16: dynamic tile counters of the QKV and FFN1 GEMMs (2 per layer) and the 128-row block
+  // readiness flags of the W_O and FFN2 outputs (2 per layer), for the tail overlap of a
+  // GEMM with the LayerNorm GEMM before it
+  L.gemm_cnt = off;
+  L.ready = off;
+  L.ready_per_launch = 0;
+  if (c.dtype == 1) {
+    off += align256(sizeof(int32_t) * 2 * static_cast<size_t>(c.num_layers));
+    L.ready = off;
+    L.ready_per_launch = align256(sizeof(int32_t) * 2 * static_cast<size_t>((M + 255) / 256));
+    off += L.ready_per_launch * 2 * static_cast<size_t>(c.num_layers);
+  }
   L.total = off;
   return L;
 }
@@ -551,6 +564,19 @@ tcb_status forward_impl(const tcb_weights* wc, const tcb_plan* plan, const int32
     if (cudaMemsetAsync(ws + L.lncnt, 0, L.total - L.lncnt, s) != cudaSuccess)
       return fail(TCB_ERR_CUDA, "tcb_encoder_forward: counter reset failed");
     int* attn_cnt = reinterpret_cast<int*>(ws + L.attn_cnt);
+    // Tail overlap (opt-in, TCB_XOVERLAP=1; TCB_XOVERLAP=dyn: dynamic tiles without the
+    // flags): FFN1 starts on the W_O + LN1 rows that are done and the next layer's QKV on the
+    // FFN2 + LN2 rows that are done, with dynamic tile order, while the LayerNorm GEMM before
+    // it finishes its last tiles.  Correct (parity tests pass with it), but measured no faster:
+    // C2 1383 vs 1382 us per step, C3 +1% -- the overlap gains ~25 us per C2
+    // step and the dynamic tile hand-off costs about as much -- so it is off by default.
+    static const char* xov_env = std::getenv("TCB_XOVERLAP");
+    const bool xov_dyn = xov_env != nullptr && L.ready_per_launch > 0;
+    const bool xov = xov_dyn && std::string(xov_env) != "dyn";
+    int* gemm_cnt = reinterpret_cast<int*>(ws + L.gemm_cnt);
+    auto ready = [&](int launch) -> int* {
+      return reinterpret_cast<int*>(ws + L.ready + L.ready_per_launch * launch);
+    };
     for (int l = 0; l < c.num_layers; ++l) {
       NvtxRange nvtx_layer("tcb encoder layer");
       const auto& mp = w->maps[l];
@@ -558,27 +584,36 @@ tcb_status forward_impl(const tcb_weights* wc, const tcb_plan* plan, const int32
       const tcb::k::GemmMaps g_o{aAtt, mp.o, cZ, cX};
       const tcb::k::GemmMaps g_1{aX1, mp.w1, cH, cH};
       const tcb::k::GemmMaps g_2{aH, mp.w2, cZ, cX1};
-      TCB_LAUNCH(TCB_K_GEMM_QKV, s, tcb::k::launch_linear_bf16_tc(g_qkv, M, 3 * d, d,
-                                                                  w->Lf(l, B_QKV), TCB_EPI_BIAS, s));
+      // the previous layer's FFN2 + LN2 signals its rows when fused (xov); layer 0 reads the embedding
+      const bool qkv_x = xov && fuse_ln && l > 0;
+      TCB_LAUNCH(TCB_K_GEMM_QKV, s, tcb::k::launch_linear_bf16_tc(
+                                        g_qkv, M, 3 * d, d, w->Lf(l, B_QKV), TCB_EPI_BIAS, s,
+                                        xov_dyn ? gemm_cnt + 2 * l : nullptr,
+                                        qkv_x ? ready(2 * (l - 1) + 1) : nullptr, 4 * d));
       TCB_LAUNCH(TCB_K_ATTN, s, attention_bf16(M, d, c.num_heads, qkv, seg, segtab, att, attn_cnt + l, s));
       if (fuse_ln) {   // W_O + bias + residual + LN1 in one kernel -> x1
         const tcb::k::GemmMaps g_o_ln{aAtt, mp.o, cX1, cX};
         TCB_LAUNCH(TCB_K_GEMM_O, s, tcb::k::launch_linear_ln_bf16_tc(
                                         g_o_ln, M, d, d, w->Lf(l, B_O), w->Lf(l, LN1_G),
-                                        w->Lf(l, LN1_B), c.ln_eps, seg, s, lnst, lncnt(2 * l)));
+                                        w->Lf(l, LN1_B), c.ln_eps, seg, s, lnst, lncnt(2 * l),
+                                        xov ? ready(2 * l) : nullptr));
       } else {
         TCB_LAUNCH(TCB_K_GEMM_O, s, tcb::k::launch_linear_bf16_tc(g_o, M, d, d, w->Lf(l, B_O),
                                                                   TCB_EPI_BIAS_RESIDUAL, s));
         TCB_LAUNCH(TCB_K_LN, s, tcb::k::launch_layernorm(1, M, d, z, w->Lf(l, LN1_G),
                                                          w->Lf(l, LN1_B), c.ln_eps, seg, x1, s));
       }
-      TCB_LAUNCH(TCB_K_GEMM_FFN1, s, tcb::k::launch_linear_bf16_tc(g_1, M, f, d, w->Lf(l, B_1),
-                                                                   act_epi, s));
+      const bool ffn1_x = xov && fuse_ln;
+      TCB_LAUNCH(TCB_K_GEMM_FFN1, s, tcb::k::launch_linear_bf16_tc(
+                                         g_1, M, f, d, w->Lf(l, B_1), act_epi, s,
+                                         xov_dyn ? gemm_cnt + 2 * l + 1 : nullptr,
+                                         ffn1_x ? ready(2 * l) : nullptr, 4 * d));
       if (fuse_ln) {   // FFN2 + bias + residual + LN2 in one kernel -> X
         const tcb::k::GemmMaps g_2_ln{aH, mp.w2, cX, cX1};
         TCB_LAUNCH(TCB_K_GEMM_FFN2, s, tcb::k::launch_linear_ln_bf16_tc(
                                            g_2_ln, M, d, f, w->Lf(l, B_2), w->Lf(l, LN2_G),
-                                           w->Lf(l, LN2_B), c.ln_eps, seg, s, lnst, lncnt(2 * l + 1)));
+                                           w->Lf(l, LN2_B), c.ln_eps, seg, s, lnst, lncnt(2 * l + 1),
+                                           (xov && l + 1 < c.num_layers) ? ready(2 * l + 1) : nullptr));
       } else {
         TCB_LAUNCH(TCB_K_GEMM_FFN2, s, tcb::k::launch_linear_bf16_tc(g_2, M, d, f, w->Lf(l, B_2),
                                                                      TCB_EPI_BIAS_RESIDUAL, s));

@@ -102,8 +102,15 @@ bool make_tmap_bf16(CUtensorMap* map, const void* ptr, uint64_t rows, uint64_t c
 bool make_gemm_a_map(CUtensorMap* map, const void* A, uint64_t M, uint64_t K);
 bool make_gemm_w_map(CUtensorMap* map, const void* W, uint64_t N, uint64_t K);
 bool make_gemm_c_map(CUtensorMap* map, const void* C, uint64_t M, uint64_t N);
+// tile_counter (one int32, zero at launch): dynamic tile order.  a_ready: readiness flags of
+// A's 128-row blocks written by the still-running previous kernel (see ready_signal in
+// linear_tc.cu; block b is complete at a_target = 4 x the producer's row width); the kernel
+// then skips griddepcontrol.wait -- only for an A produced by the immediately preceding
+// kernel, and a C no earlier kernel still reads.
 cudaError_t launch_linear_bf16_tc(const GemmMaps& maps, int64_t M, int N, int K,
-                                  const float* bias, int epi, cudaStream_t s);
+                                  const float* bias, int epi, cudaStream_t s,
+                                  int* tile_counter = nullptr, const int* a_ready = nullptr,
+                                  int a_target = 0);
 // C = LayerNorm(A W^T + bias + R) * gamma + beta over rows of N = 512 columns (pad rows 0).
 bool linear_ln_supported(int N);
 // lng_stats / lng_cnt (optional scratch, sizes below; cnt zeroed before the launch) select the
@@ -111,7 +118,8 @@ bool linear_ln_supported(int N);
 cudaError_t launch_linear_ln_bf16_tc(const GemmMaps& maps, int64_t M, int N, int K,
                                      const float* bias, const float* gamma, const float* beta,
                                      float eps, const int32_t* seg_ids, cudaStream_t s,
-                                     float2* lng_stats = nullptr, int* lng_cnt = nullptr);
+                                     float2* lng_stats = nullptr, int* lng_cnt = nullptr,
+                                     int* ready_out = nullptr);
 size_t linear_ln_scratch_stats_bytes(int64_t M, int N);
 size_t linear_ln_scratch_cnt_bytes(int64_t M);
 

@@ -54,7 +54,7 @@ struct TcCfg {
   static constexpr int kStages = (225 * 1024 - kEpiBytes) / kStageBytes > 8
                                      ? 8 : (225 * 1024 - kEpiBytes) / kStageBytes;
   static constexpr int kTmemCols = 2 * BN;                  // double-buffered accumulator
-  static constexpr int kBarBytes = 8 * (2 * kStages + 4 + kBufs * kEpiWarps) + 16;
+  static constexpr int kBarBytes = 8 * (2 * kStages + 4 + kBufs * kEpiWarps + 2 * 2 + 2 * 4) + 4 * (2 + 4) + 16;
   static constexpr int kSmemBytes = 1024 + kStages * kStageBytes + kEpiBytes + kBarBytes;
   static_assert(kSmemBytes <= 232448, "shared memory budget");
   static_assert(kTmemCols <= 512, "TMEM budget");
@@ -72,6 +72,11 @@ __device__ __forceinline__ uint32_t cluster_rank() {
 __device__ __forceinline__ uint32_t map_to_rank0(uint32_t saddr) {
   uint32_t r;
   asm volatile("mapa.shared::cluster.u32 %0, %1, 0;" : "=r"(r) : "r"(saddr));
+  return r;
+}
+__device__ __forceinline__ uint32_t mapa_u32(uint32_t saddr, uint32_t rank) {
+  uint32_t r;
+  asm volatile("mapa.shared::cluster.u32 %0, %1, %2;" : "=r"(r) : "r"(saddr), "r"(rank));
   return r;
 }
 __device__ __forceinline__ void cluster_sync() {
@@ -275,6 +280,67 @@ __device__ __forceinline__ uint4 ld_shared_v4(uint32_t addr) {
 __device__ __forceinline__ void mbar_arrive_remote(uint32_t cluster_addr) {
   asm volatile("mbarrier.arrive.shared::cluster.b64 _, [%0];" ::"r"(cluster_addr) : "memory");
 }
+// ---- cross-kernel row readiness (tail overlap of consecutive GEMMs) ------------------------
+// A producer kernel adds, per 128-row block of its output, the number of columns each
+// epilogue warp wrote (32 of the block's rows per warp) to ready[block] once those stores are
+// complete; a consumer that reads the block waits until ready[block] == 4 * N (all columns of
+// all 128 rows), then loads it with TMA.
+__device__ __forceinline__ void ready_signal(int* flag, int cols) {
+  asm volatile("cp.async.bulk.wait_group 0;" ::: "memory");      // this thread's stores landed
+  asm volatile("fence.proxy.async.global;" ::: "memory");
+  asm volatile("red.release.gpu.global.add.s32 [%0], %1;" ::"l"(flag), "r"(cols) : "memory");
+}
+__device__ __forceinline__ void ready_wait(const int* flag, int target) {
+  int v;
+  for (;;) {
+    asm volatile("ld.acquire.gpu.global.b32 %0, [%1];" : "=r"(v) : "l"(flag) : "memory");
+    if (v >= target) break;
+    __nanosleep(64);
+  }
+  asm volatile("fence.proxy.async.global;" ::: "memory");         // before the TMA reads
+}
+// all NB blocks of a tile at once: relaxed polls (no L1 invalidation per poll), then one
+// acquire load each once they are complete
+template <int NB>
+__device__ __forceinline__ void ready_wait_blocks(const int* flag, int target) {
+  for (;;) {
+    bool ok = true;
+#pragma unroll
+    for (int c = 0; c < NB; ++c) {
+      int v;
+      asm volatile("ld.relaxed.gpu.global.b32 %0, [%1];" : "=r"(v) : "l"(flag + c) : "memory");
+      ok &= v >= target;
+    }
+    if (ok) break;
+    __nanosleep(64);
+  }
+#pragma unroll
+  for (int c = 0; c < NB; ++c) {
+    int v;
+    asm volatile("ld.acquire.gpu.global.b32 %0, [%1];" : "=r"(v) : "l"(flag + c) : "memory");
+  }
+}
+// ---- dynamic tile ring (one per CTA; the even CTA of a pair fetches, both consume) ---------
+__device__ __forceinline__ void mbar_wait_acq_cluster(uint64_t* bar, uint32_t parity) {
+  const uint32_t addr = smem_u32(bar);
+  uint32_t done = 0;
+  do {
+    asm volatile(
+        "{\n\t.reg .pred p;\n\t"
+        "mbarrier.try_wait.parity.acquire.cluster.shared::cta.b64 p, [%1], %2;\n\t"
+        "selp.u32 %0, 1, 0, p;\n\t}"
+        : "=r"(done)
+        : "r"(addr), "r"(parity)
+        : "memory");
+  } while (!done);
+}
+__device__ __forceinline__ void mbar_arrive_release_cluster(uint32_t cluster_addr) {
+  asm volatile("mbarrier.arrive.release.cluster.shared::cluster.b64 _, [%0];" ::"r"(cluster_addr)
+               : "memory");
+}
+__device__ __forceinline__ void st_cluster_u32(uint32_t cluster_addr, int v) {
+  asm volatile("st.shared::cluster.u32 [%0], %1;" ::"r"(cluster_addr), "r"(v) : "memory");
+}
 
 // byte offset of 16-byte chunk c of row r in a [32 rows x 64 B] 64B-swizzled box
 __device__ __forceinline__ uint32_t sw64(int r, int c) {
@@ -302,8 +368,20 @@ template <int CG, int BN, int EPI>
 __global__ void __launch_bounds__(kThreads, 1)
 linear_tc_kernel(const __grid_constant__ CUtensorMap tmA, const __grid_constant__ CUtensorMap tmW,
                  const __grid_constant__ CUtensorMap tmC, const __grid_constant__ CUtensorMap tmR,
-                 int M, int N, int K, const float* __restrict__ bias, int raster) {
+                 int M, int N, int K, const float* __restrict__ bias, int raster,
+                 int* __restrict__ tile_counter, const int* __restrict__ a_ready, int a_target) {
+  // tile_counter != NULL: tiles are handed out dynamically (the pair's even CTA grabs the next
+  // index and publishes it through both CTAs' tile rings).  a_ready != NULL: the A rows come
+  // from the previous kernel, which is still finishing (no griddepcontrol.wait): the producer
+  // waits per 128-row block on its readiness flags instead -- with dynamic tiles, CTAs that
+  // start on SMs the previous kernel has left take the ready rows (tail overlap).
   using Cfg = TcCfg<CG, BN, EPI>;
+  // tile ring depth: the scheduler runs at most one tile ahead of the consumers (a deeper ring
+  // lets a pair hoard tiles at the end of the grid -- measured 3-5% slower)
+  constexpr int kTR = 2;
+  // the epilogue warps get their tile indices from their own CTA's producer (a local ring),
+  // so global ring slots are released as soon as the producers and the MMA warp start a tile
+  constexpr int kER = 4;
   constexpr int S = Cfg::kStages;
   constexpr int TILE_M = 128 * CG;
   extern __shared__ uint8_t smem_raw[];
@@ -317,7 +395,13 @@ linear_tc_kernel(const __grid_constant__ CUtensorMap tmA, const __grid_constant_
   uint64_t* tfull = empty + S;                          // [2]
   uint64_t* tempty = tfull + 2;                         // [2] (used on the even CTA)
   uint64_t* rbar = tempty + 2;                          // [8 warps][chunks] residual loads
-  uint32_t* tmem_slot = reinterpret_cast<uint32_t*>(rbar + Cfg::kBufs * kEpiWarps);
+  uint64_t* trf = rbar + Cfg::kBufs * kEpiWarps;        // [kTR] tile ring: index published
+  uint64_t* tre = trf + kTR;                            // [kTR] all consumers read it (even CTA)
+  uint64_t* erf = tre + kTR;                            // [kER] this CTA's producer -> its epilogue
+  uint64_t* ere = erf + kER;
+  int* tring = reinterpret_cast<int*>(ere + kER);       // [kTR]
+  int* ering = tring + kTR;                             // [kER]
+  uint32_t* tmem_slot = reinterpret_cast<uint32_t*>(ering + kER);
 
   const int warp = threadIdx.x >> 5;
   const int lane = threadIdx.x & 31;
@@ -336,6 +420,9 @@ linear_tc_kernel(const __grid_constant__ CUtensorMap tmA, const __grid_constant_
     for (int i = 0; i < S; ++i) { mbar_init(&full[i], 1); mbar_init(&empty[i], 1); }
     for (int i = 0; i < 2; ++i) { mbar_init(&tfull[i], 1); mbar_init(&tempty[i], CG * kEpiWarps); }
     for (int i = 0; i < Cfg::kBufs * kEpiWarps; ++i) mbar_init(&rbar[i], 1);
+    // consumers of a global ring slot: the producers of both CTAs + the MMA warp
+    for (int i = 0; i < kTR; ++i) { mbar_init(&trf[i], 1); mbar_init(&tre[i], CG + 1); }
+    for (int i = 0; i < kER; ++i) { mbar_init(&erf[i], 1); mbar_init(&ere[i], kEpiWarps); }
     asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
   }
   if (warp == 2) {
@@ -356,10 +443,106 @@ linear_tc_kernel(const __grid_constant__ CUtensorMap tmA, const __grid_constant_
   // A / residual come from the previous kernel and C may still be read by it: everything but
   // the producer waits for it here (PDL).  The weights are constant, so the producer issues the
   // W halves of the first S stages BEFORE its wait -- their latency hides in that kernel's tail.
-  if (warp != 0) pdl_wait();
+  const bool xover = a_ready != nullptr;
+  const bool dyn = tile_counter != nullptr;
+  // the scheduler warp touches only its tile counter (zeroed before the forward): no wait
+  if (warp != 0 && !(warp == 3 && dyn) && !xover) pdl_wait();
   pdl_trigger();
+  const uint32_t tre0 = CG == 2 ? map_to_rank0(smem_u32(tre)) : smem_u32(tre);
+  // a consumer's next tile from the ring (whole warp; lane 0 releases the slot)
+  auto ring_next = [&](int& rs, uint32_t& rph) -> int {
+    mbar_wait_acq_cluster(&trf[rs], rph);
+    const int t = *reinterpret_cast<volatile int*>(&tring[rs]);
+    __syncwarp();
+    if (lane == 0) mbar_arrive_remote(tre0 + 8u * rs);
+    if (++rs == kTR) { rs = 0; rph ^= 1; }
+    return t;
+  };
 
-  if (warp == 0) {
+  if (warp == 3 && dyn) {
+    // ===== tile scheduler (even CTA, dynamic tiles): grabs the next tile index, waits until
+    // its A rows are ready (tail overlap), publishes it into both CTAs' rings.  Kept off the
+    // TMA-issuing thread: the release fences of a cross-CTA publish would drain that
+    // thread's outstanding copies. =====
+    if (rank == 0 && lane == 0) {
+      int rs = 0;
+      uint32_t rph = 0;
+      uint32_t seen[4] = {0u, 0u, 0u, 0u};         // m-blocks already seen ready (first 128)
+      for (;;) {
+        const int t = atomicAdd(tile_counter, 1);
+        if (xover && t < num_tiles) {
+          int m_blk, n_blk;
+          tile_coords(t, m_blocks, n_blocks, raster, m_blk, n_blk);
+          const bool cached = m_blk < 128 && ((seen[m_blk >> 5] >> (m_blk & 31)) & 1u);
+          if (!cached) {
+            ready_wait_blocks<CG>(a_ready + m_blk * CG, a_target);
+            if (m_blk < 128) seen[m_blk >> 5] |= 1u << (m_blk & 31);
+          }
+        }
+        mbar_wait(&tre[rs], rph ^ 1);
+        tring[rs] = t;
+        if constexpr (CG == 2) {
+          st_cluster_u32(mapa_u32(smem_u32(&tring[rs]), 1), t);
+          mbar_arrive_release_cluster(mapa_u32(smem_u32(&trf[rs]), 1));
+        }
+        mbar_arrive_release_cluster(smem_u32(&trf[rs]));
+        if (++rs == kTR) { rs = 0; rph ^= 1; }
+        if (t >= num_tiles) break;
+      }
+    }
+  } else if (warp == 0 && dyn) {
+    // ===== TMA producer, dynamic tiles (from the ring) =====
+    if (lane == 0) {
+      const uint32_t full0 = CG == 2 ? map_to_rank0(smem_u32(full)) : smem_u32(full);
+      int stage = 0, rs = 0, es = 0;
+      uint32_t phase = 0, rph = 0, eph = 0;
+      bool first = true;
+      for (;;) {
+        mbar_wait_acq_cluster(&trf[rs], rph);
+        const int tile = *reinterpret_cast<volatile int*>(&tring[rs]);
+        mbar_arrive_remote(tre0 + 8u * rs);
+        if (++rs == kTR) { rs = 0; rph ^= 1; }
+        mbar_wait(&ere[es], eph ^ 1);             // this CTA's epilogue: local hand-off
+        ering[es] = tile;
+        asm volatile("mbarrier.arrive.shared::cta.b64 _, [%0];" ::"r"(smem_u32(&erf[es])) : "memory");
+        if (++es == kER) { es = 0; eph ^= 1; }
+        if (tile >= num_tiles) {
+          if (first && !xover) pdl_wait();
+          break;
+        }
+        int m_blk, n_blk;
+        tile_coords(tile, m_blocks, n_blocks, raster, m_blk, n_blk);
+        const int a_row = m_blk * TILE_M + static_cast<int>(rank) * 128;
+        const int b_row = n_blk * BN + static_cast<int>(rank) * Cfg::kBRows;
+        // first tile without readiness flags: its W k-blocks (constant) go out before the
+        // wait for the previous kernel, as in the static order
+        int npre = 0;
+        if (first && !xover) {
+          for (; npre < num_kb && npre < S; ++npre) {
+            if (rank == 0) mbar_expect_tx(&full[npre], CG * Cfg::kStageBytes);
+            tma_load_2d<CG>(sB + npre * Cfg::kBBytes, &tmW, full0 + 8u * npre, npre * BK, b_row);
+          }
+          pdl_wait();
+        }
+        first = false;
+        // the scheduler saw the A rows' flags (gpu-scope acquire) before publishing: order
+        // this thread's async-proxy reads after that
+        if (xover) asm volatile("fence.proxy.async.global;" ::: "memory");
+        for (int kb = 0; kb < num_kb; ++kb) {
+          const uint32_t fb = full0 + 8u * stage;
+          if (kb >= npre) {
+            mbar_wait(&empty[stage], phase ^ 1);
+            if (rank == 0) mbar_expect_tx(&full[stage], CG * Cfg::kStageBytes);
+            tma_load_2d<CG>(sB + stage * Cfg::kBBytes, &tmW, fb, kb * BK, b_row);
+          }
+          tma_load_2d<CG>(sA + stage * Cfg::kABytes, &tmA, fb, kb * BK, a_row);
+          if (++stage == S) { stage = 0; phase ^= 1; }
+        }
+      }
+    } else if (!xover) {
+      pdl_wait();
+    }
+  } else if (warp == 0) {
     // ===== TMA producer (both CTAs of a pair load their own halves) =====
     if (lane == 0) {
       const uint32_t full0 = CG == 2 ? map_to_rank0(smem_u32(full)) : smem_u32(full);
@@ -409,7 +592,11 @@ linear_tc_kernel(const __grid_constant__ CUtensorMap tmA, const __grid_constant_
       uint32_t phase = 0;
       int acc = 0;
       uint32_t acc_phase = 0;
-      for (int tile = cluster_id; tile < num_tiles; tile += num_clusters) {
+      int rs = 0;
+      uint32_t rph = 0;
+      for (int k = 0;; ++k) {
+        const int tile = dyn ? ring_next(rs, rph) : cluster_id + k * num_clusters;
+        if (tile >= num_tiles) break;
 #ifdef TCB_GEMM_PROBE
         long long t0 = clock64();
 #endif
@@ -467,7 +654,18 @@ linear_tc_kernel(const __grid_constant__ CUtensorMap tmA, const __grid_constant_
     const uint32_t tempty0 = CG == 2 ? map_to_rank0(smem_u32(tempty)) : smem_u32(tempty);
     int acc = 0;
     uint32_t acc_phase = 0;
-    for (int tile = cluster_id; tile < num_tiles; tile += num_clusters) {
+    int es = 0;
+    uint32_t eph = 0;
+    for (int k = 0;; ++k) {
+      int tile = cluster_id + k * num_clusters;
+      if (dyn) {
+        mbar_wait(&erf[es], eph);
+        tile = *reinterpret_cast<volatile int*>(&ering[es]);
+        __syncwarp();
+        if (lane == 0) asm volatile("mbarrier.arrive.shared::cta.b64 _, [%0];" ::"r"(smem_u32(&ere[es])) : "memory");
+        if (++es == kER) { es = 0; eph ^= 1; }
+      }
+      if (tile >= num_tiles) break;
       int m_blk, n_blk;
       tile_coords(tile, m_blocks, n_blocks, raster, m_blk, n_blk);
       const int row0 = m_blk * TILE_M + static_cast<int>(rank) * 128 + q * 32;
@@ -657,7 +855,7 @@ linear_ln_kernel(const __grid_constant__ CUtensorMap tmA, const __grid_constant_
                  const __grid_constant__ CUtensorMap tmC, const __grid_constant__ CUtensorMap tmR,
                  int M, int K, const float* __restrict__ bias, const float* __restrict__ gamma,
                  const float* __restrict__ beta, float eps, const int32_t* __restrict__ seg_ids,
-                 int split_kb) {
+                 int split_kb, int* __restrict__ ready_out) {
   constexpr int S = LnCfg<JOINT>::kStages;
   constexpr int kLnStageBytes = LnCfg<JOINT>::kStageBytes;
   constexpr int kHalfBytes = 128 * BK * 2;
@@ -809,6 +1007,7 @@ linear_ln_kernel(const __grid_constant__ CUtensorMap tmA, const __grid_constant_
     uint32_t tphase = 0;
     // chunk j (0..3): half j>>1, columns h*256 + part*64 + (j&1)*32
     auto col_of = [&](int j) { return (j >> 1) * 256 + part * 64 + (j & 1) * 32; };
+    int prev_blk = -1;                            // 128-row block of the previous tile
 #ifdef TCB_LN_PROBE
     long long e0 = clock64(), e_tfull = 0, e_res = 0, e_p1 = 0, e_bar = 0, e_p2 = 0, e_st = 0;
 #endif
@@ -819,7 +1018,13 @@ linear_ln_kernel(const __grid_constant__ CUtensorMap tmA, const __grid_constant_
       const int row0 = tile * 256 + static_cast<int>(rank) * 128 + q * 32;
       const int64_t grow = static_cast<int64_t>(row0) + lane;
       const bool pad = grow >= M || (seg_ids && __ldg(&seg_ids[grow]) < 0);
-      if (lane == 0) bulk_wait_read<0>();         // previous tile's stores have read the buffers
+      // previous tile's stores have read the buffers (and, when the next kernel waits per
+      // 128-row block, have landed: signal that block's 128 columns of this warp)
+      if (lane == 0) {
+        if (ready_out && prev_blk >= 0) ready_signal(ready_out + prev_blk, 128);
+        else bulk_wait_read<0>();
+      }
+      prev_blk = tile * 2 + static_cast<int>(rank);
       __syncwarp();
       if (lane == 0) {
 #pragma unroll
@@ -983,7 +1188,10 @@ linear_ln_kernel(const __grid_constant__ CUtensorMap tmA, const __grid_constant_
 #endif
       tphase ^= 1;
     }
-    if (lane == 0) bulk_wait_all();
+    if (lane == 0) {
+      if (ready_out && prev_blk >= 0) ready_signal(ready_out + prev_blk, 128);
+      else bulk_wait_all();
+    }
 #ifdef TCB_LN_PROBE
     if (lane == 0 && ew == 0 && blockIdx.x < 6)
       printf("lnprobe epi cta %d total %lld pass1 %lld (wait_tfull %lld wait_res %lld) bar %lld pass2 %lld tiles %d\n",
@@ -1078,7 +1286,8 @@ __global__ void __launch_bounds__(kLncThreads, 1)
 linear_lnc_kernel(const __grid_constant__ CUtensorMap tmA, const __grid_constant__ CUtensorMap tmW,
                   const __grid_constant__ CUtensorMap tmC, const __grid_constant__ CUtensorMap tmR,
                   int M, int K, const float* __restrict__ bias, const float* __restrict__ gamma,
-                  const float* __restrict__ beta, float eps, const int32_t* __restrict__ seg_ids) {
+                  const float* __restrict__ beta, float eps, const int32_t* __restrict__ seg_ids,
+                  int* __restrict__ ready_out) {
   using Cfg = LncCfg<P>;
   constexpr int S = Cfg::kStages;
   constexpr int kABytes = 128 * BK * 2;
@@ -1192,6 +1401,7 @@ linear_lnc_kernel(const __grid_constant__ CUtensorMap tmA, const __grid_constant
     const uint32_t tempty0 = mapa_rank(smem_u32(tempty), lead);
     int acc = 0;
     uint32_t acc_phase = 0, rphase = 0;
+    int prev_blk = -1;                            // 128-row block of the previous tile
     for (int tile = cluster_id; tile < num_tiles; tile += num_clusters) {
       const int row0 = tile * 256 + static_cast<int>(r) * 128 + q * 32;
       const int col0 = static_cast<int>(p) * 256 + cg * (32 * kLncChunks);
@@ -1200,9 +1410,14 @@ linear_lnc_kernel(const __grid_constant__ CUtensorMap tmA, const __grid_constant
       // this tile's phase of the statistics barrier completes once all 2P x 128 partials
       // (8 B each, from this CTA and its P-1 peers) have landed
       if (ew == 0 && lane == 0) mbar_expect_tx(&sfull[acc], Cfg::kContrib * 128 * 8);
-      // the previous tile's stores have read the staging buffers: prefetch this tile's
-      // residual chunks into them while the MMAs run
-      if (lane == 0) bulk_wait_read<0>();
+      // the previous tile's stores have read the staging buffers (and landed, when the next
+      // kernel waits per 128-row block: signal this warp's columns of it): prefetch this
+      // tile's residual chunks into them while the MMAs run
+      if (lane == 0) {
+        if (ready_out && prev_blk >= 0) ready_signal(ready_out + prev_blk, 32 * kLncChunks);
+        else bulk_wait_read<0>();
+      }
+      prev_blk = tile * 2 + static_cast<int>(r);
       __syncwarp();
       if (lane == 0) {
 #pragma unroll
@@ -1343,7 +1558,10 @@ linear_lnc_kernel(const __grid_constant__ CUtensorMap tmA, const __grid_constant
       acc ^= 1;
       if (acc == 0) acc_phase ^= 1;
     }
-    if (lane == 0) bulk_wait_all();
+    if (lane == 0) {
+      if (ready_out && prev_blk >= 0) ready_signal(ready_out + prev_blk, 32 * kLncChunks);
+      else bulk_wait_all();
+    }
   }
   __syncwarp();
   tc_fence_before();
@@ -1371,7 +1589,7 @@ linear_lng_kernel(const __grid_constant__ CUtensorMap tmA, const __grid_constant
                   const __grid_constant__ CUtensorMap tmC, const __grid_constant__ CUtensorMap tmR,
                   int M, int K, const float* __restrict__ bias, const float* __restrict__ gamma,
                   const float* __restrict__ beta, float eps, const int32_t* __restrict__ seg_ids,
-                  float2* __restrict__ gstats, int* __restrict__ gcnt) {
+                  float2* __restrict__ gstats, int* __restrict__ gcnt, int* __restrict__ ready_out) {
   constexpr int kStageBytes = 2 * 128 * BK * 2;
   constexpr int kEpiBytes = kLncEpiWarps * kLncChunks * kStageBufBytes;
   constexpr int S = (227 * 1024 - 1024 - kEpiBytes - 1024) / kStageBytes;
@@ -1483,6 +1701,7 @@ linear_lng_kernel(const __grid_constant__ CUtensorMap tmA, const __grid_constant
     long long e0 = clock64(), e_tfull = 0, e_p1 = 0, e_x = 0, e_p2 = 0;
     int nunits = 0;
 #endif
+    int prev_blk = -1;                            // 128-row block of the previous unit
     for (int u = pair; u < num_units; u += num_pairs) {
       const int t = u / P, p = u % P;
 #ifdef TCB_LN_PROBE
@@ -1494,7 +1713,11 @@ linear_lng_kernel(const __grid_constant__ CUtensorMap tmA, const __grid_constant
       const int col0 = p * 256 + cg * (32 * kLncChunks);
       const int64_t grow = static_cast<int64_t>(row0) + lane;
       const bool pad = grow >= M || (seg_ids && __ldg(&seg_ids[grow]) < 0);
-      if (lane == 0) bulk_wait_read<0>();
+      if (lane == 0) {
+        if (ready_out && prev_blk >= 0) ready_signal(ready_out + prev_blk, 32 * kLncChunks);
+        else bulk_wait_read<0>();
+      }
+      prev_blk = t * 2 + static_cast<int>(r);
       __syncwarp();
       if (lane == 0) {
 #pragma unroll
@@ -1650,7 +1873,10 @@ linear_lng_kernel(const __grid_constant__ CUtensorMap tmA, const __grid_constant
       acc ^= 1;
       if (acc == 0) acc_phase ^= 1;
     }
-    if (lane == 0) bulk_wait_all();
+    if (lane == 0) {
+      if (ready_out && prev_blk >= 0) ready_signal(ready_out + prev_blk, 32 * kLncChunks);
+      else bulk_wait_all();
+    }
 #ifdef TCB_LN_PROBE
     if (lane == 0 && ew == 0 && blockIdx.x < 6)
       printf("lngprobe epi cta %d total %lld wait_tfull %lld pass1 %lld exchange %lld pass2 %lld units %d\n",
@@ -1694,7 +1920,8 @@ int num_sms() {
 }
 
 template <int CG, int BN, int EPI>
-cudaError_t launch_tc(const GemmMaps& m, int M, int N, int K, const float* bias, cudaStream_t s) {
+cudaError_t launch_tc(const GemmMaps& m, int M, int N, int K, const float* bias, cudaStream_t s,
+                      int* tile_counter, const int* a_ready, int a_target) {
   using Cfg = TcCfg<CG, BN, EPI>;
   auto kern = linear_tc_kernel<CG, BN, EPI>;
   static bool attr_set = false;  // idempotent if raced
@@ -1721,17 +1948,18 @@ cudaError_t launch_tc(const GemmMaps& m, int M, int N, int K, const float* bias,
   cfg.numAttrs = 1;
   if (pdl_enabled()) pdl_attr(attr[cfg.numAttrs++]);
   static const int raster = std::getenv("TCB_GEMM_RASTER") ? std::atoi(std::getenv("TCB_GEMM_RASTER")) : 8;
-  return cudaLaunchKernelEx(&cfg, kern, m.a, m.w, m.c, m.r, M, N, K, bias, raster);
+  return cudaLaunchKernelEx(&cfg, kern, m.a, m.w, m.c, m.r, M, N, K, bias, raster, tile_counter,
+                            a_ready, a_target);
 }
 
 template <int CG, int BN>
 cudaError_t dispatch_epi(const GemmMaps& m, int M, int N, int K, const float* bias, int epi,
-                         cudaStream_t s) {
+                         cudaStream_t s, int* tc, const int* ar, int at) {
   switch (epi) {
-    case TCB_EPI_BIAS: return launch_tc<CG, BN, TCB_EPI_BIAS>(m, M, N, K, bias, s);
-    case TCB_EPI_BIAS_GELU: return launch_tc<CG, BN, TCB_EPI_BIAS_GELU>(m, M, N, K, bias, s);
-    case TCB_EPI_BIAS_RELU: return launch_tc<CG, BN, TCB_EPI_BIAS_RELU>(m, M, N, K, bias, s);
-    case TCB_EPI_BIAS_RESIDUAL: return launch_tc<CG, BN, TCB_EPI_BIAS_RESIDUAL>(m, M, N, K, bias, s);
+    case TCB_EPI_BIAS: return launch_tc<CG, BN, TCB_EPI_BIAS>(m, M, N, K, bias, s, tc, ar, at);
+    case TCB_EPI_BIAS_GELU: return launch_tc<CG, BN, TCB_EPI_BIAS_GELU>(m, M, N, K, bias, s, tc, ar, at);
+    case TCB_EPI_BIAS_RELU: return launch_tc<CG, BN, TCB_EPI_BIAS_RELU>(m, M, N, K, bias, s, tc, ar, at);
+    case TCB_EPI_BIAS_RESIDUAL: return launch_tc<CG, BN, TCB_EPI_BIAS_RESIDUAL>(m, M, N, K, bias, s, tc, ar, at);
     default: return cudaErrorInvalidValue;
   }
 }
@@ -1744,7 +1972,8 @@ bool linear_ln_supported(int N) { return N == 512 || N == 768 || N == 1024; }
 // TCB_LN_KERNEL=cluster).
 template <int P>
 cudaError_t launch_lnc(const GemmMaps& m, int M, int K, const float* bias, const float* gamma,
-                       const float* beta, float eps, const int32_t* seg_ids, cudaStream_t s) {
+                       const float* beta, float eps, const int32_t* seg_ids, cudaStream_t s,
+                       int* ready_out) {
   using Cfg = LncCfg<P>;
   auto kern = linear_lnc_kernel<P>;
   static int max_clusters = 0;
@@ -1776,7 +2005,8 @@ cudaError_t launch_lnc(const GemmMaps& m, int M, int K, const float* bias, const
   const int clusters = tiles < max_clusters ? tiles : max_clusters;
   cfg.gridDim = dim3(2 * P * clusters);
   if (pdl_enabled()) pdl_attr(attr[cfg.numAttrs++]);
-  return cudaLaunchKernelEx(&cfg, kern, m.a, m.w, m.c, m.r, M, K, bias, gamma, beta, eps, seg_ids);
+  return cudaLaunchKernelEx(&cfg, kern, m.a, m.w, m.c, m.r, M, K, bias, gamma, beta, eps, seg_ids,
+                            ready_out);
 }
 
 // The L2-exchange kernel (clusters of one pair, every pair of the GPU).  `stats` holds
@@ -1784,7 +2014,7 @@ cudaError_t launch_lnc(const GemmMaps& m, int M, int K, const float* bias, const
 template <int P>
 cudaError_t launch_lng(const GemmMaps& m, int M, int K, const float* bias, const float* gamma,
                        const float* beta, float eps, const int32_t* seg_ids, float2* stats,
-                       int* cnt, cudaStream_t s) {
+                       int* cnt, cudaStream_t s, int* ready_out) {
   constexpr int kStageBytes = 2 * 128 * BK * 2;
   constexpr int kEpiBytes = kLncEpiWarps * kLncChunks * kStageBufBytes;
   constexpr int S = (227 * 1024 - 1024 - kEpiBytes - 1024) / kStageBytes;
@@ -1818,7 +2048,7 @@ cudaError_t launch_lng(const GemmMaps& m, int M, int K, const float* bias, const
   // The P units of a tile must sit on P distinct pairs (a unit waits for its tile's other
   // units; two on one pair would wait for themselves): with fewer co-resident pairs than P
   // (an SM-limited context) use the cluster kernel instead.
-  if (max_pairs < P) return launch_lnc<P>(m, M, K, bias, gamma, beta, eps, seg_ids, s);
+  if (max_pairs < P) return launch_lnc<P>(m, M, K, bias, gamma, beta, eps, seg_ids, s, ready_out);
   const int units = ((M + 255) / 256) * P;
   const int pairs = units < max_pairs ? units : max_pairs;
   cfg.gridDim = dim3(2 * pairs);
@@ -1836,7 +2066,7 @@ cudaError_t launch_lng(const GemmMaps& m, int M, int K, const float* bias, const
     ++cfg.numAttrs;
   }
   cudaError_t e = cudaLaunchKernelEx(&cfg, kern, m.a, m.w, m.c, m.r, M, K, bias, gamma, beta, eps,
-                                     seg_ids, stats, cnt);
+                                     seg_ids, stats, cnt, ready_out);
   if (coop == -1) {
     coop = e == cudaSuccess ? 1 : 0;
     if (std::getenv("TCB_VERBOSE"))
@@ -1846,7 +2076,7 @@ cudaError_t launch_lng(const GemmMaps& m, int M, int K, const float* bias, const
       cudaGetLastError();
       --cfg.numAttrs;
       e = cudaLaunchKernelEx(&cfg, kern, m.a, m.w, m.c, m.r, M, K, bias, gamma, beta, eps, seg_ids,
-                             stats, cnt);
+                             stats, cnt, ready_out);
     }
   }
   return e;
@@ -1870,7 +2100,7 @@ bool pdl_enabled() {
 cudaError_t launch_linear_ln_bf16_tc(const GemmMaps& m, int64_t M, int N, int K,
                                      const float* bias, const float* gamma, const float* beta,
                                      float eps, const int32_t* seg_ids, cudaStream_t s,
-                                     float2* lng_stats, int* lng_cnt) {
+                                     float2* lng_stats, int* lng_cnt, int* ready_out) {
   if (M == 0) return cudaSuccess;
   // d = 512 / 1024, K >= 2d (FFN2) with scratch: the L2-exchange kernel on all 74 pairs (the
   // 4- / 8-CTA cluster kernel fits on 132 / 120 SMs only): C4/C5 FFN2 262 -> 218 us.  At K = d (W_O) the
@@ -1885,13 +2115,13 @@ cudaError_t launch_linear_ln_bf16_tc(const GemmMaps& m, int64_t M, int N, int K,
   if (lng_stats && lng_cnt && ln_env != 1) {
     if (N == 1024 && (K >= 2 * N || ln_env == 2))
       return launch_lng<4>(m, static_cast<int>(M), K, bias, gamma, beta, eps, seg_ids, lng_stats,
-                           lng_cnt, s);
+                           lng_cnt, s, ready_out);
     if (N == 512 && K >= 2 * N)             // C2 FFN2: 73.4 -> 71.0 us (148 vs 132 SMs)
       return launch_lng<2>(m, static_cast<int>(M), K, bias, gamma, beta, eps, seg_ids, lng_stats,
-                           lng_cnt, s);
+                           lng_cnt, s, ready_out);
     if (N == 768 && ln_env == 2)
       return launch_lng<3>(m, static_cast<int>(M), K, bias, gamma, beta, eps, seg_ids, lng_stats,
-                           lng_cnt, s);
+                           lng_cnt, s, ready_out);
   }
   // d = 512: the single-pair kernel measured 2% faster per forward (C2) than the 4-CTA
   // cluster kernel; TCB_LN_KERNEL=cluster selects the cluster kernel there too (A/B)
@@ -1900,12 +2130,12 @@ cudaError_t launch_linear_ln_bf16_tc(const GemmMaps& m, int64_t M, int N, int K,
     return !(e && std::string(e) == "cluster");
   }();
   const int Mi = static_cast<int>(M);
-  if (N == 768) return launch_lnc<3>(m, Mi, K, bias, gamma, beta, eps, seg_ids, s);
-  if (N == 1024) return launch_lnc<4>(m, Mi, K, bias, gamma, beta, eps, seg_ids, s);
+  if (N == 768) return launch_lnc<3>(m, Mi, K, bias, gamma, beta, eps, seg_ids, s, ready_out);
+  if (N == 1024) return launch_lnc<4>(m, Mi, K, bias, gamma, beta, eps, seg_ids, s, ready_out);
   if (N != kLnN) return cudaErrorInvalidValue;
   // K >= 1024 (FFN2): the cluster kernel measured faster (64.1 vs 66.6 us at K = 2048);
   // K = 512 (W_O): the single pair (32.3 vs 34.9 us)
-  if (!pair_512 || K >= 1024) return launch_lnc<2>(m, Mi, K, bias, gamma, beta, eps, seg_ids, s);
+  if (!pair_512 || K >= 1024) return launch_lnc<2>(m, Mi, K, bias, gamma, beta, eps, seg_ids, s, ready_out);
   const int nkb = K / BK;
   static const int split_env = [] {
     const char* e = getenv("TCB_LN_SPLIT");             // tuning override (k-blocks)
@@ -1941,7 +2171,7 @@ cudaError_t launch_linear_ln_bf16_tc(const GemmMaps& m, int64_t M, int N, int K,
   cfg.numAttrs = 1;
   if (pdl_enabled()) pdl_attr(attr[cfg.numAttrs++]);
   return cudaLaunchKernelEx(&cfg, kern, m.a, m.w, m.c, m.r, static_cast<int>(M), K, bias, gamma,
-                            beta, eps, seg_ids, split_kb);
+                            beta, eps, seg_ids, split_kb, ready_out);
 }
 
 bool make_tmap_bf16(CUtensorMap* map, const void* ptr, uint64_t rows, uint64_t cols,
@@ -1988,15 +2218,18 @@ GemmShape linear_tc_shape(int N) {
 }
 
 cudaError_t launch_linear_bf16_tc(const GemmMaps& m, int64_t M, int N, int K, const float* bias,
-                                  int epi, cudaStream_t s) {
+                                  int epi, cudaStream_t s, int* tile_counter, const int* a_ready,
+                                  int a_target) {
   if (M == 0) return cudaSuccess;
   const GemmShape g = linear_tc_shape(N);
   const int Mi = static_cast<int>(M);
-  if (g.cg == 2 && g.bn == 256) return dispatch_epi<2, 256>(m, Mi, N, K, bias, epi, s);
-  if (g.cg == 2 && g.bn == 128) return dispatch_epi<2, 128>(m, Mi, N, K, bias, epi, s);
-  if (g.cg == 1 && g.bn == 256) return dispatch_epi<1, 256>(m, Mi, N, K, bias, epi, s);
-  if (g.cg == 1 && g.bn == 128) return dispatch_epi<1, 128>(m, Mi, N, K, bias, epi, s);
-  return dispatch_epi<1, 64>(m, Mi, N, K, bias, epi, s);
+  int* tc = tile_counter;
+  const int* ar = a_ready;
+  if (g.cg == 2 && g.bn == 256) return dispatch_epi<2, 256>(m, Mi, N, K, bias, epi, s, tc, ar, a_target);
+  if (g.cg == 2 && g.bn == 128) return dispatch_epi<2, 128>(m, Mi, N, K, bias, epi, s, tc, ar, a_target);
+  if (g.cg == 1 && g.bn == 256) return dispatch_epi<1, 256>(m, Mi, N, K, bias, epi, s, tc, ar, a_target);
+  if (g.cg == 1 && g.bn == 128) return dispatch_epi<1, 128>(m, Mi, N, K, bias, epi, s, tc, ar, a_target);
+  return dispatch_epi<1, 64>(m, Mi, N, K, bias, epi, s, tc, ar, a_target);
 }
 
 }  // namespace k

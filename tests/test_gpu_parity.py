@@ -253,3 +253,20 @@ def test_internal_graph_replay_with_new_plan_contents():
     g.replay()
     torch.cuda.synchronize()
     assert torch.equal(got, rows3)
+
+
+@pytest.mark.parametrize("mode", ["1", "dyn"])
+def test_tail_overlap_option_parity(mode):
+    """The opt-in tail overlap (TCB_XOVERLAP=1: dynamic tile order + per-128-row readiness
+    flags between the LayerNorm GEMMs and the GEMM after them; =dyn: dynamic tiles only) gives
+    the same results: C2 full size and a C3 batch vs the oracle, in a subprocess (the option is
+    read once per process)."""
+    import os
+    import subprocess
+    import sys
+    code = ("import sys; sys.path.insert(0, 'tests'); import test_gpu_parity as t; "
+            "t._sampled_parity('c2', [0, -1]); t._sampled_parity('c3', [0], gpu_rows=8)")
+    env = dict(os.environ, TCB_XOVERLAP=mode)
+    r = subprocess.run([sys.executable, "-c", code], env=env, capture_output=True, text=True,
+                       cwd=os.path.dirname(os.path.dirname(os.path.abspath(__file__))), timeout=600)
+    assert r.returncode == 0, r.stderr[-2000:]
