@@ -13,10 +13,11 @@ rank 0 and broadcast once (NCCL); there is no per-step collective.
 value: device time (CUDA events on the launching stream), inputs resident in HBM, the
        forward replayed from a CUDA graph, L2 flushed (256 MiB write) between steps,
        max over ranks; value = sum of non-pad tokens over ranks / max time.
-e2e:   the same metric through the public API from host memory: per step tcb_pack (C++),
-       H2D of the segment table + token ids from pinned memory, forward, unpack, D2H of the
-       per-request outputs [T, d] into pinned memory, read by the host; two-deep pipeline (the
-       D2H of step i overlaps step i+1 on a copy stream); host wall clock.
+e2e:   the same metric through the C ABI with HOST buffers: per step tcb_pack (C++) and
+       tcb_session_run (the library uploads the segment table + pinned token ids, runs forward +
+       unpack, downloads the per-request outputs [T, d] into pinned host memory on a copy
+       stream), tcb_session_wait, the host reads the outputs; two slots (the download of step i
+       overlaps step i+1); host wall clock.
 roofline: the dominant kernel class (largest device time per step), each launch timed by CUDA
        event nodes inside a graph-replayed step (tcb_profile_*; L2 flushed per replay);
        algorithmic flops / bytes per class in DESIGN.md section 7 (GEMMs: 2 T d_in d_out per
@@ -519,59 +520,41 @@ def main():
                 "classes": classes}
     whole_tc = (gemm_flops + attn_flops) / (ms_per_step / 1e3) / 1e12
 
-    # ---- e2e: public API from host memory, every step -------------------------------------
-    # A two-deep serving pipeline: step i's outputs go device -> pinned host on a copy stream
-    # while step i+1 is packed (host C++) and computed; every step still copies its inputs
-    # host -> device and its [T, d] outputs device -> host inside the timed region, and the
-    # host reads each step's outputs once their copy has completed (before the slot is reused).
+    # ---- e2e: the C-ABI host-buffer path (tcb_session_run), every step ---------------------
+    # Per step: tcb_pack (host C++) -> tcb_session_run(plan, pinned host ids, pinned host out):
+    # the library uploads the segment table and the ids, runs forward + unpack and copies the
+    # [T, d] outputs back -- on a copy stream, so step i's download overlaps step i+1 (two
+    # slots) -- and the host reads each step's outputs once tcb_session_wait returns.
     pinned_ids = [torch.from_numpy(i).pin_memory() for _, i in batches]
     max_t = max(p.info["total_tokens"] for p in plans)
     out_host = [torch.empty((max_t, model.d_model), dtype=enc.dtype).pin_memory() for _ in range(2)]
-    e2e_out = [torch.empty((max_t, model.d_model), dtype=enc.dtype, device=dev) for _ in range(2)]
-    e2e_rows = enc.alloc_rows(M)
-    e2e_ids = torch.empty(max(len(i) for _, i in batches), dtype=torch.int32, device=dev)
-    e2e_seg = torch.empty(max(p.segtab().size for p in plans), dtype=torch.int32, device=dev)
-    seg_pin = [torch.empty(e2e_seg.numel(), dtype=torch.int32).pin_memory() for _ in range(2)]
+    sess = enc.session(B, L, max_t)
     cstream = torch.cuda.Stream(device=dev)
-    h2d_ev, copy_ev, pending = [None, None], [None, None], [0, 0]
+    tickets, pending = [None, None], [0, 0]
     h2d = d2h = 0
     checksum = 0.0
 
     def consume(k):
         nonlocal checksum
-        if copy_ev[k] is not None:
-            copy_ev[k].synchronize()                          # step's outputs are on the host
+        if tickets[k] is not None:
+            sess.wait(tickets[k])                              # step's outputs are on the host
             checksum += float(out_host[k][pending[k] - 1, 0])
-            copy_ev[k] = None
+            tickets[k] = None
 
     def e2e_step(i):
         nonlocal h2d, d2h
         k = i & 1
         lengths, ids = batches[i % len(batches)]
         p = tcb.tcb_pack(lengths, L, B)                         # host packer (C++)
-        st = p.segtab()
-        if h2d_ev[k] is not None:
-            h2d_ev[k].synchronize()                             # pinned slot k is free again
-        seg_pin[k][:st.size].copy_(torch.from_numpy(st))
         consume(k)                                              # output slot k is free again
         T = p.info["total_tokens"]
-        with torch.cuda.stream(stream):
-            e2e_seg[:st.size].copy_(seg_pin[k][:st.size], non_blocking=True)
-            e2e_ids[:len(ids)].copy_(pinned_ids[i % len(batches)], non_blocking=True)
-            h2d_ev[k] = torch.cuda.Event()
-            h2d_ev[k].record(stream)
-            enc.encoder_forward(p, e2e_seg, e2e_ids, e2e_rows, stream=stream)
-            enc.unpack(p, e2e_seg, e2e_rows, e2e_out[k], stream=stream)
-            done = torch.cuda.Event()
-            done.record(stream)
-        with torch.cuda.stream(cstream):
-            cstream.wait_event(done)
-            out_host[k][:T].copy_(e2e_out[k][:T], non_blocking=True)
-            copy_ev[k] = torch.cuda.Event()
-            copy_ev[k].record(cstream)
+        tickets[k] = sess.run(p, pinned_ids[i % len(batches)], out_host[k], stream, cstream)
         pending[k] = T
-        h2d += st.size * 4 + len(ids) * 4
-        d2h += T * model.d_model * e2e_out[k].element_size()
+        h2d += int(lib_words(p)) * 4 + len(ids) * 4
+        d2h += T * model.d_model * out_host[k].element_size()
+
+    def lib_words(p):
+        return tcb._lib.lib().tcb_plan_segtab_words(p.handle)
 
     def drain():
         consume(0)
@@ -594,6 +577,7 @@ def main():
         dist.all_reduce(e2e_t, op=dist.ReduceOp.MAX)
     e2e_tokens = sum(plans[i % len(plans)].info["placed_tokens"] for i in range(args.steps))
     e2e_value = e2e_tokens * world / float(e2e_t[0])
+    del sess
 
     cpu = None
     if rank == 0 and world == 1 and not args.no_cpu_baseline:
@@ -629,7 +613,7 @@ def main():
             "roofline": roofline,
             "e2e": {"value": e2e_value, "unit": UNIT, "h2d_bytes_per_step": h2d // args.steps,
                     "d2h_bytes_per_step": d2h // args.steps,
-                    "path": "tcb_pack + pinned H2D + tcb_encoder_forward + tcb_unpack + D2H read by the host, two-deep pipeline (D2H of step i on a copy stream overlaps step i+1)"},
+                    "path": "tcb_pack + tcb_session_run (C ABI, host buffers: pinned ids in, pinned [T, d] out; the library uploads the segment table + ids, runs forward + unpack, downloads on a copy stream) + tcb_session_wait, host reads each step's outputs; two slots (step i's download overlaps step i+1)"},
             "clocks": clk.summary(),
             "cpu_baseline": cpu,
             "paper_context": "paper reports only end-to-end serving on 1x V100 (<~4e3 tok/s incl. decoder); no encoder tokens/s",

@@ -232,6 +232,31 @@ tcb_status tcb_encoder_forward(const tcb_weights* w, const tcb_plan* plan,
 tcb_status tcb_unpack(const tcb_weights* w, const tcb_plan* plan, const int32_t* d_segtab,
                       const void* d_rows, void* d_out, tcb_stream_t stream);
 
+/* Host buffers in, host buffers out (§8(b) with host data): a session owns the device side of
+ * a fixed batch shape -- two slots of {segment table, token ids, rows, workspace, outputs}
+ * in device memory and a pinned staging copy of the segment table -- all allocated by
+ * tcb_session_create, none by tcb_session_run.
+ *   num_rows, row_len : the batch shape every plan must have (a scheduler's B x L);
+ *   max_tokens        : the largest total_tokens of a plan (outputs are [max_tokens, d]).
+ * tcb_session_run(plan, h_token_ids, h_out) enqueues on `stream`, using the slots in turn:
+ * the plan's segment table is written into the slot's pinned staging (waiting for that slot's
+ * previous upload) and copied host->device with h_token_ids ([total_tokens] int32; pinned
+ * memory makes the copies asynchronous), then tcb_encoder_forward + tcb_unpack run, then the
+ * per-request outputs are copied device->host into h_out ([total_tokens, d_model], model
+ * dtype) -- on `copy_stream` when not NULL (after an event on `stream`, so the copy overlaps
+ * the next call's compute), else on `stream`.  *ticket identifies the call;
+ * tcb_session_wait(ticket) blocks the host until that call's outputs are in h_out.
+ * Errors: a plan of another shape or with more than max_tokens tokens ->
+ * TCB_ERR_INVALID_ARGUMENT; CUDA failures -> TCB_ERR_CUDA. */
+typedef struct tcb_session tcb_session;
+tcb_status tcb_session_create(const tcb_weights* w, int32_t num_rows, int32_t row_len,
+                              int64_t max_tokens, tcb_session** out);
+tcb_status tcb_session_run(tcb_session* s, const tcb_plan* plan, const int32_t* h_token_ids,
+                           void* h_out, tcb_stream_t stream, tcb_stream_t copy_stream,
+                           int64_t* ticket);
+tcb_status tcb_session_wait(tcb_session* s, int64_t ticket);
+void tcb_session_destroy(tcb_session* s);
+
 /* ======================================================================================
  * 4. Instrumentation.
  * ==================================================================================== */

@@ -21,7 +21,7 @@ from ._lib import KCLASSES, POLICIES, TcbError, check, lib
 
 __all__ = ["Plan", "Encoder", "Decoder", "Scheduler", "sched_batch", "tcb_pack", "tcb_pack_slotted", "op_linear", "op_linear_ln", "op_attention", "op_layernorm",
            "launch_count", "profile_enable", "profile_collect", "profile_snapshot", "TcbError",
-           "KCLASSES"]
+           "KCLASSES", "Session"]
 
 _DTYPES = {"fp32": 0, "bf16": 1}
 _ACTS = {"gelu": 0, "relu": 1}
@@ -290,6 +290,11 @@ class Encoder:
                                _stream_ptr(stream)))
         return out
 
+    def session(self, num_rows: int, row_len: int, max_tokens: int) -> "Session":
+        """Host-buffer path (tcb_session_*): device buffers for a fixed B x L shape, owned by
+        the library; each run takes a host plan, host token ids and a host output buffer."""
+        return Session(self, num_rows, row_len, max_tokens)
+
     def run(self, lengths, token_ids, row_len: int, max_rows: int = 0,
             policy: str = "first_fit", slot_len: int = 0):
         """Host arrays in, device outputs out: pack -> H2D -> forward -> unpack.
@@ -304,6 +309,37 @@ class Encoder:
         rows = self.encoder_forward(plan, d_segtab, d_ids)
         out = self.unpack(plan, d_segtab, rows)
         return plan, rows, out
+
+
+class Session:
+    """tcb_session_*: host buffers in, host buffers out, two slots in turn (include/tcb.h)."""
+
+    def __init__(self, enc: Encoder, num_rows: int, row_len: int, max_tokens: int):
+        self.enc = enc
+        h = ctypes.c_void_p()
+        check(lib().tcb_session_create(enc._h, int(num_rows), int(row_len), int(max_tokens),
+                                       ctypes.byref(h)))
+        self._h = h
+
+    def run(self, plan: Plan, h_ids, h_out, stream=None, copy_stream=None) -> int:
+        """Enqueue one batch: h_ids (host int32 tensor / array, pinned for async copies) ->
+        h_out (host tensor [>= total_tokens, d_model], model dtype).  Returns the ticket."""
+        t = ctypes.c_int64(-1)
+        cs = ctypes.c_void_p(copy_stream.cuda_stream) if copy_stream is not None else ctypes.c_void_p()
+        check(lib().tcb_session_run(self._h, plan.handle, _ptr(h_ids), _ptr(h_out),
+                                    _stream_ptr(stream), cs, ctypes.byref(t)))
+        return int(t.value)
+
+    def wait(self, ticket: int) -> None:
+        check(lib().tcb_session_wait(self._h, int(ticket)))
+
+    def __del__(self):
+        try:
+            if getattr(self, "_h", None):
+                lib().tcb_session_destroy(self._h)
+                self._h = None
+        except Exception:
+            pass
 
 
 def op_linear(A, W, bias, R=None, epilogue: str = "bias", out=None, stream=None):

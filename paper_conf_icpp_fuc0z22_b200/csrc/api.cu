@@ -218,8 +218,10 @@ enum { W_QKV = 0, B_QKV, W_O, B_O, LN1_G, LN1_B, W_1, B_1, W_2, B_2, LN2_G, LN2_
 
 // bf16 attention: the tcgen05 kernel (attention_tc.cu).
 cudaError_t attention_bf16(int64_t M, int d, int heads, const void* qkv, const int32_t* seg,
-                           const int4* segtab, void* out, int* item_counter, cudaStream_t s) {
-  return tcb::k::launch_attention_bf16_tc(M, d, heads, qkv, seg, segtab, out, item_counter, s);
+                           const int4* segtab, void* out, int* item_counter, int row_len,
+                           cudaStream_t s) {
+  return tcb::k::launch_attention_bf16_tc(M, d, heads, qkv, seg, segtab, out, item_counter,
+                                          row_len, s);
 }
 
 tcb_status embed_impl(const tcb_weights* w, const tcb_plan* plan, const int32_t* d_segtab,
@@ -590,7 +592,8 @@ tcb_status forward_impl(const tcb_weights* wc, const tcb_plan* plan, const int32
                                         g_qkv, M, 3 * d, d, w->Lf(l, B_QKV), TCB_EPI_BIAS, s,
                                         xov_dyn ? gemm_cnt + 2 * l : nullptr,
                                         qkv_x ? ready(2 * (l - 1) + 1) : nullptr, 4 * d));
-      TCB_LAUNCH(TCB_K_ATTN, s, attention_bf16(M, d, c.num_heads, qkv, seg, segtab, att, attn_cnt + l, s));
+      TCB_LAUNCH(TCB_K_ATTN, s, attention_bf16(M, d, c.num_heads, qkv, seg, segtab, att, attn_cnt + l,
+                                               plan->row_len, s));
       if (fuse_ln) {   // W_O + bias + residual + LN1 in one kernel -> x1
         const tcb::k::GemmMaps g_o_ln{aAtt, mp.o, cX1, cX};
         TCB_LAUNCH(TCB_K_GEMM_O, s, tcb::k::launch_linear_ln_bf16_tc(
@@ -674,6 +677,149 @@ tcb_status tcb_unpack(const tcb_weights* w, const tcb_plan* plan, const int32_t*
                                                     w->cfg.d_model, d_rows, d_out, s));
   return TCB_OK;
 }
+
+// ---- host-buffer sessions --------------------------------------------------------------------
+}  // extern "C"
+
+struct tcb_session {
+  const tcb_weights* w = nullptr;
+  int32_t rows = 0, row_len = 0;
+  int64_t max_tokens = 0, seg_words = 0;
+  size_t ws_bytes = 0, out_bytes_per_token = 0;
+  struct Slot {
+    int32_t* d_segtab = nullptr;
+    int32_t* d_ids = nullptr;
+    void* d_rows = nullptr;
+    void* d_ws = nullptr;
+    void* d_out = nullptr;
+    int32_t* h_seg = nullptr;              // pinned
+    cudaEvent_t h2d_done = nullptr, computed = nullptr, d2h_done = nullptr;
+    int64_t ticket = -1;                   // last call that used the slot
+  } slot[2];
+  int64_t calls = 0;
+};
+
+namespace {
+void session_free(tcb_session* s) {
+  if (!s) return;
+  for (auto& sl : s->slot) {
+    cudaFree(sl.d_segtab);
+    cudaFree(sl.d_ids);
+    cudaFree(sl.d_rows);
+    cudaFree(sl.d_ws);
+    cudaFree(sl.d_out);
+    cudaFreeHost(sl.h_seg);
+    if (sl.h2d_done) cudaEventDestroy(sl.h2d_done);
+    if (sl.computed) cudaEventDestroy(sl.computed);
+    if (sl.d2h_done) cudaEventDestroy(sl.d2h_done);
+  }
+  delete s;
+}
+}  // namespace
+
+extern "C" {
+
+tcb_status tcb_session_create(const tcb_weights* w, int32_t num_rows, int32_t row_len,
+                              int64_t max_tokens, tcb_session** out) {
+  tcb::clear_error();
+  if (!out) return fail(TCB_ERR_INVALID_ARGUMENT, "tcb_session_create: out is NULL");
+  *out = nullptr;
+  if (!w || num_rows <= 0 || row_len <= 0 || row_len % 8 != 0 || max_tokens < 0 ||
+      static_cast<int64_t>(num_rows) * row_len > INT32_MAX)
+    return fail(TCB_ERR_INVALID_ARGUMENT, "tcb_session_create: bad shape");
+  if (row_len > w->cfg.max_pos)
+    return fail(TCB_ERR_UNSUPPORTED, "tcb_session_create: row_len exceeds max_pos");
+  if (tcb_status st = check_device()) return st;
+  tcb_session* s = new (std::nothrow) tcb_session();
+  if (!s) return fail(TCB_ERR_OUT_OF_MEMORY, "tcb_session_create");
+  s->w = w;
+  s->rows = num_rows;
+  s->row_len = row_len;
+  s->max_tokens = max_tokens;
+  const int64_t M = static_cast<int64_t>(num_rows) * row_len;
+  // segment table of at most one segment per slot + row index + query-block order (tcb.h)
+  s->seg_words = 4 * (1 + M) + (num_rows + 1 + 3) / 4 * 4 + ((M + 127) / 128 + 3) / 4 * 4;
+  const size_t esz = w->cfg.dtype == 0 ? 4 : 2;
+  s->out_bytes_per_token = esz * static_cast<size_t>(w->cfg.d_model);
+  s->ws_bytes = ws_layout(w->cfg, M).total;
+  bool ok = true;
+  for (auto& sl : s->slot) {
+    ok = ok && cudaMalloc(&sl.d_segtab, 4 * static_cast<size_t>(s->seg_words)) == cudaSuccess &&
+         cudaMalloc(&sl.d_ids, 4 * static_cast<size_t>(std::max<int64_t>(max_tokens, 1))) == cudaSuccess &&
+         cudaMalloc(&sl.d_rows, esz * static_cast<size_t>(M) * w->cfg.d_model) == cudaSuccess &&
+         cudaMalloc(&sl.d_ws, s->ws_bytes) == cudaSuccess &&
+         cudaMalloc(&sl.d_out, s->out_bytes_per_token * static_cast<size_t>(std::max<int64_t>(max_tokens, 1))) == cudaSuccess &&
+         cudaMallocHost(&sl.h_seg, 4 * static_cast<size_t>(s->seg_words)) == cudaSuccess &&
+         cudaEventCreateWithFlags(&sl.h2d_done, cudaEventDisableTiming) == cudaSuccess &&
+         cudaEventCreateWithFlags(&sl.computed, cudaEventDisableTiming) == cudaSuccess &&
+         cudaEventCreateWithFlags(&sl.d2h_done, cudaEventDisableTiming) == cudaSuccess;
+  }
+  if (!ok) {
+    cudaGetLastError();
+    session_free(s);
+    return fail(TCB_ERR_OUT_OF_MEMORY, "tcb_session_create: device / pinned allocation failed");
+  }
+  *out = s;
+  return TCB_OK;
+}
+
+tcb_status tcb_session_run(tcb_session* s, const tcb_plan* plan, const int32_t* h_token_ids,
+                           void* h_out, tcb_stream_t stream, tcb_stream_t copy_stream,
+                           int64_t* ticket) {
+  tcb::clear_error();
+  if (!s || !plan) return fail(TCB_ERR_INVALID_ARGUMENT, "tcb_session_run: NULL session or plan");
+  if (plan->num_rows != s->rows || plan->row_len != s->row_len)
+    return fail(TCB_ERR_INVALID_ARGUMENT, "tcb_session_run: plan shape differs from the session's");
+  const int64_t T = plan->info.total_tokens;
+  if (T > s->max_tokens)
+    return fail(TCB_ERR_INVALID_ARGUMENT, "tcb_session_run: plan has more tokens than max_tokens");
+  if (T > 0 && (!h_token_ids || !h_out))
+    return fail(TCB_ERR_INVALID_ARGUMENT, "tcb_session_run: NULL host buffer");
+  cudaStream_t st = reinterpret_cast<cudaStream_t>(stream);
+  cudaStream_t cs = copy_stream ? reinterpret_cast<cudaStream_t>(copy_stream) : st;
+  const int64_t call = s->calls++;
+  tcb_session::Slot& sl = s->slot[call & 1];
+  if (sl.ticket >= 0 && cudaEventSynchronize(sl.h2d_done) != cudaSuccess)   // staging reusable
+    return cuda_fail(cudaGetLastError(), "tcb_session_run: wait for the slot's previous upload");
+  if (tcb_status e = tcb_plan_write_segtab(plan, sl.h_seg, s->seg_words)) return e;
+  const int64_t words = tcb_plan_segtab_words(plan);
+  cudaError_t e = cudaMemcpyAsync(sl.d_segtab, sl.h_seg, 4 * static_cast<size_t>(words),
+                                  cudaMemcpyHostToDevice, st);
+  if (e == cudaSuccess && T > 0)
+    e = cudaMemcpyAsync(sl.d_ids, h_token_ids, 4 * static_cast<size_t>(T), cudaMemcpyHostToDevice, st);
+  if (e == cudaSuccess) e = cudaEventRecord(sl.h2d_done, st);
+  // the slot's outputs may still be on their way to the host (previous call of the slot)
+  if (e == cudaSuccess && sl.ticket >= 0) e = cudaStreamWaitEvent(st, sl.d2h_done, 0);
+  if (e != cudaSuccess) return cuda_fail(e, "tcb_session_run: upload");
+  if (tcb_status r = tcb_encoder_forward(s->w, plan, sl.d_segtab, sl.d_ids, sl.d_rows, sl.d_ws,
+                                         s->ws_bytes, stream))
+    return r;
+  if (tcb_status r = tcb_unpack(s->w, plan, sl.d_segtab, sl.d_rows, sl.d_out, stream)) return r;
+  if (cs != st) {
+    e = cudaEventRecord(sl.computed, st);
+    if (e == cudaSuccess) e = cudaStreamWaitEvent(cs, sl.computed, 0);
+  }
+  if (e == cudaSuccess && T > 0)
+    e = cudaMemcpyAsync(h_out, sl.d_out, s->out_bytes_per_token * static_cast<size_t>(T),
+                        cudaMemcpyDeviceToHost, cs);
+  if (e == cudaSuccess) e = cudaEventRecord(sl.d2h_done, cs);
+  if (e != cudaSuccess) return cuda_fail(e, "tcb_session_run: download");
+  sl.ticket = call;
+  if (ticket) *ticket = call;
+  return TCB_OK;
+}
+
+tcb_status tcb_session_wait(tcb_session* s, int64_t ticket) {
+  tcb::clear_error();
+  if (!s || ticket < 0 || ticket >= s->calls)
+    return fail(TCB_ERR_INVALID_ARGUMENT, "tcb_session_wait: unknown ticket");
+  const tcb_session::Slot& sl = s->slot[ticket & 1];
+  if (sl.ticket != ticket) return TCB_OK;              // the slot has been reused: long done
+  const cudaError_t e = cudaEventSynchronize(sl.d2h_done);
+  return e == cudaSuccess ? TCB_OK : cuda_fail(e, "tcb_session_wait");
+}
+
+void tcb_session_destroy(tcb_session* s) { session_free(s); }
 
 // ---- op-level entry points (include/tcb_ops.h) ---------------------------------------------
 tcb_status tcb_op_linear(int32_t dtype, int64_t M, int32_t N, int32_t K, const void* A,
@@ -778,7 +924,7 @@ tcb_status tcb_op_attention(int32_t dtype, int64_t num_slots, int32_t d_model,
     if (cudaMemsetAsync(cnt, 0, sizeof(int), s) != cudaSuccess)
       return fail(TCB_ERR_CUDA, "tcb_op_attention: counter reset failed");
     TCB_LAUNCH(TCB_K_ATTN, s, attention_bf16(num_slots, d_model, num_heads, qkv, d_seg, segtab, O,
-                                             static_cast<int*>(cnt), s));
+                                             static_cast<int*>(cnt), 0, s));
   }
   else
     TCB_LAUNCH(TCB_K_ATTN, s, tcb::k::launch_attention_f32(num_slots, d_model, num_heads,

@@ -1238,13 +1238,535 @@ attn_tc3_kernel(const __grid_constant__ CUtensorMap tmQKV, const __grid_constant
 }
 }  // namespace v3
 
+// =============================================================================================
+// v3s: v3 with an item-scheduler warp, for rows of at most 128 slots (every item one chunk).
+// A third control warp takes the next item from the counter and computes its metadata into a
+// 2-deep ring ahead of the TMA producer (8 warps: the control warpgroup hands its registers to
+// the softmax warpgroup with setmaxnreg).  With one 128 x 128 chunk per item the producer's
+// metadata latency is what the softmax warps wait for: C2 (L = 128) 46.5 -> 42.3 us per launch;
+// on multi-chunk items the extra look-ahead costs more than it gains (C3 101.5 -> 112), so the
+// launcher uses this kernel only for row_len <= 128 (r02 A/B).
+namespace v3s {
+constexpr int kWarps = 8;                    // warpgroup 0: 0 TMA producer, 1 MMA + TMEM,
+                                             // 2 item scheduler (metadata), 3 idle;
+                                             // warpgroup 1: 4..7 softmax / epilogue
+constexpr int kCtrlRegs = 56, kSoftmaxRegs = 168;   // setmaxnreg split (2 CTAs x 256 threads)
+constexpr int kThreads = kWarps * 32;
+constexpr int kQStages = 2, kKStages = 2, kVStages = 2, kInfoStages = 2;
+constexpr uint32_t kTmemCols = 256;          // S [0,128), O [128,192), P [192,256)
+constexpr uint32_t kOCol = 128, kPCol = 192;
+
+
+struct Info {
+  int2 rows[TQ];   // [start, end) of the request of query slot q0 + r (empty for pads)
+  int kbase, nch;  // first key (8-aligned), number of 128-key chunks; nch < 0: no more items
+  int qb, h;       // query block, head
+};
+constexpr int kSmemBytes = 1024 + (kQStages + kKStages + kVStages) * kTileBytes +
+                           kInfoStages * static_cast<int>(sizeof(Info)) + 256;
+
+// the segment table's query-block order (tcb.h: after the records and the row index), longest
+// key interval first
+__device__ __forceinline__ const int32_t* qblock_order(const int4* __restrict__ segtab) {
+  const int4 hd = __ldg(&segtab[0]);               // {S, num_slots, row_len, total_tokens}
+  const int num_rows = hd.z > 0 ? hd.y / hd.z : 0;
+  return reinterpret_cast<const int32_t*>(segtab) + 4 * (1 + hd.x) + (num_rows + 1 + 3) / 4 * 4;
+}
+
+__device__ __forceinline__ void tc_mma_ts(uint32_t tmem_d, uint32_t tmem_a, uint64_t bdesc,
+                                          uint32_t idesc, uint32_t accumulate) {
+  asm volatile(
+      "{\n\t.reg .pred p;\n\tsetp.ne.b32 p, %4, 0;\n\t"
+      "tcgen05.mma.cta_group::1.kind::f16 [%0], [%1], %2, %3, p;\n\t}" ::"r"(tmem_d),
+      "r"(tmem_a), "l"(bdesc), "r"(idesc), "r"(accumulate)
+      : "memory");
+}
+__device__ __forceinline__ void tmem_st8(uint32_t taddr, const uint32_t (&w)[8]) {
+  asm volatile("tcgen05.st.sync.aligned.32x32b.x8.b32 [%0], {%1,%2,%3,%4,%5,%6,%7,%8};" ::"r"(taddr),
+               "r"(w[0]), "r"(w[1]), "r"(w[2]), "r"(w[3]), "r"(w[4]), "r"(w[5]), "r"(w[6]), "r"(w[7])
+               : "memory");
+}
+
+// valid-key bit mask of 32-key group [g0, g0 + 32) for a row whose keys are [jlo, jhi)
+// (chunk-relative)
+__device__ __forceinline__ uint32_t group_mask(int jlo, int jhi, int g0) {
+  const int lo = min(max(jlo - g0, 0), 32), hi = min(max(jhi - g0, 0), 32);
+  const uint32_t below_hi = hi >= 32 ? 0xffffffffu : (1u << hi) - 1u;
+  const uint32_t from_lo = lo >= 32 ? 0u : ~((1u << lo) - 1u);   // no shift by 32
+  return below_hi & from_lo;
+}
+
+// masked max of one 64-key half (groups 2*hh, 2*hh+1) into 8 partial maxima
+__device__ __forceinline__ void half_max(const uint32_t (&sr)[64], const bool* live, const bool* inner,
+                                         const uint32_t* vm, int hh, float (&mxp)[8]) {
+#pragma unroll
+  for (int gi = 0; gi < 2; ++gi) {
+    const int g = 2 * hh + gi;
+    if (!live[g]) continue;
+    if (inner[g]) {
+#pragma unroll
+      for (int j = 32 * gi; j < 32 * gi + 32; j += 2)
+        mxp[(j >> 1) & 7] = fmax3(mxp[(j >> 1) & 7], __uint_as_float(sr[j]), __uint_as_float(sr[j + 1]));
+    } else {
+#pragma unroll
+      for (int j = 32 * gi; j < 32 * gi + 32; j += 2) {
+        const float v0 = (vm[g] & (1u << (j - 32 * gi))) ? __uint_as_float(sr[j]) : -INFINITY;
+        const float v1 = (vm[g] & (2u << (j - 32 * gi))) ? __uint_as_float(sr[j + 1]) : -INFINITY;
+        mxp[(j >> 1) & 7] = fmax3(mxp[(j >> 1) & 7], v0, v1);
+      }
+    }
+  }
+}
+
+// p = 2^(s * scale - m) of one 32-key group (0 outside the row's request when MASKED) -> 16
+// bf16 pairs (key 2j in the low half of word j).  Straight-line code: the 32 exponentials of a
+// group are independent, so their MUFU latencies overlap.
+template <bool MASKED>
+__device__ __forceinline__ void group_exp(const uint32_t* sr, uint32_t vm, float2 sc2, float2 off2,
+                                          uint32_t (&w)[16], float2 (&lp)[2]) {
+#pragma unroll
+  for (int e = 0; e < 16; ++e) {
+    const float2 x = ffma2(make_float2(__uint_as_float(sr[2 * e]), __uint_as_float(sr[2 * e + 1])), sc2, off2);
+    float2 pp = make_float2(ex2(x.x), ex2(x.y));
+    if (MASKED) {
+      pp.x = (vm & (1u << (2 * e))) ? pp.x : 0.f;
+      pp.y = (vm & (2u << (2 * e))) ? pp.y : 0.f;
+    }
+    lp[e & 1] = fadd2(lp[e & 1], pp);
+    __nv_bfloat162 hv = __floats2bfloat162_rn(pp.x, pp.y);
+    w[e] = *reinterpret_cast<uint32_t*>(&hv);
+  }
+}
+
+// the two 32-key groups of one 64-key half -> TMEM P columns [32hh, 32hh + 32); dead groups
+// (no key of the warp's rows) are written as zeros without math.  live / inner are warp-uniform.
+__device__ __forceinline__ void half_exp(const uint32_t (&sr)[64], const bool* live, const bool* inner,
+                                         const uint32_t* vm, int hh, float2 sc2, float2 off2,
+                                         uint32_t paddr, float2 (&lp)[2]) {
+#pragma unroll
+  for (int gi = 0; gi < 2; ++gi) {
+    const int g = 2 * hh + gi;
+    uint32_t w[16];
+    if (!live[g]) {
+#pragma unroll
+      for (int e = 0; e < 16; ++e) w[e] = 0u;
+    } else if (inner[g]) {
+      group_exp<false>(sr + 32 * gi, 0u, sc2, off2, w, lp);
+    } else {
+      group_exp<true>(sr + 32 * gi, vm[g], sc2, off2, w, lp);
+    }
+    const uint32_t (&w0)[8] = *reinterpret_cast<const uint32_t(*)[8]>(&w[0]);
+    const uint32_t (&w1)[8] = *reinterpret_cast<const uint32_t(*)[8]>(&w[8]);
+    tmem_st8(paddr + 32 * hh + 16 * gi, w0);
+    tmem_st8(paddr + 32 * hh + 16 * gi + 8, w1);
+  }
+}
+
+__global__ void __launch_bounds__(kThreads, 2)
+attn_tc3s_kernel(const __grid_constant__ CUtensorMap tmQKV, const __grid_constant__ CUtensorMap tmO,
+                const int32_t* __restrict__ seg_ids,
+                const int4* __restrict__ segtab, __nv_bfloat16* __restrict__ O,
+                int64_t num_slots, int d_model, int num_heads, int num_items, float scale_log2,
+                int* __restrict__ item_counter) {
+  extern __shared__ uint8_t smem_raw[];
+  const uint32_t raw = smem_u32(smem_raw);
+  const uint32_t base = (raw + 1023) & ~1023u;
+  const uint32_t sQ = base;                                    // [2][128 x 64]
+  const uint32_t sK = sQ + kQStages * kTileBytes;              // [2][128 x 64]
+  const uint32_t sV = sK + kKStages * kTileBytes;              // [2][128 x 64]
+  uint8_t* gen = smem_raw + (sV + kVStages * kTileBytes - raw);
+  Info* infos = reinterpret_cast<Info*>(gen);                  // [kInfoStages]
+  uint32_t* tmem_slot = reinterpret_cast<uint32_t*>(gen + kInfoStages * sizeof(Info));
+  const uint32_t bars = (smem_u32(tmem_slot + 2) + 7) & ~7u;
+  const uint32_t q_full = bars, q_empty = q_full + 8 * kQStages;
+  const uint32_t k_full = q_empty + 8 * kQStages, k_empty = k_full + 8 * kKStages;
+  const uint32_t v_full = k_empty + 8 * kKStages, v_empty = v_full + 8 * kVStages;
+  const uint32_t s_full = v_empty + 8 * kVStages, s_free = s_full + 8;
+  const uint32_t p_full = s_free + 8, pv_done = p_full + 8;
+  const uint32_t i_full = pv_done + 8, i_empty = i_full + 8 * kInfoStages;
+
+  const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
+  if (threadIdx.x == 0) {
+    for (int i = 0; i < kQStages; ++i) {
+      mbar_init(q_full + 8 * i, 1);
+      mbar_init(q_empty + 8 * i, 1 + 4);    // MMA (after the item's last S) + 4 softmax warps
+                                            // (after their output tile left the slot)
+    }
+    for (int i = 0; i < kKStages; ++i) { mbar_init(k_full + 8 * i, 1); mbar_init(k_empty + 8 * i, 1); }
+    for (int i = 0; i < kVStages; ++i) { mbar_init(v_full + 8 * i, 1); mbar_init(v_empty + 8 * i, 1); }
+    mbar_init(s_full, 1);
+    mbar_init(s_free, 4);
+    mbar_init(p_full, 4);
+    mbar_init(pv_done, 1);
+    for (int i = 0; i < kInfoStages; ++i) {
+      mbar_init(i_full + 8 * i, 1);
+      mbar_init(i_empty + 8 * i, 1 + 1 + 4);  // TMA producer + MMA + 4 softmax warps
+    }
+    asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
+  }
+  if (warp == 1) {
+    asm volatile("tcgen05.alloc.cta_group::1.sync.aligned.shared::cta.b32 [%0], %1;" ::"r"(
+                     smem_u32(tmem_slot)), "r"(kTmemCols) : "memory");
+    asm volatile("tcgen05.relinquish_alloc_permit.cta_group::1.sync.aligned;" ::: "memory");
+  }
+  tc_fence_before();
+  __syncthreads();
+  tc_fence_after();
+  const uint32_t tmem = *tmem_slot;
+  pdl_wait();                                 // QKV / segment ids come from earlier kernels
+  pdl_trigger();
+  // registers: the control warpgroup hands most of its share to the softmax warpgroup
+  if (warp < 4) {
+  asm volatile("setmaxnreg.dec.sync.aligned.u32 %0;" ::"n"(kCtrlRegs));
+  if (warp == 2) {
+    // ================= item scheduler: next item -> metadata ring ==========================
+    const int32_t* qorder = qblock_order(segtab);
+    int is = 0;
+    uint32_t iph = 0;
+    for (int k = 0;; ++k) {
+      int item = 0;
+      if (item_counter) {
+        if (lane == 0) item = atomicAdd(item_counter, 1);
+        item = __shfl_sync(0xffffffffu, item, 0);
+      } else {
+        item = blockIdx.x + k * gridDim.x;
+      }
+      if (lane == 0) mbar_wait(i_empty + 8 * is, iph ^ 1);
+      __syncwarp();
+      Info* inf = infos + is;
+      if (item >= num_items) {
+        if (lane == 0) {
+          inf->nch = -1;
+          mbar_arrive(i_full + 8 * is);
+        }
+        break;
+      }
+      const int qb = __ldg(&qorder[item / num_heads]);
+      compute_info(reinterpret_cast<ItemInfo*>(inf), seg_ids, segtab, static_cast<int64_t>(qb) * TQ,
+                   num_slots, lane);
+      if (lane == 0) {
+        inf->qb = qb;
+        inf->h = item % num_heads;
+        mbar_arrive(i_full + 8 * is);
+      }
+      __syncwarp();
+      if (++is == kInfoStages) { is = 0; iph ^= 1; }
+    }
+  } else if (warp == 0) {
+    // ================= TMA producer: per item its Q tile, then K one chunk ahead of V =========
+    if (lane == 0) {
+      asm volatile("prefetch.tensormap [%0];" ::"l"(reinterpret_cast<uint64_t>(&tmQKV)) : "memory");
+      int qs = 0, ks = 0, vs = 0, is = 0;
+      uint32_t qph = 0, kph = 0, vph = 0, iph = 0;
+      for (;;) {
+        mbar_wait(i_full + 8 * is, iph);
+        const Info* inf = infos + is;
+        const int nch = inf->nch, kbase = inf->kbase, qb = inf->qb, h = inf->h;
+        mbar_arrive(i_empty + 8 * is);
+        if (++is == kInfoStages) { is = 0; iph ^= 1; }
+        if (nch < 0) break;
+        mbar_wait(q_empty + 8 * qs, qph ^ 1);  // the slot is ours (also for an empty item:
+                                               // the softmax warps stage its output there)
+        if (nch == 0) {
+          mbar_arrive(q_full + 8 * qs);
+        } else {
+          mbar_expect_tx(q_full + 8 * qs, kTileBytes);
+          tma_load(sQ + qs * kTileBytes, &tmQKV, q_full + 8 * qs, h * DH, qb * TQ);
+        }
+        // K one chunk ahead of V (K is released by S, V only by P V)
+        for (int c = 0; c <= nch; ++c) {
+          if (c < nch) {
+            mbar_wait(k_empty + 8 * ks, kph ^ 1);
+            mbar_expect_tx(k_full + 8 * ks, kTileBytes);
+            tma_load(sK + ks * kTileBytes, &tmQKV, k_full + 8 * ks, d_model + h * DH, kbase + c * TK);
+            if (++ks == kKStages) { ks = 0; kph ^= 1; }
+          }
+          if (c > 0) {
+            mbar_wait(v_empty + 8 * vs, vph ^ 1);
+            mbar_expect_tx(v_full + 8 * vs, kTileBytes);
+            tma_load(sV + vs * kTileBytes, &tmQKV, v_full + 8 * vs, 2 * d_model + h * DH, kbase + (c - 1) * TK);
+            if (++vs == kVStages) { vs = 0; vph ^= 1; }
+          }
+        }
+        if (++qs == kQStages) { qs = 0; qph ^= 1; }
+      }
+    }
+  } else if (warp == 1) {
+    // ================= MMA issuer ===========================================================
+    // Chunk g: S(g) = Q K^T as soon as S(g-1) has been read (s_free) and K(g) is in; then
+    // O += P(g-1) V(g-1) once P(g-1) is written -- S of the next chunk runs while the softmax
+    // warps still work on the current one.
+    int qs = 0, ks = 0, vs = 0;
+    uint32_t qph = 0, kph = 0, vph = 0, g = 0;
+    struct Pend {
+      bool first, valid;
+    } pend{false, false};
+#ifdef TCB_ATTN_PROBE
+    long long a_q = 0, a_kv = 0, a_sf = 0, a_p = 0, a_start = clock64();
+#endif
+    auto issue_pv = [&](const Pend& pp, uint32_t gp) {
+      PRB(t3);
+      mbar_wait(v_full + 8 * vs, vph);
+      mbar_wait(p_full, gp & 1);
+      PRB_ADD(a_p, t3);
+      tc_fence_after();
+      if (lane == 0) {
+        const uint32_t va = sV + vs * kTileBytes;
+#pragma unroll
+        for (int k = 0; k < TK / 16; ++k)
+          tc_mma_ts(tmem + kOCol, tmem + kPCol + 8 * k, desc_mnmajor(va + k * 2048), kIdescPV,
+                    (!pp.first || k > 0) ? 1u : 0u);
+        tc_commit(pv_done);
+        tc_commit(v_empty + 8 * vs);
+      }
+      __syncwarp();
+      if (++vs == kVStages) { vs = 0; vph ^= 1; }
+    };
+    int is = 0;
+    uint32_t iph = 0;
+    for (;;) {
+      PRB(t0);
+      mbar_wait(i_full + 8 * is, iph);
+      const int nch = infos[is].nch;
+      __syncwarp();
+      if (lane == 0) mbar_arrive(i_empty + 8 * is);
+      if (++is == kInfoStages) { is = 0; iph ^= 1; }
+      if (nch < 0) break;
+      mbar_wait(q_full + 8 * qs, qph);
+      PRB_ADD(a_q, t0);
+      tc_fence_after();
+      const uint32_t qaddr = sQ + qs * kTileBytes;
+      if (nch == 0) {
+        // an empty item must not hold back the pending P V: the softmax warps wait for it
+        // (epilogue of the previous item) and would stop releasing Q slots -> deadlock
+        if (pend.valid) {
+          issue_pv(pend, g - 1);
+          pend.valid = false;
+        }
+        if (lane == 0) mbar_arrive(q_empty + 8 * qs);
+      }
+      for (int c = 0; c < nch; ++c) {
+        PRB(t1);
+        mbar_wait(k_full + 8 * ks, kph);
+        PRB_ADD(a_kv, t1);
+        PRB(t2);
+        if (g > 0) mbar_wait(s_free, (g - 1) & 1);
+        PRB_ADD(a_sf, t2);
+        tc_fence_after();
+        if (lane == 0) {
+          const uint32_t ka = sK + ks * kTileBytes;
+#pragma unroll
+          for (int k = 0; k < DH / 16; ++k)
+            tc_mma(tmem, desc_kmajor(qaddr + k * 32), desc_kmajor(ka + k * 32), kIdescQK, k > 0 ? 1u : 0u);
+          tc_commit(s_full);
+          tc_commit(k_empty + 8 * ks);
+          if (c == nch - 1) tc_commit(q_empty + 8 * qs);
+        }
+        __syncwarp();
+        if (pend.valid) issue_pv(pend, g - 1);
+        pend = Pend{c == 0, true};
+        ++g;
+        if (++ks == kKStages) { ks = 0; kph ^= 1; }
+      }
+      if (pend.valid) {                     // the item's last P V: its epilogue waits for it
+        issue_pv(pend, g - 1);
+        pend.valid = false;
+      }
+      if (++qs == kQStages) { qs = 0; qph ^= 1; }
+    }
+    if (pend.valid) issue_pv(pend, g - 1);
+#ifdef TCB_ATTN_PROBE
+    if (lane == 0 && blockIdx.x < 3)
+      printf("a3probe mma cta %d total %lld wait_q %lld wait_kv %lld wait_sfree %lld wait_p %lld chunks %u\n",
+             blockIdx.x, clock64() - a_start, a_q, a_kv, a_sf, a_p, g);
+#endif
+  }
+  } else {
+    asm volatile("setmaxnreg.inc.sync.aligned.u32 %0;" ::"n"(kSoftmaxRegs));
+    // ================= softmax + output (warps 4..7, thread = query row) ===================
+    const int q = warp & 3;                 // TMEM lane quarter
+    const int row = q * 32 + lane;
+    const uint32_t lane_off = static_cast<uint32_t>(q * 32) << 16;
+    const uint32_t s_addr = tmem + lane_off, o_addr = tmem + lane_off + kOCol, p_addr = tmem + lane_off + kPCol;
+    int qs = 0, is = 0;
+    uint32_t iph = 0, g = 0;
+#ifdef TCB_ATTN_PROBE
+    long long b_q = 0, b_s = 0, b_p1 = 0, b_pv = 0, b_e1 = 0, b_e0 = 0, b_epi = 0, b_start = clock64();
+#endif
+    for (;;) {
+      PRB(t0);
+      mbar_wait(i_full + 8 * is, iph);
+      PRB_ADD(b_q, t0);
+      const Info* inf = infos + is;
+      const int nch = inf->nch;
+      const int2 rr = inf->rows[row];
+      const int kbase = inf->kbase, qb = inf->qb, h = inf->h;
+      __syncwarp();
+      if (lane == 0) mbar_arrive(i_empty + 8 * is);   // metadata copied to registers
+      if (++is == kInfoStages) { is = 0; iph ^= 1; }
+      if (nch < 0) break;
+      // the item's Q slot (acquired by the producer, read by the item's S MMAs) stages the
+      // output tile; no wait needed: the epilogue runs after the item's last P V
+      const int my_qs = qs;
+      if (++qs == kQStages) { qs = 0; }
+      // key interval of this warp's 32 rows: union [ulo, uhi) and intersection [ilo, ihi)
+      const bool real = rr.y > rr.x;
+      int ulo = real ? rr.x : INT_MAX, uhi = real ? rr.y : -1;
+      int ilo = real ? rr.x : INT_MAX, ihi = real ? rr.y : -1;
+#pragma unroll
+      for (int o = 16; o > 0; o >>= 1) {
+        ulo = min(ulo, __shfl_xor_sync(0xffffffffu, ulo, o));
+        uhi = max(uhi, __shfl_xor_sync(0xffffffffu, uhi, o));
+        ilo = max(ilo, __shfl_xor_sync(0xffffffffu, ilo, o));
+        ihi = min(ihi, __shfl_xor_sync(0xffffffffu, ihi, o));
+      }
+      float m_used = -INFINITY, lsum = 0.f;
+      for (int c = 0; c < nch; ++c, ++g) {
+        // 32-key groups of the chunk: dead (no key of any of the warp's rows' requests: P = 0
+        // without math), interior (inside every row's request: no mask) or boundary (per
+        // element bit mask: key outside the row's own request -> p = 0 exactly, R11)
+        const int k0 = kbase + c * TK;
+        const int jlo = rr.x - k0, jhi = rr.y - k0;
+        bool live[4], inner[4];
+        uint32_t vm[4];
+#pragma unroll
+        for (int gi = 0; gi < 4; ++gi) {
+          const int gk = k0 + 32 * gi;
+          live[gi] = gk < uhi && gk + 32 > ulo;
+          inner[gi] = gk >= ilo && gk + 32 <= ihi;
+          vm[gi] = group_mask(jlo, jhi, 32 * gi);
+        }
+        PRB(t1);
+        mbar_wait(s_full, g & 1);
+        PRB_ADD(b_s, t1);
+        tc_fence_after();
+        PRB(t2);
+        float mxp[8];
+#pragma unroll
+        for (int t = 0; t < 8; ++t) mxp[t] = -INFINITY;
+        uint32_t sr[64];
+        tmem_ld64_sync(s_addr, sr);
+        half_max(sr, live, inner, vm, 0, mxp);
+        tmem_ld64_sync(s_addr + 64, sr);
+        half_max(sr, live, inner, vm, 1, mxp);
+        const float rmax = fmaxf(fmaxf(fmaxf(mxp[0], mxp[1]), fmaxf(mxp[2], mxp[3])),
+                                 fmaxf(fmaxf(mxp[4], mxp[5]), fmaxf(mxp[6], mxp[7])));
+        PRB_ADD(b_p1, t2);
+        // P V of the previous chunk must be done before P is overwritten (and before O is
+        // rescaled); it was issued when that chunk's P was complete, so this rarely waits
+        PRB(t3);
+        if (g > 0) mbar_wait(pv_done, (g - 1) & 1);
+        tc_fence_after();
+        PRB_ADD(b_pv, t3);
+        // lazy rescale: a row moves its max only when it grew by more than 2^8 (warp-collective
+        // TMEM access, so the decision is per warp; lanes that keep their max scale by 1)
+        bool grow = false;
+        if (rmax != -INFINITY) {
+          if (m_used == -INFINITY) m_used = rmax;
+          else grow = (rmax - m_used) * scale_log2 > kRescaleLog2;
+        }
+        if (__any_sync(0xffffffffu, grow)) {
+          const float f = grow ? ex2((m_used - rmax) * scale_log2) : 1.f;
+#pragma unroll 1
+          for (int cq = 0; cq < 2; ++cq) {
+            uint32_t o[32];
+            tmem_ld32_sync(o_addr + 32 * cq, o);
+#pragma unroll
+            for (int t = 0; t < 32; ++t) o[t] = __float_as_uint(__uint_as_float(o[t]) * f);
+            tmem_st32(o_addr + 32 * cq, o);
+          }
+          if (grow) {
+            lsum *= f;
+            m_used = rmax;
+          }
+        }
+        const float off = m_used == -INFINITY ? 0.f : -m_used * scale_log2;
+        const float2 sc2 = make_float2(scale_log2, scale_log2), off2 = make_float2(off, off);
+        float2 lp[2] = {make_float2(0.f, 0.f), make_float2(0.f, 0.f)};
+        PRB(t4);
+        half_exp(sr, live, inner, vm, 1, sc2, off2, p_addr, lp);      // keys 64-127 (in registers)
+        PRB_ADD(b_e1, t4);
+        PRB(t5);
+        tmem_ld64_sync(s_addr, sr);                                     // keys 0-63 again
+        tc_fence_before();
+        __syncwarp();
+        if (lane == 0) mbar_arrive(s_free);                            // S consumed: next S may go
+        half_exp(sr, live, inner, vm, 0, sc2, off2, p_addr, lp);
+        lsum += (lp[0].x + lp[0].y) + (lp[1].x + lp[1].y);
+        asm volatile("tcgen05.wait::st.sync.aligned;" ::: "memory");
+        tc_fence_before();
+        __syncwarp();
+        if (lane == 0) mbar_arrive(p_full);
+        PRB_ADD(b_e0, t5);
+      }
+      // ---- output: O / l -> bf16 -> this warp's 32 rows of the item's (now unused) Q slot,
+      // 128B-swizzled, -> one TMA store (pad rows and empty items: 0; rows past M clipped) ----
+      PRB(t6);
+      const float inv = (nch > 0 && lsum > 0.f) ? 1.f / lsum : 0.f;
+      if (nch > 0) {
+        mbar_wait(pv_done, (g - 1) & 1);
+        tc_fence_after();
+      }
+      const uint32_t stage = sQ + my_qs * kTileBytes + q * 32 * 128;
+#pragma unroll 1
+      for (int cq = 0; cq < 2; ++cq) {          // 32 output columns at a time
+        uint32_t o[32];
+        if (nch > 0) tmem_ld32_sync(o_addr + 32 * cq, o);
+#pragma unroll
+        for (int t = 0; t < 4; ++t) {
+          uint32_t xp[4];
+#pragma unroll
+          for (int e = 0; e < 4; ++e) {
+            const int j = 8 * t + 2 * e;
+            const float a = inv == 0.f ? 0.f : __uint_as_float(o[j]) * inv;
+            const float b = inv == 0.f ? 0.f : __uint_as_float(o[j + 1]) * inv;
+            __nv_bfloat162 hv = __floats2bfloat162_rn(a, b);
+            xp[e] = *reinterpret_cast<uint32_t*>(&hv);
+          }
+          const int chunk = 4 * cq + t;
+          asm volatile("st.shared.v4.b32 [%0], {%1, %2, %3, %4};" ::"r"(
+                           stage + lane * 128 + ((chunk ^ (lane & 7)) << 4)),
+                       "r"(xp[0]), "r"(xp[1]), "r"(xp[2]), "r"(xp[3])
+                       : "memory");
+        }
+      }
+      asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
+      __syncwarp();
+      if (lane == 0) {
+        asm volatile("cp.async.bulk.tensor.2d.global.shared::cta.bulk_group [%0, {%2, %3}], [%1];" ::"l"(
+                         reinterpret_cast<uint64_t>(&tmO)),
+                     "r"(stage), "r"(h * DH), "r"(qb * TQ + q * 32)
+                     : "memory");
+        asm volatile("cp.async.bulk.commit_group;" ::: "memory");
+        asm volatile("cp.async.bulk.wait_group.read 0;" ::: "memory");
+        mbar_arrive(q_empty + 8 * my_qs);       // the slot may take the next Q
+      }
+      __syncwarp();
+      tc_fence_before();                        // O reads done before the next item's P V
+      PRB_ADD(b_epi, t6);
+    }
+#ifdef TCB_ATTN_PROBE
+    if (lane == 0 && blockIdx.x < 3 && warp == 4)
+      printf("a3probe sm cta %d total %lld wait_q %lld wait_s %lld pass1 %lld wait_pv %lld exp1 %lld exp0 %lld epi %lld chunks %u\n",
+             blockIdx.x, clock64() - b_start, b_q, b_s, b_p1, b_pv, b_e1, b_e0, b_epi, g);
+#endif
+  }
+  __syncwarp();
+  tc_fence_before();
+  __syncthreads();
+  tc_fence_after();
+  if (warp == 1)
+    asm volatile("tcgen05.dealloc.cta_group::1.sync.aligned.b32 %0, %1;" ::"r"(tmem), "r"(kTmemCols) : "memory");
+}
+}  // namespace v3s
+
 
 }  // namespace
 
 cudaError_t launch_attention_bf16_tc(int64_t num_slots, int d_model, int num_heads,
                                      const void* qkv, const int32_t* seg_ids,
                                      const int4* segtab, void* O, int* item_counter,
-                                     cudaStream_t s) {
+                                     int row_len, cudaStream_t s) {
   if (num_slots == 0) return cudaSuccess;
   static const bool use_v1 = [] {              // TCB_ATTN=v1: the previous kernel (A/B only)
     const char* v = std::getenv("TCB_ATTN");
@@ -1258,6 +1780,9 @@ cudaError_t launch_attention_bf16_tc(int64_t num_slots, int d_model, int num_hea
     if (e == cudaSuccess)
       e = cudaFuncSetAttribute(v3::attn_tc3_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize,
                                v3::kSmemBytes);
+    if (e == cudaSuccess)
+      e = cudaFuncSetAttribute(v3s::attn_tc3s_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize,
+                               v3s::kSmemBytes);
 
     if (e != cudaSuccess) return e;
     int dev = 0;
@@ -1284,6 +1809,15 @@ cudaError_t launch_attention_bf16_tc(int64_t num_slots, int d_model, int num_hea
   CUtensorMap omap;
   if (!make_tmap_bf16(&omap, O, static_cast<uint64_t>(num_slots), static_cast<uint64_t>(d_model), 32, 64, 128))
     return cudaErrorInvalidValue;
+  static const int sched_env = [] {             // TCB_ATTN_SCHED=0/1 forces either (A/B)
+    const char* v = std::getenv("TCB_ATTN_SCHED");
+    return v ? std::atoi(v) : -1;
+  }();
+  const bool sched = sched_env >= 0 ? sched_env == 1 : (row_len > 0 && row_len <= TK);
+  if (sched)
+    return launch_ex(v3s::attn_tc3s_kernel, dim3(grid), dim3(v3s::kThreads), v3s::kSmemBytes, s, 1,
+                     map, omap, seg_ids, segtab, static_cast<__nv_bfloat16*>(O), num_slots,
+                     d_model, num_heads, items, scale_log2, item_counter);
   return launch_ex(v3::attn_tc3_kernel, dim3(grid), dim3(v3::kThreads), v3::kSmemBytes, s, 1, map,
                    omap, seg_ids, segtab, static_cast<__nv_bfloat16*>(O), num_slots, d_model,
                    num_heads, items, scale_log2, item_counter);

@@ -126,9 +126,11 @@ size_t linear_ln_scratch_cnt_bytes(int64_t M);
 // Attention ------------------------------------------------------------------------------
 // tcgen05 kernel (attention_tc.cu): S and O in TMEM, 128-query x 128-key chunks.  item_counter:
 // one int32 in device memory, zero at launch (dynamic item scheduling); NULL = static order.
+// row_len: the batch's row length when known (<= 128 selects the scheduler-warp variant for
+// one-chunk items), 0 otherwise.
 cudaError_t launch_attention_bf16_tc(int64_t num_slots, int d_model, int num_heads,
                                      const void* qkv, const int32_t* seg_ids, const int4* segtab,
-                                     void* O, int* item_counter, cudaStream_t s);
+                                     void* O, int* item_counter, int row_len, cudaStream_t s);
 cudaError_t launch_attention_f32(int64_t num_slots, int d_model, int num_heads,
                                  const float* qkv, const int32_t* seg_ids, const int4* segtab,
                                  float* O, cudaStream_t s);

@@ -362,3 +362,17 @@ def test_unpack_roundtrip_exact():
     for s, req in enumerate(a["seg_req"]):
         st = a["seg_start"][s]
         assert torch.equal(o[cu[req]:cu[req + 1]], r[st:st + lengths[req]])
+
+
+def test_attention_scheduler_variant_ops():
+    """The scheduler-warp attention kernel (v3s; the forward uses it for rows of <= 128 slots)
+    on every attention op test of this file: subprocess with TCB_ATTN_SCHED=1 (read once)."""
+    import os
+    import subprocess
+    import sys
+    root = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+    env = dict(os.environ, TCB_ATTN_SCHED="1")
+    r = subprocess.run([sys.executable, "-m", "pytest", "-q", "-x", "-p", "no:cacheprovider",
+                        "tests/test_gpu_kernels.py", "-k", "attention and not scheduler_variant"],
+                       env=env, capture_output=True, text=True, cwd=root, timeout=900)
+    assert r.returncode == 0, r.stdout[-3000:] + r.stderr[-2000:]

@@ -16,7 +16,7 @@ torch = pytest.importorskip("torch")
 pytestmark = pytest.mark.gpu
 
 import paper_conf_icpp_fuc0z22_b200 as tcb  # noqa: E402
-from _helpers import TOL, oracle_selected_rows, per_request_errors, segments_in_rows  # noqa: E402
+from _helpers import TOL, oracle_selected_rows, per_request_errors, segments_in_rows, small_model  # noqa: E402
 
 
 def _gpu_rows(enc, lengths, ids, L, max_rows=0, policy="first_fit", slot_len=0):
@@ -270,3 +270,48 @@ def test_tail_overlap_option_parity(mode):
     r = subprocess.run([sys.executable, "-c", code], env=env, capture_output=True, text=True,
                        cwd=os.path.dirname(os.path.dirname(os.path.abspath(__file__))), timeout=600)
     assert r.returncode == 0, r.stderr[-2000:]
+
+
+@pytest.mark.parametrize("copy_stream", [False, True])
+def test_session_host_buffers_equal_device_path(copy_stream):
+    """tcb_session_run (host ids in, host outputs out, two device slots used in turn): five
+    consecutive batches of different plans through one session give bitwise the outputs of
+    the device-buffer path (tcb_encoder_forward + tcb_unpack), and the first batch matches the
+    oracle at the bf16 bar."""
+    model = small_model("sess", d=512, h=8, f=2048, layers=2, dtype="bf16", act="relu",
+                        vocab=1000, max_pos=128)
+    w = wl.draw_weights(model, 21)
+    names = wl.weight_names(model)
+    enc = tcb.Encoder(model, w, names)
+    B, L = 8, 128
+    batches = []
+    for b in range(5):
+        lengths = wl.lengths_filling("paracrawl", B, L, 70 + b, 0.9)
+        ids = wl.draw_token_ids(int(lengths.sum()), model.vocab, 80 + b)
+        batches.append((lengths, ids))
+    max_t = max(int(l.sum()) for l, _ in batches)
+    sess = enc.session(B, L, max_t)
+    st = torch.cuda.Stream()
+    cs = torch.cuda.Stream() if copy_stream else None
+    outs, tickets = [], []
+    for lengths, ids in batches:
+        plan = tcb.tcb_pack(lengths, L, B)
+        h_ids = torch.from_numpy(ids).pin_memory()
+        h_out = torch.empty((max_t, model.d_model), dtype=torch.bfloat16).pin_memory()
+        tickets.append(sess.run(plan, h_ids, h_out, st, cs))
+        outs.append((plan, h_out))
+    for t in tickets:
+        sess.wait(t)
+    for (lengths, ids), (plan, h_out) in zip(batches, outs):
+        T = plan.info["total_tokens"]
+        _, _, ref = enc.run(lengths, ids, L, B)
+        torch.cuda.synchronize()
+        assert torch.equal(h_out[:T], ref.cpu()), "session output differs from the device path"
+    lengths, ids = batches[0]
+    res = oracle.run(model, w, names, lengths, ids, L, B)
+    got = outs[0][1][:int(lengths.sum())].float().numpy()
+    cu = np.concatenate([[0], np.cumsum(lengths)])
+    for r in range(len(lengths)):
+        o = res["out"][cu[r]:cu[r + 1]]
+        e = np.max(np.abs(got[cu[r]:cu[r + 1]] - o)) / np.max(np.abs(o))
+        assert e <= TOL["bf16"], (r, e)
