@@ -469,12 +469,13 @@ def main():
     }
     # the kernels that run for each class (api.cu / linear_tc.cu dispatch)
     ln_o = {512: "linear_ln_kernel<false>", 768: "linear_lnc_kernel<3>", 1024: "linear_lnc_kernel<4>"}
-    ln_2 = {512: "linear_lng_kernel<2>", 768: "linear_lnc_kernel<3>", 1024: "linear_lng_kernel<4>"}
+    ln_2 = {512: "linear_lng_kernel<2>", 768: "linear_lng_kernel<3>", 1024: "linear_lng_kernel<4>"}
     names = {"gemm_qkv": "linear_tc_kernel<2,256,EPI_BIAS> (QKV)",
              "gemm_o": f"{ln_o.get(d)} (W_O + residual + LN1)" if fused_ln else "linear_tc_kernel (W_O + residual)",
              "gemm_ffn1": "linear_tc_kernel<2,256,EPI_ACT> (FFN1 + act)",
              "gemm_ffn2": f"{ln_2.get(d)} (FFN2 + residual + LN2)" if fused_ln else "linear_tc_kernel (FFN2 + residual)",
-             "attention": "v3::attn_tc3_kernel (segment-masked attention; Q,K,V in + O out)",
+             "attention": ("v3s::attn_tc3s_kernel" if L <= 128 else "v3::attn_tc3_kernel") +
+                          " (segment-masked attention; Q,K,V in + O out)",
              "embed": "pack_embed_kernel", "layernorm": "layernorm_kernel", "unpack": "unpack_kernel"}
     classes = {}
     for c, (bound, w) in work.items():

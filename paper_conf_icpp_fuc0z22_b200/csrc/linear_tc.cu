@@ -2119,7 +2119,9 @@ cudaError_t launch_linear_ln_bf16_tc(const GemmMaps& m, int64_t M, int N, int K,
     if (N == 512 && K >= 2 * N)             // C2 FFN2: 73.4 -> 71.0 us (148 vs 132 SMs)
       return launch_lng<2>(m, static_cast<int>(M), K, bias, gamma, beta, eps, seg_ids, lng_stats,
                            lng_cnt, s, ready_out);
-    if (N == 768 && ln_env == 2)
+    // d = 768: FFN2 (K = 4d) on all pairs measured 139-142 vs 145-147 us (C3, r02al); W_O
+    // (K = d) stays on the cluster kernel (60 vs 72 us)
+    if (N == 768 && (K >= 2 * N || ln_env == 2))
       return launch_lng<3>(m, static_cast<int>(M), K, bias, gamma, beta, eps, seg_ids, lng_stats,
                            lng_cnt, s, ready_out);
   }
