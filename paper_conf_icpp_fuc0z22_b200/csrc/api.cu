@@ -179,6 +179,7 @@ struct tcb_weights {
   float* pe_table = nullptr;
   struct LayerMaps {
     CUtensorMap qkv, o, w1, w2;  // W operands (built once)
+    CUtensorMap w2h;             // W_2 with 64-row boxes (128-column LN units, TCB_LNG_UNIT)
   };
   std::vector<LayerMaps> maps;
   // activation TMA descriptors, rebuilt when the (rows, workspace) pointers change:
@@ -358,7 +359,8 @@ tcb_status tcb_weights_create(const tcb_model_config* cfg, const void* const* te
       bool ok = tcb::k::make_gemm_w_map(&w->maps[l].qkv, w->L(l, W_QKV), 3 * d, d) &&
                 tcb::k::make_gemm_w_map(&w->maps[l].o, w->L(l, W_O), d, d) &&
                 tcb::k::make_gemm_w_map(&w->maps[l].w1, w->L(l, W_1), f, d) &&
-                tcb::k::make_gemm_w_map(&w->maps[l].w2, w->L(l, W_2), d, f);
+                tcb::k::make_gemm_w_map(&w->maps[l].w2, w->L(l, W_2), d, f) &&
+                tcb::k::make_gemm_w_half_map(&w->maps[l].w2h, w->L(l, W_2), d, f);
       if (!ok) {
         if (w->pe_table) cudaFree(w->pe_table);
         delete w;
@@ -612,7 +614,9 @@ tcb_status forward_impl(const tcb_weights* wc, const tcb_plan* plan, const int32
                                          xov_dyn ? gemm_cnt + 2 * l + 1 : nullptr,
                                          ffn1_x ? ready(2 * l) : nullptr, 4 * d));
       if (fuse_ln) {   // FFN2 + bias + residual + LN2 in one kernel -> X
-        const tcb::k::GemmMaps g_2_ln{aH, mp.w2, cX, cX1};
+        tcb::k::GemmMaps g_2_ln{aH, mp.w2, cX, cX1};
+        g_2_ln.w_half = mp.w2h;
+        g_2_ln.has_w_half = true;
         TCB_LAUNCH(TCB_K_GEMM_FFN2, s, tcb::k::launch_linear_ln_bf16_tc(
                                            g_2_ln, M, d, f, w->Lf(l, B_2), w->Lf(l, LN2_G),
                                            w->Lf(l, LN2_B), c.ln_eps, seg, s, lnst, lncnt(2 * l + 1),
@@ -866,8 +870,10 @@ tcb_status tcb_op_linear_ln(int64_t M, int32_t N, int32_t K, const void* A, cons
   cudaStream_t s = reinterpret_cast<cudaStream_t>(stream);
   tcb::k::GemmMaps maps;
   if (!tcb::k::make_gemm_a_map(&maps.a, A, M, K) || !tcb::k::make_gemm_w_map(&maps.w, W, N, K) ||
+      !tcb::k::make_gemm_w_half_map(&maps.w_half, W, N, K) ||
       !tcb::k::make_gemm_c_map(&maps.c, C, M, N) || !tcb::k::make_gemm_c_map(&maps.r, R, M, N))
     return fail(TCB_ERR_CUDA, "tcb_op_linear_ln: cuTensorMapEncodeTiled failed (alignment?)");
+  maps.has_w_half = true;
   // the row-statistics scratch of the L2-exchange kernel (N = 512 / 1024 with K >= 2N, or
   // every N under TCB_LN_KERNEL=global): stream-ordered allocation per call, so calls on
   // different streams never share counters (the encoder forward uses its workspace instead)

@@ -1583,19 +1583,23 @@ linear_lnc_kernel(const __grid_constant__ CUtensorMap tmA, const __grid_constant
 // pairs, one CTA per SM) and a unit only waits for units of its own tile, each of which
 // depends only on work of lower index (its pair's previous units).  The counters of a launch
 // are zeroed by the caller (one memset per forward, a distinct region per launch).
-template <int P>
+template <int P, int UN>
 __global__ void __launch_bounds__(kLncThreads, 1)
 linear_lng_kernel(const __grid_constant__ CUtensorMap tmA, const __grid_constant__ CUtensorMap tmW,
                   const __grid_constant__ CUtensorMap tmC, const __grid_constant__ CUtensorMap tmR,
                   int M, int K, const float* __restrict__ bias, const float* __restrict__ gamma,
                   const float* __restrict__ beta, float eps, const int32_t* __restrict__ seg_ids,
                   float2* __restrict__ gstats, int* __restrict__ gcnt, int* __restrict__ ready_out) {
-  constexpr int kStageBytes = 2 * 128 * BK * 2;
-  constexpr int kEpiBytes = kLncEpiWarps * kLncChunks * kStageBufBytes;
+  // UN = the width of one unit's column block (256, or 128 for finer units: twice the units,
+  // so the last round of a grid of 74 pairs is fuller)
+  constexpr int kCh = UN / kLncColGroups / 32;              // 32-column chunks per warp
+  constexpr int kBBytes = (UN / 2) * BK * 2;                // this CTA's W rows per stage
+  constexpr int kStageBytes = 128 * BK * 2 + kBBytes;
+  constexpr int kEpiBytes = kLncEpiWarps * kCh * kStageBufBytes;
   constexpr int S = (227 * 1024 - 1024 - kEpiBytes - 1024) / kStageBytes;
   constexpr int kABytes = 128 * BK * 2;
   constexpr int kContrib = P * kLncColGroups;
-  constexpr float kInvN = 1.f / (P * 256);
+  constexpr float kInvN = 1.f / (P * UN);
   extern __shared__ uint8_t smem_raw[];
   uint8_t* smem = reinterpret_cast<uint8_t*>((reinterpret_cast<uintptr_t>(smem_raw) + 1023) &
                                              ~static_cast<uintptr_t>(1023));
@@ -1607,7 +1611,7 @@ linear_lng_kernel(const __grid_constant__ CUtensorMap tmA, const __grid_constant
   uint64_t* tfull = empty + S;                               // [2]
   uint64_t* tempty = tfull + 2;                              // [2] (pair leader)
   uint64_t* rbar = tempty + 2;                               // [warps][chunks] residual loads
-  uint32_t* tmem_slot = reinterpret_cast<uint32_t*>(rbar + kLncEpiWarps * kLncChunks);
+  uint32_t* tmem_slot = reinterpret_cast<uint32_t*>(rbar + kLncEpiWarps * kCh);
 
   const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
   const uint32_t r = cluster_rank() & 1u;
@@ -1621,7 +1625,7 @@ linear_lng_kernel(const __grid_constant__ CUtensorMap tmA, const __grid_constant
     asm volatile("prefetch.tensormap [%0];" ::"l"(reinterpret_cast<uint64_t>(&tmC)) : "memory");
     for (int i = 0; i < S; ++i) { mbar_init(&full[i], 1); mbar_init(&empty[i], 1); }
     for (int i = 0; i < 2; ++i) { mbar_init(&tfull[i], 1); mbar_init(&tempty[i], 2 * kLncEpiWarps); }
-    for (int i = 0; i < kLncEpiWarps * kLncChunks; ++i) mbar_init(&rbar[i], 1);
+    for (int i = 0; i < kLncEpiWarps * kCh; ++i) mbar_init(&rbar[i], 1);
     asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
   }
   if (warp == 2) {
@@ -1645,13 +1649,13 @@ linear_lng_kernel(const __grid_constant__ CUtensorMap tmA, const __grid_constant
       for (int u = pair; u < num_units; u += num_pairs) {
         const int t = u / P, p = u % P;
         const int a_row = t * 256 + static_cast<int>(r) * 128;
-        const int b_row = p * 256 + static_cast<int>(r) * 128;
+        const int b_row = p * UN + static_cast<int>(r) * (UN / 2);
         for (int kb = 0; kb < num_kb; ++kb) {
           mbar_wait(&empty[stage], phase ^ 1);
           if (r == 0) mbar_expect_tx(&full[stage], 2 * kStageBytes);
           const uint32_t fb = full0 + 8u * stage;
           tma_load_2d<2>(sA + stage * kABytes, &tmA, fb, kb * BK, a_row);
-          tma_load_2d<2>(sB + stage * kABytes, &tmW, fb, kb * BK, b_row);
+          tma_load_2d<2>(sB + stage * kBBytes, &tmW, fb, kb * BK, b_row);
           if (++stage == S) { stage = 0; phase ^= 1; }
         }
       }
@@ -1659,19 +1663,19 @@ linear_lng_kernel(const __grid_constant__ CUtensorMap tmA, const __grid_constant
   } else if (warp == 1) {
     // ===== MMA issuer: the pair leader drives M=256 x N=256 into accumulator acc =====
     if (r == 0) {
-      constexpr uint32_t idesc = idesc_bf16<2, 256>();
+      constexpr uint32_t idesc = idesc_bf16<2, UN>();
       int stage = 0, acc = 0;
       uint32_t phase = 0, acc_phase = 0;
       for (int u = pair; u < num_units; u += num_pairs) {
         mbar_wait(&tempty[acc], acc_phase ^ 1);
         tc_fence_after();
-        const uint32_t d_tmem = tmem_base + static_cast<uint32_t>(acc * 256);
+        const uint32_t d_tmem = tmem_base + static_cast<uint32_t>(acc * UN);
         for (int kb = 0; kb < num_kb; ++kb) {
           mbar_wait(&full[stage], phase);
           tc_fence_after();
           if (lane == 0) {
             const uint32_t a0 = smem_u32(sA + stage * kABytes);
-            const uint32_t b0 = smem_u32(sB + stage * kABytes);
+            const uint32_t b0 = smem_u32(sB + stage * kBBytes);
 #pragma unroll
             for (int k = 0; k < BK / 16; ++k)
               tc_mma<2>(d_tmem, sdesc_sw128(a0 + k * 32), sdesc_sw128(b0 + k * 32), idesc,
@@ -1692,8 +1696,8 @@ linear_lng_kernel(const __grid_constant__ CUtensorMap tmA, const __grid_constant
     const int q = warp & 3;                       // TMEM lane quarter
     const int cg = ew >> 2;                       // column group of the unit's 256 columns
     const int srow = q * 32 + lane;               // row within this CTA's 128
-    const uint32_t bufs = smem_u32(sEpi) + ew * kLncChunks * kStageBufBytes;
-    uint64_t* my_rbar = rbar + kLncChunks * ew;
+    const uint32_t bufs = smem_u32(sEpi) + ew * kCh * kStageBufBytes;
+    uint64_t* my_rbar = rbar + kCh * ew;
     const uint32_t tempty0 = mapa_rank(smem_u32(tempty), 0);
     int acc = 0;
     uint32_t acc_phase = 0, rphase = 0;
@@ -1710,18 +1714,18 @@ linear_lng_kernel(const __grid_constant__ CUtensorMap tmA, const __grid_constant
 #endif
       const int wid = p * kLncColGroups + cg;     // contribution slot of this warp
       const int row0 = t * 256 + static_cast<int>(r) * 128 + q * 32;
-      const int col0 = p * 256 + cg * (32 * kLncChunks);
+      const int col0 = p * UN + cg * (32 * kCh);
       const int64_t grow = static_cast<int64_t>(row0) + lane;
       const bool pad = grow >= M || (seg_ids && __ldg(&seg_ids[grow]) < 0);
       if (lane == 0) {
-        if (ready_out && prev_blk >= 0) ready_signal(ready_out + prev_blk, 32 * kLncChunks);
+        if (ready_out && prev_blk >= 0) ready_signal(ready_out + prev_blk, 32 * kCh);
         else bulk_wait_read<0>();
       }
       prev_blk = t * 2 + static_cast<int>(r);
       __syncwarp();
       if (lane == 0) {
 #pragma unroll
-        for (int j = 0; j < kLncChunks; ++j) {
+        for (int j = 0; j < kCh; ++j) {
           mbar_expect_tx(&my_rbar[j], kStageBufBytes);
           tma_load_res(bufs + j * kStageBufBytes, &tmR, &my_rbar[j], col0 + 32 * j, row0);
         }
@@ -1733,11 +1737,11 @@ linear_lng_kernel(const __grid_constant__ CUtensorMap tmA, const __grid_constant
       e_tfull += tb - ta;
 #endif
       const uint32_t tbase = tmem_base + (static_cast<uint32_t>(q * 32) << 16) +
-                             static_cast<uint32_t>(acc * 256 + cg * (32 * kLncChunks));
+                             static_cast<uint32_t>(acc * UN + cg * (32 * kCh));
       // pass 1: z = acc + bias + residual -> TMEM; row partial moments
       float sum = 0.f, sumsq = 0.f;
 #pragma unroll 1
-      for (int j = 0; j < kLncChunks; ++j) {
+      for (int j = 0; j < kCh; ++j) {
         uint32_t rr[32];
         tmem_ld32_nowait(tbase + 32 * j, rr);
         tmem_wait_ld();
@@ -1821,11 +1825,11 @@ linear_lng_kernel(const __grid_constant__ CUtensorMap tmA, const __grid_constant
 #endif
       // pass 2: normalise -> bf16 -> staging -> TMA store
 #pragma unroll 1
-      for (int j = 0; j < kLncChunks; ++j) {
+      for (int j = 0; j < kCh; ++j) {
         uint32_t rr[32];
         tmem_ld32_nowait(tbase + 32 * j, rr);
         tmem_wait_ld();
-        if (j == kLncChunks - 1) {
+        if (j == kCh - 1) {
           tc_fence_before();
           __syncwarp();
           if (lane == 0) mbar_arrive_remote(tempty0 + 8u * acc);
@@ -1874,7 +1878,7 @@ linear_lng_kernel(const __grid_constant__ CUtensorMap tmA, const __grid_constant
       if (acc == 0) acc_phase ^= 1;
     }
     if (lane == 0) {
-      if (ready_out && prev_blk >= 0) ready_signal(ready_out + prev_blk, 32 * kLncChunks);
+      if (ready_out && prev_blk >= 0) ready_signal(ready_out + prev_blk, 32 * kCh);
       else bulk_wait_all();
     }
 #ifdef TCB_LN_PROBE
@@ -2011,16 +2015,16 @@ cudaError_t launch_lnc(const GemmMaps& m, int M, int K, const float* bias, const
 
 // The L2-exchange kernel (clusters of one pair, every pair of the GPU).  `stats` holds
 // ceil(M/256) * 2P * 256 float2, `cnt` ceil(M/256) * 8 int32 zeroed before the launch.
-template <int P>
+template <int P, int UN>
 cudaError_t launch_lng(const GemmMaps& m, int M, int K, const float* bias, const float* gamma,
                        const float* beta, float eps, const int32_t* seg_ids, float2* stats,
                        int* cnt, cudaStream_t s, int* ready_out) {
-  constexpr int kStageBytes = 2 * 128 * BK * 2;
-  constexpr int kEpiBytes = kLncEpiWarps * kLncChunks * kStageBufBytes;
+  constexpr int kStageBytes = 128 * BK * 2 + (UN / 2) * BK * 2;
+  constexpr int kEpiBytes = kLncEpiWarps * (UN / kLncColGroups / 32) * kStageBufBytes;
   constexpr int S = (227 * 1024 - 1024 - kEpiBytes - 1024) / kStageBytes;
   constexpr int kSmem = 1024 + S * kStageBytes + kEpiBytes + 1024;
   static_assert(kSmem <= 232448, "shared memory budget");
-  auto kern = linear_lng_kernel<P>;
+  auto kern = linear_lng_kernel<P, UN>;
   static int max_pairs = 0;
   cudaLaunchConfig_t cfg{};
   cfg.blockDim = dim3(kLncThreads);
@@ -2048,7 +2052,7 @@ cudaError_t launch_lng(const GemmMaps& m, int M, int K, const float* bias, const
   // The P units of a tile must sit on P distinct pairs (a unit waits for its tile's other
   // units; two on one pair would wait for themselves): with fewer co-resident pairs than P
   // (an SM-limited context) use the cluster kernel instead.
-  if (max_pairs < P) return launch_lnc<P>(m, M, K, bias, gamma, beta, eps, seg_ids, s, ready_out);
+  if (max_pairs < P) return launch_lnc<P * UN / 256>(m, M, K, bias, gamma, beta, eps, seg_ids, s, ready_out);
   const int units = ((M + 255) / 256) * P;
   const int pairs = units < max_pairs ? units : max_pairs;
   cfg.gridDim = dim3(2 * pairs);
@@ -2082,8 +2086,8 @@ cudaError_t launch_lng(const GemmMaps& m, int M, int K, const float* bias, const
   return e;
 }
 
-size_t linear_ln_scratch_stats_bytes(int64_t M, int N) {
-  return static_cast<size_t>((M + 255) / 256) * (N / 256) * kLncColGroups * 256 * sizeof(float2);
+size_t linear_ln_scratch_stats_bytes(int64_t M, int N) {   // room for 128-column units
+  return static_cast<size_t>((M + 255) / 256) * (N / 128) * kLncColGroups * 256 * sizeof(float2);
 }
 size_t linear_ln_scratch_cnt_bytes(int64_t M) {
   return static_cast<size_t>((M + 255) / 256) * 8 * sizeof(int);
@@ -2114,15 +2118,23 @@ cudaError_t launch_linear_ln_bf16_tc(const GemmMaps& m, int64_t M, int N, int K,
   }();
   if (lng_stats && lng_cnt && ln_env != 1) {
     if (N == 1024 && (K >= 2 * N || ln_env == 2))
-      return launch_lng<4>(m, static_cast<int>(M), K, bias, gamma, beta, eps, seg_ids, lng_stats,
+      return launch_lng<4, 256>(m, static_cast<int>(M), K, bias, gamma, beta, eps, seg_ids, lng_stats,
                            lng_cnt, s, ready_out);
-    if (N == 512 && K >= 2 * N)             // C2 FFN2: 73.4 -> 71.0 us (148 vs 132 SMs)
-      return launch_lng<2>(m, static_cast<int>(M), K, bias, gamma, beta, eps, seg_ids, lng_stats,
-                           lng_cnt, s, ready_out);
+    if (N == 512 && (K >= 2 * N || ln_env == 2)) {   // C2 FFN2: 73.4 -> 71.0 us (148 vs 132 SMs)
+      static const int unit = [] {          // TCB_LNG_UNIT=128: 128-column units (A/B)
+        const char* e = std::getenv("TCB_LNG_UNIT");
+        return e ? std::atoi(e) : 256;
+      }();
+      if (unit == 128 && m.has_w_half)
+        return launch_lng<4, 128>(m.with_w_half(), static_cast<int>(M), K, bias, gamma, beta, eps,
+                                  seg_ids, lng_stats, lng_cnt, s, ready_out);
+      return launch_lng<2, 256>(m, static_cast<int>(M), K, bias, gamma, beta, eps, seg_ids, lng_stats,
+                                lng_cnt, s, ready_out);
+    }
     // d = 768: FFN2 (K = 4d) on all pairs measured 139-142 vs 145-147 us (C3, r02al); W_O
     // (K = d) stays on the cluster kernel (60 vs 72 us)
     if (N == 768 && (K >= 2 * N || ln_env == 2))
-      return launch_lng<3>(m, static_cast<int>(M), K, bias, gamma, beta, eps, seg_ids, lng_stats,
+      return launch_lng<3, 256>(m, static_cast<int>(M), K, bias, gamma, beta, eps, seg_ids, lng_stats,
                            lng_cnt, s, ready_out);
   }
   // d = 512: the single-pair kernel measured 2% faster per forward (C2) than the 4-CTA
@@ -2199,6 +2211,9 @@ bool make_gemm_a_map(CUtensorMap* map, const void* A, uint64_t M, uint64_t K) {
 bool make_gemm_w_map(CUtensorMap* map, const void* W, uint64_t N, uint64_t K) {
   const GemmShape g = linear_tc_shape(static_cast<int>(N));
   return make_tmap_bf16(map, W, N, K, static_cast<uint32_t>(g.bn / g.cg), BK, 128);
+}
+bool make_gemm_w_half_map(CUtensorMap* map, const void* W, uint64_t N, uint64_t K) {
+  return make_tmap_bf16(map, W, N, K, 64, BK, 128);
 }
 bool make_gemm_c_map(CUtensorMap* map, const void* C, uint64_t M, uint64_t N) {
   return make_tmap_bf16(map, C, M, N, kStageRows, kStageCols, 64);

@@ -41,11 +41,13 @@ def one(path):
 
 if __name__ == "__main__":
     allr = []
-    for p in sorted(glob.glob(sys.argv[1] + "/full_*.ncu-rep")):
-        allr += one(p)
+    for p in sorted(glob.glob(sys.argv[1] + "/*.ncu-rep")):
+        for d in one(p):
+            d["capture"] = p.split("/")[-1].replace(".ncu-rep", "")
+            allr.append(d)
     print("# ncu --set full --clock-control none (cold cache, kernel replayed): bytes in MB, time in us")
     cols = ["time", "sm_clk", "dram_rd", "dram_wr", "dram_%", "tensor_%", "sm_%", "occ_%", "regs", "grid"]
     print("%-62s " % "kernel" + " ".join("%9s" % c for c in cols))
     for d in allr:
-        print("%-62s " % d["kernel"] + " ".join("%9.2f" % d.get(c, float("nan")) for c in cols))
+        print("%-62s " % (d["capture"][:3] + d["kernel"][:58]) + " ".join("%9.2f" % d.get(c, float("nan")) for c in cols))
     json.dump(allr, open(sys.argv[2], "w"), indent=1) if len(sys.argv) > 2 else None

@@ -111,6 +111,19 @@ def test_linear_ln_l2_exchange_kernel_everywhere():
     assert r.returncode == 0, r.stderr[-2000:]
 
 
+def test_linear_ln_l2_exchange_128_column_units():
+    """TCB_LNG_UNIT=128: the L2-exchange kernel at N = 512 with four 128-column units per row
+    tile (eight partials per row through L2) instead of two 256-column ones."""
+    import subprocess, sys, os
+    code = ("import sys; sys.path.insert(0, 'tests'); import test_gpu_kernels as t; "
+            "t.test_linear_ln_fused_vs_oracle(4133, 2048, 512); t.test_linear_ln_fused_vs_oracle(1, 2048, 512); "
+            "t.test_linear_ln_fused_vs_oracle(32768, 2048, 512); t.test_linear_ln_fused_vs_oracle(513, 4096, 512)")
+    env = dict(os.environ, TCB_LNG_UNIT="128")
+    r = subprocess.run([sys.executable, "-c", code], env=env, capture_output=True, text=True,
+                       cwd=os.path.dirname(os.path.dirname(os.path.abspath(__file__))), timeout=300)
+    assert r.returncode == 0, r.stderr[-2000:]
+
+
 @pytest.mark.parametrize("M,N,K", [(64, 192, 64), (130, 256, 64), (37, 64, 256)])
 @pytest.mark.parametrize("epi", ["bias", "bias_gelu", "bias_residual"])
 def test_linear_f32_simt_vs_oracle(M, N, K, epi):
