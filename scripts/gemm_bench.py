@@ -7,7 +7,11 @@ import paper_conf_icpp_fuc0z22_b200 as tcb
 
 SHAPES = [(32768, 1536, 512, "bias"), (32768, 512, 512, "bias_residual"),
           (32768, 2048, 512, "bias_relu"), (32768, 512, 2048, "bias_residual"),
+          (32768, 2304, 768, "bias"), (32768, 3072, 768, "bias_gelu"),
+          (32768, 3072, 1024, "bias"), (32768, 4096, 1024, "bias_gelu"),
           (8192, 8192, 8192, "bias")]
+if os.environ.get("SHAPES"):
+    SHAPES = [tuple(int(x) for x in s.split(",")[:3]) + (s.split(",")[3],) for s in os.environ["SHAPES"].split()]
 
 def t_ms(fn, it=20):
     for _ in range(3): fn()

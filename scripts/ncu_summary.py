@@ -14,9 +14,14 @@ SCALE = {"byte": 1, "Kbyte": 1e3, "Mbyte": 1e6, "Gbyte": 1e9, "nsecond": 1e-3, "
 
 
 def one(path):
-    out = subprocess.run(["ncu", "-i", path, "--page", "raw", "--csv"], capture_output=True,
-                         text=True).stdout
+    if path.endswith(".csv"):           # raw page exported on the GPU box
+        out = open(path).read()
+    else:
+        out = subprocess.run(["ncu", "-i", path, "--page", "raw", "--csv"], capture_output=True,
+                             text=True).stdout
     rows = list(csv.reader(io.StringIO(out)))
+    if len(rows) < 3 or "Kernel Name" not in rows[0]:
+        return []
     hdr, units = rows[0], rows[1]
     res = []
     for r in rows[2:]:
@@ -41,13 +46,14 @@ def one(path):
 
 if __name__ == "__main__":
     allr = []
-    for p in sorted(glob.glob(sys.argv[1] + "/*.ncu-rep")):
+    paths = sorted(glob.glob(sys.argv[1] + "/*.ncu-rep")) + sorted(glob.glob(sys.argv[1] + "/*.csv"))
+    for p in paths:
         for d in one(p):
-            d["capture"] = p.split("/")[-1].replace(".ncu-rep", "")
+            d["capture"] = p.split("/")[-1].replace(".ncu-rep", "").replace(".csv", "")
             allr.append(d)
     print("# ncu --set full --clock-control none (cold cache, kernel replayed): bytes in MB, time in us")
     cols = ["time", "sm_clk", "dram_rd", "dram_wr", "dram_%", "tensor_%", "sm_%", "occ_%", "regs", "grid"]
     print("%-62s " % "kernel" + " ".join("%9s" % c for c in cols))
     for d in allr:
-        print("%-62s " % (d["capture"][:3] + d["kernel"][:58]) + " ".join("%9.2f" % d.get(c, float("nan")) for c in cols))
+        print("%-62s " % (d["capture"][:16] + " " + d["kernel"].split("::")[-1][:45]) + " ".join("%9.2f" % d.get(c, float("nan")) for c in cols))
     json.dump(allr, open(sys.argv[2], "w"), indent=1) if len(sys.argv) > 2 else None

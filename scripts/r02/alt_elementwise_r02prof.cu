@@ -57,138 +57,17 @@ __device__ __forceinline__ float warp_sum(float v) {
   return v;
 }
 
-// One CTA per (batch row, kRowChunk-slot chunk of it).  The row's segment records (row_first[]
-// of the device segment table gives them in O(1)) are staged in shared memory; one thread per
-// slot of the chunk resolves (segment, position, token id) by a binary search in smem, so the
-// dependent-load chain (table header -> row_first -> records -> token id -> embedding row) is
-// paid once per chunk, every id load of the chunk in flight together.  Each warp then owns
-// kRowChunk / 8 slots and streams them kSB at a time: all of a batch's embedding-row and
-// position-row loads are issued before the first is consumed, so a lane keeps kSB * NV
-// 16-byte HBM loads in flight (the chain, not the bandwidth, bounded the one-slot-per-step
-// version: 0.27-0.39 of HBM).
+// One CTA per (batch row, 64-slot chunk of it).  The row's segment records (row_first[] of
+// the device segment table gives them in O(1)) are staged in shared memory; each warp then
+// owns slots j = chunk*64 + warp, +8, ... and finds its segment by a binary search in smem.
 #ifndef TCB_ROW_CHUNK
-#define TCB_ROW_CHUNK 64
+#define TCB_ROW_CHUNK 16
 #endif
-constexpr int kRowChunk = TCB_ROW_CHUNK;   // slots per CTA
+constexpr int kRowChunk = TCB_ROW_CHUNK;   // slots per CTA (64 measured slower: fewer CTAs in flight)
 static_assert(kRowChunk <= kWarpsPerBlock * 32, "one metadata thread per slot of a chunk");
-static_assert(kRowChunk % kWarpsPerBlock == 0, "whole slots per warp");
-
-// raw 16-byte vectors of a slot's embedding row and position row, loaded before any use
-template <typename T, int NV, bool PE_TABLE> struct SlotRaw {
-  static constexpr int V = Vec<T>::N;
-  static constexpr int kPeVec = PE_TABLE ? V / 4 : 1;   // float4 (table) or one T-vector per vector
-  uint4 e[NV];
-  uint4 p[NV][kPeVec];
-};
-
-template <typename T, int NV, bool PE_TABLE>
-__device__ __forceinline__ void slot_load(const EmbedArgs& a, int lane, int pos, int id,
-                                          SlotRaw<T, NV, PE_TABLE>& r) {
+template <typename T, int NV>
+__global__ void __launch_bounds__(kWarpsPerBlock * 32) pack_embed_kernel(EmbedArgs a) {
   constexpr int V = Vec<T>::N;
-  const int nvec = a.d / V;
-  if (pos < 0) return;
-  const uint4* e = reinterpret_cast<const uint4*>(reinterpret_cast<const T*>(a.tok_emb) +
-                                                  static_cast<int64_t>(id) * a.d);
-#pragma unroll
-  for (int jv = 0; jv < NV; ++jv) {
-    const int i = lane + 32 * jv;
-    if (i < nvec) {
-      r.e[jv] = __ldg(e + i);
-      if constexpr (PE_TABLE) {
-        const uint4* pt = reinterpret_cast<const uint4*>(a.pe_table + static_cast<int64_t>(pos) * a.d + i * V);
-#pragma unroll
-        for (int c = 0; c < SlotRaw<T, NV, PE_TABLE>::kPeVec; ++c) r.p[jv][c] = __ldg(pt + c);
-      } else {
-        r.p[jv][0] = __ldg(reinterpret_cast<const uint4*>(reinterpret_cast<const T*>(a.pos_emb) +
-                                                          static_cast<int64_t>(pos) * a.d) + i);
-      }
-    }
-  }
-}
-
-template <typename T, int NV, bool PE_TABLE>
-__device__ __forceinline__ void slot_finish(const EmbedArgs& a, int lane, int pos, T* x,
-                                            const SlotRaw<T, NV, PE_TABLE>& r, const float* s_type,
-                                            const float* s_g, const float* s_b) {
-  constexpr int V = Vec<T>::N;
-  const int nvec = a.d / V;
-  if (pos < 0) {                                  // pad slot: zeros (R12)
-    float z[V] = {};
-    for (int i = lane; i < nvec; i += 32) Vec<T>::store(x + i * V, z);
-    return;
-  }
-  float v[NV][V];
-  float sum = 0.f;
-#pragma unroll
-  for (int jv = 0; jv < NV; ++jv) {
-    const int i = lane + 32 * jv;
-    if (i < nvec) {
-      Vec<T>::load(reinterpret_cast<const T*>(&r.e[jv]), v[jv]);
-      float p[V];
-      if constexpr (PE_TABLE) {
-        const float* pf = reinterpret_cast<const float*>(&r.p[jv][0]);
-#pragma unroll
-        for (int c = 0; c < V; ++c) p[c] = pf[c];
-      } else {
-        Vec<T>::load(reinterpret_cast<const T*>(&r.p[jv][0]), p);
-      }
-      if (a.type_emb) {
-#pragma unroll
-        for (int c = 0; c < V; c += 4) {
-          const float4 ty = *reinterpret_cast<const float4*>(s_type + i * V + c);
-          p[c] += ty.x; p[c + 1] += ty.y; p[c + 2] += ty.z; p[c + 3] += ty.w;
-        }
-      }
-#pragma unroll
-      for (int c = 0; c < V; ++c) {
-        const float t = v[jv][c] * a.emb_scale + p[c];
-        v[jv][c] = t;
-        sum += t;
-      }
-    }
-  }
-  if (a.ln_g) {
-    const float mean = warp_sum(sum) / a.d;
-    float sq = 0.f;
-#pragma unroll
-    for (int jv = 0; jv < NV; ++jv)
-      if (lane + 32 * jv < nvec)
-#pragma unroll
-        for (int c = 0; c < V; ++c) { const float t = v[jv][c] - mean; sq += t * t; }
-    const float rstd = rsqrtf(warp_sum(sq) / a.d + a.ln_eps);
-#pragma unroll
-    for (int jv = 0; jv < NV; ++jv) {
-      const int i = lane + 32 * jv;
-      if (i < nvec)
-#pragma unroll
-        for (int c = 0; c < V; c += 4) {
-          const float4 g4 = *reinterpret_cast<const float4*>(s_g + i * V + c);
-          const float4 b4 = *reinterpret_cast<const float4*>(s_b + i * V + c);
-          v[jv][c] = (v[jv][c] - mean) * rstd * g4.x + b4.x;
-          v[jv][c + 1] = (v[jv][c + 1] - mean) * rstd * g4.y + b4.y;
-          v[jv][c + 2] = (v[jv][c + 2] - mean) * rstd * g4.z + b4.z;
-          v[jv][c + 3] = (v[jv][c + 3] - mean) * rstd * g4.w + b4.w;
-        }
-    }
-  }
-#pragma unroll
-  for (int jv = 0; jv < NV; ++jv) {
-    const int i = lane + 32 * jv;
-    if (i < nvec) Vec<T>::store(x + i * V, v[jv]);
-  }
-}
-
-template <typename T, int NV, bool PE_TABLE>
-__global__ void __launch_bounds__(kWarpsPerBlock * 32, 2) pack_embed_kernel(EmbedArgs a) {
-  // slots in flight per warp: the raw registers of a batch stay near 64 per lane
-  constexpr int kRawRegs = NV * 4 * (1 + (PE_TABLE ? Vec<T>::N / 4 : 1));
-#ifdef TCB_EMB_SB
-  constexpr int kSB = TCB_EMB_SB;
-#else
-  constexpr int kSB = kRawRegs <= 16 ? 4 : kRawRegs <= 32 ? 2 : 1;
-#endif
-  constexpr int kPerWarp = kRowChunk / kWarpsPerBlock;
-  static_assert(kPerWarp % kSB == 0, "whole batches per warp");
   extern __shared__ int4 row_recs[];
   const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
   const int row = blockIdx.x;
@@ -210,9 +89,14 @@ __global__ void __launch_bounds__(kWarpsPerBlock * 32, 2) pack_embed_kernel(Embe
     }
   }
   __syncthreads();
+  const int d = a.d;
+  const int nvec = d / V;
   const int64_t row0 = static_cast<int64_t>(row) * a.row_len;
   const int jc0 = static_cast<int>(blockIdx.y) * kRowChunk;
   const int j_end = min(a.row_len, jc0 + kRowChunk);
+  // one thread per slot of the chunk resolves (segment, position, token id) -- every id load
+  // of the chunk in flight together -- and writes the slot metadata coalesced; the warps then
+  // wait on only the embedding-row load per slot
   __shared__ int2 s_meta[kRowChunk];   // (position, token id); position -1 at pad
   if (jc0 + static_cast<int>(threadIdx.x) < j_end) {
     const int64_t slot = row0 + jc0 + threadIdx.x;
@@ -232,23 +116,78 @@ __global__ void __launch_bounds__(kWarpsPerBlock * 32, 2) pack_embed_kernel(Embe
     s_meta[threadIdx.x] = make_int2(pos, id);
   }
   __syncthreads();
-  // warp w: slots jc0 + w * kPerWarp + [0, kPerWarp), kSB at a time
-  for (int b = 0; b < kPerWarp; b += kSB) {
-    SlotRaw<T, NV, PE_TABLE> raw[kSB];
-    int pos[kSB];
+  for (int j = jc0 + warp; j < j_end; j += kWarpsPerBlock) {
+    const int64_t slot = row0 + j;
+    T* x = reinterpret_cast<T*>(a.X) + slot * d;
+    const int2 m = s_meta[j - jc0];
+    const int pos = m.x, id = m.y;
+    if (pos < 0) {                        // pad slot: zeros
+      float z[V] = {};
+      for (int i = lane; i < nvec; i += 32) Vec<T>::store(x + i * V, z);
+      continue;
+    }
+    const T* e = reinterpret_cast<const T*>(a.tok_emb) + static_cast<int64_t>(id) * d;
+    float v[NV][V];
+    float sum = 0.f;
 #pragma unroll
-    for (int u = 0; u < kSB; ++u) {
-      const int jl = warp * kPerWarp + b + u;
-      const int2 m = jc0 + jl < j_end ? s_meta[jl] : make_int2(-2, 0);
-      pos[u] = m.x;
-      slot_load<T, NV, PE_TABLE>(a, lane, m.x, m.y, raw[u]);
+    for (int jv = 0; jv < NV; ++jv) {
+      const int i = lane + 32 * jv;
+      if (i < nvec) {
+        Vec<T>::load(e + i * V, v[jv]);
+        float p[V];
+        if (a.pe_table) {
+          const float* pt = a.pe_table + static_cast<int64_t>(pos) * d + i * V;
+#pragma unroll
+          for (int c = 0; c < V; c += 4) {
+            float4 q = __ldg(reinterpret_cast<const float4*>(pt + c));
+            p[c] = q.x; p[c + 1] = q.y; p[c + 2] = q.z; p[c + 3] = q.w;
+          }
+        } else {
+          Vec<T>::load(reinterpret_cast<const T*>(a.pos_emb) + static_cast<int64_t>(pos) * d + i * V, p);
+        }
+        if (a.type_emb) {
+#pragma unroll
+          for (int c = 0; c < V; c += 4) {
+            const float4 ty = *reinterpret_cast<const float4*>(s_type + i * V + c);
+            p[c] += ty.x; p[c + 1] += ty.y; p[c + 2] += ty.z; p[c + 3] += ty.w;
+          }
+        }
+#pragma unroll
+        for (int c = 0; c < V; ++c) {
+          const float t = v[jv][c] * a.emb_scale + p[c];
+          v[jv][c] = t;
+          sum += t;
+        }
+      }
+    }
+    if (a.ln_g) {
+      const float mean = warp_sum(sum) / d;
+      float sq = 0.f;
+#pragma unroll
+      for (int jv = 0; jv < NV; ++jv)
+        if (lane + 32 * jv < nvec)
+#pragma unroll
+          for (int c = 0; c < V; ++c) { const float t = v[jv][c] - mean; sq += t * t; }
+      const float rstd = rsqrtf(warp_sum(sq) / d + a.ln_eps);
+#pragma unroll
+      for (int jv = 0; jv < NV; ++jv) {
+        const int i = lane + 32 * jv;
+        if (i < nvec)
+#pragma unroll
+          for (int c = 0; c < V; c += 4) {
+            const float4 g4 = *reinterpret_cast<const float4*>(s_g + i * V + c);
+            const float4 b4 = *reinterpret_cast<const float4*>(s_b + i * V + c);
+            v[jv][c] = (v[jv][c] - mean) * rstd * g4.x + b4.x;
+            v[jv][c + 1] = (v[jv][c + 1] - mean) * rstd * g4.y + b4.y;
+            v[jv][c + 2] = (v[jv][c + 2] - mean) * rstd * g4.z + b4.z;
+            v[jv][c + 3] = (v[jv][c + 3] - mean) * rstd * g4.w + b4.w;
+          }
+      }
     }
 #pragma unroll
-    for (int u = 0; u < kSB; ++u) {
-      if (pos[u] == -2) continue;        // beyond the row
-      const int64_t slot = row0 + jc0 + warp * kPerWarp + b + u;
-      slot_finish<T, NV, PE_TABLE>(a, lane, pos[u], reinterpret_cast<T*>(a.X) + slot * a.d, raw[u],
-                                   s_type, s_g, s_b);
+    for (int jv = 0; jv < NV; ++jv) {
+      const int i = lane + 32 * jv;
+      if (i < nvec) Vec<T>::store(x + i * V, v[jv]);
     }
   }
 }
@@ -442,17 +381,17 @@ cudaError_t launch_embed(int dtype, const EmbedArgs& a, cudaStream_t s) {
   cudaError_t attr_err = cudaSuccess, launch_err = cudaSuccess;
   auto go = [&](auto tag) {
     constexpr int NV = decltype(tag)::value;
-    auto run = [&](auto kern) {
-      if (smem > 48 * 1024)
-        attr_err = cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, static_cast<int>(smem));
-      launch_err = launch_ex(kern, grid, dim3(kWarpsPerBlock * 32), smem, s, 1, a);
-    };
     if (dtype == 0) {
-      if (a.pe_table) run(pack_embed_kernel<float, NV, true>);
-      else run(pack_embed_kernel<float, NV, false>);
+      if (smem > 48 * 1024)
+        attr_err = cudaFuncSetAttribute(pack_embed_kernel<float, NV>,
+                                        cudaFuncAttributeMaxDynamicSharedMemorySize, static_cast<int>(smem));
+      launch_err = launch_ex(pack_embed_kernel<float, NV>, grid, dim3(kWarpsPerBlock * 32), smem, s, 1, a);
     } else {
-      if (a.pe_table) run(pack_embed_kernel<__nv_bfloat16, NV, true>);
-      else run(pack_embed_kernel<__nv_bfloat16, NV, false>);
+      if (smem > 48 * 1024)
+        attr_err = cudaFuncSetAttribute(pack_embed_kernel<__nv_bfloat16, NV>,
+                                        cudaFuncAttributeMaxDynamicSharedMemorySize, static_cast<int>(smem));
+      launch_err = launch_ex(pack_embed_kernel<__nv_bfloat16, NV>, grid, dim3(kWarpsPerBlock * 32), smem, s,
+                             1, a);
     }
   };
   if (!dispatch_nv(nv, go)) return cudaErrorInvalidValue;

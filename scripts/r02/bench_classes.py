@@ -11,4 +11,4 @@ for w in sys.argv[1:] or ["c2"]:
     d = json.loads(line[-1])
     print(json.dumps({"workload": f"{w}:step_ms", "us": d["ms_per_step"] * 1e3}), flush=True)
     for c, v in d["roofline"]["classes"].items():
-        print(json.dumps({"workload": f"{w}:{c}", "us": v["us_per_launch"]}), flush=True)
+        print(json.dumps({"workload": f"{w}:{c}", "us": v["us_per_launch"], "iso_us": v.get("isolated", {}).get("us_per_launch")}), flush=True)

@@ -297,7 +297,12 @@ def _scaled(mkey, pe, scale):
                                              # both sinusoidal readings (R1) with emb_scale != 1 (R3)
                                              ("transformer-base", 128, "sin_paper", 22.627416997969522),
                                              ("transformer-base", 128, "sin_vaswani", 2.5),
-                                             ("toy", 32, "sin_vaswani", 8.0)])
+                                             ("toy", 32, "sin_vaswani", 8.0),
+                                             # 64-slot chunks, slots in batches of 2 per warp:
+                                             # ragged last chunk (104 = 64 + 40, 72 = 64 + 8)
+                                             ("transformer-base", 104, None, None),
+                                             ("bert-large", 72, None, None),
+                                             ("transformer-big", 72, None, None)])
 def test_pack_embed_metadata_bit_exact_and_values(mkey, L, pe, scale):
     model = wl.MODELS[mkey] if pe is None else _scaled(mkey, pe, scale)
     w = wl.draw_weights(model, 2)
