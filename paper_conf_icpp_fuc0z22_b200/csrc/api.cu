@@ -179,7 +179,7 @@ struct tcb_weights {
   float* pe_table = nullptr;
   struct LayerMaps {
     CUtensorMap qkv, o, w1, w2;  // W operands (built once)
-    CUtensorMap w2h;             // W_2 with 64-row boxes (128-column LN units, TCB_LNG_UNIT)
+    CUtensorMap w2h;             // W_2 with 64-row boxes (half-width tail units of the LN GEMM)
   };
   std::vector<LayerMaps> maps;
   // activation TMA descriptors, rebuilt when the (rows, workspace) pointers change:

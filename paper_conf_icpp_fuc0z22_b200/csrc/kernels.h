@@ -92,14 +92,9 @@ cudaError_t launch_linear_f32(int64_t M, int N, int K, const float* A, const flo
 // 64B swizzle; R is read only by the residual epilogue).
 struct GemmMaps {
   CUtensorMap a, w, c, r;
-  // optional: W with 64-row boxes (the 128-column units of the L2-exchange LayerNorm GEMM)
+  // optional: W with 64-row boxes (the half-width tail units of the L2-exchange LayerNorm GEMM)
   CUtensorMap w_half;
   bool has_w_half = false;
-  GemmMaps with_w_half() const {
-    GemmMaps g = *this;
-    g.w = w_half;
-    return g;
-  }
 };
 struct GemmShape {
   int cg, bn;  // CTAs per MMA tile (cta_group) and tile width in N
@@ -109,7 +104,7 @@ bool make_tmap_bf16(CUtensorMap* map, const void* ptr, uint64_t rows, uint64_t c
                     uint32_t box_rows, uint32_t box_cols, int swizzle_bytes);
 bool make_gemm_a_map(CUtensorMap* map, const void* A, uint64_t M, uint64_t K);
 bool make_gemm_w_map(CUtensorMap* map, const void* W, uint64_t N, uint64_t K);
-// W with 64-row boxes: the 128-column units of the L2-exchange LayerNorm GEMM (TCB_LNG_UNIT)
+// W with 64-row boxes: the half-width tail units of the L2-exchange LayerNorm GEMM
 bool make_gemm_w_half_map(CUtensorMap* map, const void* W, uint64_t N, uint64_t K);
 bool make_gemm_c_map(CUtensorMap* map, const void* C, uint64_t M, uint64_t N);
 // tile_counter (one int32, zero at launch): dynamic tile order.  a_ready: readiness flags of

@@ -1583,23 +1583,25 @@ linear_lnc_kernel(const __grid_constant__ CUtensorMap tmA, const __grid_constant
 // pairs, one CTA per SM) and a unit only waits for units of its own tile, each of which
 // depends only on work of lower index (its pair's previous units).  The counters of a launch
 // are zeroed by the caller (one memset per forward, a distinct region per launch).
-template <int P, int UN>
+template <int P>
 __global__ void __launch_bounds__(kLncThreads, 1)
 linear_lng_kernel(const __grid_constant__ CUtensorMap tmA, const __grid_constant__ CUtensorMap tmW,
                   const __grid_constant__ CUtensorMap tmC, const __grid_constant__ CUtensorMap tmR,
+                  const __grid_constant__ CUtensorMap tmWh,
                   int M, int K, const float* __restrict__ bias, const float* __restrict__ gamma,
                   const float* __restrict__ beta, float eps, const int32_t* __restrict__ seg_ids,
-                  float2* __restrict__ gstats, int* __restrict__ gcnt, int* __restrict__ ready_out) {
-  // UN = the width of one unit's column block (256, or 128 for finer units: twice the units,
-  // so the last round of a grid of 74 pairs is fuller)
-  constexpr int kCh = UN / kLncColGroups / 32;              // 32-column chunks per warp
-  constexpr int kBBytes = (UN / 2) * BK * 2;                // this CTA's W rows per stage
+                  float2* __restrict__ gstats, int* __restrict__ gcnt, int* __restrict__ ready_out,
+                  int full_units) {
+  // Units u < full_units are 256 columns wide (P per row tile); the row tiles after them
+  // (the last, partial round of the grid) are split into 2P units of 128 columns (W via
+  // tmWh's 64-row boxes, N = 128 MMAs), so that round spreads over twice as many pairs.
+  constexpr int kCh = 256 / kLncColGroups / 32;             // 32-column chunks per warp (full unit)
+  constexpr int kBBytes = 128 * BK * 2;                     // this CTA's W rows per stage (full unit)
   constexpr int kStageBytes = 128 * BK * 2 + kBBytes;
   constexpr int kEpiBytes = kLncEpiWarps * kCh * kStageBufBytes;
   constexpr int S = (227 * 1024 - 1024 - kEpiBytes - 1024) / kStageBytes;
   constexpr int kABytes = 128 * BK * 2;
-  constexpr int kContrib = P * kLncColGroups;
-  constexpr float kInvN = 1.f / (P * UN);
+  constexpr float kInvN = 1.f / (P * 256);
   extern __shared__ uint8_t smem_raw[];
   uint8_t* smem = reinterpret_cast<uint8_t*>((reinterpret_cast<uintptr_t>(smem_raw) + 1023) &
                                              ~static_cast<uintptr_t>(1023));
@@ -1616,13 +1618,21 @@ linear_lng_kernel(const __grid_constant__ CUtensorMap tmA, const __grid_constant
   const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
   const uint32_t r = cluster_rank() & 1u;
   const int pair = blockIdx.x >> 1, num_pairs = gridDim.x >> 1;
-  const int num_units = ((M + 255) / 256) * P;
+  const int tiles_full = full_units / P;
+  const int num_units = full_units + ((M + 255) / 256 - tiles_full) * 2 * P;
+  // unit -> (row tile, column block, half width?)
+  auto unit_of = [&](int u, int& t, int& p, bool& half) {
+    if (u < full_units) { t = u / P; p = u % P; half = false; }
+    else { const int v = u - full_units; t = tiles_full + v / (2 * P); p = v % (2 * P); half = true; }
+  };
   const int num_kb = K / BK;
 
   if (warp == 0 && lane == 0) {
     asm volatile("prefetch.tensormap [%0];" ::"l"(reinterpret_cast<uint64_t>(&tmA)) : "memory");
     asm volatile("prefetch.tensormap [%0];" ::"l"(reinterpret_cast<uint64_t>(&tmW)) : "memory");
     asm volatile("prefetch.tensormap [%0];" ::"l"(reinterpret_cast<uint64_t>(&tmC)) : "memory");
+    if (full_units < num_units)
+      asm volatile("prefetch.tensormap [%0];" ::"l"(reinterpret_cast<uint64_t>(&tmWh)) : "memory");
     for (int i = 0; i < S; ++i) { mbar_init(&full[i], 1); mbar_init(&empty[i], 1); }
     for (int i = 0; i < 2; ++i) { mbar_init(&tfull[i], 1); mbar_init(&tempty[i], 2 * kLncEpiWarps); }
     for (int i = 0; i < kLncEpiWarps * kCh; ++i) mbar_init(&rbar[i], 1);
@@ -1647,15 +1657,19 @@ linear_lng_kernel(const __grid_constant__ CUtensorMap tmA, const __grid_constant
       int stage = 0;
       uint32_t phase = 0;
       for (int u = pair; u < num_units; u += num_pairs) {
-        const int t = u / P, p = u % P;
+        int t, p;
+        bool half;
+        unit_of(u, t, p, half);
         const int a_row = t * 256 + static_cast<int>(r) * 128;
-        const int b_row = p * UN + static_cast<int>(r) * (UN / 2);
+        const int b_row = half ? p * 128 + static_cast<int>(r) * 64 : p * 256 + static_cast<int>(r) * 128;
+        const CUtensorMap* wmap = half ? &tmWh : &tmW;
+        const uint32_t tx = 2 * (kABytes + (half ? kBBytes / 2 : kBBytes));
         for (int kb = 0; kb < num_kb; ++kb) {
           mbar_wait(&empty[stage], phase ^ 1);
-          if (r == 0) mbar_expect_tx(&full[stage], 2 * kStageBytes);
+          if (r == 0) mbar_expect_tx(&full[stage], tx);
           const uint32_t fb = full0 + 8u * stage;
           tma_load_2d<2>(sA + stage * kABytes, &tmA, fb, kb * BK, a_row);
-          tma_load_2d<2>(sB + stage * kBBytes, &tmW, fb, kb * BK, b_row);
+          tma_load_2d<2>(sB + stage * kBBytes, wmap, fb, kb * BK, b_row);
           if (++stage == S) { stage = 0; phase ^= 1; }
         }
       }
@@ -1663,13 +1677,14 @@ linear_lng_kernel(const __grid_constant__ CUtensorMap tmA, const __grid_constant
   } else if (warp == 1) {
     // ===== MMA issuer: the pair leader drives M=256 x N=256 into accumulator acc =====
     if (r == 0) {
-      constexpr uint32_t idesc = idesc_bf16<2, UN>();
+      constexpr uint32_t idesc_full = idesc_bf16<2, 256>(), idesc_half = idesc_bf16<2, 128>();
       int stage = 0, acc = 0;
       uint32_t phase = 0, acc_phase = 0;
       for (int u = pair; u < num_units; u += num_pairs) {
+        const uint32_t idesc = u < full_units ? idesc_full : idesc_half;
         mbar_wait(&tempty[acc], acc_phase ^ 1);
         tc_fence_after();
-        const uint32_t d_tmem = tmem_base + static_cast<uint32_t>(acc * UN);
+        const uint32_t d_tmem = tmem_base + static_cast<uint32_t>(acc * 256);
         for (int kb = 0; kb < num_kb; ++kb) {
           mbar_wait(&full[stage], phase);
           tc_fence_after();
@@ -1705,27 +1720,31 @@ linear_lng_kernel(const __grid_constant__ CUtensorMap tmA, const __grid_constant
     long long e0 = clock64(), e_tfull = 0, e_p1 = 0, e_x = 0, e_p2 = 0;
     int nunits = 0;
 #endif
-    int prev_blk = -1;                            // 128-row block of the previous unit
+    int prev_blk = -1, prev_cols = 0;             // 128-row block / columns of the previous unit
     for (int u = pair; u < num_units; u += num_pairs) {
-      const int t = u / P, p = u % P;
+      int t, p;
+      bool half;
+      unit_of(u, t, p, half);
+      const int nch = half ? kCh / 2 : kCh;       // 32-column chunks of this warp in this unit
+      const int kContrib = (half ? 2 * P : P) * kLncColGroups;   // partials per row of tile t
 #ifdef TCB_LN_PROBE
       long long ta = clock64();
       ++nunits;
 #endif
       const int wid = p * kLncColGroups + cg;     // contribution slot of this warp
       const int row0 = t * 256 + static_cast<int>(r) * 128 + q * 32;
-      const int col0 = p * UN + cg * (32 * kCh);
+      const int col0 = half ? p * 128 + cg * (32 * nch) : p * 256 + cg * (32 * nch);
       const int64_t grow = static_cast<int64_t>(row0) + lane;
       const bool pad = grow >= M || (seg_ids && __ldg(&seg_ids[grow]) < 0);
       if (lane == 0) {
-        if (ready_out && prev_blk >= 0) ready_signal(ready_out + prev_blk, 32 * kCh);
+        if (ready_out && prev_blk >= 0) ready_signal(ready_out + prev_blk, prev_cols);
         else bulk_wait_read<0>();
       }
       prev_blk = t * 2 + static_cast<int>(r);
+      prev_cols = 32 * nch;
       __syncwarp();
       if (lane == 0) {
-#pragma unroll
-        for (int j = 0; j < kCh; ++j) {
+        for (int j = 0; j < nch; ++j) {
           mbar_expect_tx(&my_rbar[j], kStageBufBytes);
           tma_load_res(bufs + j * kStageBufBytes, &tmR, &my_rbar[j], col0 + 32 * j, row0);
         }
@@ -1737,11 +1756,11 @@ linear_lng_kernel(const __grid_constant__ CUtensorMap tmA, const __grid_constant
       e_tfull += tb - ta;
 #endif
       const uint32_t tbase = tmem_base + (static_cast<uint32_t>(q * 32) << 16) +
-                             static_cast<uint32_t>(acc * UN + cg * (32 * kCh));
+                             static_cast<uint32_t>(acc * 256 + cg * (32 * nch));
       // pass 1: z = acc + bias + residual -> TMEM; row partial moments
       float sum = 0.f, sumsq = 0.f;
 #pragma unroll 1
-      for (int j = 0; j < kCh; ++j) {
+      for (int j = 0; j < nch; ++j) {
         uint32_t rr[32];
         tmem_ld32_nowait(tbase + 32 * j, rr);
         tmem_wait_ld();
@@ -1790,7 +1809,7 @@ linear_lng_kernel(const __grid_constant__ CUtensorMap tmA, const __grid_constant
       e_p1 += tc2 - tb;
 #endif
       // publish this warp's partials of its 32 rows, then wait for all kContrib of them
-      float2* tst = gstats + static_cast<size_t>(t) * kContrib * 256 + static_cast<int>(r) * 128 + srow;
+      float2* tst = gstats + static_cast<size_t>(t) * (4 * P) * 256 + static_cast<int>(r) * 128 + srow;
       tst[wid * 256] = make_float2(sum, sumsq);
       int* cnt = gcnt + t * 8 + static_cast<int>(r) * 4 + q;
       __syncwarp();
@@ -1804,7 +1823,6 @@ linear_lng_kernel(const __grid_constant__ CUtensorMap tmA, const __grid_constant
       }
       __syncwarp();
       float s1 = 0.f, s2 = 0.f;
-#pragma unroll
       for (int k = 0; k < kContrib; ++k) {
         float2 st;
         asm volatile("ld.relaxed.gpu.global.v2.f32 {%0, %1}, [%2];"
@@ -1825,11 +1843,11 @@ linear_lng_kernel(const __grid_constant__ CUtensorMap tmA, const __grid_constant
 #endif
       // pass 2: normalise -> bf16 -> staging -> TMA store
 #pragma unroll 1
-      for (int j = 0; j < kCh; ++j) {
+      for (int j = 0; j < nch; ++j) {
         uint32_t rr[32];
         tmem_ld32_nowait(tbase + 32 * j, rr);
         tmem_wait_ld();
-        if (j == kCh - 1) {
+        if (j == nch - 1) {
           tc_fence_before();
           __syncwarp();
           if (lane == 0) mbar_arrive_remote(tempty0 + 8u * acc);
@@ -1878,7 +1896,7 @@ linear_lng_kernel(const __grid_constant__ CUtensorMap tmA, const __grid_constant
       if (acc == 0) acc_phase ^= 1;
     }
     if (lane == 0) {
-      if (ready_out && prev_blk >= 0) ready_signal(ready_out + prev_blk, 32 * kCh);
+      if (ready_out && prev_blk >= 0) ready_signal(ready_out + prev_blk, prev_cols);
       else bulk_wait_all();
     }
 #ifdef TCB_LN_PROBE
@@ -2014,17 +2032,18 @@ cudaError_t launch_lnc(const GemmMaps& m, int M, int K, const float* bias, const
 }
 
 // The L2-exchange kernel (clusters of one pair, every pair of the GPU).  `stats` holds
-// ceil(M/256) * 2P * 256 float2, `cnt` ceil(M/256) * 8 int32 zeroed before the launch.
-template <int P, int UN>
+// ceil(M/256) * 4P * 256 float2 (room for half-width units), `cnt` ceil(M/256) * 8 int32
+// zeroed before the launch.
+template <int P>
 cudaError_t launch_lng(const GemmMaps& m, int M, int K, const float* bias, const float* gamma,
                        const float* beta, float eps, const int32_t* seg_ids, float2* stats,
                        int* cnt, cudaStream_t s, int* ready_out) {
-  constexpr int kStageBytes = 128 * BK * 2 + (UN / 2) * BK * 2;
-  constexpr int kEpiBytes = kLncEpiWarps * (UN / kLncColGroups / 32) * kStageBufBytes;
+  constexpr int kStageBytes = 2 * 128 * BK * 2;
+  constexpr int kEpiBytes = kLncEpiWarps * kLncChunks * kStageBufBytes;
   constexpr int S = (227 * 1024 - 1024 - kEpiBytes - 1024) / kStageBytes;
   constexpr int kSmem = 1024 + S * kStageBytes + kEpiBytes + 1024;
   static_assert(kSmem <= 232448, "shared memory budget");
-  auto kern = linear_lng_kernel<P, UN>;
+  auto kern = linear_lng_kernel<P>;
   static int max_pairs = 0;
   cudaLaunchConfig_t cfg{};
   cfg.blockDim = dim3(kLncThreads);
@@ -2052,8 +2071,24 @@ cudaError_t launch_lng(const GemmMaps& m, int M, int K, const float* bias, const
   // The P units of a tile must sit on P distinct pairs (a unit waits for its tile's other
   // units; two on one pair would wait for themselves): with fewer co-resident pairs than P
   // (an SM-limited context) use the cluster kernel instead.
-  if (max_pairs < P) return launch_lnc<P * UN / 256>(m, M, K, bias, gamma, beta, eps, seg_ids, s, ready_out);
-  const int units = ((M + 255) / 256) * P;
+  if (max_pairs < P) return launch_lnc<P>(m, M, K, bias, gamma, beta, eps, seg_ids, s, ready_out);
+  // Tail split: when the last round of full units is partial, the row tiles after the last
+  // complete round are cut into 2P half-width units -- if they then fit in one round of the
+  // grid (C2: 256 units = 3 x 74 + 34 -> 222 full + 68 half; C3: 384 = 5 x 74 + 14 -> 369
+  // full + 30 half; C4 / C5: 512 = 6 x 74 + 68 -> no split).  TCB_LNG_TAIL=0 disables it.
+  static const bool tail_env = [] {
+    const char* e = std::getenv("TCB_LNG_TAIL");
+    return !(e && std::atoi(e) == 0);
+  }();
+  const int tiles = (M + 255) / 256;
+  int full_units = tiles * P;
+  if (tail_env && m.has_w_half && max_pairs >= 2 * P) {
+    const int rounds = full_units / max_pairs;
+    const int aligned = (rounds * max_pairs / P) * P;
+    const int halves = (tiles - aligned / P) * 2 * P;
+    if (rounds > 0 && aligned < full_units && halves <= max_pairs) full_units = aligned;
+  }
+  const int units = full_units + (tiles - full_units / P) * 2 * P;
   const int pairs = units < max_pairs ? units : max_pairs;
   cfg.gridDim = dim3(2 * pairs);
   // cooperative: the runtime guarantees every CTA of the grid is co-resident (the kernel's
@@ -2069,8 +2104,9 @@ cudaError_t launch_lng(const GemmMaps& m, int M, int K, const float* bias, const
     attr3[cfg.numAttrs].val.cooperative = 1;
     ++cfg.numAttrs;
   }
-  cudaError_t e = cudaLaunchKernelEx(&cfg, kern, m.a, m.w, m.c, m.r, M, K, bias, gamma, beta, eps,
-                                     seg_ids, stats, cnt, ready_out);
+  const CUtensorMap& wh = m.has_w_half ? m.w_half : m.w;
+  cudaError_t e = cudaLaunchKernelEx(&cfg, kern, m.a, m.w, m.c, m.r, wh, M, K, bias, gamma, beta, eps,
+                                     seg_ids, stats, cnt, ready_out, full_units);
   if (coop == -1) {
     coop = e == cudaSuccess ? 1 : 0;
     if (std::getenv("TCB_VERBOSE"))
@@ -2079,8 +2115,8 @@ cudaError_t launch_lng(const GemmMaps& m, int M, int K, const float* bias, const
     if (e != cudaSuccess) {       // not supported with these attributes: plain launch
       cudaGetLastError();
       --cfg.numAttrs;
-      e = cudaLaunchKernelEx(&cfg, kern, m.a, m.w, m.c, m.r, M, K, bias, gamma, beta, eps, seg_ids,
-                             stats, cnt, ready_out);
+      e = cudaLaunchKernelEx(&cfg, kern, m.a, m.w, m.c, m.r, wh, M, K, bias, gamma, beta, eps,
+                             seg_ids, stats, cnt, ready_out, full_units);
     }
   }
   return e;
@@ -2118,23 +2154,15 @@ cudaError_t launch_linear_ln_bf16_tc(const GemmMaps& m, int64_t M, int N, int K,
   }();
   if (lng_stats && lng_cnt && ln_env != 1) {
     if (N == 1024 && (K >= 2 * N || ln_env == 2))
-      return launch_lng<4, 256>(m, static_cast<int>(M), K, bias, gamma, beta, eps, seg_ids, lng_stats,
+      return launch_lng<4>(m, static_cast<int>(M), K, bias, gamma, beta, eps, seg_ids, lng_stats,
                            lng_cnt, s, ready_out);
-    if (N == 512 && (K >= 2 * N || ln_env == 2)) {   // C2 FFN2: 73.4 -> 71.0 us (148 vs 132 SMs)
-      static const int unit = [] {          // TCB_LNG_UNIT=128: 128-column units (A/B)
-        const char* e = std::getenv("TCB_LNG_UNIT");
-        return e ? std::atoi(e) : 256;
-      }();
-      if (unit == 128 && m.has_w_half)
-        return launch_lng<4, 128>(m.with_w_half(), static_cast<int>(M), K, bias, gamma, beta, eps,
-                                  seg_ids, lng_stats, lng_cnt, s, ready_out);
-      return launch_lng<2, 256>(m, static_cast<int>(M), K, bias, gamma, beta, eps, seg_ids, lng_stats,
-                                lng_cnt, s, ready_out);
-    }
+    if (N == 512 && (K >= 2 * N || ln_env == 2))   // C2 FFN2: 73.4 -> 71.0 us (148 vs 132 SMs)
+      return launch_lng<2>(m, static_cast<int>(M), K, bias, gamma, beta, eps, seg_ids, lng_stats,
+                           lng_cnt, s, ready_out);
     // d = 768: FFN2 (K = 4d) on all pairs measured 139-142 vs 145-147 us (C3, r02al); W_O
     // (K = d) stays on the cluster kernel (60 vs 72 us)
     if (N == 768 && (K >= 2 * N || ln_env == 2))
-      return launch_lng<3, 256>(m, static_cast<int>(M), K, bias, gamma, beta, eps, seg_ids, lng_stats,
+      return launch_lng<3>(m, static_cast<int>(M), K, bias, gamma, beta, eps, seg_ids, lng_stats,
                            lng_cnt, s, ready_out);
   }
   // d = 512: the single-pair kernel measured 2% faster per forward (C2) than the 4-CTA

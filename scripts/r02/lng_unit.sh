@@ -1,3 +1,4 @@
+# HISTORICAL (r02): the TCB_LNG_UNIT=128 option this script A/Bs was measured slower and removed
 # TCB_LNG_UNIT=128 vs 256: parity (op tests + forward parity) then per-class timing on c2
 cd $GRAFT_REPO_ROOT; T=gpurun_out/${TAG:-lngu}; mkdir -p $T
 python -c "import __graft_entry__ as g; g.build()" > $T/build.log 2>&1; echo build rc $?

@@ -57,7 +57,10 @@ def test_linear_bf16_tcgen05_vs_oracle(M, N, K, epi):
                                    (3001, 3072, 768), (32768, 768, 768), (32768, 3072, 768),
                                    (300, 1024, 1024), (2049, 4096, 1024),
                                    (1, 4096, 1024), (300, 2048, 1024), (32768, 1024, 1024),
-                                   (32768, 4096, 1024)])
+                                   (32768, 4096, 1024),
+                                   # tail split of the L2-exchange kernel (half-width units for
+                                   # the row tiles after the last complete round), ragged M
+                                   (32668, 2048, 512), (26000, 3072, 768)])
 def test_linear_ln_fused_vs_oracle(M, K, N):
     """W_O / FFN2 + bias + residual + LayerNorm in one tcgen05 kernel (N = 512, 768, 1024:
     clusters of N / 256 CTA pairs exchanging the row statistics over DSMEM; N = 1024 with
@@ -111,14 +114,13 @@ def test_linear_ln_l2_exchange_kernel_everywhere():
     assert r.returncode == 0, r.stderr[-2000:]
 
 
-def test_linear_ln_l2_exchange_128_column_units():
-    """TCB_LNG_UNIT=128: the L2-exchange kernel at N = 512 with four 128-column units per row
-    tile (eight partials per row through L2) instead of two 256-column ones."""
+def test_linear_ln_l2_exchange_without_tail_split():
+    """TCB_LNG_TAIL=0: the L2-exchange kernel with full-width units only (the default splits
+    the row tiles after the last complete round of the grid into half-width units)."""
     import subprocess, sys, os
     code = ("import sys; sys.path.insert(0, 'tests'); import test_gpu_kernels as t; "
-            "t.test_linear_ln_fused_vs_oracle(4133, 2048, 512); t.test_linear_ln_fused_vs_oracle(1, 2048, 512); "
-            "t.test_linear_ln_fused_vs_oracle(32768, 2048, 512); t.test_linear_ln_fused_vs_oracle(513, 4096, 512)")
-    env = dict(os.environ, TCB_LNG_UNIT="128")
+            "t.test_linear_ln_fused_vs_oracle(32668, 2048, 512); t.test_linear_ln_fused_vs_oracle(26000, 3072, 768)")
+    env = dict(os.environ, TCB_LNG_TAIL="0")
     r = subprocess.run([sys.executable, "-c", code], env=env, capture_output=True, text=True,
                        cwd=os.path.dirname(os.path.dirname(os.path.abspath(__file__))), timeout=300)
     assert r.returncode == 0, r.stderr[-2000:]
