@@ -302,6 +302,8 @@ def main():
     ap.add_argument("--warmup", type=int, default=5)
     ap.add_argument("--impl", default="ours", choices=["ours", "reference"])
     ap.add_argument("--workload", default="c2", choices=sorted(wl.WORKLOADS))
+    ap.add_argument("--rows", type=int, default=0,
+                    help="batch rows per GPU (default: the workload's B; a sweep knob, not the bench line)")
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--no-graph", action="store_true")
     ap.add_argument("--online", action="store_true",
@@ -326,6 +328,9 @@ def main():
     torch.cuda.set_device(local)
     dev = torch.device("cuda", local)
     key = args.workload
+    if args.rows > 0:                     # batch-size sweep: same workload, B rows per GPU
+        import dataclasses
+        wl.WORKLOADS[key] = dataclasses.replace(wl.WORKLOADS[key], rows=args.rows)
     wlc = wl.WORKLOADS[key]
     model = wlc.model
     names = wl.weight_names(model)
