@@ -241,7 +241,9 @@ tcb_status tcb_unpack(const tcb_weights* w, const tcb_plan* plan, const int32_t*
  * tcb_session_run(plan, h_token_ids, h_out) enqueues on `stream`, using the slots in turn:
  * the plan's segment table is written into the slot's pinned staging (waiting for that slot's
  * previous upload) and copied host->device with h_token_ids ([total_tokens] int32; pinned
- * memory makes the copies asynchronous), then tcb_encoder_forward + tcb_unpack run, then the
+ * memory makes the copies asynchronous) on a stream the session owns -- after the slot's
+ * previous forward, so the upload overlaps the compute of the other slot -- then `stream`
+ * waits for the upload and tcb_encoder_forward + tcb_unpack run, then the
  * per-request outputs are copied device->host into h_out ([total_tokens, d_model], model
  * dtype) -- on `copy_stream` when not NULL (after an event on `stream`, so the copy overlaps
  * the next call's compute), else on `stream`.  *ticket identifies the call;

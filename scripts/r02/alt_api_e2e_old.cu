@@ -701,7 +701,6 @@ struct tcb_session {
     int64_t ticket = -1;                   // last call that used the slot
   } slot[2];
   int64_t calls = 0;
-  cudaStream_t up = nullptr;               // uploads: ahead of the compute stream
 };
 
 namespace {
@@ -718,7 +717,6 @@ void session_free(tcb_session* s) {
     if (sl.computed) cudaEventDestroy(sl.computed);
     if (sl.d2h_done) cudaEventDestroy(sl.d2h_done);
   }
-  if (s->up) cudaStreamDestroy(s->up);
   delete s;
 }
 }  // namespace
@@ -760,7 +758,6 @@ tcb_status tcb_session_create(const tcb_weights* w, int32_t num_rows, int32_t ro
          cudaEventCreateWithFlags(&sl.computed, cudaEventDisableTiming) == cudaSuccess &&
          cudaEventCreateWithFlags(&sl.d2h_done, cudaEventDisableTiming) == cudaSuccess;
   }
-  ok = ok && cudaStreamCreateWithFlags(&s->up, cudaStreamNonBlocking) == cudaSuccess;
   if (!ok) {
     cudaGetLastError();
     session_free(s);
@@ -790,16 +787,11 @@ tcb_status tcb_session_run(tcb_session* s, const tcb_plan* plan, const int32_t* 
     return cuda_fail(cudaGetLastError(), "tcb_session_run: wait for the slot's previous upload");
   if (tcb_status e = tcb_plan_write_segtab(plan, sl.h_seg, s->seg_words)) return e;
   const int64_t words = tcb_plan_segtab_words(plan);
-  // the uploads run on the session's own stream, so they overlap the previous call's forward:
-  // they only wait for the slot's previous forward to have finished reading its buffers
-  cudaError_t e = cudaSuccess;
-  if (sl.ticket >= 0) e = cudaStreamWaitEvent(s->up, sl.computed, 0);
-  if (e == cudaSuccess)
-    e = cudaMemcpyAsync(sl.d_segtab, sl.h_seg, 4 * static_cast<size_t>(words), cudaMemcpyHostToDevice, s->up);
+  cudaError_t e = cudaMemcpyAsync(sl.d_segtab, sl.h_seg, 4 * static_cast<size_t>(words),
+                                  cudaMemcpyHostToDevice, st);
   if (e == cudaSuccess && T > 0)
-    e = cudaMemcpyAsync(sl.d_ids, h_token_ids, 4 * static_cast<size_t>(T), cudaMemcpyHostToDevice, s->up);
-  if (e == cudaSuccess) e = cudaEventRecord(sl.h2d_done, s->up);
-  if (e == cudaSuccess) e = cudaStreamWaitEvent(st, sl.h2d_done, 0);
+    e = cudaMemcpyAsync(sl.d_ids, h_token_ids, 4 * static_cast<size_t>(T), cudaMemcpyHostToDevice, st);
+  if (e == cudaSuccess) e = cudaEventRecord(sl.h2d_done, st);
   // the slot's outputs may still be on their way to the host (previous call of the slot)
   if (e == cudaSuccess && sl.ticket >= 0) e = cudaStreamWaitEvent(st, sl.d2h_done, 0);
   if (e != cudaSuccess) return cuda_fail(e, "tcb_session_run: upload");
@@ -807,8 +799,10 @@ tcb_status tcb_session_run(tcb_session* s, const tcb_plan* plan, const int32_t* 
                                          s->ws_bytes, stream))
     return r;
   if (tcb_status r = tcb_unpack(s->w, plan, sl.d_segtab, sl.d_rows, sl.d_out, stream)) return r;
-  e = cudaEventRecord(sl.computed, st);
-  if (e == cudaSuccess && cs != st) e = cudaStreamWaitEvent(cs, sl.computed, 0);
+  if (cs != st) {
+    e = cudaEventRecord(sl.computed, st);
+    if (e == cudaSuccess) e = cudaStreamWaitEvent(cs, sl.computed, 0);
+  }
   if (e == cudaSuccess && T > 0)
     e = cudaMemcpyAsync(h_out, sl.d_out, s->out_bytes_per_token * static_cast<size_t>(T),
                         cudaMemcpyDeviceToHost, cs);
