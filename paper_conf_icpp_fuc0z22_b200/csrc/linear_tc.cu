@@ -656,6 +656,10 @@ linear_tc_kernel(const __grid_constant__ CUtensorMap tmA, const __grid_constant_
     uint32_t acc_phase = 0;
     int es = 0;
     uint32_t eph = 0;
+#ifdef TCB_GEMM_PROBE
+    long long pe_start = clock64(), pe_wait = 0, pe_work = 0;
+    int pe_tiles = 0;
+#endif
     for (int k = 0;; ++k) {
       int tile = cluster_id + k * num_clusters;
       if (dyn) {
@@ -688,8 +692,16 @@ linear_tc_kernel(const __grid_constant__ CUtensorMap tmA, const __grid_constant_
           }
         }
       }
+#ifdef TCB_GEMM_PROBE
+      long long pw0 = clock64();
+#endif
       mbar_wait(&tfull[acc], acc_phase);
       tc_fence_after();
+#ifdef TCB_GEMM_PROBE
+      long long pw1 = clock64();
+      pe_wait += pw1 - pw0;
+      ++pe_tiles;
+#endif
       const uint32_t tbase = tmem_base + (static_cast<uint32_t>(q * 32) << 16) +
                              static_cast<uint32_t>(acc * BN + half * (BN / 2));
       uint32_t ra[32], rb[32];
@@ -769,9 +781,17 @@ linear_tc_kernel(const __grid_constant__ CUtensorMap tmA, const __grid_constant_
       tc_fence_before();
       __syncwarp();
       if (lane == 0) mbar_arrive_remote(tempty0 + 8u * acc);
+#ifdef TCB_GEMM_PROBE
+      pe_work += clock64() - pw1;
+#endif
       acc ^= 1;
       if (acc == 0) acc_phase ^= 1;
     }
+#ifdef TCB_GEMM_PROBE
+    if (lane == 0 && blockIdx.x < 4 && (warp == 4 || warp == 11))
+      printf("probe epi cta %d warp %d total %lld wait_tfull %lld work %lld tiles %d\n", blockIdx.x, warp,
+             clock64() - pe_start, pe_wait, pe_work, pe_tiles);
+#endif
     if (lane == 0) bulk_wait_all();
   }
   __syncwarp();
