@@ -226,6 +226,18 @@ tcb_status tcb_encoder_forward(const tcb_weights* w, const tcb_plan* plan,
                                void* d_rows, void* d_workspace, size_t workspace_bytes,
                                tcb_stream_t stream);
 
+/* tcb_encoder_forward followed by tcb_unpack into d_out, with the unpack fused into the last
+ * layer's FFN2 + LN2 where the L2-exchange LayerNorm GEMM runs (bf16, d in {512, 768, 1024}):
+ * its epilogue writes each real slot's row to d_out[token_offset(seg) + position] (Concat of
+ * Eq. (8)) instead of to d_rows, so the packed rows are not written back and read
+ * again.  Elsewhere (fp32, other d) it is the two calls.  d_out as for tcb_unpack; d_rows is
+ * used as the layer buffer and holds no defined result afterwards.  Graph replay as for
+ * tcb_encoder_forward (d_out is part of the cache key). */
+tcb_status tcb_encoder_forward_unpacked(const tcb_weights* w, const tcb_plan* plan,
+                                        const int32_t* d_segtab, const int32_t* d_token_ids,
+                                        void* d_rows, void* d_out, void* d_workspace,
+                                        size_t workspace_bytes, tcb_stream_t stream);
+
 /* unpack: out[token_offset(seg) + j] = rows[slot_start(seg) + j] for every segment -- the
  * per-request responses (Concat of Eq. (8)).  d_out is
  * [total_tokens, d_model] in the model dtype; rows of unplaced requests are not written. */
@@ -243,7 +255,7 @@ tcb_status tcb_unpack(const tcb_weights* w, const tcb_plan* plan, const int32_t*
  * previous upload) and copied host->device with h_token_ids ([total_tokens] int32; pinned
  * memory makes the copies asynchronous) on a stream the session owns -- after the slot's
  * previous forward, so the upload overlaps the compute of the other slot -- then `stream`
- * waits for the upload and tcb_encoder_forward + tcb_unpack run, then the
+ * waits for the upload and tcb_encoder_forward_unpacked runs, then the
  * per-request outputs are copied device->host into h_out ([total_tokens, d_model], model
  * dtype) -- on `copy_stream` when not NULL (after an event on `stream`, so the copy overlaps
  * the next call's compute), else on `stream`.  *ticket identifies the call;

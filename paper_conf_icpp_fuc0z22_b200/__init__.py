@@ -281,6 +281,23 @@ class Encoder:
                                         _ptr(rows), _ptr(ws), ws.numel(), _stream_ptr(stream)))
         return rows
 
+    def encoder_forward_unpacked(self, plan: Plan, d_segtab, d_ids, out=None, rows=None,
+                                 stream=None):
+        """tcb_encoder_forward + tcb_unpack in one call (the unpack fused into the last
+        FFN2 + LN2 where possible); returns out [total_tokens, d_model]."""
+        import torch
+        M = plan.num_slots
+        if rows is None:
+            rows = self.alloc_rows(M)
+        if out is None:
+            out = torch.zeros((plan.info["total_tokens"], self.model.d_model), dtype=self.dtype,
+                              device=self.device)
+        ws = self.workspace(M)
+        check(lib().tcb_encoder_forward_unpacked(self._h, plan.handle, _ptr(d_segtab), _ptr(d_ids),
+                                                 _ptr(rows), _ptr(out), _ptr(ws), ws.numel(),
+                                                 _stream_ptr(stream)))
+        return out
+
     def unpack(self, plan: Plan, d_segtab, rows, out=None, stream=None):
         import torch
         if out is None:

@@ -27,6 +27,7 @@ EXPORTS = ["tcb_last_error", "tcb_version", "tcb_pack", "tcb_pack_slotted", "tcb
            "tcb_plan_info_get", "tcb_plan_copy", "tcb_plan_segtab_words",
            "tcb_plan_write_segtab", "tcb_weights_count", "tcb_weights_create",
            "tcb_weights_destroy", "tcb_workspace_size", "tcb_embed", "tcb_encoder_forward",
+           "tcb_encoder_forward_unpacked",
            "tcb_unpack", "tcb_session_create", "tcb_session_run", "tcb_session_wait",
            "tcb_session_destroy", "tcb_launch_count", "tcb_profile_enable", "tcb_profile_collect", "tcb_profile_snapshot",
            "tcb_op_linear", "tcb_op_linear_ln", "tcb_op_attention", "tcb_op_layernorm",
@@ -118,6 +119,7 @@ def lib() -> ctypes.CDLL:
                                      ctypes.POINTER(ctypes.c_size_t)]),
         "tcb_embed": (I32, [P, P, P, P, P, P, P, P]),
         "tcb_encoder_forward": (I32, [P, P, P, P, P, P, ctypes.c_size_t, P]),
+        "tcb_encoder_forward_unpacked": (I32, [P, P, P, P, P, P, P, ctypes.c_size_t, P]),
         "tcb_unpack": (I32, [P, P, P, P, P, P]),
         "tcb_session_create": (I32, [P, I32, I32, I64, ctypes.POINTER(P)]),
         "tcb_session_run": (I32, [P, P, P, P, P, P, ctypes.POINTER(I64)]),

@@ -194,7 +194,7 @@ struct tcb_weights {
   struct FwdGraph {
     int64_t M;
     int32_t rows, row_len;
-    const void *segtab, *ids, *drows, *ws;
+    const void *segtab, *ids, *drows, *ws, *dout;
     cudaGraphExec_t exec;
     uint64_t launches, last_use;
   };
@@ -395,8 +395,8 @@ tcb_status tcb_embed(const tcb_weights* w, const tcb_plan* plan, const int32_t* 
 
 namespace {
 tcb_status forward_impl(const tcb_weights* wc, const tcb_plan* plan, const int32_t* d_segtab,
-                        const int32_t* d_token_ids, void* d_rows, void* d_ws, size_t ws_bytes,
-                        tcb_stream_t stream);
+                        const int32_t* d_token_ids, void* d_rows, void* d_out, void* d_ws,
+                        size_t ws_bytes, tcb_stream_t stream);
 }  // namespace
 
 // The public forward replays a CUDA graph of its own launch sequence when it can: on a
@@ -405,10 +405,11 @@ tcb_status forward_impl(const tcb_weights* wc, const tcb_plan* plan, const int32
 // set of buffers (LRU of 4 per weights handle) and replayed for any later plan of the same
 // B x L (every plan-specific value is read from the device segment table); otherwise the
 // kernels are launched directly.  Either way the work is the same.
-tcb_status tcb_encoder_forward(const tcb_weights* wc, const tcb_plan* plan,
-                               const int32_t* d_segtab, const int32_t* d_token_ids,
-                               void* d_rows, void* d_ws, size_t ws_bytes, tcb_stream_t stream) {
-  tcb::clear_error();
+namespace {
+// d_out == NULL: tcb_encoder_forward; else tcb_encoder_forward_unpacked
+tcb_status forward_entry(const tcb_weights* wc, const tcb_plan* plan, const int32_t* d_segtab,
+                         const int32_t* d_token_ids, void* d_rows, void* d_out, void* d_ws,
+                         size_t ws_bytes, tcb_stream_t stream) {
   static const bool no_graph =
       std::getenv("TCB_NO_FWD_GRAPH") != nullptr || std::getenv("TCB_DEBUG_SYNC") != nullptr;
   cudaStream_t s = reinterpret_cast<cudaStream_t>(stream);
@@ -426,7 +427,7 @@ tcb_status tcb_encoder_forward(const tcb_weights* wc, const tcb_plan* plan,
     }
   }
   if (!use_graph)
-    return forward_impl(wc, plan, d_segtab, d_token_ids, d_rows, d_ws, ws_bytes, stream);
+    return forward_impl(wc, plan, d_segtab, d_token_ids, d_rows, d_out, d_ws, ws_bytes, stream);
   if (tcb_status st = validate_plan_for(wc, plan)) return st;
   // the same argument checks as forward_impl BEFORE a cache hit can replay (a graph captured
   // for an all-pad plan with NULL ids must not serve a plan that has tokens)
@@ -437,7 +438,8 @@ tcb_status tcb_encoder_forward(const tcb_weights* wc, const tcb_plan* plan,
   std::lock_guard<std::mutex> gl(w->graph_mu);
   for (auto& e : w->fwd_graphs) {
     if (e.M == M && e.rows == plan->num_rows && e.row_len == plan->row_len &&
-        e.segtab == d_segtab && e.ids == d_token_ids && e.drows == d_rows && e.ws == d_ws) {
+        e.segtab == d_segtab && e.ids == d_token_ids && e.drows == d_rows && e.ws == d_ws &&
+        e.dout == d_out) {
       if (ws_bytes < ws_layout(w->cfg, M).total)
         break;                                   // let forward_impl report it
       e.last_use = ++w->fwd_tick;
@@ -451,30 +453,30 @@ tcb_status tcb_encoder_forward(const tcb_weights* wc, const tcb_plan* plan,
   if (!w->cap_stream && cudaStreamCreateWithFlags(&w->cap_stream, cudaStreamNonBlocking) != cudaSuccess) {
     cudaGetLastError();
     w->cap_stream = nullptr;
-    return forward_impl(wc, plan, d_segtab, d_token_ids, d_rows, d_ws, ws_bytes, stream);
+    return forward_impl(wc, plan, d_segtab, d_token_ids, d_rows, d_out, d_ws, ws_bytes, stream);
   }
   cudaStream_t cap = w->cap_stream;
   if (cudaStreamBeginCapture(cap, cudaStreamCaptureModeThreadLocal) != cudaSuccess) {
     cudaGetLastError();
-    return forward_impl(wc, plan, d_segtab, d_token_ids, d_rows, d_ws, ws_bytes, stream);
+    return forward_impl(wc, plan, d_segtab, d_token_ids, d_rows, d_out, d_ws, ws_bytes, stream);
   }
   const uint64_t c0 = g_launches.load();
-  const tcb_status st = forward_impl(wc, plan, d_segtab, d_token_ids, d_rows, d_ws, ws_bytes,
-                                     reinterpret_cast<tcb_stream_t>(cap));
+  const tcb_status st = forward_impl(wc, plan, d_segtab, d_token_ids, d_rows, d_out, d_ws,
+                                     ws_bytes, reinterpret_cast<tcb_stream_t>(cap));
   cudaGraph_t graph = nullptr;
   const cudaError_t ce = cudaStreamEndCapture(cap, &graph);
   if (st != TCB_OK || ce != cudaSuccess || !graph) {
     if (graph) cudaGraphDestroy(graph);
     cudaGetLastError();
     if (st != TCB_OK) return st;
-    return forward_impl(wc, plan, d_segtab, d_token_ids, d_rows, d_ws, ws_bytes, stream);
+    return forward_impl(wc, plan, d_segtab, d_token_ids, d_rows, d_out, d_ws, ws_bytes, stream);
   }
   cudaGraphExec_t exec = nullptr;
   const cudaError_t ie = cudaGraphInstantiate(&exec, graph, 0);
   cudaGraphDestroy(graph);
   if (ie != cudaSuccess) {
     cudaGetLastError();
-    return forward_impl(wc, plan, d_segtab, d_token_ids, d_rows, d_ws, ws_bytes, stream);
+    return forward_impl(wc, plan, d_segtab, d_token_ids, d_rows, d_out, d_ws, ws_bytes, stream);
   }
   if (w->fwd_graphs.size() >= 4) {               // evict the least recently used
     auto lru = std::min_element(w->fwd_graphs.begin(), w->fwd_graphs.end(),
@@ -483,10 +485,27 @@ tcb_status tcb_encoder_forward(const tcb_weights* wc, const tcb_plan* plan,
     w->fwd_graphs.erase(lru);
   }
   w->fwd_graphs.push_back({M, plan->num_rows, plan->row_len, d_segtab, d_token_ids, d_rows, d_ws,
-                           exec, g_launches.load() - c0, ++w->fwd_tick});
+                           d_out, exec, g_launches.load() - c0, ++w->fwd_tick});
   const cudaError_t le = cudaGraphLaunch(exec, s);
   if (le != cudaSuccess) return cuda_fail(le, "tcb_encoder_forward: graph launch");
   return TCB_OK;
+}
+}  // namespace
+
+tcb_status tcb_encoder_forward(const tcb_weights* wc, const tcb_plan* plan,
+                               const int32_t* d_segtab, const int32_t* d_token_ids,
+                               void* d_rows, void* d_ws, size_t ws_bytes, tcb_stream_t stream) {
+  tcb::clear_error();
+  return forward_entry(wc, plan, d_segtab, d_token_ids, d_rows, nullptr, d_ws, ws_bytes, stream);
+}
+
+tcb_status tcb_encoder_forward_unpacked(const tcb_weights* wc, const tcb_plan* plan,
+                                        const int32_t* d_segtab, const int32_t* d_token_ids,
+                                        void* d_rows, void* d_out, void* d_ws, size_t ws_bytes,
+                                        tcb_stream_t stream) {
+  tcb::clear_error();
+  if (!d_out) return fail(TCB_ERR_INVALID_ARGUMENT, "tcb_encoder_forward_unpacked: d_out is NULL");
+  return forward_entry(wc, plan, d_segtab, d_token_ids, d_rows, d_out, d_ws, ws_bytes, stream);
 }
 
 namespace {
@@ -496,8 +515,8 @@ struct NvtxRange {
 };
 
 tcb_status forward_impl(const tcb_weights* wc, const tcb_plan* plan, const int32_t* d_segtab,
-                        const int32_t* d_token_ids, void* d_rows, void* d_ws, size_t ws_bytes,
-                        tcb_stream_t stream) {
+                        const int32_t* d_token_ids, void* d_rows, void* d_out, void* d_ws,
+                        size_t ws_bytes, tcb_stream_t stream) {
   NvtxRange nvtx_fwd("tcb_encoder_forward");
   if (tcb_status st = validate_plan_for(wc, plan)) return st;
   tcb_weights* w = const_cast<tcb_weights*>(wc);
@@ -524,6 +543,7 @@ tcb_status forward_impl(const tcb_weights* wc, const tcb_plan* plan, const int32
   const int4* segtab = reinterpret_cast<const int4*>(d_segtab);
 
   if (tcb_status st = embed_impl(w, plan, d_segtab, d_token_ids, d_rows, seg, nullptr, s)) return st;
+  bool out_done = false;                         // d_out written by the fused last FFN2
 
   if (c.dtype == 1) {
     // Activation TMA descriptors: cached per weights handle for the last (rows, workspace, M)
@@ -617,10 +637,27 @@ tcb_status forward_impl(const tcb_weights* wc, const tcb_plan* plan, const int32
         tcb::k::GemmMaps g_2_ln{aH, mp.w2, cX, cX1};
         g_2_ln.w_half = mp.w2h;
         g_2_ln.has_w_half = true;
-        TCB_LAUNCH(TCB_K_GEMM_FFN2, s, tcb::k::launch_linear_ln_bf16_tc(
-                                           g_2_ln, M, d, f, w->Lf(l, B_2), w->Lf(l, LN2_G),
-                                           w->Lf(l, LN2_B), c.ln_eps, seg, s, lnst, lncnt(2 * l + 1),
-                                           (xov && l + 1 < c.num_layers) ? ready(2 * l + 1) : nullptr));
+        bool scattered = false;
+        if (d_out && l + 1 == c.num_layers && lnst) {
+          // the unpack fused into the last FFN2 + LN2: rows go straight to d_out[token]
+          ProfScope ps_(TCB_K_GEMM_FFN2, s);
+          const cudaError_t e = tcb::k::launch_linear_ln_bf16_tc(
+              g_2_ln, M, d, f, w->Lf(l, B_2), w->Lf(l, LN2_G), w->Lf(l, LN2_B), c.ln_eps, seg, s,
+              lnst, lncnt(2 * l + 1), nullptr, d_out, segtab);
+          if (e == cudaSuccess) {
+            g_launches.fetch_add(1, std::memory_order_relaxed);
+            scattered = out_done = true;
+          } else if (e == cudaErrorNotSupported) {
+            cudaGetLastError();                  // packed rows + a separate unpack below
+          } else {
+            return cuda_fail(e, "tcb_encoder_forward_unpacked: last FFN2");
+          }
+        }
+        if (!scattered)
+          TCB_LAUNCH(TCB_K_GEMM_FFN2, s, tcb::k::launch_linear_ln_bf16_tc(
+                                             g_2_ln, M, d, f, w->Lf(l, B_2), w->Lf(l, LN2_G),
+                                             w->Lf(l, LN2_B), c.ln_eps, seg, s, lnst, lncnt(2 * l + 1),
+                                             (xov && l + 1 < c.num_layers) ? ready(2 * l + 1) : nullptr));
       } else {
         TCB_LAUNCH(TCB_K_GEMM_FFN2, s, tcb::k::launch_linear_bf16_tc(g_2, M, d, f, w->Lf(l, B_2),
                                                                      TCB_EPI_BIAS_RESIDUAL, s));
@@ -657,6 +694,9 @@ tcb_status forward_impl(const tcb_weights* wc, const tcb_plan* plan, const int32
                                                        w->Lf(l, LN2_B), c.ln_eps, seg, X, s));
     }
   }
+  if (d_out && !out_done)
+    TCB_LAUNCH(TCB_K_UNPACK, s, tcb::k::launch_unpack(c.dtype, segtab, plan->num_rows,
+                                                      plan->row_len, c.d_model, d_rows, d_out, s));
   if (std::getenv("TCB_DEBUG_SYNC")) {
     cudaError_t e = cudaStreamSynchronize(s);
     if (e != cudaSuccess) return cuda_fail(e, "tcb_encoder_forward (TCB_DEBUG_SYNC)");
@@ -803,10 +843,10 @@ tcb_status tcb_session_run(tcb_session* s, const tcb_plan* plan, const int32_t* 
   // the slot's outputs may still be on their way to the host (previous call of the slot)
   if (e == cudaSuccess && sl.ticket >= 0) e = cudaStreamWaitEvent(st, sl.d2h_done, 0);
   if (e != cudaSuccess) return cuda_fail(e, "tcb_session_run: upload");
-  if (tcb_status r = tcb_encoder_forward(s->w, plan, sl.d_segtab, sl.d_ids, sl.d_rows, sl.d_ws,
-                                         s->ws_bytes, stream))
+  // forward + unpack (fused into the last FFN2 + LN2 where the L2-exchange kernel runs)
+  if (tcb_status r = tcb_encoder_forward_unpacked(s->w, plan, sl.d_segtab, sl.d_ids, sl.d_rows,
+                                                  sl.d_out, sl.d_ws, s->ws_bytes, stream))
     return r;
-  if (tcb_status r = tcb_unpack(s->w, plan, sl.d_segtab, sl.d_rows, sl.d_out, stream)) return r;
   e = cudaEventRecord(sl.computed, st);
   if (e == cudaSuccess && cs != st) e = cudaStreamWaitEvent(cs, sl.computed, 0);
   if (e == cudaSuccess && T > 0)

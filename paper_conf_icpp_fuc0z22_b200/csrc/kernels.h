@@ -124,7 +124,12 @@ cudaError_t launch_linear_ln_bf16_tc(const GemmMaps& maps, int64_t M, int N, int
                                      const float* bias, const float* gamma, const float* beta,
                                      float eps, const int32_t* seg_ids, cudaStream_t s,
                                      float2* lng_stats = nullptr, int* lng_cnt = nullptr,
-                                     int* ready_out = nullptr);
+                                     int* ready_out = nullptr, void* scatter_out = nullptr,
+                                     const int4* segtab = nullptr);
+// scatter_out (with the device segment table): the LayerNorm output of every real slot goes to
+// scatter_out[token, :] in request order (the unpack fused into the encoder's last FFN2 + LN2);
+// the packed C is not written.  The L2-exchange kernel only; cudaErrorNotSupported otherwise
+// (the caller then writes the packed rows and unpacks separately).
 size_t linear_ln_scratch_stats_bytes(int64_t M, int N);
 size_t linear_ln_scratch_cnt_bytes(int64_t M);
 

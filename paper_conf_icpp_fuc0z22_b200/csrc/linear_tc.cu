@@ -1603,7 +1603,11 @@ linear_lnc_kernel(const __grid_constant__ CUtensorMap tmA, const __grid_constant
 // pairs, one CTA per SM) and a unit only waits for units of its own tile, each of which
 // depends only on work of lower index (its pair's previous units).  The counters of a launch
 // are zeroed by the caller (one memset per forward, a distinct region per launch).
-template <int P>
+// SCATTER (the encoder's last FFN2 + LN2 with the unpack fused, Concat of Eq. (8)):
+// instead of the packed rows, each lane writes its row's LayerNorm output straight to the
+// request-order output out_rows[token] (token = the slot's segment record token offset +
+// position; pad slots are not written), 64 B per 32-column chunk.
+template <int P, bool SCATTER = false>
 __global__ void __launch_bounds__(kLncThreads, 1)
 linear_lng_kernel(const __grid_constant__ CUtensorMap tmA, const __grid_constant__ CUtensorMap tmW,
                   const __grid_constant__ CUtensorMap tmC, const __grid_constant__ CUtensorMap tmR,
@@ -1611,7 +1615,8 @@ linear_lng_kernel(const __grid_constant__ CUtensorMap tmA, const __grid_constant
                   int M, int K, const float* __restrict__ bias, const float* __restrict__ gamma,
                   const float* __restrict__ beta, float eps, const int32_t* __restrict__ seg_ids,
                   float2* __restrict__ gstats, int* __restrict__ gcnt, int* __restrict__ ready_out,
-                  int full_units) {
+                  int full_units, __nv_bfloat16* __restrict__ out_rows,
+                  const int4* __restrict__ segtab) {
   // Units u < full_units are 256 columns wide (P per row tile); the row tiles after them
   // (the last, partial round of the grid) are split into 2P units of 128 columns (W via
   // tmWh's 64-row boxes, N = 128 MMAs), so that round spreads over twice as many pairs.
@@ -1755,7 +1760,13 @@ linear_lng_kernel(const __grid_constant__ CUtensorMap tmA, const __grid_constant
       const int row0 = t * 256 + static_cast<int>(r) * 128 + q * 32;
       const int col0 = half ? p * 128 + cg * (32 * nch) : p * 256 + cg * (32 * nch);
       const int64_t grow = static_cast<int64_t>(row0) + lane;
-      const bool pad = grow >= M || (seg_ids && __ldg(&seg_ids[grow]) < 0);
+      const int seg_row = grow < M && seg_ids ? __ldg(&seg_ids[grow]) : -1;
+      const bool pad = grow >= M || (seg_ids && seg_row < 0);
+      int64_t tok_row = -1;                       // SCATTER: the row's request-order token
+      if (SCATTER && !pad) {
+        const int4 rec = __ldg(&segtab[1 + seg_row]);
+        tok_row = static_cast<int64_t>(rec.z) + (grow - rec.x);
+      }
       if (lane == 0) {
         if (ready_out && prev_blk >= 0) ready_signal(ready_out + prev_blk, prev_cols);
         else bulk_wait_read<0>();
@@ -1888,6 +1899,21 @@ linear_lng_kernel(const __grid_constant__ CUtensorMap tmA, const __grid_constant
           y[4 * tt + 1] = z0.y;
           y[4 * tt + 2] = z1.x;
           y[4 * tt + 3] = z1.y;
+        }
+        if constexpr (SCATTER) {
+          if (tok_row >= 0) {
+            uint4* dst = reinterpret_cast<uint4*>(out_rows + tok_row * (P * 256) + gc);
+#pragma unroll
+            for (int tt = 0; tt < 4; ++tt) {
+              uint4 x;
+              __nv_bfloat162* hh = reinterpret_cast<__nv_bfloat162*>(&x);
+#pragma unroll
+              for (int e = 0; e < 4; ++e)
+                hh[e] = __floats2bfloat162_rn(y[8 * tt + 2 * e], y[8 * tt + 2 * e + 1]);
+              dst[tt] = x;
+            }
+          }
+          continue;
         }
         const uint32_t buf = bufs + j * kStageBufBytes;
 #pragma unroll
@@ -2054,16 +2080,17 @@ cudaError_t launch_lnc(const GemmMaps& m, int M, int K, const float* bias, const
 // The L2-exchange kernel (clusters of one pair, every pair of the GPU).  `stats` holds
 // ceil(M/256) * 4P * 256 float2 (room for half-width units), `cnt` ceil(M/256) * 8 int32
 // zeroed before the launch.
-template <int P>
+template <int P, bool SCATTER = false>
 cudaError_t launch_lng(const GemmMaps& m, int M, int K, const float* bias, const float* gamma,
                        const float* beta, float eps, const int32_t* seg_ids, float2* stats,
-                       int* cnt, cudaStream_t s, int* ready_out) {
+                       int* cnt, cudaStream_t s, int* ready_out, void* out_rows = nullptr,
+                       const int4* segtab = nullptr) {
   constexpr int kStageBytes = 2 * 128 * BK * 2;
   constexpr int kEpiBytes = kLncEpiWarps * kLncChunks * kStageBufBytes;
   constexpr int S = (227 * 1024 - 1024 - kEpiBytes - 1024) / kStageBytes;
   constexpr int kSmem = 1024 + S * kStageBytes + kEpiBytes + 1024;
   static_assert(kSmem <= 232448, "shared memory budget");
-  auto kern = linear_lng_kernel<P>;
+  auto kern = linear_lng_kernel<P, SCATTER>;
   static int max_pairs = 0;
   cudaLaunchConfig_t cfg{};
   cfg.blockDim = dim3(kLncThreads);
@@ -2091,7 +2118,11 @@ cudaError_t launch_lng(const GemmMaps& m, int M, int K, const float* bias, const
   // The P units of a tile must sit on P distinct pairs (a unit waits for its tile's other
   // units; two on one pair would wait for themselves): with fewer co-resident pairs than P
   // (an SM-limited context) use the cluster kernel instead.
-  if (max_pairs < P) return launch_lnc<P>(m, M, K, bias, gamma, beta, eps, seg_ids, s, ready_out);
+  if (max_pairs < P) {
+    if (SCATTER) return cudaErrorNotSupported;   // the caller unpacks separately
+    return launch_lnc<P>(m, M, K, bias, gamma, beta, eps, seg_ids, s, ready_out);
+  }
+  __nv_bfloat16* orow = static_cast<__nv_bfloat16*>(out_rows);
   // Tail split: when the last round of full units is partial, the row tiles after the last
   // complete round are cut into 2P half-width units -- if they then fit in one round of the
   // grid (C2: 256 units = 3 x 74 + 34 -> 222 full + 68 half; C3: 384 = 5 x 74 + 14 -> 369
@@ -2126,7 +2157,7 @@ cudaError_t launch_lng(const GemmMaps& m, int M, int K, const float* bias, const
   }
   const CUtensorMap& wh = m.has_w_half ? m.w_half : m.w;
   cudaError_t e = cudaLaunchKernelEx(&cfg, kern, m.a, m.w, m.c, m.r, wh, M, K, bias, gamma, beta, eps,
-                                     seg_ids, stats, cnt, ready_out, full_units);
+                                     seg_ids, stats, cnt, ready_out, full_units, orow, segtab);
   if (coop == -1) {
     coop = e == cudaSuccess ? 1 : 0;
     if (std::getenv("TCB_VERBOSE"))
@@ -2136,7 +2167,7 @@ cudaError_t launch_lng(const GemmMaps& m, int M, int K, const float* bias, const
       cudaGetLastError();
       --cfg.numAttrs;
       e = cudaLaunchKernelEx(&cfg, kern, m.a, m.w, m.c, m.r, wh, M, K, bias, gamma, beta, eps,
-                             seg_ids, stats, cnt, ready_out, full_units);
+                             seg_ids, stats, cnt, ready_out, full_units, orow, segtab);
     }
   }
   return e;
@@ -2160,8 +2191,17 @@ bool pdl_enabled() {
 cudaError_t launch_linear_ln_bf16_tc(const GemmMaps& m, int64_t M, int N, int K,
                                      const float* bias, const float* gamma, const float* beta,
                                      float eps, const int32_t* seg_ids, cudaStream_t s,
-                                     float2* lng_stats, int* lng_cnt, int* ready_out) {
+                                     float2* lng_stats, int* lng_cnt, int* ready_out,
+                                     void* scatter_out, const int4* segtab) {
   if (M == 0) return cudaSuccess;
+  if (scatter_out) {   // fused unpack: the L2-exchange kernel only (FFN2, K >= 2N)
+    if (!lng_stats || !lng_cnt || !segtab || !seg_ids || K < 2 * N) return cudaErrorNotSupported;
+    const int Mi = static_cast<int>(M);
+    if (N == 512) return launch_lng<2, true>(m, Mi, K, bias, gamma, beta, eps, seg_ids, lng_stats, lng_cnt, s, nullptr, scatter_out, segtab);
+    if (N == 768) return launch_lng<3, true>(m, Mi, K, bias, gamma, beta, eps, seg_ids, lng_stats, lng_cnt, s, nullptr, scatter_out, segtab);
+    if (N == 1024) return launch_lng<4, true>(m, Mi, K, bias, gamma, beta, eps, seg_ids, lng_stats, lng_cnt, s, nullptr, scatter_out, segtab);
+    return cudaErrorNotSupported;
+  }
   // d = 512 / 1024, K >= 2d (FFN2) with scratch: the L2-exchange kernel on all 74 pairs (the
   // 4- / 8-CTA cluster kernel fits on 132 / 120 SMs only): C4/C5 FFN2 262 -> 218 us.  At K = d (W_O) the
   // epilogue bounds the kernel and the L2 round trip of the statistics costs more than the

@@ -195,6 +195,42 @@ def test_forward_deterministic_and_graph_replay():
     assert torch.equal(rows, r1)
 
 
+@pytest.mark.parametrize("key,rows", [("c1", 0), ("c2", 256), ("c3", 8), ("c5", 16)])
+def test_forward_unpacked_equals_forward_plus_unpack(key, rows):
+    """tcb_encoder_forward_unpacked (the unpack fused into the last FFN2 + LN2 for bf16
+    d = 512 / 768 / 1024; the two calls for the fp32 toy) == tcb_encoder_forward + tcb_unpack,
+    bit for bit: same arithmetic, only the last layer's store goes to the request-order output.
+    Also through a stream (the internal graph) and with the output pre-filled with garbage (every
+    token row must be written)."""
+    wlc = wl.WORKLOADS[key]
+    model = wlc.model
+    if rows:
+        lengths, ids, w = wl.workload_inputs(key, rows=rows)
+    else:
+        lengths, ids, w = wl.workload_inputs(key)
+    enc = tcb.Encoder(model, w, wl.weight_names(model))
+    plan = tcb.tcb_pack(lengths, wlc.row_len, rows)
+    segtab = torch.from_numpy(plan.segtab()).cuda()
+    d_ids = torch.from_numpy(ids).cuda()
+    # both outputs pre-filled with NaN: rows of requests the plan could not place stay NaN in
+    # both (neither call writes them); any other unwritten row would differ
+    T = plan.info["total_tokens"]
+    nan = lambda: torch.full((T, model.d_model), float("nan"), device="cuda", dtype=enc.dtype)
+    ref = enc.unpack(plan, segtab, enc.encoder_forward(plan, segtab, d_ids), out=nan())
+    out = enc.encoder_forward_unpacked(plan, segtab, d_ids, nan())
+    torch.cuda.synchronize()
+    assert torch.equal(out.isnan(), ref.isnan())
+    assert torch.equal(torch.nan_to_num(out), torch.nan_to_num(ref))
+    s = torch.cuda.Stream()
+    out2 = nan()
+    with torch.cuda.stream(s):
+        for _ in range(2):                       # first call captures, second replays
+            enc.encoder_forward_unpacked(plan, segtab, d_ids, out2, stream=s)
+    torch.cuda.synchronize()
+    assert torch.equal(out2.isnan(), ref.isnan())
+    assert torch.equal(torch.nan_to_num(out2), torch.nan_to_num(ref))
+
+
 def test_empty_and_tiny_batches():
     model = wl.MODELS["transformer-base"]
     w = wl.draw_weights(model, 1)
