@@ -34,5 +34,6 @@ for wl in traffic:
                            "writes still resident in the 126 MB L2 when the kernel ends are not counted, so "
                            "the write side is a lower bound")
 json.dump(traffic, open(os.path.join(ROOT, "profiles", "traffic.json"), "w"), indent=1, sort_keys=True)
-open(os.path.join(ROOT, "profiles", "r02", "r02full_ncu_summary.txt"), "w").write("\n".join(lines) + "\n")
+summary = os.environ.get("SUMMARY", os.path.join("profiles", "r02", "r02full_ncu_summary.txt"))
+open(os.path.join(ROOT, summary), "w").write("\n".join(lines) + "\n")
 print("\n".join(lines))

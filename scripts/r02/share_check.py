@@ -16,14 +16,23 @@ ours = {k: v for k, v in agg.items() if any(m in k for m in match.values())}
 tot_n = sum(v[1] for v in ours.values())
 tot_b = sum(v["ms_per_step"] for v in r["classes"].values())
 print("%-10s %-34s %9s %9s %9s %9s" % ("class", "ncu kernel", "bench_sh", "ncu_sh", "bench_us", "ncu_us"))
+
+
+def agg_class(c):
+    """(launches, total us, names) over every ncu kernel of class c (e.g. both FFN2 variants:
+    the last layer's fused-unpack instantiation and the others)."""
+    ks = [k for k in ours if match[c] in k]
+    return sum(ours[k][0] for k in ks), sum(ours[k][1] for k in ks), "+".join(ks)
+
+
 for c, v in r["classes"].items():
-    k = next((k for k in ours if match[c] in k), None)
-    if k is None:
+    n, tot, name = agg_class(c)
+    if n == 0:
         continue
-    print("%-10s %-34s %9.4f %9.4f %9.2f %9.2f" % (c, k[:34], v["ms_per_step"] / tot_b, ours[k][1] / tot_n,
-                                                 v["us_per_launch"], ours[k][1] / ours[k][0]))
-k = next(k for k in ours if match[r["class"]] in k)
-ncu_us = ours[k][1] / ours[k][0]
+    print("%-10s %-34s %9.4f %9.4f %9.2f %9.2f" % (c, name[:34], v["ms_per_step"] / tot_b, tot / tot_n,
+                                                 v["us_per_launch"], tot / n))
+n, tot, _ = agg_class(r["class"])
+ncu_us = tot / n
 print("dominant %s: bench frac %.4f (%.2f us per launch in the graph-timed step); frac from the ncu "
       "average launch (%.2f us, cold cache) %.4f" % (r["class"], r["frac"], r["us_per_launch"], ncu_us,
                                                       r["work_per_launch"] / (ncu_us * 1e-6) / 1e12 / r["peak"]))
