@@ -504,7 +504,10 @@ tcb_status tcb_encoder_forward_unpacked(const tcb_weights* wc, const tcb_plan* p
                                         void* d_rows, void* d_out, void* d_ws, size_t ws_bytes,
                                         tcb_stream_t stream) {
   tcb::clear_error();
-  if (!d_out) return fail(TCB_ERR_INVALID_ARGUMENT, "tcb_encoder_forward_unpacked: d_out is NULL");
+  if (plan && plan->info.total_tokens > 0 && !d_out)
+    return fail(TCB_ERR_INVALID_ARGUMENT, "tcb_encoder_forward_unpacked: d_out is NULL");
+  if (plan && plan->info.total_tokens == 0)      // nothing to write: the plain forward
+    return forward_entry(wc, plan, d_segtab, d_token_ids, d_rows, nullptr, d_ws, ws_bytes, stream);
   return forward_entry(wc, plan, d_segtab, d_token_ids, d_rows, d_out, d_ws, ws_bytes, stream);
 }
 

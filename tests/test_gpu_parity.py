@@ -231,6 +231,28 @@ def test_forward_unpacked_equals_forward_plus_unpack(key, rows):
     assert torch.equal(torch.nan_to_num(out2), torch.nan_to_num(ref))
 
 
+@pytest.mark.parametrize("lengths,L", [([1], 8), ([7, 2, 3], 8), ([13, 1, 16, 5], 16), ([], 128)])
+def test_forward_unpacked_tiny_and_empty(lengths, L):
+    """The fused-unpack forward on one-slot requests, rows full to the last slot, a ragged
+    last tile and an empty batch: equal to forward + unpack."""
+    model = wl.MODELS["transformer-base"]
+    w = wl.draw_weights(model, 1)
+    enc = tcb.Encoder(model, w, wl.weight_names(model))
+    lengths = np.array(lengths, np.int32)
+    ids = wl.draw_token_ids(int(lengths.sum()), model.vocab, 3)
+    plan = tcb.tcb_pack(lengths, L, 0)
+    segtab = torch.from_numpy(plan.segtab()).cuda()
+    d_ids = torch.from_numpy(ids).cuda()
+    T = plan.info["total_tokens"]
+    out = torch.full((T, model.d_model), float("nan"), device="cuda", dtype=enc.dtype)
+    enc.encoder_forward_unpacked(plan, segtab, d_ids, out)
+    if T == 0:
+        return
+    ref = enc.unpack(plan, segtab, enc.encoder_forward(plan, segtab, d_ids))
+    torch.cuda.synchronize()
+    assert torch.equal(out, ref)
+
+
 def test_empty_and_tiny_batches():
     model = wl.MODELS["transformer-base"]
     w = wl.draw_weights(model, 1)
