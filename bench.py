@@ -410,6 +410,8 @@ def main():
     if world > 1:
         dist.barrier()
     step_ms = [a.elapsed_time(b) for a, b in ev]
+    if os.environ.get("TCB_BENCH_DUMP_STEPS"):            # diagnostics: per-step device times
+        print("step_ms " + " ".join("%.4f" % t for t in step_ms), file=sys.stderr, flush=True)
     ms = sum(step_ms)
     t_local = torch.tensor([ms, float(tokens_rank)], dtype=torch.float64, device=dev)
     if world > 1:
