@@ -33,7 +33,11 @@ namespace k {
 namespace {
 
 constexpr int BK = 64;                  // 64 bf16 = 128 bytes = one swizzle-128B row
-constexpr int kEpiWarps = 8;
+#ifndef TCB_GEMM_EPI_WARPS
+#define TCB_GEMM_EPI_WARPS 8
+#endif
+constexpr int kEpiWarps = TCB_GEMM_EPI_WARPS;          // 8 or 16: kEpiWarps / 4 column groups
+constexpr int kEpiGroups = kEpiWarps / 4;
 constexpr int kThreads = (4 + kEpiWarps) * 32;
 constexpr int kStageRows = 32, kStageCols = 32;            // epilogue staging box
 constexpr int kStageBufBytes = kStageRows * kStageCols * 2;  // 2 KB
@@ -45,7 +49,7 @@ struct TcCfg {
   static constexpr int kABytes = kRowsPerCta * BK * 2;
   static constexpr int kBBytes = kBRows * BK * 2;
   static constexpr int kStageBytes = kABytes + kBBytes;
-  static constexpr int kChunksPerWarp = BN / 64;             // 32-column chunks per warp/tile
+  static constexpr int kChunksPerWarp = BN / (32 * kEpiGroups);   // 32-column chunks per warp/tile
   // staging buffers per epilogue warp: one per chunk when the residual tile is prefetched,
   // else two (double-buffered TMA stores) so the freed smem deepens the operand ring
   static constexpr int kBufs = EPI == TCB_EPI_BIAS_RESIDUAL ? kChunksPerWarp
@@ -647,7 +651,7 @@ linear_tc_kernel(const __grid_constant__ CUtensorMap tmA, const __grid_constant_
     constexpr int NB = Cfg::kBufs;
     const int ew = warp - 4;
     const int q = warp & 3;                 // TMEM lane quarter this warp may access
-    const int half = ew >> 2;               // which half of the BN columns
+    const int half = ew >> 2;               // which column group (BN / kEpiGroups wide)
     const uint32_t bufs = smem_u32(sEpi) + ew * NB * kStageBufBytes;
     uint64_t* my_rbar = rbar + NB * ew;
     uint32_t rphase = 0;                    // phase of this warp's residual barriers
@@ -673,7 +677,7 @@ linear_tc_kernel(const __grid_constant__ CUtensorMap tmA, const __grid_constant_
       int m_blk, n_blk;
       tile_coords(tile, m_blocks, n_blocks, raster, m_blk, n_blk);
       const int row0 = m_blk * TILE_M + static_cast<int>(rank) * 128 + q * 32;
-      const int col0 = n_blk * BN + half * (BN / 2);
+      const int col0 = n_blk * BN + half * (BN / kEpiGroups);
       if constexpr (EPI == TCB_EPI_BIAS_RESIDUAL) {
         // every staging buffer is free once the previous tile's stores have read it; then
         // prefetch this tile's residual chunks while the MMAs run
@@ -703,7 +707,7 @@ linear_tc_kernel(const __grid_constant__ CUtensorMap tmA, const __grid_constant_
       ++pe_tiles;
 #endif
       const uint32_t tbase = tmem_base + (static_cast<uint32_t>(q * 32) << 16) +
-                             static_cast<uint32_t>(acc * BN + half * (BN / 2));
+                             static_cast<uint32_t>(acc * BN + half * (BN / kEpiGroups));
       uint32_t ra[32], rb[32];
       tmem_ld32_nowait(tbase, ra);
 #pragma unroll
