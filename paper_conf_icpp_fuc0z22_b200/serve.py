@@ -71,13 +71,11 @@ class Server:
         s.wait_stream(torch.cuda.current_stream())
         with torch.cuda.stream(s):
             for _ in range(2):
-                self.enc.encoder_forward(plan, self.d_segtab, self.d_ids, self.rows, stream=s)
-                self.enc.unpack(plan, self.d_segtab, self.rows, self.out, stream=s)
+                self.enc.encoder_forward_unpacked(plan, self.d_segtab, self.d_ids, self.out, self.rows, stream=s)
         s.synchronize()
         self.graph = torch.cuda.CUDAGraph()
         with torch.cuda.graph(self.graph, stream=s):
-            self.enc.encoder_forward(plan, self.d_segtab, self.d_ids, self.rows, stream=s)
-            self.enc.unpack(plan, self.d_segtab, self.rows, self.out, stream=s)
+            self.enc.encoder_forward_unpacked(plan, self.d_segtab, self.d_ids, self.out, self.rows, stream=s)
 
     def _capture_slot(self, k, plan) -> None:
         import torch
@@ -86,13 +84,11 @@ class Server:
         s.wait_stream(torch.cuda.current_stream())
         with torch.cuda.stream(s):
             for _ in range(2):
-                self.enc.encoder_forward(plan, d_seg, d_ids, self.rows, stream=s)
-                self.enc.unpack(plan, d_seg, self.rows, out, stream=s)
+                self.enc.encoder_forward_unpacked(plan, d_seg, d_ids, out, self.rows, stream=s)
         s.synchronize()
         g = torch.cuda.CUDAGraph()
         with torch.cuda.graph(g, stream=s):
-            self.enc.encoder_forward(plan, d_seg, d_ids, self.rows, stream=s)
-            self.enc.unpack(plan, d_seg, self.rows, out, stream=s)
+            self.enc.encoder_forward_unpacked(plan, d_seg, d_ids, out, self.rows, stream=s)
         self.graphs[k] = g
 
     def _run_overlap(self, lengths, arrival, deadline, token_ids, tok_offsets, horizon):
